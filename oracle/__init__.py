@@ -1,0 +1,219 @@
+"""oracle — TEST INFRASTRUCTURE ONLY.
+
+Plain CPU implementation of the OLAP hot path (Malik et al., IPDPSW 2012,
+/root/reference/PAPER.md), used to prove parity of the CUDA path.  Only
+``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline`` /
+``--impl reference`` legs may import this package.  It shares no code with
+``paper_conf_ipps_malikrse12_b200`` and never imports it.
+
+Functions (all cite the passage they follow in oracle.cpp):
+  query()      Eq. 1 / Eq. 3 / PAPER.md:25 — odometer sub-cube aggregation.
+  Dict         PAPER.md:252-256 — one std::map dictionary per text column.
+  factscan()   PAPER.md:206-208 — filtered aggregation over a fact table.
+  fill()       the counter-based cell generator (independent re-implementation).
+
+Parity of every function is pinned in tests/test_oracle_*.py against brute
+force (numpy slicing), an independent summed-area-table algorithm, the affine
+closed form, a hand-worked example and invariants; none is "parity unpinned".
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "oracle.cpp")
+_LIB = os.path.join(_HERE, "liboracle.so")
+
+INT32, FLOAT32 = 1, 2
+SUM, COUNT, MIN, MAX, AVG = 0, 1, 2, 3, 4
+GEN_UNIFORM, GEN_AFFINE = 1, 2
+RESULT_EMPTY = 1
+
+RESULT_DTYPE = np.dtype([("i", "<i8"), ("d", "<f8"), ("flags", "<u4"), ("pad", "<u4")])
+
+
+def build(force: bool = False) -> str:
+    """Compile oracle.cpp -> liboracle.so (g++ -O2 -fopenmp)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        cmd = ["g++", "-O2", "-std=c++17", "-fopenmp", "-shared", "-fPIC", _SRC, "-o", _LIB + ".tmp"]
+        subprocess.check_call(cmd)
+        os.replace(_LIB + ".tmp", _LIB)
+    return _LIB
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        L = ctypes.CDLL(build())
+        c_i64p = ctypes.POINTER(ctypes.c_int64)
+        L.oracle_splitmix64.restype = ctypes.c_uint64
+        L.oracle_splitmix64.argtypes = [ctypes.c_uint64, ctypes.c_uint64]
+        L.oracle_fill.restype = ctypes.c_int
+        L.oracle_fill.argtypes = [ctypes.c_int, c_i64p, ctypes.c_int, ctypes.c_int, ctypes.c_uint64,
+                                  ctypes.c_void_p, ctypes.c_int64, ctypes.c_int64, ctypes.c_void_p]
+        L.oracle_query.restype = ctypes.c_int
+        L.oracle_query.argtypes = [ctypes.c_int, c_i64p, ctypes.c_int, ctypes.c_void_p,
+                                   ctypes.c_int, ctypes.c_uint64, ctypes.c_void_p,
+                                   ctypes.c_int64, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                   ctypes.c_int, c_i64p]
+        L.oracle_max_threads.restype = ctypes.c_int
+        L.oracle_dict_build.restype = ctypes.c_void_p
+        L.oracle_dict_build.argtypes = [ctypes.c_char_p, c_i64p, ctypes.c_int64]
+        L.oracle_dict_size.restype = ctypes.c_int64
+        L.oracle_dict_size.argtypes = [ctypes.c_void_p]
+        L.oracle_dict_translate.restype = ctypes.c_int64
+        L.oracle_dict_translate.argtypes = [ctypes.c_void_p, ctypes.c_char_p, c_i64p, ctypes.c_int64,
+                                            ctypes.c_void_p]
+        L.oracle_dict_bound.restype = ctypes.c_int64
+        L.oracle_dict_bound.argtypes = [ctypes.c_void_p, ctypes.c_char_p, ctypes.c_int64, ctypes.c_int]
+        L.oracle_dict_lookup.restype = ctypes.c_int
+        L.oracle_dict_lookup.argtypes = [ctypes.c_void_p, ctypes.c_int32,
+                                         ctypes.POINTER(ctypes.c_char_p), c_i64p]
+        L.oracle_dict_destroy.restype = None
+        L.oracle_dict_destroy.argtypes = [ctypes.c_void_p]
+        L.oracle_factscan.restype = ctypes.c_int
+        L.oracle_factscan.argtypes = [ctypes.c_int64, ctypes.c_int, ctypes.c_void_p, ctypes.c_int,
+                                      ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p,
+                                      ctypes.c_void_p, ctypes.c_void_p]
+        _lib = L
+    return _lib
+
+
+def _i64(a):
+    a = np.ascontiguousarray(a, dtype=np.int64)
+    return a, a.ctypes.data_as(ctypes.POINTER(ctypes.c_int64))
+
+
+def _dtype_code(dt) -> int:
+    dt = np.dtype(dt)
+    if dt == np.int32:
+        return INT32
+    if dt == np.float32:
+        return FLOAT32
+    raise ValueError(f"unsupported cube dtype {dt}")
+
+
+def splitmix64(seed: int, idx: int) -> int:
+    return int(lib().oracle_splitmix64(seed, idx))
+
+
+def fill(extents, dtype, gen: int, seed: int = 0, params=None, first: int = 0, count: int | None = None):
+    """Cells [first, first+count) of a procedural cube, row-major."""
+    ext, ext_p = _i64(extents)
+    n = int(np.prod(ext)) if count is None else int(count)
+    out = np.empty(n, dtype=np.dtype(dtype))
+    par = np.ascontiguousarray(params if params is not None else np.zeros(len(ext) + 1), dtype=np.float64)
+    rc = lib().oracle_fill(len(ext), ext_p, _dtype_code(dtype), gen, seed, par.ctypes.data,
+                           first, n, out.ctypes.data)
+    if rc:
+        raise ValueError("oracle_fill failed")
+    return out
+
+
+def query(extents, ranges, ops, cells=None, *, dtype=None, gen: int = 0, seed: int = 0,
+          params=None, nthreads: int = 1):
+    """Answer queries on a host cube (cells: ndarray, row-major) or a procedural one.
+
+    ranges: int64 array (nq, nd, 2) of inclusive [lo, hi]; ops: int32 (nq,).
+    Returns a structured array with fields i, d, flags (RESULT_DTYPE).
+    """
+    ext, ext_p = _i64(extents)
+    nd = len(ext)
+    rng = np.ascontiguousarray(ranges, dtype=np.int64).reshape(-1, nd, 2)
+    nq = rng.shape[0]
+    opa = np.ascontiguousarray(ops, dtype=np.int32).reshape(nq)
+    out = np.zeros(nq, dtype=RESULT_DTYPE)
+    if cells is not None:
+        cells = np.ascontiguousarray(cells)
+        dt = _dtype_code(cells.dtype)
+        if cells.size != int(np.prod(ext)):
+            raise ValueError("cells size does not match extents")
+        cptr = cells.ctypes.data
+    else:
+        dt = _dtype_code(dtype)
+        cptr = None
+    par = np.ascontiguousarray(params if params is not None else np.zeros(nd + 1), dtype=np.float64)
+    bad = ctypes.c_int64(-1)
+    rc = lib().oracle_query(nd, ext_p, dt, cptr, gen, seed, par.ctypes.data, nq, rng.ctypes.data,
+                            opa.ctypes.data, out.ctypes.data, nthreads, ctypes.byref(bad))
+    if rc == -2:
+        raise IndexError(f"query {bad.value} out of bounds")
+    if rc:
+        raise ValueError("oracle_query: invalid arguments")
+    return out
+
+
+def max_threads() -> int:
+    return int(lib().oracle_max_threads())
+
+
+def _pack(keys):
+    keys = [k.encode() if isinstance(k, str) else bytes(k) for k in keys]
+    offs = np.zeros(len(keys) + 1, dtype=np.int64)
+    if keys:
+        offs[1:] = np.cumsum([len(k) for k in keys])
+    return b"".join(keys), offs
+
+
+class Dict:
+    """std::map text-to-integer dictionary of one text column."""
+
+    def __init__(self, keys):
+        blob, offs = _pack(keys)
+        self._h = lib().oracle_dict_build(blob, offs.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
+                                          len(offs) - 1)
+
+    def __len__(self):
+        return int(lib().oracle_dict_size(self._h))
+
+    def translate(self, keys):
+        blob, offs = _pack(keys)
+        ids = np.empty(len(offs) - 1, dtype=np.int32)
+        lib().oracle_dict_translate(self._h, blob, offs.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
+                                    len(ids), ids.ctypes.data)
+        return ids
+
+    def bound(self, key, upper: bool = False) -> int:
+        k = key.encode() if isinstance(key, str) else bytes(key)
+        return int(lib().oracle_dict_bound(self._h, k, len(k), 1 if upper else 0))
+
+    def lookup(self, i: int) -> bytes:
+        p = ctypes.c_char_p()
+        n = ctypes.c_int64()
+        if lib().oracle_dict_lookup(self._h, i, ctypes.byref(p), ctypes.byref(n)):
+            raise KeyError(i)
+        return ctypes.string_at(p, n.value)
+
+    def close(self):
+        if self._h:
+            lib().oracle_dict_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def factscan(dims, data, ranges):
+    """SUM and fact COUNT over rows of dims (nd, nrows) int32 whose values lie in ranges (nq, nd, 2)."""
+    dims = np.ascontiguousarray(dims, dtype=np.int32)
+    nd, nrows = dims.shape
+    data = np.ascontiguousarray(data)
+    rng = np.ascontiguousarray(ranges, dtype=np.int64).reshape(-1, nd, 2)
+    nq = rng.shape[0]
+    s = np.zeros(nq, dtype=np.int64)
+    c = np.zeros(nq, dtype=np.int64)
+    lib().oracle_factscan(nrows, nd, dims.ctypes.data, _dtype_code(data.dtype), data.ctypes.data, nq,
+                          rng.ctypes.data, s.ctypes.data, c.ctypes.data)
+    if data.dtype == np.float32:
+        s = s.view(np.float64)
+    return s, c
