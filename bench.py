@@ -1,0 +1,333 @@
+#!/usr/bin/env python3
+"""bench.py — OLAP sub-cube query throughput on B200 (BASELINE.json metric:
+"OLAP queries/sec and achieved HBM GB/s vs 8 TB/s at 1/2/4/8 B200").
+
+Workload (N=1): config C2a — 6-D float32 cube (16,16,16,16,16,256) = 1 GiB,
+device-filled with the counter-hash generator; every step answers one batch of
+4,096 synthetic queries (target fraction log-uniform in [1e-4,1], ops SUM 40% /
+MIN 20% / MAX 20% / AVG 10% / COUNT 10%) with inputs resident in HBM: plan ->
+persistent range-reduce -> finalize.  Each step draws a different batch.
+N>1 (torchrun, one rank per GPU): weak scaling — the global cube grows to
+(16N,16,16,16,16,256), block-cyclic dim-0 shards of 1 GiB per GPU, the same
+4,096-query batch recipe over the global cube; partials cross GPUs through one
+pair of NCCL all-reduces per batch.
+
+Prints ONE JSON line (rank 0).  `--impl reference` times the CPU oracle (the
+paper's OpenMP partition analogue) on the host cores instead.
+"""
+from __future__ import annotations
+
+import argparse
+import functools
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+METRIC = "OLAP queries/sec and achieved HBM GB/s vs 8 TB/s at 1/2/4/8 B200"
+NOMINAL_HBM_GBS = 8000.0
+
+
+def env_int(k, d):
+    try:
+        return int(os.environ.get(k, d))
+    except ValueError:
+        return d
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            j = json.load(f)
+        return float(j["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def workload(name: str, world: int):
+    cfg = synth.CONFIGS[name]
+    ext = list(cfg["extents"])
+    ext[0] *= world
+    return tuple(ext), cfg
+
+
+def batches(name, ext, nq, count, seed0):
+    out = []
+    for k in range(count):
+        b, o = synth.config_queries(name, nq=nq, seed=seed0 + 1000 + k, extents=ext)
+        out.append((b, o))
+    return out
+
+
+class Clocks:
+    """nvidia-smi sampler running during the timed region."""
+
+    def __init__(self, index: int):
+        self.proc = None
+        self.path = os.path.join(ROOT, "gpurun_out", f"clocks_{os.getpid()}.csv")
+        try:
+            os.makedirs(os.path.dirname(self.path), exist_ok=True)
+            self.f = open(self.path, "w")
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(index),
+                 "--query-gpu=clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+                 "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
+                 "--format=csv,noheader,nounits", "-lms", "100"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.f.close()
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in open(self.path):
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) < 8:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx = max(mx, float(parts[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[4:8]):
+                if v.lower() in ("active", "1"):
+                    reasons.add(n)
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def cpu_baseline(name, ext_global, cfg, seed, target_s=12.0, max_queries=None):
+    """The oracle as it stands, OpenMP over queries on all host cores, on a bounded
+    sample (the first n queries of the first batch, stopping after ~target_s)."""
+    import oracle
+    ext = cfg["extents"]  # a one-GPU cube; the oracle evaluates the global cube semantics on it
+    cells = _host_cells(tuple(ext), np.dtype(cfg["dtype"]).str, cfg["seed"])
+    b, o = synth.config_queries(name, nq=cfg["nq"], seed=seed, extents=ext)
+    threads = oracle.max_threads()
+    done, cells_read, t_used = 0, 0, 0.0
+    chunk = max(threads, 8)
+    t0 = time.perf_counter()
+    while done < len(b) and (time.perf_counter() - t0) < target_s:
+        if max_queries is not None and done >= max_queries:
+            break
+        bb, oo = b[done:done + chunk], o[done:done + chunk]
+        oracle.query(ext, bb, oo, cells, nthreads=threads)
+        vol = np.prod(bb[:, :, 1] - bb[:, :, 0] + 1, axis=1)
+        cells_read += int(vol[oo != synth.COUNT].sum())
+        done += len(bb)
+    t_used = time.perf_counter() - t0
+    return {
+        "value": done / t_used, "unit": "queries/s", "cores": threads, "kind": "oracle",
+        "gbs": cells_read * 4 / t_used / 1e9,
+        "sample": f"first {done} queries of a {name} batch on the 1-GPU cube {tuple(ext)}, "
+                  f"{cells_read * 4 / 2**30:.1f} GiB read, {t_used:.1f} s, OpenMP over queries",
+        "host": host_info(),
+    }
+
+
+@functools.lru_cache(maxsize=2)
+def _host_cells(ext, dtype_str, seed):
+    return synth.uniform_cells(int(np.prod(ext)), np.dtype(dtype_str), seed)
+
+
+def host_info():
+    model = ""
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"nproc": os.cpu_count(), "cpu": model, "OMP_NUM_THREADS": os.environ.get("OMP_NUM_THREADS")}
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return 0
+    ext, cfg = workload(args.workload, 1)
+    steps, warm = args.steps, args.warmup
+    # each step: a bounded sample of one batch (the full batch is ~444 GiB of reads)
+    vals = []
+    per_step = max(1.0, 60.0 / max(1, steps + warm))
+    for k in range(warm + steps):
+        cb = cpu_baseline(args.workload, ext, cfg, seed=cfg["seed"] + 1000 + k, target_s=per_step)
+        if k >= warm:
+            vals.append(cb)
+    q = sum(v["value"] for v in vals) / len(vals)
+    gbs = sum(v["gbs"] for v in vals) / len(vals)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": q, "unit": "queries/s", "n_gpus": world,
+        "steps": steps, "warmup": warm, "ms_per_step": 1000.0 / q * cfg["nq"], "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": args.workload, "extents": list(ext), "batch": cfg["nq"],
+                   "note": "oracle on a bounded sample per step; ms_per_step extrapolated to a full batch"},
+        "gbs": gbs,
+        "cpu_baseline": {"value": q, "unit": "queries/s", "cores": vals[0]["cores"], "kind": "oracle",
+                         "sample": vals[0]["sample"]},
+        "e2e": {"value": q, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="C2a", choices=["C2a", "C2b", "C3", "C1"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    args = ap.parse_args()
+
+    rank, world, local = env_int("RANK", 0), env_int("WORLD_SIZE", 1), env_int("LOCAL_RANK", 0)
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_malikrse12_b200 as olap
+    from paper_conf_ipps_malikrse12_b200.dist import exchange_partials
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    ext, cfg = workload(args.workload, world)
+    nq = cfg["nq"]
+    dtype = cfg["dtype"]
+    nd = len(ext)
+    cube = olap.Cube(ext, dtype, shard=(world, rank, 1) if world > 1 else None, device=local)
+    cube.fill(olap.GEN_UNIFORM, cfg["seed"])
+    host_batches = batches(args.workload, ext, nq, args.warmup + args.steps, cfg["seed"])
+    d_batches = [(torch.from_numpy(b).to(dev), torch.from_numpy(o).to(dev)) for b, o in host_batches]
+    res = torch.empty(nq * olap.RESULT_DTYPE.itemsize, dtype=torch.uint8, device=dev)
+    psum = torch.empty(nq, dtype=torch.int64, device=dev)
+    pext = torch.empty(2 * nq, dtype=torch.int32, device=dev)
+    stream = torch.cuda.Stream(device=dev)
+
+    def step(k):
+        dr, do = d_batches[k]
+        if world == 1:
+            cube.query_device(dr, do, res, nq=nq, stream=stream)
+        else:
+            cube.partials_device(dr, do, psum, pext, nq=nq, stream=stream)
+            with torch.cuda.stream(stream):
+                exchange_partials(psum, pext, cube.dtype_code)
+            olap.finalize_device(ext, cube.dtype_code, nq, dr, do, psum, pext, res, stream=stream)
+
+    with torch.cuda.stream(stream):
+        for k in range(args.warmup):
+            step(k)
+    stream.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    cube.profile(True)
+    clocks = Clocks(local)
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    with torch.cuda.stream(stream):
+        for k in range(args.warmup, args.warmup + args.steps):
+            step(k)
+    e1.record(stream)
+    e1.synchronize()
+    torch.cuda.synchronize()
+    elapsed_ms = e0.elapsed_time(e1)
+    clk = clocks.stop()
+    reduce_ms, launches, alg_bytes = cube.profile_read()
+    cube.profile(False)
+    t = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev)
+    tb = torch.tensor([alg_bytes], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(tb, op=dist.ReduceOp.SUM)
+    elapsed_ms = float(t.item())
+    total_bytes = float(tb.item())
+    total_q = nq * args.steps
+    qps = total_q / (elapsed_ms / 1e3)
+    gbs_total = total_bytes / (elapsed_ms / 1e3) / 1e9
+    peak, peak_src = measured_peaks()
+    achieved = (alg_bytes / max(launches, 1)) / (reduce_ms / max(launches, 1) / 1e3) / 1e9 if reduce_ms else 0.0
+
+    # end to end through the public host-buffer C-ABI (H2D of ranges/ops, D2H of results inside)
+    e2e = None
+    if world == 1 and args.e2e_steps > 0:
+        outs = np.zeros(nq, dtype=olap.RESULT_DTYPE)
+        b0, o0 = host_batches[0]
+        cube.query(b0, o0, out=outs)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for k in range(args.e2e_steps):
+            b, o = host_batches[args.warmup + (k % args.steps)]
+            cube.query(b, o, out=outs)
+        e2e_s = time.perf_counter() - t0
+        e2e = {"value": nq * args.e2e_steps / e2e_s, "unit": "queries/s",
+               "h2d_bytes_per_step": int(nq * nd * 16 + nq * 4), "d2h_bytes_per_step": int(nq * 24),
+               "api": "olap_query_batch (host buffers; pinned staging inside the library)"}
+    elif world > 1:
+        e2e = {"value": None, "unit": "queries/s", "h2d_bytes_per_step": int(nq * nd * 16 + nq * 4),
+               "d2h_bytes_per_step": int(nq * 24), "note": "host-buffer e2e measured at N=1 only"}
+
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        with open(tp) as f:
+            traffic = json.load(f).get(args.workload)
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(args.workload, ext, cfg, seed=cfg["seed"] + 1000 + args.warmup)
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": qps, "unit": "queries/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": args.workload, "extents": list(ext), "cube_gib_per_gpu":
+                       cube.info()[1] * 4 / 2**30, "batch": nq,
+                       "queries": "phi log-uniform [1e-4,1], l_d=max(1,round(n_d*phi^(1/6))); ops 40/20/20/10/10",
+                       "l2": "no flush: inputs > L2 (1 GiB cube/GPU, ~0.4 TiB read per step)",
+                       "accumulation": "f32 cells, f64 SUM", "parallelism": f"shard{world}" if world > 1 else "1gpu"},
+            "gbs": gbs_total, "frac_of_nominal_8tbs": gbs_total / world / NOMINAL_HBM_GBS,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic, "kernel": "reduce_kernel",
+                         "peak_source": peak_src,
+                         "reduce_share_of_step": reduce_ms / elapsed_ms if elapsed_ms else None},
+            "gpu_launches": int(args.steps * 3),
+            "clocks": clk,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,208 @@
+/*
+ * include/olap.h — C-ABI of the B200-native OLAP hot path.
+ *
+ * Method: Malik, Riha, Shea, El-Ghazawi, "Task Scheduling for GPU Accelerated
+ * Hybrid OLAP Systems with Multi-core Support and Text-to-Integer Translation",
+ * IPDPS Workshops 2012 (text at /root/reference/PAPER.md, cited as PAPER.md:line).
+ *
+ * The library answers batches of OLAP queries against a dense MOLAP cube held in
+ * B200 HBM.  A query is Eq. 1
+ *       Q(C_1(f_1,t_1), ..., C_N(f_N,t_N))
+ * restricted to one cube resolution (reading R14): one inclusive index range
+ * [f_i, t_i] per dimension plus one aggregate op from "count, sum, average,
+ * maximum etc." (MIN added per reading R4).  The answer aggregates
+ * every cell of the sub-cube ("area of limited search", PAPER.md:109-112,
+ * Fig. 2), whose volume is Eq. 3 (corrected to
+ * V = prod_i (t_i - f_i + 1), reading R1).  Text predicates are first translated
+ * to integer member ids through one dictionary per text column (§III-F,
+ * PAPER.md:252-256).
+ *
+ * Conventions (all functions):
+ *   - return an olap_status; out-parameters are written only on OLAP_OK;
+ *     olap_last_error() gives a thread-local message for the last failure.
+ *   - the caller owns every buffer it passes; the library copies what it keeps
+ *     before returning (the *_device variants are asynchronous on `stream` and
+ *     their buffers must stay live until that stream reaches the call).
+ *   - handles are owned by the library and released by *_destroy (NULL-safe).
+ *   - a handle is bound to the CUDA device it was created on; device pointers
+ *     passed to *_device calls must live on that device.
+ *   - a CUDA error maps to OLAP_E_CUDA (message names the call); bad arguments
+ *     to OLAP_E_INVALID; a query outside the cube to OLAP_E_RANGE (host-buffer
+ *     calls fail the whole batch and name the first bad query and dimension).
+ *   - the library never falls back to the CPU: without a usable CUDA device
+ *     every compute entry point returns OLAP_E_CUDA.
+ */
+#ifndef OLAP_H_
+#define OLAP_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct olap_cube olap_cube; /* opaque: one (shard of a) dense cube on one GPU */
+typedef struct olap_dict olap_dict; /* opaque: one text column's dictionary, immutable */
+
+typedef enum {
+    OLAP_OK = 0,
+    OLAP_E_INVALID = -1,     /* bad argument (NULL, ndims, dtype, op, sizes) */
+    OLAP_E_RANGE = -2,       /* a query range lies outside the cube */
+    OLAP_E_NOMEM = -3,       /* device or host allocation failed */
+    OLAP_E_CUDA = -4,        /* CUDA runtime error / no device */
+    OLAP_E_STATE = -6,       /* handle in the wrong state */
+    OLAP_E_UNSUPPORTED = -7
+} olap_status;
+
+typedef enum { OLAP_INT32 = 1, OLAP_FLOAT32 = 2 } olap_dtype; /* cell type, E_size = 4 B (Eq. 3) */
+
+typedef enum { OLAP_SUM = 0, OLAP_COUNT = 1, OLAP_MIN = 2, OLAP_MAX = 3, OLAP_AVG = 4 } olap_agg;
+
+typedef enum { OLAP_GEN_UNIFORM = 1, OLAP_GEN_AFFINE = 2 } olap_generator;
+
+#define OLAP_RESULT_EMPTY 1u   /* some f_i > t_i: the box is empty (COUNT 0, SUM 0)        */
+#define OLAP_RESULT_INVALID 2u /* *_device calls only: range out of bounds or bad op code    */
+
+/* One condition C_i(f_i, t_i) of Eq. 1: inclusive index range; lo > hi => empty box. */
+typedef struct { int64_t lo, hi; } olap_range;
+
+/* One answer.  int32 cube: i = SUM, COUNT, MIN, MAX (exact; SUM is int64 with
+ * two's-complement wraparound, reading R7), d = AVG.  float32 cube: d = SUM
+ * (fp64 accumulation), MIN, MAX, AVG; i = COUNT.  AVG = (double)SUM/(double)V.
+ * Fields not named for an op are 0. */
+typedef struct { int64_t i; double d; uint32_t flags; uint32_t _pad; } olap_result;
+
+/* Block-cyclic sharding of dimension 0 (reading R3 / DESIGN.md "layout"): global
+ * row r belongs to shard (r / block) % nshards and is stored at local row
+ * (r / (block*nshards))*block + r % block.  {1, 0, 1} (or NULL) = whole cube. */
+typedef struct { int64_t nshards, shard, block; } olap_shard;
+
+/* Per-query partial aggregates of one shard, structure-of-arrays in device
+ * memory, combinable across shards with two element-wise reductions:
+ *   sum[q]        int64: int32 cube -> wraparound sum (combine: +),
+ *                         float32 cube -> the bits of a double (combine: + as float64)
+ *   ext[2q+0]     int32: order-preserving code of the shard's MAX  (combine: max)
+ *   ext[2q+1]     int32: bitwise NOT of the code of its MIN        (combine: max)
+ * Identity (shard holds no cell of the box): sum 0, ext INT32_MIN.  The code of
+ * an int32 cell is the cell; of a float32 cell, its bits b ^ ((b >> 31) & 0x7fffffff). */
+
+/* ---------------------------------------------------------------- cube */
+
+/* Create an uninitialised cube (or one shard of it) of ndims in [1,8] with the
+ * given global extents (each >= 1), cell dtype, on CUDA `device`.  Layout:
+ * row-major, dimension 0 outermost (PAPER.md:111-112 leaves the structure open;
+ * reading R3).  OLAP_E_NOMEM if the shard does not fit in HBM. */
+int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_shard* shard,
+                     int device, olap_cube** out);
+
+/* Local geometry: owned dim-0 rows, owned cells, device pointer of the cells. */
+int olap_cube_info(const olap_cube* c, int64_t* local_rows, int64_t* local_cells, void** d_cells);
+
+/* Copy cells from a HOST array holding the FULL global cube in row-major order
+ * (ncells must equal the product of the extents); a shard copies its own rows. */
+int olap_cube_load(olap_cube* c, const void* cells, int64_t ncells);
+
+/* Copy global dim-0 rows [row_lo, row_hi) from a HOST buffer holding exactly
+ * those rows (row-major); rows not owned by this shard are skipped. */
+int olap_cube_load_rows(olap_cube* c, int64_t row_lo, int64_t row_hi, const void* cells);
+
+/* Fill on the device with a counter-based generator of the GLOBAL linear index i:
+ *   OLAP_GEN_UNIFORM: z = splitmix64(seed, i); int32 -> (z >> 43) - 2^20,
+ *                     float32 -> (z >> 40) * 2^-24
+ *   OLAP_GEN_AFFINE:  v(x) = params[0] + sum_d params[1+d] * x_d  (ndims+1 params). */
+int olap_cube_fill(olap_cube* c, int generator, uint64_t seed, const double* params);
+
+int olap_cube_destroy(olap_cube* c);
+
+/* ---------------------------------------------------------------- queries */
+
+/* Whole path on HOST buffers: validate, copy ranges (nq*ndims, query-major) and
+ * ops in, plan + range-reduce + finalize on the GPU, copy results out, sync.
+ * Only valid on an unsharded cube (nshards == 1).  nq == 0 is a no-op. */
+int olap_query_batch(olap_cube* c, int64_t nq, const olap_range* ranges, const int32_t* ops,
+                     olap_result* results);
+
+/* Same path on DEVICE buffers, asynchronous on `stream` (cudaStream_t, NULL =
+ * legacy default stream).  Invalid queries are flagged OLAP_RESULT_INVALID in
+ * their result instead of failing the batch.  Unsharded cubes only. */
+int olap_query_batch_device(olap_cube* c, int64_t nq, const olap_range* d_ranges,
+                            const int32_t* d_ops, olap_result* d_results, void* stream);
+
+/* Shard-local half of the path: plan + range-reduce of this shard's part of
+ * every query into partials (d_sum[nq], d_ext[2*nq], see above).  COUNT queries
+ * and boxes that miss the shard produce the identity.  Asynchronous. */
+int olap_query_partials_device(olap_cube* c, int64_t nq, const olap_range* d_ranges,
+                               const int32_t* d_ops, int64_t* d_sum, int32_t* d_ext, void* stream);
+
+/* Fold partials `in` into `acc` element-wise (the exchange's reduction, for
+ * shards that live on one device).  Asynchronous. */
+int olap_partials_combine_device(int dtype, int64_t nq, const int64_t* d_sum_in,
+                                 const int32_t* d_ext_in, int64_t* d_sum_acc, int32_t* d_ext_acc,
+                                 void* stream);
+
+/* Turn fully-combined partials into results: COUNT = V (global volume, Eq. 3),
+ * AVG = SUM/V, EMPTY / INVALID flags.  `extents` is a HOST array of the global
+ * extents.  Asynchronous. */
+int olap_finalize_device(int ndims, const int64_t* extents, int dtype, int64_t nq,
+                         const olap_range* d_ranges, const int32_t* d_ops, const int64_t* d_sum,
+                         const int32_t* d_ext, olap_result* d_results, void* stream);
+
+/* Host-only helper (no GPU needed): the local dim-0 range [*llo, *lhi] of global
+ * rows [lo, hi] on a shard of a dimension of n0 rows; *llo > *lhi if none. */
+int olap_shard_local_rows(int64_t n0, const olap_shard* shard, int64_t lo, int64_t hi,
+                          int64_t* llo, int64_t* lhi);
+
+/* Accumulated device time (CUDA events on the launching stream) and launch
+ * count of the range-reduce kernel since the last reset, plus the algorithmic
+ * bytes it read (sum over non-COUNT queries of V_local * 4, Eq. 3).  Timing is
+ * recorded only while enabled; enabling resets the counters. */
+int olap_cube_profile(olap_cube* c, int enable);
+int olap_cube_profile_read(olap_cube* c, double* reduce_ms, int64_t* launches, int64_t* bytes);
+
+/* ---------------------------------------------------------------- dictionaries */
+
+/* Build one text column's dictionary from n keys (key i = bytes[offsets[i],
+ * offsets[i+1]), HOST buffers, length-delimited, NUL not special, duplicates
+ * allowed).  Ids are the ranks of the distinct keys in byte-lexicographic
+ * (memcmp, shorter-prefix-first) order (reading R11).  The sorted arena and an
+ * open-addressing hash table are uploaded to `device`. */
+int olap_dict_build(const char* bytes, const int64_t* offsets, int64_t n, int device,
+                    olap_dict** out);
+
+int olap_dict_size(const olap_dict* d, int64_t* n_distinct);
+
+/* Translate n keys (HOST buffers) to ids on the GPU, key i looked up in
+ * dicts[dict_of_key[i]] (dict_of_key NULL => dicts[0]); ids_out[i] = -1 when
+ * absent (reading R13).  *n_missing (optional) = number of misses.  All dicts
+ * must live on one device. */
+int olap_dict_translate(const olap_dict* const* dicts, int ndicts, const int32_t* dict_of_key,
+                        const char* bytes, const int64_t* offsets, int64_t n, int32_t* ids_out,
+                        int64_t* n_missing);
+
+/* Same on DEVICE buffers (bytes, offsets[n+1], dict_of_key or NULL, ids_out),
+ * asynchronous on `stream`; d_n_missing (device int64, optional) is incremented. */
+int olap_dict_translate_device(const olap_dict* const* dicts, int ndicts,
+                               const int32_t* d_dict_of_key, const char* d_bytes,
+                               const int64_t* d_offsets, int64_t n, int32_t* d_ids_out,
+                               int64_t* d_n_missing, void* stream);
+
+/* For string-range conditions: out[i] = number of members < key i (upper = 0,
+ * lower_bound) or <= key i (upper = 1, upper_bound), by binary search on the
+ * GPU; HOST buffers.  A range [s1, s2] maps to ids [lower(s1), upper(s2) - 1]. */
+int olap_dict_bound(const olap_dict* d, const char* bytes, const int64_t* offsets, int64_t n,
+                    int upper, int32_t* out);
+
+/* Inverse: bytes of member `id` (pointer valid until the dict is destroyed). */
+int olap_dict_lookup(const olap_dict* d, int32_t id, const char** bytes, int64_t* len);
+
+int olap_dict_destroy(olap_dict* d);
+
+/* ---------------------------------------------------------------- misc */
+
+const char* olap_last_error(void); /* thread-local; valid until the next olap_* call */
+const char* olap_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* OLAP_H_ */

@@ -1,0 +1,333 @@
+"""paper_conf_ipps_malikrse12_b200 — B200-native OLAP sub-cube query hot path.
+
+Thin ctypes binding over ``libolap_b200.so`` whose C-ABI is ``include/olap.h``
+(Malik, Riha, Shea, El-Ghazawi, IPDPSW 2012; Eq. 1, Eq. 3, §III-F).
+This module only marshals arguments: every step of the path (planning,
+range-reduce, combine, finalize, dictionary translation) runs in the library's
+CUDA kernels.  There is no CPU fallback: if the library is missing, importing
+this package raises; if no GPU is usable, the compute calls raise OlapError.
+
+torch is used only for device memory and streams (tensors are passed by
+``data_ptr()``; streams by ``torch.cuda.Stream.cuda_stream``).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+__all__ = ["Cube", "Dict", "OlapError", "translate", "shard_local_rows", "combine_partials_device",
+           "finalize_device", "translate_device", "RESULT_DTYPE", "lib", "LIB_PATH",
+           "INT32", "FLOAT32", "SUM", "COUNT", "MIN", "MAX", "AVG", "GEN_UNIFORM", "GEN_AFFINE",
+           "RESULT_EMPTY", "RESULT_INVALID", "EXPORTS"]
+
+LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libolap_b200.so")
+
+INT32, FLOAT32 = 1, 2
+SUM, COUNT, MIN, MAX, AVG = 0, 1, 2, 3, 4
+GEN_UNIFORM, GEN_AFFINE = 1, 2
+RESULT_EMPTY, RESULT_INVALID = 1, 2
+
+OK, E_INVALID, E_RANGE, E_NOMEM, E_CUDA, E_STATE, E_UNSUPPORTED = 0, -1, -2, -3, -4, -6, -7
+
+# olap_result: {int64 i; double d; uint32 flags; uint32 _pad}
+RESULT_DTYPE = np.dtype([("i", "<i8"), ("d", "<f8"), ("flags", "<u4"), ("pad", "<u4")])
+
+_p = ctypes.c_void_p
+_i64 = ctypes.c_int64
+_i64p = ctypes.POINTER(ctypes.c_int64)
+_int = ctypes.c_int
+
+# every function declared in include/olap.h: name -> (restype, argtypes)
+EXPORTS = {
+    "olap_cube_create": (_int, [_int, _i64p, _int, _p, _int, ctypes.POINTER(_p)]),
+    "olap_cube_info": (_int, [_p, _i64p, _i64p, ctypes.POINTER(_p)]),
+    "olap_cube_load": (_int, [_p, _p, _i64]),
+    "olap_cube_load_rows": (_int, [_p, _i64, _i64, _p]),
+    "olap_cube_fill": (_int, [_p, _int, ctypes.c_uint64, _p]),
+    "olap_cube_destroy": (_int, [_p]),
+    "olap_query_batch": (_int, [_p, _i64, _p, _p, _p]),
+    "olap_query_batch_device": (_int, [_p, _i64, _p, _p, _p, _p]),
+    "olap_query_partials_device": (_int, [_p, _i64, _p, _p, _p, _p, _p]),
+    "olap_partials_combine_device": (_int, [_int, _i64, _p, _p, _p, _p, _p]),
+    "olap_finalize_device": (_int, [_int, _i64p, _int, _i64, _p, _p, _p, _p, _p, _p]),
+    "olap_shard_local_rows": (_int, [_i64, _p, _i64, _i64, _i64p, _i64p]),
+    "olap_cube_profile": (_int, [_p, _int]),
+    "olap_cube_profile_read": (_int, [_p, ctypes.POINTER(ctypes.c_double), _i64p, _i64p]),
+    "olap_dict_build": (_int, [_p, _i64p, _i64, _int, ctypes.POINTER(_p)]),
+    "olap_dict_size": (_int, [_p, _i64p]),
+    "olap_dict_translate": (_int, [_p, _int, _p, _p, _i64p, _i64, _p, _i64p]),
+    "olap_dict_translate_device": (_int, [_p, _int, _p, _p, _p, _i64, _p, _p, _p]),
+    "olap_dict_bound": (_int, [_p, _p, _i64p, _i64, _int, _p]),
+    "olap_dict_lookup": (_int, [_p, ctypes.c_int32, ctypes.POINTER(ctypes.c_char_p), _i64p]),
+    "olap_dict_destroy": (_int, [_p]),
+    "olap_last_error": (ctypes.c_char_p, []),
+    "olap_version": (ctypes.c_char_p, []),
+}
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_ipps_malikrse12_b200.build` "
+                          "(there is no CPU fallback)")
+    L = ctypes.CDLL(LIB_PATH)
+    for name, (res, args) in EXPORTS.items():
+        f = getattr(L, name)
+        f.restype = res
+        f.argtypes = args
+    L.olap_selftest_fastdiv.restype = _int
+    L.olap_selftest_fastdiv.argtypes = [ctypes.c_uint32, _p, _i64, _p]
+    L.olap_selftest_hash.restype = ctypes.c_uint64
+    L.olap_selftest_hash.argtypes = [ctypes.c_char_p, _i64]
+    return L
+
+
+lib = _load()
+
+
+class OlapError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        msg = lib.olap_last_error().decode(errors="replace")
+        super().__init__(f"{where}: status {status}: {msg}")
+
+
+def _check(rc: int, where: str):
+    if rc != OK:
+        raise OlapError(rc, where)
+
+
+def _ptr(x):
+    """device or host address of a torch tensor / numpy array / int / None"""
+    if x is None:
+        return None
+    if isinstance(x, int):
+        return x
+    if isinstance(x, np.ndarray):
+        return x.ctypes.data
+    return x.data_ptr()
+
+
+def _stream(stream):
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+def _dtype_code(dtype) -> int:
+    if isinstance(dtype, int):
+        return dtype
+    if isinstance(dtype, (type, np.dtype)):
+        dt = np.dtype(dtype)
+    else:
+        dt = np.dtype(str(dtype).replace("torch.", ""))
+    if dt == np.int32:
+        return INT32
+    if dt == np.float32:
+        return FLOAT32
+    raise ValueError(f"unsupported cell dtype {dtype}")
+
+
+class _Shard(ctypes.Structure):
+    _fields_ = [("nshards", ctypes.c_int64), ("shard", ctypes.c_int64), ("block", ctypes.c_int64)]
+
+
+def _shard(shard):
+    if shard is None:
+        return None
+    G, g, b = shard
+    return _Shard(G, g, b)
+
+
+def _i64arr(a):
+    a = np.ascontiguousarray(a, dtype=np.int64)
+    return a, a.ctypes.data_as(_i64p)
+
+
+class Cube:
+    """A dense cube (or one block-cyclic dim-0 shard of it) resident in one GPU's HBM."""
+
+    def __init__(self, extents, dtype, shard=None, device: int = 0):
+        self.extents = tuple(int(e) for e in extents)
+        self.ndims = len(self.extents)
+        self.dtype_code = _dtype_code(dtype)
+        self.np_dtype = np.int32 if self.dtype_code == INT32 else np.float32
+        self.shard = tuple(shard) if shard is not None else (1, 0, 1)
+        self.device = device
+        ext, extp = _i64arr(self.extents)
+        h = ctypes.c_void_p()
+        sh = _shard(shard)
+        _check(lib.olap_cube_create(self.ndims, extp, self.dtype_code, ctypes.byref(sh) if sh else None, device,
+                                    ctypes.byref(h)), "olap_cube_create")
+        self._h = h
+
+    @property
+    def handle(self):
+        return self._h
+
+    def info(self):
+        rows, cells, ptr = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_void_p()
+        _check(lib.olap_cube_info(self._h, ctypes.byref(rows), ctypes.byref(cells), ctypes.byref(ptr)),
+               "olap_cube_info")
+        return rows.value, cells.value, ptr.value
+
+    def load(self, cells: np.ndarray):
+        cells = np.ascontiguousarray(cells, dtype=self.np_dtype).reshape(-1)
+        _check(lib.olap_cube_load(self._h, cells.ctypes.data, cells.size), "olap_cube_load")
+
+    def load_rows(self, row_lo: int, row_hi: int, cells: np.ndarray):
+        cells = np.ascontiguousarray(cells, dtype=self.np_dtype).reshape(-1)
+        _check(lib.olap_cube_load_rows(self._h, row_lo, row_hi, cells.ctypes.data), "olap_cube_load_rows")
+
+    def fill(self, generator: int = GEN_UNIFORM, seed: int = 0, params=None):
+        par = None
+        if params is not None:
+            par = np.ascontiguousarray(params, dtype=np.float64)
+        _check(lib.olap_cube_fill(self._h, generator, seed & 0xFFFFFFFFFFFFFFFF,
+                                  par.ctypes.data if par is not None else None), "olap_cube_fill")
+
+    def query(self, ranges, ops, out: np.ndarray | None = None) -> np.ndarray:
+        """Host-buffer path (olap_query_batch): ranges (nq, ndims, 2) int64, ops (nq,) int32."""
+        rng = np.ascontiguousarray(ranges, dtype=np.int64).reshape(-1, self.ndims, 2)
+        nq = rng.shape[0]
+        opa = np.ascontiguousarray(ops, dtype=np.int32).reshape(nq)
+        res = out if out is not None else np.zeros(nq, dtype=RESULT_DTYPE)
+        _check(lib.olap_query_batch(self._h, nq, rng.ctypes.data, opa.ctypes.data, res.ctypes.data),
+               "olap_query_batch")
+        return res
+
+    def query_device(self, d_ranges, d_ops, d_results, nq: int | None = None, stream=None):
+        nq = d_ops.numel() if nq is None else nq
+        _check(lib.olap_query_batch_device(self._h, nq, _ptr(d_ranges), _ptr(d_ops), _ptr(d_results),
+                                           _stream(stream)), "olap_query_batch_device")
+
+    def partials_device(self, d_ranges, d_ops, d_sum, d_ext, nq: int | None = None, stream=None):
+        nq = d_ops.numel() if nq is None else nq
+        _check(lib.olap_query_partials_device(self._h, nq, _ptr(d_ranges), _ptr(d_ops), _ptr(d_sum), _ptr(d_ext),
+                                              _stream(stream)), "olap_query_partials_device")
+
+    def profile(self, enable: bool = True):
+        _check(lib.olap_cube_profile(self._h, 1 if enable else 0), "olap_cube_profile")
+
+    def profile_read(self):
+        ms, n, b = ctypes.c_double(), ctypes.c_int64(), ctypes.c_int64()
+        _check(lib.olap_cube_profile_read(self._h, ctypes.byref(ms), ctypes.byref(n), ctypes.byref(b)),
+               "olap_cube_profile_read")
+        return ms.value, n.value, b.value
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib.olap_cube_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def combine_partials_device(dtype, nq: int, sum_in, ext_in, sum_acc, ext_acc, stream=None):
+    _check(lib.olap_partials_combine_device(_dtype_code(dtype), nq, _ptr(sum_in), _ptr(ext_in), _ptr(sum_acc),
+                                            _ptr(ext_acc), _stream(stream)), "olap_partials_combine_device")
+
+
+def finalize_device(extents, dtype, nq: int, d_ranges, d_ops, d_sum, d_ext, d_results, stream=None):
+    ext, extp = _i64arr(extents)
+    _check(lib.olap_finalize_device(len(ext), extp, _dtype_code(dtype), nq, _ptr(d_ranges), _ptr(d_ops),
+                                    _ptr(d_sum), _ptr(d_ext), _ptr(d_results), _stream(stream)),
+           "olap_finalize_device")
+
+
+def shard_local_rows(n0: int, shard, lo: int, hi: int):
+    """(llo, lhi) local dim-0 range of global rows [lo, hi]; llo > lhi if the shard owns none."""
+    a, b = ctypes.c_int64(), ctypes.c_int64()
+    sh = _shard(shard)
+    _check(lib.olap_shard_local_rows(n0, ctypes.byref(sh) if sh else None, lo, hi, ctypes.byref(a), ctypes.byref(b)),
+           "olap_shard_local_rows")
+    return a.value, b.value
+
+
+def _pack(keys):
+    keys = [k.encode() if isinstance(k, str) else bytes(k) for k in keys]
+    offs = np.zeros(len(keys) + 1, dtype=np.int64)
+    if keys:
+        offs[1:] = np.cumsum([len(k) for k in keys])
+    blob = b"".join(keys)
+    buf = np.frombuffer(blob, dtype=np.uint8) if blob else np.zeros(1, np.uint8)
+    return np.ascontiguousarray(buf), offs
+
+
+class Dict:
+    """One text column's dictionary, resident on a GPU."""
+
+    def __init__(self, keys, device: int = 0):
+        buf, offs = _pack(keys)
+        h = ctypes.c_void_p()
+        _check(lib.olap_dict_build(buf.ctypes.data, offs.ctypes.data_as(_i64p), len(offs) - 1, device,
+                                   ctypes.byref(h)), "olap_dict_build")
+        self._h = h
+        self.device = device
+
+    @property
+    def handle(self):
+        return self._h
+
+    def __len__(self):
+        n = ctypes.c_int64()
+        _check(lib.olap_dict_size(self._h, ctypes.byref(n)), "olap_dict_size")
+        return n.value
+
+    def translate(self, keys):
+        return translate([self], None, keys)[0]
+
+    def bound(self, keys, upper: bool = False) -> np.ndarray:
+        buf, offs = _pack(keys)
+        out = np.empty(len(offs) - 1, dtype=np.int32)
+        _check(lib.olap_dict_bound(self._h, buf.ctypes.data, offs.ctypes.data_as(_i64p), len(out),
+                                   1 if upper else 0, out.ctypes.data), "olap_dict_bound")
+        return out
+
+    def lookup(self, i: int) -> bytes:
+        p, n = ctypes.c_char_p(), ctypes.c_int64()
+        _check(lib.olap_dict_lookup(self._h, i, ctypes.byref(p), ctypes.byref(n)), "olap_dict_lookup")
+        return ctypes.string_at(p, n.value)
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib.olap_dict_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def _dict_array(dicts):
+    arr = (ctypes.c_void_p * len(dicts))(*[d.handle.value for d in dicts])
+    return arr
+
+
+def translate(dicts, dict_of_key, keys):
+    """ids[i] of key i in dicts[dict_of_key[i]] (-1 if absent) and the number of misses."""
+    buf, offs = _pack(keys)
+    n = len(offs) - 1
+    ids = np.empty(n, dtype=np.int32)
+    dk = None if dict_of_key is None else np.ascontiguousarray(dict_of_key, dtype=np.int32)
+    miss = ctypes.c_int64()
+    _check(lib.olap_dict_translate(_dict_array(dicts), len(dicts), dk.ctypes.data if dk is not None else None,
+                                   buf.ctypes.data, offs.ctypes.data_as(_i64p), n, ids.ctypes.data,
+                                   ctypes.byref(miss)), "olap_dict_translate")
+    return ids, miss.value
+
+
+def translate_device(dicts, d_dict_of_key, d_bytes, d_offsets, n: int, d_ids, d_n_missing=None, stream=None):
+    _check(lib.olap_dict_translate_device(_dict_array(dicts), len(dicts), _ptr(d_dict_of_key), _ptr(d_bytes),
+                                          _ptr(d_offsets), n, _ptr(d_ids), _ptr(d_n_missing), _stream(stream)),
+           "olap_dict_translate_device")

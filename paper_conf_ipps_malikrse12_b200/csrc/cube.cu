@@ -1,0 +1,1207 @@
+// cube.cu — dense MOLAP cube in B200 HBM and the batched sub-cube range-reduce.
+//
+// Hot path per batch:
+//   plan_kernel      a1/a3/a4/a5  per query: validate, intersect with the shard,
+//                    linearise the box into runs (Fig. 2 "area of limited search",
+//                    PAPER.md:143,151), size work units and items, scan -> item table
+//   reduce_kernel    a6/a7        persistent grid, items popped from a device
+//                    counter; streams runs with 128-bit / 32-bit loads; per-item
+//                    partials, fixed-order per-query combine by the last block
+//   finalize_kernel  a9           COUNT = V (Eq. 3), AVG = SUM/V, flags
+// The per-query partial format (olap.h) is what crosses GPUs (a8).
+#include <algorithm>
+#include <climits>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <vector>
+
+#include "common.cuh"
+
+namespace olap {
+
+constexpr int kMaxDims = 8;
+constexpr int kMaxRunDims = 7;
+constexpr int kWarps = 8;                   // warps per reduce block
+constexpr int kThreads = kWarps * 32;
+constexpr int kPieceCells = 2048;           // MODE_VEC unit: <= 2048 cells (8 KiB) inside one run
+constexpr int kRunsPerBatch = 32;           // MODE_RUNS unit: 32 consecutive runs (one per lane)
+constexpr int64_t kVectorMinRun = 128;      // runs of >= 128 cells stream as 16-B vectors
+constexpr int64_t kItemCells = 262144;      // target item: 1 MiB of 4-byte cells
+constexpr int64_t kMaxExtent = (1ll << 30); // per-dimension limit (32-bit digit arithmetic)
+constexpr int64_t kMaxCells = (1ll << 42);
+
+enum : int32_t { MODE_NONE = 0, MODE_VEC = 1, MODE_RUNS = 2 };
+
+// Per-query plan (shard-local).  Run r of the box starts at
+//   base + sum_e digit_e(r) * rs[e]       (digits of r in radix frl[e].d, innermost first)
+// and covers L consecutive cells (all dims after the split dim k are full and merge).
+struct QDesc {
+    int64_t base;
+    int64_t L;
+    int64_t R;
+    int64_t units;
+    int64_t vlocal;
+    uint32_t upi;   // units per item
+    uint32_t ppr;   // pieces per run (MODE_VEC)
+    int32_t mode, nrd, op, pad;
+    FastDiv fL;     // / L (MODE_RUNS; L < 128)
+    FastDiv fppr;   // / ppr (MODE_VEC)
+    FastDiv frl[kMaxRunDims];
+    int64_t rs[kMaxRunDims];
+};
+
+struct Geo {
+    int nd, dtype;
+    int64_t G, g, b;
+    int64_t n[kMaxDims];       // global extents
+    int64_t stride[kMaxDims];  // local strides (cells)
+    int64_t local_rows;
+};
+
+struct Extents {
+    int64_t n[kMaxDims];
+};
+
+// ------------------------------------------------------------------ device helpers
+
+__device__ __forceinline__ uint4 ld_stream4(const void* p) {
+    uint4 r;
+    asm("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+        : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+        : "l"(p));
+    return r;
+}
+__device__ __forceinline__ uint32_t ld_stream1(const void* p) {
+    uint32_t r;
+    asm("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
+    return r;
+}
+
+__device__ __forceinline__ int32_t f32_code(float f) {
+    int32_t b = __float_as_int(f);
+    return b ^ ((b >> 31) & 0x7fffffff);
+}
+__host__ __device__ __forceinline__ float f32_decode(int32_t c) {
+    int32_t b = c ^ ((c >> 31) & 0x7fffffff);
+#ifdef __CUDA_ARCH__
+    return __int_as_float(b);
+#else
+    float f;
+    std::memcpy(&f, &b, 4);
+    return f;
+#endif
+}
+
+// Per-lane accumulators.  int32 cells: SUM in uint64 (wraparound, reading R7),
+// MIN/MAX in int32.  float32 cells: SUM in double (reading R8), MIN/MAX in float.
+struct AccI {
+    unsigned long long s;
+    int32_t mn, mx;
+    __device__ void init() { s = 0ull; mn = INT_MAX; mx = INT_MIN; }
+    __device__ __forceinline__ void add1(uint32_t bits) {
+        int32_t v = (int32_t)bits;
+        s += (unsigned long long)(long long)v;
+        mn = min(mn, v);
+        mx = max(mx, v);
+    }
+    __device__ __forceinline__ void add4(uint4 v) { add1(v.x); add1(v.y); add1(v.z); add1(v.w); }
+    __device__ __forceinline__ long long sum_bits() const { return (long long)s; }
+    __device__ __forceinline__ int32_t code_max() const { return mx; }
+    __device__ __forceinline__ int32_t code_min() const { return mn; }
+};
+struct AccF {
+    double s;
+    float mn, mx;
+    __device__ void init() { s = 0.0; mn = __int_as_float(0x7f800000); mx = __int_as_float(0xff800000); }
+    __device__ __forceinline__ void add1(uint32_t bits) {
+        float v = __uint_as_float(bits);
+        s += (double)v;
+        mn = fminf(mn, v);
+        mx = fmaxf(mx, v);
+    }
+    __device__ __forceinline__ void add4(uint4 v) { add1(v.x); add1(v.y); add1(v.z); add1(v.w); }
+    __device__ __forceinline__ long long sum_bits() const { return __double_as_longlong(s); }
+    __device__ __forceinline__ int32_t code_max() const { return f32_code(mx); }
+    __device__ __forceinline__ int32_t code_min() const { return f32_code(mn); }
+};
+
+template <class Acc> struct SumOps;
+template <> struct SumOps<AccI> {
+    __device__ static long long add(long long a, long long b) {
+        return (long long)((unsigned long long)a + (unsigned long long)b);
+    }
+};
+template <> struct SumOps<AccF> {
+    __device__ static long long add(long long a, long long b) {
+        return __double_as_longlong(__longlong_as_double(a) + __longlong_as_double(b));
+    }
+};
+
+// Advance a run cursor by `inc` runs (inc < 2^20): add to the mixed-radix digits with carry.
+__device__ __forceinline__ void advance_runs(const QDesc& d, uint32_t (&dig)[kMaxRunDims], int64_t& addr,
+                                             uint32_t inc) {
+    uint32_t c = inc;
+#pragma unroll
+    for (int e = 0; e < kMaxRunDims; ++e) {
+        if (e < d.nrd && c != 0u) {
+            uint32_t t = dig[e] + c;
+            uint32_t q = fdiv(t, d.frl[e]);
+            uint32_t nd = t - q * d.frl[e].d;
+            addr += ((int64_t)nd - (int64_t)dig[e]) * d.rs[e];
+            dig[e] = nd;
+            c = q;
+        }
+    }
+}
+
+// Full decode of run index r (64-bit divisions; once per item).
+__device__ void decode_run(const QDesc& d, int64_t r, uint32_t (&dig)[kMaxRunDims], int64_t& addr) {
+    addr = d.base;
+#pragma unroll
+    for (int e = 0; e < kMaxRunDims; ++e) {
+        dig[e] = 0u;
+        if (e < d.nrd) {
+            uint32_t l = d.frl[e].d;
+            int64_t q = r / l;
+            uint32_t di = (uint32_t)(r - q * l);
+            dig[e] = di;
+            addr += (int64_t)di * d.rs[e];
+            r = q;
+        }
+    }
+}
+
+// One warp streams cells [a, a+len) (len <= kPieceCells): scalar head to 16-B
+// alignment, 16-B vector body (4 independent loads in flight per lane), scalar tail.
+template <class Acc, typename T>
+__device__ __forceinline__ void stream_piece(const T* __restrict__ cube, int64_t a, int len, Acc& acc,
+                                             int lane) {
+    int head = (int)((4 - (a & 3)) & 3);
+    if (head > len) head = len;
+    if (lane < head) acc.add1(ld_stream1(cube + a + lane));
+    a += head;
+    len -= head;
+    const int nvec = len >> 2;
+    const uint4* v = reinterpret_cast<const uint4*>(cube + a);
+    int i = lane;
+    for (; i + 96 < nvec; i += 128) {
+        uint4 x0 = ld_stream4(v + i);
+        uint4 x1 = ld_stream4(v + i + 32);
+        uint4 x2 = ld_stream4(v + i + 64);
+        uint4 x3 = ld_stream4(v + i + 96);
+        acc.add4(x0);
+        acc.add4(x1);
+        acc.add4(x2);
+        acc.add4(x3);
+    }
+    for (; i < nvec; i += 32) acc.add4(ld_stream4(v + i));
+    const int tail = len & 3;
+    if (lane < tail) acc.add1(ld_stream1(cube + a + 4 * (int64_t)nvec + lane));
+}
+
+// Largest q in [0,nq) with item_start[q] <= item (32-ary warp search).
+__device__ __forceinline__ int64_t find_query(const int64_t* __restrict__ item_start, int64_t nq, int64_t item,
+                                              int lane) {
+    int64_t lo = 0, hi = nq;
+    while (hi - lo > 32) {
+        const int64_t step = (hi - lo + 31) / 32;
+        const int64_t idx = lo + lane * step;
+        const bool ok = idx < hi && __ldg(item_start + idx) <= item;
+        const unsigned m = __ballot_sync(0xffffffffu, ok);
+        const int l = 31 - __clz(m);
+        lo = lo + l * step;
+        hi = min(hi, lo + step);
+    }
+    const int64_t idx = lo + lane;
+    const bool ok = idx < hi && __ldg(item_start + idx) <= item;
+    const unsigned m = __ballot_sync(0xffffffffu, ok);
+    return lo + (31 - __clz(m));
+}
+
+// ------------------------------------------------------------------ plan
+
+__device__ void build_desc(const Geo& g, const olap_range* r, int32_t op, QDesc& d) {
+    d.mode = MODE_NONE;
+    d.op = op;
+    d.vlocal = 0;
+    d.units = 0;
+    d.nrd = 0;
+    d.upi = 1;
+    if (op < OLAP_SUM || op > OLAP_AVG) return;
+    int64_t lo[kMaxDims], hi[kMaxDims];
+    bool empty = false;
+    for (int k = 0; k < g.nd; ++k) {
+        lo[k] = r[k].lo;
+        hi[k] = r[k].hi;
+        if (lo[k] < 0 || hi[k] >= g.n[k]) return;  // invalid: flagged by finalize
+        if (lo[k] > hi[k]) empty = true;
+    }
+    if (empty || op == OLAP_COUNT) return;
+    int64_t llo, lhi;
+    if (!shard_local_range(g.n[0], g.G, g.g, g.b, lo[0], hi[0], &llo, &lhi)) return;
+    lo[0] = llo;
+    hi[0] = lhi;
+    int64_t ell[kMaxDims];
+    for (int k = 0; k < g.nd; ++k) ell[k] = hi[k] - lo[k] + 1;
+    int ks = g.nd - 1;  // split dim: innermost dim not fully covered
+    while (ks > 0 && ell[ks] == (ks == 0 ? g.local_rows : g.n[ks])) --ks;
+    d.L = ell[ks] * g.stride[ks];
+    int64_t R = 1, base = 0;
+    for (int k = 0; k < g.nd; ++k) base += lo[k] * g.stride[k];
+    int nrd = 0;
+    for (int k = ks - 1; k >= 0; --k) {
+        R *= ell[k];
+        if (ell[k] > 1) {
+            d.frl[nrd] = FastDiv{};
+            uint32_t l = (uint32_t)ell[k];
+            // device-side make_fastdiv
+            FastDiv f;
+            f.d = l;
+            if (l <= 1) {
+                f.m = 0;
+                f.s = 0xffffffffu;
+            } else {
+                uint32_t lg = 32 - __clz(l - 1);
+                uint32_t p = 31 + lg;
+                f.m = (uint32_t)(((1ull << p) + l - 1) / l);
+                f.s = p - 32;
+            }
+            d.frl[nrd] = f;
+            d.rs[nrd] = g.stride[k];
+            ++nrd;
+        }
+    }
+    d.nrd = nrd;
+    d.R = R;
+    d.base = base;
+    d.vlocal = R * d.L;
+    if (d.L >= kVectorMinRun) {
+        d.mode = MODE_VEC;
+        int64_t ppr = (d.L + kPieceCells - 1) / kPieceCells;
+        d.ppr = (uint32_t)ppr;
+        uint32_t l = (uint32_t)ppr;
+        FastDiv f;
+        f.d = l;
+        if (l <= 1) {
+            f.m = 0;
+            f.s = 0xffffffffu;
+        } else {
+            uint32_t lg = 32 - __clz(l - 1);
+            uint32_t p = 31 + lg;
+            f.m = (uint32_t)(((1ull << p) + l - 1) / l);
+            f.s = p - 32;
+        }
+        d.fppr = f;
+        d.units = R * ppr;
+    } else {
+        d.mode = MODE_RUNS;
+        uint32_t l = (uint32_t)d.L;
+        FastDiv f;
+        f.d = l;
+        if (l <= 1) {
+            f.m = 0;
+            f.s = 0xffffffffu;
+        } else {
+            uint32_t lg = 32 - __clz(l - 1);
+            uint32_t p = 31 + lg;
+            f.m = (uint32_t)(((1ull << p) + l - 1) / l);
+            f.s = p - 32;
+        }
+        d.fL = f;
+        d.ppr = 1;
+        d.units = (R + kRunsPerBatch - 1) / kRunsPerBatch;
+    }
+}
+
+constexpr int kPlanThreads = 1024;
+
+template <typename V>
+__device__ V block_sum(V v, V* sh) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if (lane == 0) sh[w] = v;
+    __syncthreads();
+    V t = 0;
+    if (threadIdx.x < 32) {
+        t = threadIdx.x < (blockDim.x >> 5) ? sh[threadIdx.x] : V(0);
+#pragma unroll
+        for (int o = 16; o; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+        if (threadIdx.x == 0) sh[0] = t;
+    }
+    __syncthreads();
+    t = sh[0];
+    __syncthreads();
+    return t;
+}
+
+// One block: descriptors, adaptive item size, exclusive scan of item counts.
+__global__ void __launch_bounds__(kPlanThreads) plan_kernel(Geo geo, int64_t nq, const olap_range* __restrict__ ranges,
+                                                            const int32_t* __restrict__ ops, QDesc* desc,
+                                                            int64_t* item_start, int32_t* done,
+                                                            unsigned long long* counter, int64_t* psum,
+                                                            int32_t* pext, int64_t items_cap,
+                                                            unsigned long long* bytes_acc) {
+    __shared__ int64_t sh[32];
+    const int tid = threadIdx.x;
+    const int64_t per = (nq + kPlanThreads - 1) / kPlanThreads;
+    const int64_t q0 = min(nq, (int64_t)tid * per), q1 = min(nq, q0 + per);
+    int64_t my_cells = 0;
+    for (int64_t q = q0; q < q1; ++q) {
+        QDesc d;
+        build_desc(geo, ranges + q * geo.nd, ops[q], d);
+        desc[q] = d;
+        done[q] = 0;
+        if (d.mode == MODE_NONE) {
+            psum[q] = 0;
+            pext[2 * q] = INT_MIN;
+            pext[2 * q + 1] = INT_MIN;
+        }
+        my_cells += d.vlocal;
+    }
+    const int64_t total_cells = block_sum<int64_t>(my_cells, sh);
+    const int64_t cap_left = items_cap - 2 * nq;
+    int64_t teff = (4 * total_cells + cap_left - 1) / cap_left;
+    if (teff < kItemCells) teff = kItemCells;
+    int64_t my_items = 0;
+    for (int64_t q = q0; q < q1; ++q) {
+        QDesc& d = desc[q];
+        int64_t items = 0;
+        if (d.mode != MODE_NONE) {
+            const int64_t unit_cells = d.mode == MODE_VEC ? (int64_t)kPieceCells : kRunsPerBatch * d.L;
+            int64_t upi = teff / unit_cells;
+            if (upi < 1) upi = 1;
+            if (upi > (1ll << 30)) upi = (1ll << 30);
+            d.upi = (uint32_t)upi;
+            items = (d.units + upi - 1) / upi;
+        }
+        item_start[q] = items;
+        my_items += items;
+    }
+    // exclusive scan of my_items over the block
+    __shared__ int64_t scan[kPlanThreads];
+    scan[tid] = my_items;
+    __syncthreads();
+    for (int o = 1; o < kPlanThreads; o <<= 1) {
+        int64_t v = tid >= o ? scan[tid - o] : 0;
+        __syncthreads();
+        scan[tid] += v;
+        __syncthreads();
+    }
+    int64_t off = scan[tid] - my_items;
+    for (int64_t q = q0; q < q1; ++q) {
+        const int64_t items = item_start[q];
+        item_start[q] = off;
+        off += items;
+    }
+    if (tid == kPlanThreads - 1) {
+        item_start[nq] = scan[tid];
+        *counter = 0ull;
+        atomicAdd(bytes_acc, (unsigned long long)(total_cells * 4));
+    }
+}
+
+// ------------------------------------------------------------------ reduce (the hot loop)
+
+template <typename T, class Acc>
+__global__ void __launch_bounds__(kThreads) reduce_kernel(const T* __restrict__ cube, int64_t nq,
+                                                          const QDesc* __restrict__ desc,
+                                                          const int64_t* __restrict__ item_start,
+                                                          unsigned long long* counter, int32_t* done,
+                                                          long long* item_sum, int32_t* item_ext,
+                                                          int64_t* psum, int32_t* pext) {
+    __shared__ QDesc sd;
+    __shared__ int64_t s_item, s_q, s_r0, s_addr0;
+    __shared__ uint32_t s_p0, s_dig0[kMaxRunDims];
+    __shared__ long long s_wsum[kWarps];
+    __shared__ int32_t s_wmx[kWarps], s_wmn[kWarps];
+    __shared__ int s_last;
+
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t total = __ldg(item_start + nq);
+
+    for (;;) {
+        if (threadIdx.x == 0) s_item = (int64_t)atomicAdd(counter, 1ull);
+        __syncthreads();
+        const int64_t item = s_item;
+        if (item >= total) break;
+        if (w == 0) {
+            const int64_t q = find_query(item_start, nq, item, lane);
+            if (lane == 0) s_q = q;
+        }
+        __syncthreads();
+        const int64_t q = s_q;
+        {
+            const int* src = reinterpret_cast<const int*>(desc + q);
+            int* dst = reinterpret_cast<int*>(&sd);
+            for (int i = threadIdx.x; i < (int)(sizeof(QDesc) / 4); i += kThreads) dst[i] = __ldg(src + i);
+        }
+        __syncthreads();
+        const int64_t first_item = __ldg(item_start + q);
+        const int64_t u0 = (item - first_item) * (int64_t)sd.upi;
+        const int64_t u1 = min(sd.units, u0 + (int64_t)sd.upi);
+        if (threadIdx.x == 0) {
+            uint32_t dig[kMaxRunDims];
+            int64_t addr, r0;
+            if (sd.mode == MODE_VEC) {
+                r0 = u0 / sd.ppr;
+                s_p0 = (uint32_t)(u0 - r0 * sd.ppr);
+            } else {
+                r0 = u0 * kRunsPerBatch;
+                s_p0 = 0;
+            }
+            decode_run(sd, r0, dig, addr);
+            s_r0 = r0;
+            s_addr0 = addr;
+#pragma unroll
+            for (int e = 0; e < kMaxRunDims; ++e) s_dig0[e] = dig[e];
+        }
+        __syncthreads();
+
+        Acc acc;
+        acc.init();
+        uint32_t dig[kMaxRunDims];
+#pragma unroll
+        for (int e = 0; e < kMaxRunDims; ++e) dig[e] = s_dig0[e];
+        int64_t addr = s_addr0;
+
+        if (sd.mode == MODE_VEC) {
+            const uint32_t ppr = sd.ppr;
+            uint32_t p = s_p0 + (uint32_t)w;
+            if (p >= ppr) {
+                const uint32_t dr = fdiv(p, sd.fppr);
+                p -= dr * ppr;
+                advance_runs(sd, dig, addr, dr);
+            }
+            for (int64_t u = u0 + w; u < u1; u += kWarps) {
+                const int64_t off = (int64_t)p * kPieceCells;
+                const int64_t rem = sd.L - off;
+                const int len = rem < kPieceCells ? (int)rem : kPieceCells;
+                stream_piece(cube, addr + off, len, acc, lane);
+                p += kWarps;
+                if (p >= ppr) {
+                    const uint32_t dr = fdiv(p, sd.fppr);
+                    p -= dr * ppr;
+                    advance_runs(sd, dig, addr, dr);
+                }
+            }
+        } else {
+            // lane owns run (first run of the warp's batch) + lane
+            const int64_t R = sd.R;
+            const int L = (int)sd.L;
+            advance_runs(sd, dig, addr, (uint32_t)(w * kRunsPerBatch + lane));
+            for (int64_t u = u0 + w; u < u1; u += kWarps) {
+                const int64_t rfirst = u * kRunsPerBatch;
+                const int64_t nr64 = R - rfirst;
+                const int nr = nr64 < kRunsPerBatch ? (int)nr64 : kRunsPerBatch;
+                const int ncell = nr * L;
+                for (int c0 = 0; c0 < ncell; c0 += 128) {
+                    uint32_t v[4];
+                    bool ok[4];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const int c = c0 + j * 32 + lane;
+                        ok[j] = c < ncell;
+                        const int cc = ok[j] ? c : 0;
+                        const uint32_t ri = fdiv((uint32_t)cc, sd.fL);
+                        const int o = cc - (int)ri * L;
+                        const int64_t a = __shfl_sync(0xffffffffu, addr, (int)ri) + o;
+                        v[j] = ok[j] ? ld_stream1(cube + a) : 0u;
+                    }
+#pragma unroll
+                    for (int j = 0; j < 4; ++j)
+                        if (ok[j]) acc.add1(v[j]);
+                }
+                advance_runs(sd, dig, addr, (uint32_t)(kWarps * kRunsPerBatch));
+            }
+        }
+
+        // warp -> block -> item partial (fixed order: deterministic)
+        long long s = acc.sum_bits();
+        int32_t cmx = acc.code_max(), cmn = ~acc.code_min();
+#pragma unroll
+        for (int o = 16; o; o >>= 1) s = SumOps<Acc>::add(s, __shfl_xor_sync(0xffffffffu, s, o));
+        cmx = __reduce_max_sync(0xffffffffu, cmx);
+        cmn = __reduce_max_sync(0xffffffffu, cmn);
+        if (lane == 0) {
+            s_wsum[w] = s;
+            s_wmx[w] = cmx;
+            s_wmn[w] = cmn;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            long long ts = s_wsum[0];
+            int32_t tmx = s_wmx[0], tmn = s_wmn[0];
+#pragma unroll
+            for (int i = 1; i < kWarps; ++i) {
+                ts = SumOps<Acc>::add(ts, s_wsum[i]);
+                tmx = max(tmx, s_wmx[i]);
+                tmn = max(tmn, s_wmn[i]);
+            }
+            item_sum[item] = ts;
+            item_ext[2 * item] = tmx;
+            item_ext[2 * item + 1] = tmn;
+            __threadfence();
+            const int64_t nitems = (sd.units + sd.upi - 1) / sd.upi;
+            const int prev = atomicAdd(done + q, 1);
+            s_last = (prev == (int)nitems - 1);
+        }
+        __syncthreads();
+        if (s_last) {
+            // last finisher of query q: fold its item partials in fixed order
+            __threadfence();
+            const int64_t nitems = (sd.units + sd.upi - 1) / sd.upi;
+            long long ts = 0;
+            int32_t tmx = INT_MIN, tmn = INT_MIN;
+            for (int64_t i = threadIdx.x; i < nitems; i += kThreads) {
+                const int64_t it = first_item + i;
+                ts = SumOps<Acc>::add(ts, __ldcg(item_sum + it));
+                tmx = max(tmx, __ldcg(item_ext + 2 * it));
+                tmn = max(tmn, __ldcg(item_ext + 2 * it + 1));
+            }
+#pragma unroll
+            for (int o = 16; o; o >>= 1) ts = SumOps<Acc>::add(ts, __shfl_xor_sync(0xffffffffu, ts, o));
+            tmx = __reduce_max_sync(0xffffffffu, tmx);
+            tmn = __reduce_max_sync(0xffffffffu, tmn);
+            if (lane == 0) {
+                s_wsum[w] = ts;
+                s_wmx[w] = tmx;
+                s_wmn[w] = tmn;
+            }
+            __syncthreads();
+            if (threadIdx.x == 0) {
+                long long fs = s_wsum[0];
+                int32_t fmx = s_wmx[0], fmn = s_wmn[0];
+#pragma unroll
+                for (int i = 1; i < kWarps; ++i) {
+                    fs = SumOps<Acc>::add(fs, s_wsum[i]);
+                    fmx = max(fmx, s_wmx[i]);
+                    fmn = max(fmn, s_wmn[i]);
+                }
+                psum[q] = fs;
+                pext[2 * q] = fmx;
+                pext[2 * q + 1] = fmn;
+            }
+        }
+        __syncthreads();
+    }
+}
+
+// ------------------------------------------------------------------ finalize / combine
+
+__global__ void finalize_kernel(int nd, Extents ext, int dtype, int64_t nq, const olap_range* __restrict__ ranges,
+                                const int32_t* __restrict__ ops, const int64_t* __restrict__ psum,
+                                const int32_t* __restrict__ pext, olap_result* __restrict__ out) {
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nq; q += (int64_t)gridDim.x * blockDim.x) {
+        olap_result r;
+        r.i = 0;
+        r.d = 0.0;
+        r.flags = 0;
+        r._pad = 0;
+        const int32_t op = ops[q];
+        bool invalid = op < OLAP_SUM || op > OLAP_AVG, empty = false;
+        int64_t V = 1;
+        for (int k = 0; k < nd; ++k) {
+            const olap_range rg = ranges[q * nd + k];
+            if (rg.lo < 0 || rg.hi >= ext.n[k]) invalid = true;
+            if (rg.lo > rg.hi) empty = true;
+            else V *= rg.hi - rg.lo + 1;
+        }
+        if (invalid) r.flags = OLAP_RESULT_INVALID;
+        else if (empty) r.flags = OLAP_RESULT_EMPTY;
+        else if (op == OLAP_COUNT) r.i = V;
+        else {
+            const int64_t s = psum[q];
+            const int32_t cmx = pext[2 * q], cmn = ~pext[2 * q + 1];
+            if (dtype == OLAP_INT32) {
+                if (op == OLAP_SUM) r.i = s;
+                else if (op == OLAP_MIN) r.i = cmn;
+                else if (op == OLAP_MAX) r.i = cmx;
+                else r.d = (double)s / (double)V;
+            } else {
+                const double ds = __longlong_as_double(s);
+                if (op == OLAP_SUM) r.d = ds;
+                else if (op == OLAP_MIN) r.d = (double)f32_decode(cmn);
+                else if (op == OLAP_MAX) r.d = (double)f32_decode(cmx);
+                else r.d = ds / (double)V;
+            }
+        }
+        out[q] = r;
+    }
+}
+
+__global__ void combine_kernel(int dtype, int64_t nq, const int64_t* __restrict__ s_in, const int32_t* __restrict__ e_in,
+                               int64_t* s_acc, int32_t* e_acc) {
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nq; q += (int64_t)gridDim.x * blockDim.x) {
+        if (dtype == OLAP_INT32)
+            s_acc[q] = (int64_t)((uint64_t)s_acc[q] + (uint64_t)s_in[q]);
+        else
+            s_acc[q] = __double_as_longlong(__longlong_as_double(s_acc[q]) + __longlong_as_double(s_in[q]));
+        e_acc[2 * q] = max(e_acc[2 * q], e_in[2 * q]);
+        e_acc[2 * q + 1] = max(e_acc[2 * q + 1], e_in[2 * q + 1]);
+    }
+}
+
+// ------------------------------------------------------------------ fill (support, not timed)
+
+__device__ __forceinline__ uint64_t splitmix64_at(uint64_t seed, uint64_t idx) {
+    uint64_t z = seed + (idx + 1ull) * 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+struct FillParams {
+    double c[kMaxDims + 1];
+};
+
+template <typename T>
+__global__ void fill_kernel(T* cells, Geo geo, int64_t row_cells, int gen, uint64_t seed, FillParams fp) {
+    const int64_t n = geo.local_rows * row_cells;
+    for (int64_t li = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; li < n; li += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t lr = li / row_cells, off = li - lr * row_cells;
+        const int64_t gr = shard_global_of(lr, geo.G, geo.g, geo.b);
+        const int64_t gi = gr * row_cells + off;
+        if (gen == OLAP_GEN_UNIFORM) {
+            const uint64_t z = splitmix64_at(seed, (uint64_t)gi);
+            if (sizeof(T) == 4 && geo.dtype == OLAP_INT32)
+                reinterpret_cast<int32_t*>(cells)[li] = (int32_t)(z >> 43) - (1 << 20);
+            else
+                reinterpret_cast<float*>(cells)[li] = (float)(z >> 40) * (1.0f / 16777216.0f);
+        } else {
+            double v = fp.c[0] + fp.c[1] * (double)gr;
+            int64_t rem = off;
+            for (int k = geo.nd - 1; k >= 1; --k) {
+                const int64_t x = rem % geo.n[k];
+                rem /= geo.n[k];
+                v += fp.c[1 + k] * (double)x;
+            }
+            if (geo.dtype == OLAP_INT32) reinterpret_cast<int32_t*>(cells)[li] = (int32_t)v;
+            else reinterpret_cast<float*>(cells)[li] = (float)v;
+        }
+    }
+}
+
+}  // namespace olap
+
+// ====================================================================== host runtime
+
+using namespace olap;
+
+struct olap_cube {
+    int nd = 0, dtype = 0, device = 0;
+    int64_t n[kMaxDims] = {};
+    olap_shard sh{1, 0, 1};
+    int64_t local_rows = 0, row_cells = 0, local_cells = 0;
+    int64_t stride[kMaxDims] = {};
+    void* d_cells = nullptr;
+
+    std::mutex mu;
+    cudaStream_t stream = nullptr;   // host-buffer calls
+    cudaEvent_t ws_done = nullptr;   // last batch that used the workspace
+    int num_sms = 0, blocks_per_sm = 0;
+
+    int64_t nq_cap = 0, items_cap = 0;
+    QDesc* d_desc = nullptr;
+    int64_t* d_item_start = nullptr;
+    int32_t* d_done = nullptr;
+    unsigned long long* d_counter = nullptr;  // [0] item counter, [1] algorithmic bytes
+    long long* d_item_sum = nullptr;
+    int32_t* d_item_ext = nullptr;
+    // host-path staging
+    olap_range* d_ranges = nullptr;
+    int32_t* d_ops = nullptr;
+    olap_result* d_results = nullptr;
+    int64_t* d_psum = nullptr;
+    int32_t* d_pext = nullptr;
+    void* h_pinned = nullptr;
+    size_t h_pinned_cap = 0;
+    int64_t stage_cap = 0;
+
+    bool prof = false;
+    std::vector<cudaEvent_t> ev;
+    size_t ev_used = 0;
+    int64_t launches = 0;
+    unsigned long long bytes_base = 0;
+};
+
+namespace {
+
+struct DeviceGuard {
+    int prev = -1;
+    bool ok = false;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) == cudaSuccess && cudaSetDevice(dev) == cudaSuccess) ok = true;
+    }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
+Geo make_geo(const olap_cube* c) {
+    Geo g;
+    std::memset(&g, 0, sizeof(g));
+    g.nd = c->nd;
+    g.dtype = c->dtype;
+    g.G = c->sh.nshards;
+    g.g = c->sh.shard;
+    g.b = c->sh.block;
+    for (int k = 0; k < c->nd; ++k) {
+        g.n[k] = c->n[k];
+        g.stride[k] = c->stride[k];
+    }
+    g.local_rows = c->local_rows;
+    return g;
+}
+
+void free_ws(olap_cube* c) {
+    cudaFree(c->d_desc);
+    cudaFree(c->d_item_start);
+    cudaFree(c->d_done);
+    cudaFree(c->d_item_sum);
+    cudaFree(c->d_item_ext);
+    c->d_desc = nullptr;
+    c->d_item_start = nullptr;
+    c->d_done = nullptr;
+    c->d_item_sum = nullptr;
+    c->d_item_ext = nullptr;
+    c->nq_cap = c->items_cap = 0;
+}
+
+int ensure_ws(olap_cube* c, int64_t nq) {
+    if (nq <= c->nq_cap) return OLAP_OK;
+    OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
+    free_ws(c);
+    int64_t cap = std::max<int64_t>(nq, 1024);
+    int64_t items = std::max<int64_t>(1ll << 20, 4 * cap);
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_desc, sizeof(QDesc) * cap));
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_item_start, sizeof(int64_t) * (cap + 1)));
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_done, sizeof(int32_t) * cap));
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_item_sum, sizeof(long long) * items));
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_item_ext, sizeof(int32_t) * 2 * items));
+    c->nq_cap = cap;
+    c->items_cap = items;
+    return OLAP_OK;
+}
+
+int ensure_stage(olap_cube* c, int64_t nq) {
+    if (nq <= c->stage_cap) return OLAP_OK;
+    OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
+    cudaFree(c->d_ranges);
+    cudaFree(c->d_ops);
+    cudaFree(c->d_results);
+    cudaFree(c->d_psum);
+    cudaFree(c->d_pext);
+    cudaFreeHost(c->h_pinned);
+    c->d_ranges = nullptr;
+    c->d_ops = nullptr;
+    c->d_results = nullptr;
+    c->d_psum = nullptr;
+    c->d_pext = nullptr;
+    c->h_pinned = nullptr;
+    c->stage_cap = 0;
+    int64_t cap = std::max<int64_t>(nq, 1024);
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_ranges, sizeof(olap_range) * c->nd * cap));
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_ops, sizeof(int32_t) * cap));
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_results, sizeof(olap_result) * cap));
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_psum, sizeof(int64_t) * cap));
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_pext, sizeof(int32_t) * 2 * cap));
+    c->h_pinned_cap = (sizeof(olap_range) * c->nd + sizeof(int32_t) + sizeof(olap_result)) * cap;
+    OLAP_CUDA_TRY(cudaHostAlloc(&c->h_pinned, c->h_pinned_cap, cudaHostAllocDefault));
+    c->stage_cap = cap;
+    return OLAP_OK;
+}
+
+// plan + reduce for nq queries already on the device; writes partials
+int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int32_t* d_ops, int64_t* d_psum,
+                 int32_t* d_pext, cudaStream_t st) {
+    int rc = ensure_ws(c, nq);
+    if (rc) return rc;
+    OLAP_CUDA_TRY(cudaStreamWaitEvent(st, c->ws_done, 0));
+    plan_kernel<<<1, kPlanThreads, 0, st>>>(make_geo(c), nq, d_ranges, d_ops, c->d_desc, c->d_item_start, c->d_done,
+                                            c->d_counter, d_psum, d_pext, c->items_cap, c->d_counter + 1);
+    OLAP_CUDA_TRY(cudaGetLastError());
+    const int grid = c->num_sms * c->blocks_per_sm;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    if (c->prof) {
+        while (c->ev.size() < c->ev_used + 2) {
+            cudaEvent_t e;
+            OLAP_CUDA_TRY(cudaEventCreate(&e));
+            c->ev.push_back(e);
+        }
+        e0 = c->ev[c->ev_used];
+        e1 = c->ev[c->ev_used + 1];
+        c->ev_used += 2;
+        OLAP_CUDA_TRY(cudaEventRecord(e0, st));
+    }
+    if (c->dtype == OLAP_INT32)
+        reduce_kernel<int32_t, AccI><<<grid, kThreads, 0, st>>>(
+            static_cast<const int32_t*>(c->d_cells), nq, c->d_desc, c->d_item_start, c->d_counter, c->d_done,
+            c->d_item_sum, c->d_item_ext, d_psum, d_pext);
+    else
+        reduce_kernel<float, AccF><<<grid, kThreads, 0, st>>>(
+            static_cast<const float*>(c->d_cells), nq, c->d_desc, c->d_item_start, c->d_counter, c->d_done,
+            c->d_item_sum, c->d_item_ext, d_psum, d_pext);
+    OLAP_CUDA_TRY(cudaGetLastError());
+    if (c->prof) {
+        OLAP_CUDA_TRY(cudaEventRecord(e1, st));
+        ++c->launches;
+    }
+    OLAP_CUDA_TRY(cudaEventRecord(c->ws_done, st));
+    return OLAP_OK;
+}
+
+int launch_finalize(int nd, const int64_t* ext, int dtype, int64_t nq, const olap_range* d_ranges, const int32_t* d_ops,
+                    const int64_t* d_psum, const int32_t* d_pext, olap_result* d_results, cudaStream_t st) {
+    Extents e;
+    std::memset(&e, 0, sizeof(e));
+    for (int k = 0; k < nd; ++k) e.n[k] = ext[k];
+    const int grid = (int)std::min<int64_t>((nq + 255) / 256, 4096);
+    finalize_kernel<<<grid, 256, 0, st>>>(nd, e, dtype, nq, d_ranges, d_ops, d_psum, d_pext, d_results);
+    OLAP_CUDA_TRY(cudaGetLastError());
+    return OLAP_OK;
+}
+
+int check_cube(const olap_cube* c) {
+    if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    if (!c->d_cells) return set_error(OLAP_E_STATE, "cube has no device storage");
+    return OLAP_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_shard* shard, int device,
+                     olap_cube** out) {
+    clear_error();
+    if (!out || !extents) return set_error(OLAP_E_INVALID, "olap_cube_create: NULL argument");
+    if (ndims < 1 || ndims > kMaxDims) return set_error(OLAP_E_INVALID, "ndims %d not in [1,8]", ndims);
+    if (dtype != OLAP_INT32 && dtype != OLAP_FLOAT32) return set_error(OLAP_E_INVALID, "bad dtype %d", dtype);
+    olap_shard sh{1, 0, 1};
+    if (shard) sh = *shard;
+    if (sh.nshards < 1 || sh.shard < 0 || sh.shard >= sh.nshards || sh.block < 1)
+        return set_error(OLAP_E_INVALID, "bad shard {%lld,%lld,%lld}", (long long)sh.nshards, (long long)sh.shard,
+                         (long long)sh.block);
+    int64_t cells = 1;
+    for (int k = 0; k < ndims; ++k) {
+        if (extents[k] < 1) return set_error(OLAP_E_INVALID, "extent[%d] = %lld < 1", k, (long long)extents[k]);
+        if (extents[k] > kMaxExtent)
+            return set_error(OLAP_E_UNSUPPORTED, "extent[%d] = %lld exceeds 2^30", k, (long long)extents[k]);
+        cells *= extents[k];
+        if (cells > kMaxCells) return set_error(OLAP_E_UNSUPPORTED, "cube exceeds 2^42 cells");
+    }
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
+        return set_error(OLAP_E_CUDA, "no CUDA device available (the library has no CPU fallback)");
+    if (device < 0 || device >= ndev) return set_error(OLAP_E_INVALID, "device %d not in [0,%d)", device, ndev);
+    DeviceGuard dg(device);
+    if (!dg.ok) return set_error(OLAP_E_CUDA, "cudaSetDevice(%d) failed", device);
+
+    olap_cube* c = new (std::nothrow) olap_cube();
+    if (!c) return set_error(OLAP_E_NOMEM, "host allocation failed");
+    c->nd = ndims;
+    c->dtype = dtype;
+    c->device = device;
+    c->sh = sh;
+    for (int k = 0; k < ndims; ++k) c->n[k] = extents[k];
+    c->stride[ndims - 1] = 1;
+    for (int k = ndims - 2; k >= 0; --k) c->stride[k] = c->stride[k + 1] * c->n[k + 1];
+    c->row_cells = c->stride[0];
+    c->local_rows = shard_rows(c->n[0], sh.nshards, sh.shard, sh.block);
+    c->local_cells = c->local_rows * c->row_cells;
+    int rc = OLAP_OK;
+    cudaError_t e = cudaMalloc(&c->d_cells, std::max<int64_t>(c->local_cells, 1) * 4);
+    if (e != cudaSuccess) {
+        rc = set_error(e == cudaErrorMemoryAllocation ? OLAP_E_NOMEM : OLAP_E_CUDA, "cudaMalloc of %lld cells: %s",
+                       (long long)c->local_cells, cudaGetErrorString(e));
+        cudaGetLastError();
+        delete c;
+        return rc;
+    }
+    if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&c->ws_done, cudaEventDisableTiming) != cudaSuccess ||
+        cudaMalloc(&c->d_counter, 2 * sizeof(unsigned long long)) != cudaSuccess ||
+        cudaMemset(c->d_counter, 0, 2 * sizeof(unsigned long long)) != cudaSuccess) {
+        rc = set_error(OLAP_E_CUDA, "stream/event/counter setup failed");
+        olap_cube_destroy(c);
+        return rc;
+    }
+    cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device);
+    int bps = 0;
+    if (dtype == OLAP_INT32)
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, reduce_kernel<int32_t, AccI>, kThreads, 0);
+    else
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, reduce_kernel<float, AccF>, kThreads, 0);
+    if (const char* s = getenv("OLAP_BLOCKS_PER_SM")) {
+        int v = atoi(s);
+        if (v > 0 && v < bps) bps = v;
+    }
+    c->blocks_per_sm = std::max(bps, 1);
+    *out = c;
+    return OLAP_OK;
+}
+
+int olap_cube_info(const olap_cube* c, int64_t* local_rows, int64_t* local_cells, void** d_cells) {
+    clear_error();
+    if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    if (local_rows) *local_rows = c->local_rows;
+    if (local_cells) *local_cells = c->local_cells;
+    if (d_cells) *d_cells = c->d_cells;
+    return OLAP_OK;
+}
+
+int olap_cube_load_rows(olap_cube* c, int64_t row_lo, int64_t row_hi, const void* cells) {
+    clear_error();
+    int rc = check_cube(c);
+    if (rc) return rc;
+    if (!cells || row_lo < 0 || row_hi > c->n[0] || row_lo > row_hi)
+        return set_error(OLAP_E_INVALID, "olap_cube_load_rows: bad rows [%lld,%lld)", (long long)row_lo,
+                         (long long)row_hi);
+    std::lock_guard<std::mutex> lk(c->mu);
+    DeviceGuard dg(c->device);
+    OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
+    const int64_t rb = c->row_cells * 4;
+    const char* src = static_cast<const char*>(cells);
+    char* dst = static_cast<char*>(c->d_cells);
+    const int64_t G = c->sh.nshards, g = c->sh.shard, b = c->sh.block;
+    int64_t r = row_lo;
+    while (r < row_hi) {
+        // run of consecutive owned rows starting at r (or skip the unowned ones)
+        const int64_t blk_end = (r / b + 1) * b;
+        const int64_t end = std::min(blk_end, row_hi);
+        if ((r / b) % G == g) {
+            const int64_t lr = shard_local_of(r, G, b);
+            OLAP_CUDA_TRY(cudaMemcpy(dst + lr * rb, src + (r - row_lo) * rb, (end - r) * rb, cudaMemcpyHostToDevice));
+        }
+        r = end;
+        if (G == 1) {  // whole remainder is owned and contiguous
+            if (r < row_hi)
+                OLAP_CUDA_TRY(cudaMemcpy(dst + r * rb, src + (r - row_lo) * rb, (row_hi - r) * rb,
+                                         cudaMemcpyHostToDevice));
+            break;
+        }
+    }
+    return OLAP_OK;
+}
+
+int olap_cube_load(olap_cube* c, const void* cells, int64_t ncells) {
+    clear_error();
+    int rc = check_cube(c);
+    if (rc) return rc;
+    if (ncells != c->n[0] * c->row_cells)
+        return set_error(OLAP_E_INVALID, "olap_cube_load: ncells %lld != %lld", (long long)ncells,
+                         (long long)(c->n[0] * c->row_cells));
+    return olap_cube_load_rows(c, 0, c->n[0], cells);
+}
+
+int olap_cube_fill(olap_cube* c, int generator, uint64_t seed, const double* params) {
+    clear_error();
+    int rc = check_cube(c);
+    if (rc) return rc;
+    if (generator != OLAP_GEN_UNIFORM && generator != OLAP_GEN_AFFINE)
+        return set_error(OLAP_E_INVALID, "unknown generator %d", generator);
+    if (generator == OLAP_GEN_AFFINE && !params) return set_error(OLAP_E_INVALID, "affine generator needs params");
+    std::lock_guard<std::mutex> lk(c->mu);
+    DeviceGuard dg(c->device);
+    FillParams fp;
+    std::memset(&fp, 0, sizeof(fp));
+    if (params)
+        for (int k = 0; k <= c->nd; ++k) fp.c[k] = params[k];
+    const int grid = c->num_sms * 8;
+    if (c->dtype == OLAP_INT32)
+        fill_kernel<int32_t><<<grid, 256, 0, c->stream>>>(static_cast<int32_t*>(c->d_cells), make_geo(c), c->row_cells,
+                                                          generator, seed, fp);
+    else
+        fill_kernel<float><<<grid, 256, 0, c->stream>>>(static_cast<float*>(c->d_cells), make_geo(c), c->row_cells,
+                                                        generator, seed, fp);
+    OLAP_CUDA_TRY(cudaGetLastError());
+    OLAP_CUDA_TRY(cudaStreamSynchronize(c->stream));
+    return OLAP_OK;
+}
+
+int olap_cube_destroy(olap_cube* c) {
+    clear_error();
+    if (!c) return OLAP_OK;
+    DeviceGuard dg(c->device);
+    if (c->ws_done) cudaEventSynchronize(c->ws_done);
+    if (c->stream) cudaStreamSynchronize(c->stream);
+    free_ws(c);
+    cudaFree(c->d_ranges);
+    cudaFree(c->d_ops);
+    cudaFree(c->d_results);
+    cudaFree(c->d_psum);
+    cudaFree(c->d_pext);
+    cudaFreeHost(c->h_pinned);
+    cudaFree(c->d_counter);
+    cudaFree(c->d_cells);
+    for (auto e : c->ev) cudaEventDestroy(e);
+    if (c->ws_done) cudaEventDestroy(c->ws_done);
+    if (c->stream) cudaStreamDestroy(c->stream);
+    delete c;
+    return OLAP_OK;
+}
+
+int olap_query_batch(olap_cube* c, int64_t nq, const olap_range* ranges, const int32_t* ops, olap_result* results) {
+    clear_error();
+    int rc = check_cube(c);
+    if (rc) return rc;
+    if (nq < 0) return set_error(OLAP_E_INVALID, "nq < 0");
+    if (nq == 0) return OLAP_OK;
+    if (!ranges || !ops || !results) return set_error(OLAP_E_INVALID, "olap_query_batch: NULL buffer");
+    if (c->sh.nshards != 1)
+        return set_error(OLAP_E_STATE, "olap_query_batch needs an unsharded cube; use olap_query_partials_device");
+    for (int64_t q = 0; q < nq; ++q) {
+        if (ops[q] < OLAP_SUM || ops[q] > OLAP_AVG)
+            return set_error(OLAP_E_INVALID, "query %lld: unknown op %d", (long long)q, ops[q]);
+        for (int k = 0; k < c->nd; ++k) {
+            const olap_range r = ranges[q * c->nd + k];
+            if (r.lo < 0 || r.hi >= c->n[k])
+                return set_error(OLAP_E_RANGE, "query %lld dimension %d: range [%lld,%lld] outside [0,%lld)",
+                                 (long long)q, k, (long long)r.lo, (long long)r.hi, (long long)c->n[k]);
+        }
+    }
+    std::lock_guard<std::mutex> lk(c->mu);
+    DeviceGuard dg(c->device);
+    rc = ensure_stage(c, nq);
+    if (rc) return rc;
+    const size_t rbytes = sizeof(olap_range) * c->nd * nq, obytes = sizeof(int32_t) * nq,
+                 res_bytes = sizeof(olap_result) * nq;
+    char* hp = static_cast<char*>(c->h_pinned);
+    OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));  // pinned staging reuse
+    std::memcpy(hp, ranges, rbytes);
+    std::memcpy(hp + rbytes, ops, obytes);
+    cudaStream_t st = c->stream;
+    OLAP_CUDA_TRY(cudaMemcpyAsync(c->d_ranges, hp, rbytes, cudaMemcpyHostToDevice, st));
+    OLAP_CUDA_TRY(cudaMemcpyAsync(c->d_ops, hp + rbytes, obytes, cudaMemcpyHostToDevice, st));
+    rc = run_partials(c, nq, c->d_ranges, c->d_ops, c->d_psum, c->d_pext, st);
+    if (rc) return rc;
+    rc = launch_finalize(c->nd, c->n, c->dtype, nq, c->d_ranges, c->d_ops, c->d_psum, c->d_pext, c->d_results, st);
+    if (rc) return rc;
+    char* hres = hp + rbytes + obytes;
+    OLAP_CUDA_TRY(cudaMemcpyAsync(hres, c->d_results, res_bytes, cudaMemcpyDeviceToHost, st));
+    OLAP_CUDA_TRY(cudaEventRecord(c->ws_done, st));
+    OLAP_CUDA_TRY(cudaStreamSynchronize(st));
+    std::memcpy(results, hres, res_bytes);
+    return OLAP_OK;
+}
+
+int olap_query_partials_device(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int32_t* d_ops,
+                               int64_t* d_sum, int32_t* d_ext, void* stream) {
+    clear_error();
+    int rc = check_cube(c);
+    if (rc) return rc;
+    if (nq < 0) return set_error(OLAP_E_INVALID, "nq < 0");
+    if (nq == 0) return OLAP_OK;
+    if (!d_ranges || !d_ops || !d_sum || !d_ext) return set_error(OLAP_E_INVALID, "NULL device buffer");
+    std::lock_guard<std::mutex> lk(c->mu);
+    DeviceGuard dg(c->device);
+    return run_partials(c, nq, d_ranges, d_ops, d_sum, d_ext, static_cast<cudaStream_t>(stream));
+}
+
+int olap_query_batch_device(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int32_t* d_ops,
+                            olap_result* d_results, void* stream) {
+    clear_error();
+    int rc = check_cube(c);
+    if (rc) return rc;
+    if (nq < 0) return set_error(OLAP_E_INVALID, "nq < 0");
+    if (nq == 0) return OLAP_OK;
+    if (!d_ranges || !d_ops || !d_results) return set_error(OLAP_E_INVALID, "NULL device buffer");
+    if (c->sh.nshards != 1) return set_error(OLAP_E_STATE, "olap_query_batch_device needs an unsharded cube");
+    std::lock_guard<std::mutex> lk(c->mu);
+    DeviceGuard dg(c->device);
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    rc = ensure_stage(c, nq);
+    if (rc) return rc;
+    rc = run_partials(c, nq, d_ranges, d_ops, c->d_psum, c->d_pext, st);
+    if (rc) return rc;
+    rc = launch_finalize(c->nd, c->n, c->dtype, nq, d_ranges, d_ops, c->d_psum, c->d_pext, d_results, st);
+    if (rc) return rc;
+    OLAP_CUDA_TRY(cudaEventRecord(c->ws_done, st));
+    return OLAP_OK;
+}
+
+int olap_partials_combine_device(int dtype, int64_t nq, const int64_t* d_sum_in, const int32_t* d_ext_in,
+                                 int64_t* d_sum_acc, int32_t* d_ext_acc, void* stream) {
+    clear_error();
+    if (dtype != OLAP_INT32 && dtype != OLAP_FLOAT32) return set_error(OLAP_E_INVALID, "bad dtype %d", dtype);
+    if (nq < 0) return set_error(OLAP_E_INVALID, "nq < 0");
+    if (nq == 0) return OLAP_OK;
+    if (!d_sum_in || !d_ext_in || !d_sum_acc || !d_ext_acc) return set_error(OLAP_E_INVALID, "NULL device buffer");
+    const int grid = (int)std::min<int64_t>((nq + 255) / 256, 4096);
+    combine_kernel<<<grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(dtype, nq, d_sum_in, d_ext_in, d_sum_acc,
+                                                                         d_ext_acc);
+    OLAP_CUDA_TRY(cudaGetLastError());
+    return OLAP_OK;
+}
+
+int olap_finalize_device(int ndims, const int64_t* extents, int dtype, int64_t nq, const olap_range* d_ranges,
+                         const int32_t* d_ops, const int64_t* d_sum, const int32_t* d_ext, olap_result* d_results,
+                         void* stream) {
+    clear_error();
+    if (ndims < 1 || ndims > kMaxDims || !extents) return set_error(OLAP_E_INVALID, "bad ndims/extents");
+    if (dtype != OLAP_INT32 && dtype != OLAP_FLOAT32) return set_error(OLAP_E_INVALID, "bad dtype %d", dtype);
+    if (nq < 0) return set_error(OLAP_E_INVALID, "nq < 0");
+    if (nq == 0) return OLAP_OK;
+    if (!d_ranges || !d_ops || !d_sum || !d_ext || !d_results) return set_error(OLAP_E_INVALID, "NULL device buffer");
+    return launch_finalize(ndims, extents, dtype, nq, d_ranges, d_ops, d_sum, d_ext, d_results,
+                           static_cast<cudaStream_t>(stream));
+}
+
+int olap_shard_local_rows(int64_t n0, const olap_shard* s, int64_t lo, int64_t hi, int64_t* llo, int64_t* lhi) {
+    clear_error();
+    if (!llo || !lhi || n0 < 1) return set_error(OLAP_E_INVALID, "olap_shard_local_rows: bad argument");
+    olap_shard sh{1, 0, 1};
+    if (s) sh = *s;
+    if (sh.nshards < 1 || sh.shard < 0 || sh.shard >= sh.nshards || sh.block < 1)
+        return set_error(OLAP_E_INVALID, "bad shard");
+    if (lo < 0 || hi >= n0) return set_error(OLAP_E_RANGE, "rows [%lld,%lld] outside [0,%lld)", (long long)lo,
+                                             (long long)hi, (long long)n0);
+    int64_t a = 1, b = 0;
+    if (lo <= hi && shard_local_range(n0, sh.nshards, sh.shard, sh.block, lo, hi, &a, &b)) {
+        *llo = a;
+        *lhi = b;
+    } else {
+        *llo = 1;
+        *lhi = 0;
+    }
+    return OLAP_OK;
+}
+
+int olap_cube_profile(olap_cube* c, int enable) {
+    clear_error();
+    if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    std::lock_guard<std::mutex> lk(c->mu);
+    DeviceGuard dg(c->device);
+    OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
+    c->prof = enable != 0;
+    c->ev_used = 0;
+    c->launches = 0;
+    OLAP_CUDA_TRY(cudaMemcpy(&c->bytes_base, c->d_counter + 1, sizeof(unsigned long long), cudaMemcpyDeviceToHost));
+    return OLAP_OK;
+}
+
+int olap_cube_profile_read(olap_cube* c, double* reduce_ms, int64_t* launches, int64_t* bytes) {
+    clear_error();
+    if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    std::lock_guard<std::mutex> lk(c->mu);
+    DeviceGuard dg(c->device);
+    OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
+    double ms = 0.0;
+    for (size_t i = 0; i + 1 < c->ev_used; i += 2) {
+        float t = 0.f;
+        OLAP_CUDA_TRY(cudaEventSynchronize(c->ev[i + 1]));
+        OLAP_CUDA_TRY(cudaEventElapsedTime(&t, c->ev[i], c->ev[i + 1]));
+        ms += t;
+    }
+    unsigned long long b = 0;
+    OLAP_CUDA_TRY(cudaMemcpy(&b, c->d_counter + 1, sizeof(b), cudaMemcpyDeviceToHost));
+    if (reduce_ms) *reduce_ms = ms;
+    if (launches) *launches = c->launches;
+    if (bytes) *bytes = (int64_t)(b - c->bytes_base);
+    return OLAP_OK;
+}
+
+}  // extern "C"

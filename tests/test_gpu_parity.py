@@ -1,0 +1,335 @@
+"""GPU parity: the CUDA path (through the C-ABI) vs the oracle, element by element.
+
+Bars (BASELINE.json north_star):
+  * int32 cubes: every field bit-exact (SUM int64 wraparound, COUNT, MIN, MAX, AVG as
+    (double)SUM/(double)V computed identically);
+  * float32 cubes: COUNT/MIN/MAX exact; SUM/AVG within 1e-6 relative of the fp64
+    oracle (north_star), and bit-exact on integer-valued (affine) cubes where every
+    fp64 partial sum is exact in any order.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_ipps_malikrse12_b200 as olap
+import synth
+
+pytestmark = pytest.mark.gpu
+
+REL = 1e-6   # north_star float tolerance
+
+
+def compare(gpu, ref, ops, dtype, exact_float=False, rel=REL):
+    assert gpu.shape == ref.shape
+    assert np.array_equal(gpu["flags"], ref["flags"]), np.nonzero(gpu["flags"] != ref["flags"])[0][:10]
+    if dtype == np.int32 or exact_float:
+        bad = np.nonzero((gpu["i"] != ref["i"]) | (gpu["d"] != ref["d"]))[0]
+        assert bad.size == 0, f"{bad.size} mismatches, first {bad[:5]}: gpu {gpu[bad[:3]]} ref {ref[bad[:3]]}"
+        return
+    assert np.array_equal(gpu["i"], ref["i"])
+    exact = (ops == oracle.MIN) | (ops == oracle.MAX) | (ops == oracle.COUNT)
+    assert np.array_equal(gpu["d"][exact], ref["d"][exact])
+    tol = rel * np.abs(ref["d"]) + 1e-300
+    bad = np.nonzero(np.abs(gpu["d"] - ref["d"]) > tol)[0]
+    assert bad.size == 0, f"{bad.size} beyond {rel}: {gpu['d'][bad[:5]]} vs {ref['d'][bad[:5]]}"
+
+
+def test_hand_example_fig2():
+    cells = np.arange(64, dtype=np.int32)
+    c = olap.Cube((4, 4, 4), np.int32)
+    c.load(cells)
+    box = np.array([[[1, 2], [1, 3], [0, 1]]] * 5)
+    ops = np.array([olap.COUNT, olap.SUM, olap.MIN, olap.MAX, olap.AVG], np.int32)
+    r = c.query(box, ops)
+    assert list(r["i"][:4]) == [12, 390, 20, 45] and r["d"][4] == 32.5
+
+
+def test_c1_full_bit_exact():
+    """Config C1: 4-D int32 32^4, 1,000 random boxes, 1 GPU vs the CPU oracle — all bit-exact."""
+    cfg = synth.CONFIGS["C1"]
+    cells = synth.uniform_cells(int(np.prod(cfg["extents"])), np.int32, cfg["seed"])
+    boxes, ops = synth.config_queries("C1")
+    c = olap.Cube(cfg["extents"], np.int32)
+    c.load(cells)
+    gpu = c.query(boxes, ops)
+    ref = oracle.query(cfg["extents"], boxes, ops, cells)
+    compare(gpu, ref, ops, np.int32)
+    # every op on every box
+    for op in range(5):
+        o = np.full(len(boxes), op, np.int32)
+        compare(c.query(boxes, o), oracle.query(cfg["extents"], boxes, o, cells), o, np.int32)
+
+
+SHAPES = [
+    ((8, 8, 8, 8, 8, 64), "C2a-like, runs >= 128 cells merge"),
+    ((8, 8, 16, 16, 16, 16), "C2b-like, short runs"),
+    ((3, 1000), "long rows, vector path with ragged heads/tails"),
+    ((5000,), "1-D"),
+    ((2, 3, 2, 3, 2, 3, 2, 3), "8-D"),
+    ((1, 1, 37), "extent-1 dims"),
+    ((64, 129, 7), "odd inner extents"),
+    ((17, 4099), "piece boundaries (2048-cell pieces) + tail"),
+]
+
+
+@pytest.mark.parametrize("dtype", [np.int32, np.float32])
+@pytest.mark.parametrize("ext,why", SHAPES)
+def test_shapes_random_and_fraction_boxes(ext, why, dtype):
+    n = int(np.prod(ext))
+    seed = 0x5EED1000 + n
+    cells = synth.uniform_cells(n, dtype, seed)
+    rng = np.random.default_rng(seed)
+    b1 = synth.random_boxes(ext, 300, rng)
+    b2 = synth.fraction_boxes(ext, 300, rng, 1e-4)
+    full = np.array([[[0, e - 1] for e in ext]])
+    boxes = np.concatenate([b1, b2, full, full])
+    ops = synth.ops_uniform(len(boxes), rng)
+    ops[-2:] = [olap.SUM, olap.MIN]
+    c = olap.Cube(ext, dtype)
+    c.load(cells)
+    compare(c.query(boxes, ops), oracle.query(ext, boxes, ops, cells), ops, dtype)
+
+
+@pytest.mark.parametrize("dtype", [np.int32, np.float32])
+def test_affine_integer_valued_bit_exact(dtype):
+    """Integer-valued affine cube: fp64 sums are exact in any order -> float32 SUM/AVG bit-exact too."""
+    ext = (12, 10, 9, 300)
+    params = np.array([7, 3, -2, 5, 1], float)
+    c = olap.Cube(ext, dtype)
+    c.fill(olap.GEN_AFFINE, 0, params)
+    rng = np.random.default_rng(5)
+    boxes = np.concatenate([synth.random_boxes(ext, 400, rng), synth.fraction_boxes(ext, 400, rng, 1e-4)])
+    ops = synth.ops_uniform(len(boxes), rng)
+    ref = oracle.query(ext, boxes, ops, dtype=dtype, gen=oracle.GEN_AFFINE, params=params)
+    compare(c.query(boxes, ops), ref, ops, dtype, exact_float=True)
+
+
+def test_fill_matches_inputs_generator():
+    """The device generator equals the seeded input generator (same published splitmix64
+    formula), read back cell by cell through 1-cell MAX queries."""
+    for dtype in (np.int32, np.float32):
+        ext = (33, 70)
+        c = olap.Cube(ext, dtype)
+        c.fill(olap.GEN_UNIFORM, 0x5EED0001)
+        xs, ys = np.meshgrid(np.arange(33), np.arange(70), indexing="ij")
+        boxes = np.stack([np.stack([xs.ravel(), xs.ravel()], -1), np.stack([ys.ravel(), ys.ravel()], -1)], 1)
+        r = c.query(boxes, np.full(len(boxes), olap.MAX, np.int32))
+        got = r["i"].astype(np.int32) if dtype == np.int32 else r["d"].astype(np.float32)
+        assert np.array_equal(got, synth.uniform_cells(33 * 70, dtype, 0x5EED0001))
+
+
+def test_c2_full_size_sampled():
+    """Config C2a at full size (1 GiB float32, 4,096-query batch, the bench's launch
+    configuration): GPU vs oracle on a sample of queries the oracle recomputes one by one."""
+    cfg = synth.CONFIGS["C2a"]
+    ext = cfg["extents"]
+    c = olap.Cube(ext, np.float32)
+    c.fill(olap.GEN_UNIFORM, cfg["seed"])
+    boxes, ops = synth.config_queries("C2a")
+    gpu = c.query(boxes, ops)
+    rng = np.random.default_rng(0)
+    # sample: smallest, largest and random queries (bounded oracle work)
+    vol = np.prod(boxes[:, :, 1] - boxes[:, :, 0] + 1, axis=1)
+    idx = np.unique(np.concatenate([np.argsort(vol)[:12], rng.choice(len(boxes), 24, replace=False)]))
+    idx = idx[vol[idx] < 60_000_000][:30]
+    ref = oracle.query(ext, boxes[idx], ops[idx], dtype=np.float32, gen=oracle.GEN_UNIFORM, seed=cfg["seed"],
+                       nthreads=oracle.max_threads())
+    compare(gpu[idx], ref, ops[idx], np.float32)
+    # the full-cube answer of an integer-valued affine fill is exact
+    params = np.array([1, 3, 5, 7, 11, 13, 1], float)
+    c.fill(olap.GEN_AFFINE, 0, params)
+    full = np.array([[[0, e - 1] for e in ext]] * 3)
+    o3 = np.array([olap.SUM, olap.MIN, olap.MAX], np.int32)
+    V = int(np.prod(ext))
+    s = V * 1 + sum(int(params[1 + d]) * (V // ext[d]) * ((ext[d] - 1) * ext[d] // 2) for d in range(6))
+    g3 = c.query(full, o3)
+    assert g3["d"][0] == float(s) and g3["d"][1] == 1.0
+    assert g3["d"][2] == 1 + sum(int(params[1 + d]) * (ext[d] - 1) for d in range(6))
+    # and on a sample of the batch against the oracle, bit-exact
+    gpu = c.query(boxes, ops)
+    idx2 = idx[:12]
+    ref2 = oracle.query(ext, boxes[idx2], ops[idx2], dtype=np.float32, gen=oracle.GEN_AFFINE, params=params,
+                        nthreads=oracle.max_threads())
+    compare(gpu[idx2], ref2, ops[idx2], np.float32, exact_float=True)
+
+
+def test_determinism_float_sums():
+    ext = (16, 16, 16, 16, 16, 16)
+    c = olap.Cube(ext, np.float32)
+    c.fill(olap.GEN_UNIFORM, 99)
+    boxes, ops = synth.config_queries("C2a", nq=512, extents=ext)
+    a = c.query(boxes, ops)
+    b = c.query(boxes, ops)
+    assert a.tobytes() == b.tobytes()
+
+
+def test_empty_invalid_and_errors():
+    ext = (6, 7, 8)
+    cells = synth.uniform_cells(6 * 7 * 8, np.int32, 3)
+    c = olap.Cube(ext, np.int32)
+    c.load(cells)
+    boxes = np.array([[[2, 1], [0, 6], [0, 7]], [[0, 5], [3, 3], [8, 7]], [[0, 0], [0, 0], [0, 0]]])
+    ops = np.array([olap.SUM, olap.MAX, olap.MIN], np.int32)
+    r = c.query(boxes, ops)
+    assert list(r["flags"]) == [olap.RESULT_EMPTY, olap.RESULT_EMPTY, 0]
+    assert r["i"][2] == cells[0]
+    with pytest.raises(olap.OlapError) as ei:
+        c.query(np.array([[[0, 6], [0, 6], [0, 7]]]), [olap.SUM])
+    assert ei.value.status == olap.E_RANGE and "query 0 dimension 0" in str(ei.value)
+    with pytest.raises(olap.OlapError):
+        c.query(np.array([[[0, 1], [0, 1], [0, 1]]]), [9])
+    assert c.query(np.zeros((0, 3, 2), np.int64), np.zeros(0, np.int32)).shape == (0,)
+    # device path flags invalid queries instead of failing the batch
+    dr = torch.tensor(np.array([[[0, 6], [0, 6], [0, 7]], [[0, 5], [0, 6], [0, 7]], [[0, 1], [0, 1], [0, 1]]]),
+                      dtype=torch.int64, device="cuda")
+    do = torch.tensor([olap.SUM, olap.SUM, 7], dtype=torch.int32, device="cuda")
+    res = torch.empty(3 * 24, dtype=torch.uint8, device="cuda")
+    c.query_device(dr, do, res)
+    out = res.cpu().numpy().view(olap.RESULT_DTYPE)
+    assert list(out["flags"]) == [olap.RESULT_INVALID, 0, olap.RESULT_INVALID]
+    assert out["i"][1] == int(cells.astype(np.int64).sum())
+
+
+@pytest.mark.parametrize("G,b", [(2, 1), (3, 2), (4, 1), (8, 16), (5, 3)])
+@pytest.mark.parametrize("dtype", [np.int32, np.float32])
+def test_virtual_shards_combine_to_global(G, b, dtype):
+    """G shards of one cube on one GPU: shard partials + the exchange's reduction
+    (olap_partials_combine_device) + finalize == the unsharded answer / the oracle."""
+    ext = (64, 9, 130)
+    n = int(np.prod(ext))
+    cells = synth.uniform_cells(n, dtype, 0x5EED2000 + G)
+    rng = np.random.default_rng(G * 10 + b)
+    boxes = np.concatenate([synth.random_boxes(ext, 400, rng), synth.fraction_boxes(ext, 200, rng, 1e-3)])
+    ops = synth.ops_uniform(len(boxes), rng)
+    nq = len(boxes)
+    dr = torch.from_numpy(boxes.astype(np.int64)).cuda()
+    do = torch.from_numpy(ops).cuda()
+    acc_s = torch.zeros(nq, dtype=torch.int64, device="cuda")
+    acc_e = torch.full((2 * nq,), -(2 ** 31), dtype=torch.int32, device="cuda")
+    shards = []
+    for g in range(G):
+        cg = olap.Cube(ext, dtype, shard=(G, g, b))
+        cg.load(cells)
+        shards.append(cg)
+        s = torch.empty(nq, dtype=torch.int64, device="cuda")
+        e = torch.empty(2 * nq, dtype=torch.int32, device="cuda")
+        cg.partials_device(dr, do, s, e)
+        olap.combine_partials_device(dtype, nq, s, e, acc_s, acc_e)
+    res = torch.empty(nq * 24, dtype=torch.uint8, device="cuda")
+    olap.finalize_device(ext, dtype, nq, dr, do, acc_s, acc_e, res)
+    got = res.cpu().numpy().view(olap.RESULT_DTYPE)
+    ref = oracle.query(ext, boxes, ops, cells)
+    compare(got, ref, ops, dtype, rel=1e-12)
+    # a shard filled on the device holds the right global cells
+    cg = olap.Cube(ext, dtype, shard=(G, G - 1, b))
+    cg.fill(olap.GEN_UNIFORM, 0x5EED2000 + G)
+    s = torch.empty(nq, dtype=torch.int64, device="cuda")
+    e = torch.empty(2 * nq, dtype=torch.int32, device="cuda")
+    cg.partials_device(dr, do, s, e)
+    s2 = torch.empty_like(s)
+    e2 = torch.empty_like(e)
+    shards[G - 1].partials_device(dr, do, s2, e2)
+    assert torch.equal(s, s2) and torch.equal(e, e2)
+
+
+# ------------------------------------------------------------------ dictionaries
+
+def test_dict_translate_parity():
+    keys = synth.random_keys(20000, seed=1, min_len=0, max_len=40)
+    d = olap.Dict(keys)
+    od = oracle.Dict(keys)
+    assert len(d) == len(od)
+    probes = keys[::3] + synth.random_keys(5000, seed=2, min_len=0, max_len=40) + [k + b"\0" for k in keys[:200]]
+    ids, miss = d.translate(probes)
+    ref = od.translate(probes)
+    assert np.array_equal(ids, ref)
+    assert miss == int((ref < 0).sum())
+    for i in [0, 1, len(d) // 2, len(d) - 1]:
+        assert d.lookup(i) == od.lookup(i)
+
+
+def test_dict_multi_and_bounds():
+    members = synth.tpcds_members()
+    cols = list(members)
+    dg = [olap.Dict(members[c]) for c in cols]
+    do = [oracle.Dict(members[c]) for c in cols]
+    rng = np.random.default_rng(4)
+    which = rng.integers(0, 4, size=3000).astype(np.int32)
+    keys = []
+    for w in which:
+        m = members[cols[w]]
+        k = m[rng.integers(0, len(m))]
+        keys.append(k if rng.random() < 0.9 else k[:-1])
+    ids, miss = olap.translate(dg, which, keys)
+    ref = np.array([do[w].translate([k])[0] for w, k in zip(which, keys)], np.int32)
+    assert np.array_equal(ids, ref) and miss == int((ref < 0).sum())
+    probes = ["1997-01-01", "1998-01-01", "1999-02-29", "2000-02-29", "2002-12-31", "2003", "", "2001-06-15x"]
+    for upper in (False, True):
+        got = dg[0].bound(probes, upper=upper)
+        assert list(got) == [do[0].bound(p, upper=upper) for p in probes]
+
+
+def test_dict_stress_1e6():
+    keys = synth.random_keys(1_000_000, seed=7, min_len=4, max_len=20, alphabet=b"abcdefghij")
+    d = olap.Dict(keys)
+    od = oracle.Dict(keys)
+    probes = keys[::5] + synth.random_keys(100_000, seed=8, min_len=4, max_len=20, alphabet=b"abcdefghij")
+    ids, _ = d.translate(probes)
+    assert np.array_equal(ids, od.translate(probes))
+
+
+def test_c4_tpcds_pipeline():
+    """C4 end to end: string predicates -> GPU translation (4 dictionaries) -> cube queries
+    on cubes built from the fact rows == the oracle's fact scan over the raw rows."""
+    members = synth.tpcds_members()
+    cols = ["ca_state", "i_class", "s_store_id", "d_date"]   # layout: date innermost
+    nrows = 400_000
+    facts, qty, cents = synth.tpcds_facts(nrows, members)
+    dg = {c: olap.Dict(members[c]) for c in cols}
+    do = {c: oracle.Dict(members[c]) for c in cols}
+    # fact rows -> ids (GPU translation of the raw strings, checked against the oracle)
+    ids = []
+    for c in cols:
+        strs = [members[c][i] for i in facts[c][:20000]]
+        g, _ = dg[c].translate(strs)
+        assert np.array_equal(g, do[c].translate(strs))
+        ids.append(do[c].translate([members[c][i] for i in range(len(members[c]))])[facts[c]])
+    ids = np.stack(ids).astype(np.int32)
+    ext = tuple(len(members[c]) for c in cols)
+    cube_q = np.zeros(ext, np.int64)
+    np.add.at(cube_q, tuple(ids), qty)
+    cube_n = np.zeros(ext, np.int64)
+    np.add.at(cube_n, tuple(ids), 1)
+    cq = olap.Cube(ext, np.int32)
+    cq.load(cube_q.astype(np.int32))
+    cn = olap.Cube(ext, np.int32)
+    cn.load(cube_n.astype(np.int32))
+    queries = synth.tpcds_queries(300, members)
+    keys, which = [], []
+    for q in queries:
+        for c in cols:
+            if c == "d_date":
+                keys += [q[c][0], q[c][1]]
+                which += [cols.index(c)] * 2
+            elif c in q:
+                keys.append(q[c])
+                which.append(cols.index(c))
+    tid, _ = olap.translate([dg[c] for c in cols], np.array(which, np.int32), keys)
+    boxes = np.zeros((len(queries), 4, 2), np.int64)
+    k = 0
+    for qi, q in enumerate(queries):
+        for di, c in enumerate(cols):
+            if c == "d_date":
+                boxes[qi, di] = (tid[k], tid[k + 1])
+                k += 2
+            elif c in q:
+                boxes[qi, di] = (tid[k], tid[k]) if tid[k] >= 0 else (1, 0)   # miss -> empty box
+                k += 1
+            else:
+                boxes[qi, di] = (0, ext[di] - 1)
+    sums = cq.query(boxes, np.full(len(boxes), olap.SUM, np.int32))
+    cnts = cn.query(boxes, np.full(len(boxes), olap.SUM, np.int32))
+    ref_s, ref_c = oracle.factscan(ids, qty, boxes)
+    assert np.array_equal(sums["i"], ref_s)
+    assert np.array_equal(cnts["i"], ref_c)

@@ -1,0 +1,96 @@
+"""Host-side logic of the product library, CPU only: block-cyclic shard geometry
+(brute force against the definition), the fast division used by the kernels'
+address generation, and the dictionary hash's host implementation."""
+import ctypes
+
+import numpy as np
+import pytest
+
+import paper_conf_ipps_malikrse12_b200 as olap
+
+
+def _owned(r, G, g, b):
+    return (r // b) % G == g
+
+
+def _local(r, G, b):
+    return (r // (b * G)) * b + r % b
+
+
+@pytest.mark.parametrize("n0", [1, 7, 64, 100, 2048])
+@pytest.mark.parametrize("G,b", [(1, 1), (2, 1), (3, 2), (4, 4), (8, 1), (8, 16), (5, 3)])
+def test_shard_local_rows_brute_force(n0, G, b):
+    rng = np.random.default_rng(n0 * 131 + G * 7 + b)
+    pairs = [(lo, hi) for lo in range(min(n0, 24)) for hi in range(lo, min(n0, 24))]
+    pairs += [tuple(sorted(rng.integers(0, n0, size=2))) for _ in range(300)]
+    for g in range(G):
+        for lo, hi in pairs:
+            lo, hi = int(lo), int(hi)
+            owned = [r for r in range(lo, hi + 1) if _owned(r, G, g, b)]
+            llo, lhi = olap.shard_local_rows(n0, (G, g, b), lo, hi)
+            if not owned:
+                assert llo > lhi
+            else:
+                loc = [_local(r, G, b) for r in owned]
+                assert loc == list(range(loc[0], loc[-1] + 1))     # one contiguous local range
+                assert (llo, lhi) == (loc[0], loc[-1])
+    # every row owned by exactly one shard; local indices dense per shard
+    for g in range(G):
+        rows = [r for r in range(n0) if _owned(r, G, g, b)]
+        assert [_local(r, G, b) for r in rows] == list(range(len(rows)))
+
+
+def test_shard_local_rows_errors():
+    with pytest.raises(olap.OlapError):
+        olap.shard_local_rows(10, (2, 0, 1), 0, 10)
+    with pytest.raises(olap.OlapError):
+        olap.shard_local_rows(10, (2, 2, 1), 0, 3)
+    assert olap.shard_local_rows(10, (2, 1, 1), 4, 3)[0] > olap.shard_local_rows(10, (2, 1, 1), 4, 3)[1]
+
+
+def _fastdiv(d, n):
+    n = np.ascontiguousarray(n, dtype=np.uint32)
+    q = np.empty_like(n)
+    assert olap.lib.olap_selftest_fastdiv(d, n.ctypes.data, n.size, q.ctypes.data) == 0
+    return q
+
+
+def test_fastdiv_exact():
+    rng = np.random.default_rng(0)
+    small = np.arange(0, 1 << 16, dtype=np.uint32)
+    for d in list(range(1, 300)) + [1023, 1024, 1025, 4095, 65535, 65536]:
+        assert np.array_equal(_fastdiv(d, small), small // d)
+    big = np.concatenate([rng.integers(0, 1 << 31, size=20000, dtype=np.int64),
+                          [(1 << 31) - 1, (1 << 31) - 2, 0, 1]]).astype(np.uint32)
+    for d in list(rng.integers(1, 1 << 31, size=200)) + [(1 << 30) + 1, (1 << 31) - 1, 3, 7, 1 << 20]:
+        d = int(d)
+        assert np.array_equal(_fastdiv(d, big), big // d), d
+        edge = np.array([k * d - 1 for k in range(1, 40) if k * d - 1 < (1 << 31)] +
+                        [k * d for k in range(1, 40) if k * d < (1 << 31)], dtype=np.uint32)
+        assert np.array_equal(_fastdiv(d, edge), edge // d), d
+
+
+def _ref_hash(key: bytes) -> int:
+    """The documented hash (common.cuh): fmix64(sum_j fmix64((j<<32|w_j)+K1) + len*K2) mod 2^64."""
+    M = (1 << 64) - 1
+
+    def fmix(k):
+        k ^= k >> 33
+        k = (k * 0xff51afd7ed558ccd) & M
+        k ^= k >> 33
+        k = (k * 0xc4ceb9fe1a85ec53) & M
+        k ^= k >> 33
+        return k
+
+    s = 0
+    for j in range(0, (len(key) + 3) // 4):
+        w = int.from_bytes(key[4 * j:4 * j + 4].ljust(4, b"\0"), "little")
+        s = (s + fmix((((j << 32) | w) + 0x9E3779B97F4A7C15) & M)) & M
+    return fmix((s + len(key) * 0xD6E8FEB86659FD93) & M)
+
+
+def test_dict_hash_host_matches_definition():
+    for key in [b"", b"a", b"abcd", b"abcde", b"2001-01-01", bytes(range(256)), b"\0\0\0", b"\0\0\0\0"]:
+        assert olap.lib.olap_selftest_hash(key, len(key)) == _ref_hash(key)
+    # zero padding must not collide keys of different lengths
+    assert olap.lib.olap_selftest_hash(b"ab", 2) != olap.lib.olap_selftest_hash(b"ab\0", 3)
