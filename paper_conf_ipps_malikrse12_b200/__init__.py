@@ -283,7 +283,8 @@ class Dict:
         return n.value
 
     def translate(self, keys):
-        return translate([self], None, keys)[0]
+        """(ids, n_missing) of keys in this dictionary; -1 = absent."""
+        return translate([self], None, keys)
 
     def bound(self, keys, upper: bool = False) -> np.ndarray:
         buf, offs = _pack(keys)

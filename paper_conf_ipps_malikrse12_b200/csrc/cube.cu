@@ -370,7 +370,9 @@ __global__ void __launch_bounds__(kPlanThreads) plan_kernel(Geo geo, int64_t nq,
         QDesc& d = desc[q];
         int64_t items = 0;
         if (d.mode != MODE_NONE) {
-            const int64_t unit_cells = d.mode == MODE_VEC ? (int64_t)kPieceCells : kRunsPerBatch * d.L;
+            // cells a unit holds: a piece (<= L/ppr rounded up) or a batch of 32 runs
+            const int64_t unit_cells =
+                d.mode == MODE_VEC ? (d.L + (int64_t)d.ppr - 1) / (int64_t)d.ppr : kRunsPerBatch * d.L;
             int64_t upi = teff / unit_cells;
             if (upi < 1) upi = 1;
             if (upi > (1ll << 30)) upi = (1ll << 30);
@@ -397,6 +399,9 @@ __global__ void __launch_bounds__(kPlanThreads) plan_kernel(Geo geo, int64_t nq,
         off += items;
     }
     if (tid == kPlanThreads - 1) {
+        // sum_q items_q <= 2*total/teff + 2*nq <= items_cap by construction;
+        // never write past the item-partial arrays: fail loudly instead
+        if (scan[tid] > items_cap) __trap();
         item_start[nq] = scan[tid];
         *counter = 0ull;
         atomicAdd(bytes_acc, (unsigned long long)(total_cells * 4));
