@@ -25,29 +25,36 @@ constexpr int kMaxDims = 8;
 constexpr int kMaxRunDims = 7;
 constexpr int kWarps = 8;                   // warps per reduce block
 constexpr int kThreads = kWarps * 32;
-constexpr int kPieceCells = 2048;           // MODE_VEC unit: <= 2048 cells (8 KiB) inside one run
-constexpr int kRunsPerBatch = 32;           // MODE_RUNS unit: 32 consecutive runs (one per lane)
-constexpr int64_t kVectorMinRun = 128;      // runs of >= 128 cells stream as 16-B vectors
-constexpr int64_t kItemCells = 262144;      // target item: 1 MiB of 4-byte cells
+constexpr int kTaskSlots = 256;             // slots per warp task (a task spans <= 31 runs)
+constexpr int kUnroll = 4;                  // independent loads in flight per lane
+constexpr int64_t kItemCells = 262144;      // minimum item: 1 MiB of 4-byte cells
 constexpr int64_t kMaxExtent = (1ll << 30); // per-dimension limit (32-bit digit arithmetic)
 constexpr int64_t kMaxCells = (1ll << 42);
 
-enum : int32_t { MODE_NONE = 0, MODE_VEC = 1, MODE_RUNS = 2 };
+// op class of a query: which accumulator the hot loop keeps (SUM and AVG share one)
+enum : int32_t { OPC_NONE = 0, OPC_SUM = 1, OPC_MIN = 2, OPC_MAX = 3 };
 
-// Per-query plan (shard-local).  Run r of the box starts at
-//   base + sum_e digit_e(r) * rs[e]       (digits of r in radix frl[e].d, innermost first)
-// and covers L consecutive cells (all dims after the split dim k are full and merge).
+// Per-query plan (shard-local).  The box is R runs of L consecutive cells (all dims
+// after the split dim k are full and merge into the run, Fig. 2 / DESIGN.md "runs").
+// Run r starts at cell  base + sum_e digit_e(r) * rs[e]  (digits of r in radix
+// frl[e].d, innermost first).  When every run stride is a multiple of 4 cells all runs
+// share the same 16-B misalignment h0, so each run is covered by nslot aligned 16-B
+// "slots" (V = 4 cells) whose first h0 and trailing cells are masked; otherwise V = 1.
+// Slots of all runs are flattened (G = R * nslot) and cut into warp tasks of T slots.
 struct QDesc {
-    int64_t base;
-    int64_t L;
-    int64_t R;
-    int64_t units;
-    int64_t vlocal;
-    uint32_t upi;   // units per item
-    uint32_t ppr;   // pieces per run (MODE_VEC)
-    int32_t mode, nrd, op, pad;
-    FastDiv fL;     // / L (MODE_RUNS; L < 128)
-    FastDiv fppr;   // / ppr (MODE_VEC)
+    int64_t base_al;  // first slot of run 0 (cells, multiple of V)
+    int64_t L;        // run length (cells)
+    int64_t R;        // number of runs
+    int64_t nslot;    // slots per run
+    int64_t G;        // slots in the box
+    int64_t tasks;    // ceil(G / T)
+    int64_t vlocal;   // cells of the box on this shard (R * L)
+    int32_t T;        // slots per task
+    int32_t tpi;      // tasks per item
+    int32_t h0;       // masked leading cells of each run's first slot
+    int32_t V;        // cells per slot (4 or 1)
+    int32_t opc, nrd, op, pad;
+    FastDiv fnslot;   // / nslot (valid when nslot < 2^31)
     FastDiv frl[kMaxRunDims];
     int64_t rs[kMaxRunDims];
 };
@@ -94,34 +101,51 @@ __host__ __device__ __forceinline__ float f32_decode(int32_t c) {
 #endif
 }
 
+__device__ __forceinline__ FastDiv dev_fastdiv(uint32_t l) {
+    FastDiv f;
+    f.d = l;
+    if (l <= 1) {
+        f.m = 0;
+        f.s = 0xffffffffu;
+    } else {
+        const uint32_t lg = 32 - __clz(l - 1);  // ceil(log2 l)
+        const uint32_t p = 31 + lg;
+        f.m = (uint32_t)(((1ull << p) + l - 1) / l);
+        f.s = p - 32;
+    }
+    return f;
+}
+
 // Per-lane accumulators.  int32 cells: SUM in uint64 (wraparound, reading R7),
 // MIN/MAX in int32.  float32 cells: SUM in double (reading R8), MIN/MAX in float.
+// add<OPC>(bits, valid): invalid (masked) cells contribute the op's identity.
 struct AccI {
     unsigned long long s;
     int32_t mn, mx;
     __device__ void init() { s = 0ull; mn = INT_MAX; mx = INT_MIN; }
-    __device__ __forceinline__ void add1(uint32_t bits) {
-        int32_t v = (int32_t)bits;
-        s += (unsigned long long)(long long)v;
-        mn = min(mn, v);
-        mx = max(mx, v);
+    template <int OPC>
+    __device__ __forceinline__ void add(uint32_t bits, bool valid) {
+        const int32_t v = (int32_t)bits;
+        if (OPC == OPC_SUM) s += (unsigned long long)(long long)(valid ? v : 0);
+        if (OPC == OPC_MIN) mn = min(mn, valid ? v : INT_MAX);
+        if (OPC == OPC_MAX) mx = max(mx, valid ? v : INT_MIN);
     }
-    __device__ __forceinline__ void add4(uint4 v) { add1(v.x); add1(v.y); add1(v.z); add1(v.w); }
     __device__ __forceinline__ long long sum_bits() const { return (long long)s; }
     __device__ __forceinline__ int32_t code_max() const { return mx; }
     __device__ __forceinline__ int32_t code_min() const { return mn; }
+    __device__ __forceinline__ bool has_max() const { return mx != INT_MIN; }
 };
 struct AccF {
     double s;
     float mn, mx;
     __device__ void init() { s = 0.0; mn = __int_as_float(0x7f800000); mx = __int_as_float(0xff800000); }
-    __device__ __forceinline__ void add1(uint32_t bits) {
-        float v = __uint_as_float(bits);
-        s += (double)v;
-        mn = fminf(mn, v);
-        mx = fmaxf(mx, v);
+    template <int OPC>
+    __device__ __forceinline__ void add(uint32_t bits, bool valid) {
+        const float v = __uint_as_float(bits);
+        if (OPC == OPC_SUM) s += (double)(valid ? v : 0.0f);
+        if (OPC == OPC_MIN) mn = fminf(mn, valid ? v : __int_as_float(0x7f800000));
+        if (OPC == OPC_MAX) mx = fmaxf(mx, valid ? v : __int_as_float(0xff800000));
     }
-    __device__ __forceinline__ void add4(uint4 v) { add1(v.x); add1(v.y); add1(v.z); add1(v.w); }
     __device__ __forceinline__ long long sum_bits() const { return __double_as_longlong(s); }
     __device__ __forceinline__ int32_t code_max() const { return f32_code(mx); }
     __device__ __forceinline__ int32_t code_min() const { return f32_code(mn); }
@@ -139,66 +163,28 @@ template <> struct SumOps<AccF> {
     }
 };
 
-// Advance a run cursor by `inc` runs (inc < 2^20): add to the mixed-radix digits with carry.
-__device__ __forceinline__ void advance_runs(const QDesc& d, uint32_t (&dig)[kMaxRunDims], int64_t& addr,
-                                             uint32_t inc) {
-    uint32_t c = inc;
+// First slot of run r: base_al + sum_e digit_e(r) * rs[e].  32-bit fast-division
+// chain when r < 2^31 (the common case), 64-bit divisions otherwise.
+__device__ __forceinline__ int64_t run_addr(const QDesc& d, int64_t r) {
+    int64_t a = d.base_al;
+    if (r < (1ll << 31)) {
+        uint32_t x = (uint32_t)r;
 #pragma unroll
-    for (int e = 0; e < kMaxRunDims; ++e) {
-        if (e < d.nrd && c != 0u) {
-            uint32_t t = dig[e] + c;
-            uint32_t q = fdiv(t, d.frl[e]);
-            uint32_t nd = t - q * d.frl[e].d;
-            addr += ((int64_t)nd - (int64_t)dig[e]) * d.rs[e];
-            dig[e] = nd;
-            c = q;
+        for (int e = 0; e < kMaxRunDims; ++e) {
+            if (e < d.nrd) {
+                const uint32_t q = fdiv(x, d.frl[e]);
+                a += (int64_t)(x - q * d.frl[e].d) * d.rs[e];
+                x = q;
+            }
         }
-    }
-}
-
-// Full decode of run index r (64-bit divisions; once per item).
-__device__ void decode_run(const QDesc& d, int64_t r, uint32_t (&dig)[kMaxRunDims], int64_t& addr) {
-    addr = d.base;
-#pragma unroll
-    for (int e = 0; e < kMaxRunDims; ++e) {
-        dig[e] = 0u;
-        if (e < d.nrd) {
-            uint32_t l = d.frl[e].d;
-            int64_t q = r / l;
-            uint32_t di = (uint32_t)(r - q * l);
-            dig[e] = di;
-            addr += (int64_t)di * d.rs[e];
+    } else {
+        for (int e = 0; e < d.nrd; ++e) {
+            const int64_t l = d.frl[e].d, q = r / l;
+            a += (r - q * l) * d.rs[e];
             r = q;
         }
     }
-}
-
-// One warp streams cells [a, a+len) (len <= kPieceCells): scalar head to 16-B
-// alignment, 16-B vector body (4 independent loads in flight per lane), scalar tail.
-template <class Acc, typename T>
-__device__ __forceinline__ void stream_piece(const T* __restrict__ cube, int64_t a, int len, Acc& acc,
-                                             int lane) {
-    int head = (int)((4 - (a & 3)) & 3);
-    if (head > len) head = len;
-    if (lane < head) acc.add1(ld_stream1(cube + a + lane));
-    a += head;
-    len -= head;
-    const int nvec = len >> 2;
-    const uint4* v = reinterpret_cast<const uint4*>(cube + a);
-    int i = lane;
-    for (; i + 96 < nvec; i += 128) {
-        uint4 x0 = ld_stream4(v + i);
-        uint4 x1 = ld_stream4(v + i + 32);
-        uint4 x2 = ld_stream4(v + i + 64);
-        uint4 x3 = ld_stream4(v + i + 96);
-        acc.add4(x0);
-        acc.add4(x1);
-        acc.add4(x2);
-        acc.add4(x3);
-    }
-    for (; i < nvec; i += 32) acc.add4(ld_stream4(v + i));
-    const int tail = len & 3;
-    if (lane < tail) acc.add1(ld_stream1(cube + a + 4 * (int64_t)nvec + lane));
+    return a;
 }
 
 // Largest q in [0,nq) with item_start[q] <= item (32-ary warp search).
@@ -220,15 +206,83 @@ __device__ __forceinline__ int64_t find_query(const int64_t* __restrict__ item_s
     return lo + (31 - __clz(m));
 }
 
+// The hot loop: warp w of the block streams tasks t0+w, t0+w+8, ... < t1 of one query.
+// Lane i holds the first-slot address of run (j0 + i); slot g of the task maps to run
+// j = (rem + g) / nslot (fast division) and slot s within it; the warp reads 32
+// consecutive slots per load instruction, kUnroll loads in flight per lane.
+template <typename T, class Acc, int OPC, int V>
+__device__ __forceinline__ void stream_tasks(const T* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
+                                             Acc& acc, int lane, int w) {
+    int64_t t = t0 + w;
+    if (t >= t1) return;
+    const int64_t T_ = d.T, nslot = d.nslot, L = d.L, G = d.G, R = d.R;
+    const int h0 = d.h0;
+    const bool long_runs = nslot >= T_;
+    int64_t g0 = t * T_;
+    int64_t j0 = g0 / nslot;
+    int64_t rem = g0 - j0 * nslot;
+    const int64_t step = (int64_t)kWarps * T_;
+    for (; t < t1; t += kWarps) {
+        const int64_t left = G - t * T_;
+        const int n = left < T_ ? (int)left : (int)T_;
+        int64_t ra = 0;
+        if (j0 + lane < R) ra = run_addr(d, j0 + lane);
+        for (int i0 = 0; i0 < n; i0 += 32 * kUnroll) {
+            uint32_t v[kUnroll][V];
+            int lo[kUnroll], hi[kUnroll];
+#pragma unroll
+            for (int u = 0; u < kUnroll; ++u) {
+                const int idx = i0 + 32 * u + lane;
+                const bool ok = idx < n;
+                const int64_t gr = rem + (ok ? idx : 0);
+                int j;
+                int64_t s;
+                if (long_runs) {
+                    j = gr >= nslot ? 1 : 0;
+                    s = gr - (j ? nslot : 0);
+                } else {
+                    j = (int)fdiv((uint32_t)gr, d.fnslot);
+                    s = gr - (int64_t)j * nslot;
+                }
+                const int64_t a = __shfl_sync(0xffffffffu, ra, j) + s * V;
+                const int64_t c0 = s * V - h0;  // run-relative cell index of the slot's first cell
+                lo[u] = c0 < 0 ? (int)(-c0) : 0;
+                hi[u] = ok ? (L - c0 >= V ? V : (int)(L - c0)) : 0;
+                if constexpr (V == 4) {
+                    uint4 x = make_uint4(0u, 0u, 0u, 0u);
+                    if (ok) x = ld_stream4(cube + a);
+                    v[u][0] = x.x;
+                    v[u][1] = x.y;
+                    v[u][2] = x.z;
+                    v[u][3] = x.w;
+                } else {
+                    v[u][0] = ok ? ld_stream1(cube + a) : 0u;
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < kUnroll; ++u)
+#pragma unroll
+                for (int k = 0; k < V; ++k) acc.template add<OPC>(v[u][k], k >= lo[u] && k < hi[u]);
+        }
+        rem += step;
+        if (rem >= nslot) {
+            const int64_t dj = nslot < (1ll << 30) ? (int64_t)fdiv((uint32_t)rem, d.fnslot) : (rem >= nslot ? 1 : 0);
+            j0 += dj;
+            rem -= dj * nslot;
+        }
+    }
+}
+
 // ------------------------------------------------------------------ plan
 
 __device__ void build_desc(const Geo& g, const olap_range* r, int32_t op, QDesc& d) {
-    d.mode = MODE_NONE;
+    d.opc = OPC_NONE;
     d.op = op;
     d.vlocal = 0;
-    d.units = 0;
+    d.tasks = 0;
+    d.G = 0;
     d.nrd = 0;
-    d.upi = 1;
+    d.tpi = 1;
     if (op < OLAP_SUM || op > OLAP_AVG) return;
     int64_t lo[kMaxDims], hi[kMaxDims];
     bool empty = false;
@@ -238,81 +292,41 @@ __device__ void build_desc(const Geo& g, const olap_range* r, int32_t op, QDesc&
         if (lo[k] < 0 || hi[k] >= g.n[k]) return;  // invalid: flagged by finalize
         if (lo[k] > hi[k]) empty = true;
     }
-    if (empty || op == OLAP_COUNT) return;
+    if (empty || op == OLAP_COUNT) return;  // COUNT = V needs no cell (Eq. 3, reading R5)
     int64_t llo, lhi;
     if (!shard_local_range(g.n[0], g.G, g.g, g.b, lo[0], hi[0], &llo, &lhi)) return;
     lo[0] = llo;
     hi[0] = lhi;
     int64_t ell[kMaxDims];
     for (int k = 0; k < g.nd; ++k) ell[k] = hi[k] - lo[k] + 1;
-    int ks = g.nd - 1;  // split dim: innermost dim not fully covered
-    while (ks > 0 && ell[ks] == (ks == 0 ? g.local_rows : g.n[ks])) --ks;
+    int ks = g.nd - 1;  // split dim: innermost dim not fully covered (dims after it merge into runs)
+    while (ks > 0 && ell[ks] == g.n[ks]) --ks;
     d.L = ell[ks] * g.stride[ks];
     int64_t R = 1, base = 0;
     for (int k = 0; k < g.nd; ++k) base += lo[k] * g.stride[k];
     int nrd = 0;
+    bool aligned = true;
     for (int k = ks - 1; k >= 0; --k) {
         R *= ell[k];
         if (ell[k] > 1) {
-            d.frl[nrd] = FastDiv{};
-            uint32_t l = (uint32_t)ell[k];
-            // device-side make_fastdiv
-            FastDiv f;
-            f.d = l;
-            if (l <= 1) {
-                f.m = 0;
-                f.s = 0xffffffffu;
-            } else {
-                uint32_t lg = 32 - __clz(l - 1);
-                uint32_t p = 31 + lg;
-                f.m = (uint32_t)(((1ull << p) + l - 1) / l);
-                f.s = p - 32;
-            }
-            d.frl[nrd] = f;
+            d.frl[nrd] = dev_fastdiv((uint32_t)ell[k]);
             d.rs[nrd] = g.stride[k];
+            if (g.stride[k] & 3) aligned = false;
             ++nrd;
         }
     }
     d.nrd = nrd;
     d.R = R;
-    d.base = base;
     d.vlocal = R * d.L;
-    if (d.L >= kVectorMinRun) {
-        d.mode = MODE_VEC;
-        int64_t ppr = (d.L + kPieceCells - 1) / kPieceCells;
-        d.ppr = (uint32_t)ppr;
-        uint32_t l = (uint32_t)ppr;
-        FastDiv f;
-        f.d = l;
-        if (l <= 1) {
-            f.m = 0;
-            f.s = 0xffffffffu;
-        } else {
-            uint32_t lg = 32 - __clz(l - 1);
-            uint32_t p = 31 + lg;
-            f.m = (uint32_t)(((1ull << p) + l - 1) / l);
-            f.s = p - 32;
-        }
-        d.fppr = f;
-        d.units = R * ppr;
-    } else {
-        d.mode = MODE_RUNS;
-        uint32_t l = (uint32_t)d.L;
-        FastDiv f;
-        f.d = l;
-        if (l <= 1) {
-            f.m = 0;
-            f.s = 0xffffffffu;
-        } else {
-            uint32_t lg = 32 - __clz(l - 1);
-            uint32_t p = 31 + lg;
-            f.m = (uint32_t)(((1ull << p) + l - 1) / l);
-            f.s = p - 32;
-        }
-        d.fL = f;
-        d.ppr = 1;
-        d.units = (R + kRunsPerBatch - 1) / kRunsPerBatch;
-    }
+    d.V = aligned ? 4 : 1;
+    d.h0 = aligned ? (int32_t)(base & 3) : 0;
+    d.base_al = base - d.h0;
+    d.nslot = (d.h0 + d.L + d.V - 1) / d.V;
+    d.G = R * d.nslot;
+    d.T = d.nslot < 9 ? (int32_t)(32 * d.nslot) : kTaskSlots;
+    d.tasks = (d.G + d.T - 1) / d.T;
+    d.fnslot = dev_fastdiv(d.nslot < (1ll << 31) ? (uint32_t)d.nslot : 1u);
+    d.opc = (op == OLAP_MIN) ? OPC_MIN : (op == OLAP_MAX) ? OPC_MAX : OPC_SUM;
 }
 
 constexpr int kPlanThreads = 1024;
@@ -348,41 +362,42 @@ __global__ void __launch_bounds__(kPlanThreads) plan_kernel(Geo geo, int64_t nq,
     const int tid = threadIdx.x;
     const int64_t per = (nq + kPlanThreads - 1) / kPlanThreads;
     const int64_t q0 = min(nq, (int64_t)tid * per), q1 = min(nq, q0 + per);
-    int64_t my_cells = 0;
+    int64_t my_cells = 0, my_slot_cells = 0;
     for (int64_t q = q0; q < q1; ++q) {
         QDesc d;
         build_desc(geo, ranges + q * geo.nd, ops[q], d);
         desc[q] = d;
         done[q] = 0;
-        if (d.mode == MODE_NONE) {
+        if (d.opc == OPC_NONE) {
             psum[q] = 0;
             pext[2 * q] = INT_MIN;
             pext[2 * q + 1] = INT_MIN;
+        } else {
+            my_cells += d.vlocal;
+            my_slot_cells += d.G * d.V;
         }
-        my_cells += d.vlocal;
     }
     const int64_t total_cells = block_sum<int64_t>(my_cells, sh);
+    const int64_t total_slot_cells = block_sum<int64_t>(my_slot_cells, sh);
+    // item size: >= 1 MiB, and large enough that sum_q items_q <= items_cap:
+    // items_q <= tasks_q/tpi_q + 1 <= 2*G_q*V_q/teff + 2 (tpi_q*T_q*V_q >= teff/2)
     const int64_t cap_left = items_cap - 2 * nq;
-    int64_t teff = (4 * total_cells + cap_left - 1) / cap_left;
+    int64_t teff = (4 * total_slot_cells + cap_left - 1) / cap_left;
     if (teff < kItemCells) teff = kItemCells;
     int64_t my_items = 0;
     for (int64_t q = q0; q < q1; ++q) {
         QDesc& d = desc[q];
         int64_t items = 0;
-        if (d.mode != MODE_NONE) {
-            // cells a unit holds: a piece (<= L/ppr rounded up) or a batch of 32 runs
-            const int64_t unit_cells =
-                d.mode == MODE_VEC ? (d.L + (int64_t)d.ppr - 1) / (int64_t)d.ppr : kRunsPerBatch * d.L;
-            int64_t upi = teff / unit_cells;
-            if (upi < 1) upi = 1;
-            if (upi > (1ll << 30)) upi = (1ll << 30);
-            d.upi = (uint32_t)upi;
-            items = (d.units + upi - 1) / upi;
+        if (d.opc != OPC_NONE) {
+            int64_t tpi = teff / ((int64_t)d.T * d.V);
+            if (tpi < 1) tpi = 1;
+            if (tpi > (1ll << 30)) tpi = (1ll << 30);
+            d.tpi = (int32_t)tpi;
+            items = (d.tasks + tpi - 1) / tpi;
         }
         item_start[q] = items;
         my_items += items;
     }
-    // exclusive scan of my_items over the block
     __shared__ int64_t scan[kPlanThreads];
     scan[tid] = my_items;
     __syncthreads();
@@ -399,8 +414,7 @@ __global__ void __launch_bounds__(kPlanThreads) plan_kernel(Geo geo, int64_t nq,
         off += items;
     }
     if (tid == kPlanThreads - 1) {
-        // sum_q items_q <= 2*total/teff + 2*nq <= items_cap by construction;
-        // never write past the item-partial arrays: fail loudly instead
+        // never write past the item-partial arrays: fail loudly instead (cannot happen by the bound above)
         if (scan[tid] > items_cap) __trap();
         item_start[nq] = scan[tid];
         *counter = 0ull;
@@ -411,15 +425,14 @@ __global__ void __launch_bounds__(kPlanThreads) plan_kernel(Geo geo, int64_t nq,
 // ------------------------------------------------------------------ reduce (the hot loop)
 
 template <typename T, class Acc>
-__global__ void __launch_bounds__(kThreads) reduce_kernel(const T* __restrict__ cube, int64_t nq,
-                                                          const QDesc* __restrict__ desc,
-                                                          const int64_t* __restrict__ item_start,
-                                                          unsigned long long* counter, int32_t* done,
-                                                          long long* item_sum, int32_t* item_ext,
-                                                          int64_t* psum, int32_t* pext) {
+__global__ void __launch_bounds__(kThreads, 4) reduce_kernel(const T* __restrict__ cube, int64_t nq,
+                                                             const QDesc* __restrict__ desc,
+                                                             const int64_t* __restrict__ item_start,
+                                                             unsigned long long* counter, int32_t* done,
+                                                             long long* item_sum, int32_t* item_ext, int64_t* psum,
+                                                             int32_t* pext) {
     __shared__ QDesc sd;
-    __shared__ int64_t s_item, s_q, s_r0, s_addr0;
-    __shared__ uint32_t s_p0, s_dig0[kMaxRunDims];
+    __shared__ int64_t s_item, s_q;
     __shared__ long long s_wsum[kWarps];
     __shared__ int32_t s_wmx[kWarps], s_wmn[kWarps];
     __shared__ int s_last;
@@ -445,87 +458,27 @@ __global__ void __launch_bounds__(kThreads) reduce_kernel(const T* __restrict__ 
         }
         __syncthreads();
         const int64_t first_item = __ldg(item_start + q);
-        const int64_t u0 = (item - first_item) * (int64_t)sd.upi;
-        const int64_t u1 = min(sd.units, u0 + (int64_t)sd.upi);
-        if (threadIdx.x == 0) {
-            uint32_t dig[kMaxRunDims];
-            int64_t addr, r0;
-            if (sd.mode == MODE_VEC) {
-                r0 = u0 / sd.ppr;
-                s_p0 = (uint32_t)(u0 - r0 * sd.ppr);
-            } else {
-                r0 = u0 * kRunsPerBatch;
-                s_p0 = 0;
-            }
-            decode_run(sd, r0, dig, addr);
-            s_r0 = r0;
-            s_addr0 = addr;
-#pragma unroll
-            for (int e = 0; e < kMaxRunDims; ++e) s_dig0[e] = dig[e];
-        }
-        __syncthreads();
+        const int64_t t0 = (item - first_item) * (int64_t)sd.tpi;
+        const int64_t t1 = min(sd.tasks, t0 + (int64_t)sd.tpi);
 
         Acc acc;
         acc.init();
-        uint32_t dig[kMaxRunDims];
-#pragma unroll
-        for (int e = 0; e < kMaxRunDims; ++e) dig[e] = s_dig0[e];
-        int64_t addr = s_addr0;
-
-        if (sd.mode == MODE_VEC) {
-            const uint32_t ppr = sd.ppr;
-            uint32_t p = s_p0 + (uint32_t)w;
-            if (p >= ppr) {
-                const uint32_t dr = fdiv(p, sd.fppr);
-                p -= dr * ppr;
-                advance_runs(sd, dig, addr, dr);
-            }
-            for (int64_t u = u0 + w; u < u1; u += kWarps) {
-                const int64_t off = (int64_t)p * kPieceCells;
-                const int64_t rem = sd.L - off;
-                const int len = rem < kPieceCells ? (int)rem : kPieceCells;
-                stream_piece(cube, addr + off, len, acc, lane);
-                p += kWarps;
-                if (p >= ppr) {
-                    const uint32_t dr = fdiv(p, sd.fppr);
-                    p -= dr * ppr;
-                    advance_runs(sd, dig, addr, dr);
-                }
-            }
+        const int opc = sd.opc;
+        if (sd.V == 4) {
+            if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 4>(cube, sd, t0, t1, acc, lane, w);
+            else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 4>(cube, sd, t0, t1, acc, lane, w);
+            else stream_tasks<T, Acc, OPC_MAX, 4>(cube, sd, t0, t1, acc, lane, w);
         } else {
-            // lane owns run (first run of the warp's batch) + lane
-            const int64_t R = sd.R;
-            const int L = (int)sd.L;
-            advance_runs(sd, dig, addr, (uint32_t)(w * kRunsPerBatch + lane));
-            for (int64_t u = u0 + w; u < u1; u += kWarps) {
-                const int64_t rfirst = u * kRunsPerBatch;
-                const int64_t nr64 = R - rfirst;
-                const int nr = nr64 < kRunsPerBatch ? (int)nr64 : kRunsPerBatch;
-                const int ncell = nr * L;
-                for (int c0 = 0; c0 < ncell; c0 += 128) {
-                    uint32_t v[4];
-                    bool ok[4];
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) {
-                        const int c = c0 + j * 32 + lane;
-                        ok[j] = c < ncell;
-                        const int cc = ok[j] ? c : 0;
-                        const uint32_t ri = fdiv((uint32_t)cc, sd.fL);
-                        const int o = cc - (int)ri * L;
-                        const int64_t a = __shfl_sync(0xffffffffu, addr, (int)ri) + o;
-                        v[j] = ok[j] ? ld_stream1(cube + a) : 0u;
-                    }
-#pragma unroll
-                    for (int j = 0; j < 4; ++j)
-                        if (ok[j]) acc.add1(v[j]);
-                }
-                advance_runs(sd, dig, addr, (uint32_t)(kWarps * kRunsPerBatch));
-            }
+            if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 1>(cube, sd, t0, t1, acc, lane, w);
+            else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 1>(cube, sd, t0, t1, acc, lane, w);
+            else stream_tasks<T, Acc, OPC_MAX, 1>(cube, sd, t0, t1, acc, lane, w);
         }
 
         // warp -> block -> item partial (fixed order: deterministic)
         long long s = acc.sum_bits();
         int32_t cmx = acc.code_max(), cmn = ~acc.code_min();
+        if (opc != OPC_MAX) cmx = INT_MIN;
+        if (opc != OPC_MIN) cmn = INT_MIN;
 #pragma unroll
         for (int o = 16; o; o >>= 1) s = SumOps<Acc>::add(s, __shfl_xor_sync(0xffffffffu, s, o));
         cmx = __reduce_max_sync(0xffffffffu, cmx);
@@ -549,7 +502,7 @@ __global__ void __launch_bounds__(kThreads) reduce_kernel(const T* __restrict__ 
             item_ext[2 * item] = tmx;
             item_ext[2 * item + 1] = tmn;
             __threadfence();
-            const int64_t nitems = (sd.units + sd.upi - 1) / sd.upi;
+            const int64_t nitems = (sd.tasks + sd.tpi - 1) / sd.tpi;
             const int prev = atomicAdd(done + q, 1);
             s_last = (prev == (int)nitems - 1);
         }
@@ -557,7 +510,7 @@ __global__ void __launch_bounds__(kThreads) reduce_kernel(const T* __restrict__ 
         if (s_last) {
             // last finisher of query q: fold its item partials in fixed order
             __threadfence();
-            const int64_t nitems = (sd.units + sd.upi - 1) / sd.upi;
+            const int64_t nitems = (sd.tasks + sd.tpi - 1) / sd.tpi;
             long long ts = 0;
             int32_t tmx = INT_MIN, tmn = INT_MIN;
             for (int64_t i = threadIdx.x; i < nitems; i += kThreads) {
@@ -918,7 +871,8 @@ int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_sh
     c->local_rows = shard_rows(c->n[0], sh.nshards, sh.shard, sh.block);
     c->local_cells = c->local_rows * c->row_cells;
     int rc = OLAP_OK;
-    cudaError_t e = cudaMalloc(&c->d_cells, std::max<int64_t>(c->local_cells, 1) * 4);
+    // +64 B: a run's last 16-B slot may extend up to 3 cells past the final cell (masked)
+    cudaError_t e = cudaMalloc(&c->d_cells, std::max<int64_t>(c->local_cells, 1) * 4 + 64);
     if (e != cudaSuccess) {
         rc = set_error(e == cudaErrorMemoryAllocation ? OLAP_E_NOMEM : OLAP_E_CUDA, "cudaMalloc of %lld cells: %s",
                        (long long)c->local_cells, cudaGetErrorString(e));
