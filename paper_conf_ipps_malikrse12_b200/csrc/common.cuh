@@ -32,36 +32,30 @@ void clear_error();
     } while (0)
 
 // ------------------------------------------------------------------ fast division
-// q = n / d for 0 <= n < 2^31 and 1 <= d < 2^31 via one mul-hi and one shift
-// (round-up reciprocal, Granlund-Montgomery): p = 31 + ceil(log2 d),
-// m = ceil(2^p / d) < 2^32.  Verified exhaustively for small d and randomly for
-// large d by tests/test_host_logic.py (through olap_selftest_fastdiv).
+// q = n / d for 0 <= n < 2^31 and 1 <= d < 2^31, branch-free (Granlund-Montgomery,
+// 33-bit magic): l = ceil(log2 d), m = floor(2^32 (2^l - d) / d) + 1,
+// q = (mulhi(n, m) + n) >> l   (no overflow: mulhi(n,m) + n < 2n < 2^32).
+// Verified exhaustively for small d and randomly for large d by
+// tests/test_host_logic.py (through olap_selftest_fastdiv).
 struct FastDiv {
-    uint32_t d, m, s;  // s = p - 32 (or 0xffffffff for d == 1)
+    uint32_t d, m, l;
 };
 
 inline FastDiv make_fastdiv(uint32_t d) {
     FastDiv f;
     f.d = d;
-    if (d <= 1) {
-        f.m = 0;
-        f.s = 0xffffffffu;
-        return f;
-    }
     uint32_t l = 0;
     while ((1ull << l) < d) ++l;  // ceil(log2 d)
-    uint32_t p = 31 + l;
-    f.m = (uint32_t)(((1ull << p) + d - 1) / d);
-    f.s = p - 32;
+    f.l = l;
+    f.m = (uint32_t)(((1ull << 32) * ((1ull << l) - d)) / d + 1);
     return f;
 }
 
 OLAP_HD uint32_t fdiv(uint32_t n, const FastDiv& f) {
-    if (f.s == 0xffffffffu) return n;
 #ifdef __CUDA_ARCH__
-    return __umulhi(n, f.m) >> f.s;
+    return (__umulhi(n, f.m) + n) >> f.l;
 #else
-    return (uint32_t)(((uint64_t)n * f.m) >> 32) >> f.s;
+    return (uint32_t)((((uint64_t)n * f.m) >> 32) + n) >> f.l;
 #endif
 }
 

@@ -27,6 +27,10 @@ constexpr int kWarps = 8;                   // warps per reduce block
 constexpr int kThreads = kWarps * 32;
 constexpr int kTaskSlots = 256;             // slots per warp task (a task spans <= 31 runs)
 constexpr int kUnroll = 4;                  // independent loads in flight per lane
+#ifndef OLAP_MIN_BLOCKS
+#define OLAP_MIN_BLOCKS 3
+#endif
+constexpr int kMinBlocks = OLAP_MIN_BLOCKS;  // resident reduce blocks per SM the register budget targets
 constexpr int64_t kItemCells = 262144;      // minimum item: 1 MiB of 4-byte cells
 constexpr int64_t kMaxExtent = (1ll << 30); // per-dimension limit (32-bit digit arithmetic)
 constexpr int64_t kMaxCells = (1ll << 42);
@@ -101,18 +105,11 @@ __host__ __device__ __forceinline__ float f32_decode(int32_t c) {
 #endif
 }
 
-__device__ __forceinline__ FastDiv dev_fastdiv(uint32_t l) {
+__device__ __forceinline__ FastDiv dev_fastdiv(uint32_t d) {
     FastDiv f;
-    f.d = l;
-    if (l <= 1) {
-        f.m = 0;
-        f.s = 0xffffffffu;
-    } else {
-        const uint32_t lg = 32 - __clz(l - 1);  // ceil(log2 l)
-        const uint32_t p = 31 + lg;
-        f.m = (uint32_t)(((1ull << p) + l - 1) / l);
-        f.s = p - 32;
-    }
+    f.d = d;
+    f.l = d <= 1 ? 0u : 32u - __clz(d - 1);  // ceil(log2 d)
+    f.m = (uint32_t)(((1ull << 32) * ((1ull << f.l) - d)) / d + 1);
     return f;
 }
 
@@ -126,7 +123,10 @@ struct AccI {
     template <int OPC>
     __device__ __forceinline__ void add(uint32_t bits, bool valid) {
         const int32_t v = (int32_t)bits;
-        if (OPC == OPC_SUM) s += (unsigned long long)(long long)(valid ? v : 0);
+        if (OPC == OPC_SUM) {
+            const int32_t x = valid ? v : 0;
+            asm("mad.wide.s32 %0, %1, 1, %0;" : "+l"(s) : "r"(x));  // s += sext(x): one IMAD.WIDE
+        }
         if (OPC == OPC_MIN) mn = min(mn, valid ? v : INT_MAX);
         if (OPC == OPC_MAX) mx = max(mx, valid ? v : INT_MIN);
     }
@@ -165,7 +165,7 @@ template <> struct SumOps<AccF> {
 
 // First slot of run r: base_al + sum_e digit_e(r) * rs[e].  32-bit fast-division
 // chain when r < 2^31 (the common case), 64-bit divisions otherwise.
-__device__ __forceinline__ int64_t run_addr(const QDesc& d, int64_t r) {
+__device__ __noinline__ int64_t run_addr(const QDesc& d, int64_t r) {
     int64_t a = d.base_al;
     if (r < (1ll << 31)) {
         uint32_t x = (uint32_t)r;
@@ -206,27 +206,50 @@ __device__ __forceinline__ int64_t find_query(const int64_t* __restrict__ item_s
     return lo + (31 - __clz(m));
 }
 
-// The hot loop: warp w of the block streams tasks t0+w, t0+w+8, ... < t1 of one query.
-// Lane i holds the first-slot address of run (j0 + i); slot g of the task maps to run
-// j = (rem + g) / nslot (fast division) and slot s within it; the warp reads 32
-// consecutive slots per load instruction, kUnroll loads in flight per lane.
+// Load kUnroll slots (V cells each) and fold them into the accumulator.  Masks:
+// cells [lo, hi) of a slot are the box's; the rest of the slot is skipped.
+template <typename T, class Acc, int OPC, int V, bool MASKED>
+__device__ __forceinline__ void fold(Acc& acc, const uint32_t (&v)[kUnroll][V], const int (&lo)[kUnroll],
+                                     const int (&hi)[kUnroll]) {
+#pragma unroll
+    for (int u = 0; u < kUnroll; ++u)
+#pragma unroll
+        for (int k = 0; k < V; ++k) acc.template add<OPC>(v[u][k], MASKED ? (k >= lo[u] && k < hi[u]) : true);
+}
+
+template <int V>
+__device__ __forceinline__ void load_slot(const uint32_t* p, bool ok, uint32_t (&dst)[V]) {
+    if constexpr (V == 4) {
+        uint4 x = make_uint4(0u, 0u, 0u, 0u);
+        if (ok) x = ld_stream4(p);
+        dst[0] = x.x;
+        dst[1] = x.y;
+        dst[2] = x.z;
+        dst[3] = x.w;
+    } else {
+        dst[0] = ok ? ld_stream1(p) : 0u;
+    }
+}
+
+// Short runs (nslot < T): a task spans <= 31 runs.  Lane i holds the first-slot
+// address of run j0+i; slot g of the task is run j = (rem+g)/nslot, slot s of it;
+// all index math is 32-bit, the run address comes from a shuffle.
 template <typename T, class Acc, int OPC, int V>
-__device__ __forceinline__ void stream_tasks(const T* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
+__device__ __forceinline__ void stream_short(const uint32_t* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
                                              Acc& acc, int lane, int w) {
     int64_t t = t0 + w;
     if (t >= t1) return;
-    const int64_t T_ = d.T, nslot = d.nslot, L = d.L, G = d.G, R = d.R;
-    const int h0 = d.h0;
-    const bool long_runs = nslot >= T_;
-    int64_t g0 = t * T_;
-    int64_t j0 = g0 / nslot;
-    int64_t rem = g0 - j0 * nslot;
-    const int64_t step = (int64_t)kWarps * T_;
+    const int T_ = d.T, nslot = (int)d.nslot, h0 = d.h0;
+    const int tail = (int)(d.h0 + d.L - (int64_t)V * (nslot - 1));  // valid cells of a run's last slot
+    const FastDiv fn = d.fnslot;
+    const int64_t G = d.G, R = d.R;
+    int64_t j0 = (t * T_) / nslot;
+    int rem = (int)(t * T_ - j0 * nslot);
+    const int step = kWarps * T_;
     for (; t < t1; t += kWarps) {
         const int64_t left = G - t * T_;
-        const int n = left < T_ ? (int)left : (int)T_;
-        int64_t ra = 0;
-        if (j0 + lane < R) ra = run_addr(d, j0 + lane);
+        const int n = left < T_ ? (int)left : T_;
+        const int64_t ra = (j0 + lane < R) ? run_addr(d, j0 + lane) : 0;
         for (int i0 = 0; i0 < n; i0 += 32 * kUnroll) {
             uint32_t v[kUnroll][V];
             int lo[kUnroll], hi[kUnroll];
@@ -234,43 +257,82 @@ __device__ __forceinline__ void stream_tasks(const T* __restrict__ cube, const Q
             for (int u = 0; u < kUnroll; ++u) {
                 const int idx = i0 + 32 * u + lane;
                 const bool ok = idx < n;
-                const int64_t gr = rem + (ok ? idx : 0);
-                int j;
-                int64_t s;
-                if (long_runs) {
-                    j = gr >= nslot ? 1 : 0;
-                    s = gr - (j ? nslot : 0);
-                } else {
-                    j = (int)fdiv((uint32_t)gr, d.fnslot);
-                    s = gr - (int64_t)j * nslot;
-                }
-                const int64_t a = __shfl_sync(0xffffffffu, ra, j) + s * V;
-                const int64_t c0 = s * V - h0;  // run-relative cell index of the slot's first cell
-                lo[u] = c0 < 0 ? (int)(-c0) : 0;
-                hi[u] = ok ? (L - c0 >= V ? V : (int)(L - c0)) : 0;
-                if constexpr (V == 4) {
-                    uint4 x = make_uint4(0u, 0u, 0u, 0u);
-                    if (ok) x = ld_stream4(cube + a);
-                    v[u][0] = x.x;
-                    v[u][1] = x.y;
-                    v[u][2] = x.z;
-                    v[u][3] = x.w;
-                } else {
-                    v[u][0] = ok ? ld_stream1(cube + a) : 0u;
-                }
+                const uint32_t gr = (uint32_t)(rem + (ok ? idx : 0));
+                const int j = (int)fdiv(gr, fn);
+                const int s = (int)gr - j * nslot;
+                const int64_t a = __shfl_sync(0xffffffffu, ra, j) + (int64_t)s * V;
+                lo[u] = s == 0 ? h0 : 0;
+                hi[u] = ok ? (s == nslot - 1 ? tail : V) : 0;
+                load_slot<V>(cube + a, ok, v[u]);
             }
-#pragma unroll
-            for (int u = 0; u < kUnroll; ++u)
-#pragma unroll
-                for (int k = 0; k < V; ++k) acc.template add<OPC>(v[u][k], k >= lo[u] && k < hi[u]);
+            fold<T, Acc, OPC, V, true>(acc, v, lo, hi);
         }
         rem += step;
+        const int dj = (int)fdiv((uint32_t)rem, fn);
+        j0 += dj;
+        rem -= dj * nslot;
+    }
+}
+
+// Stream slots [0, count) of one run segment starting at slot address p (cells).
+// first: slot 0 is the run's first slot (mask h0 leading cells); last: slot
+// count-1 is the run's last slot (keep `tail` cells).  Interior steps skip masking.
+template <typename T, class Acc, int OPC, int V>
+__device__ __forceinline__ void stream_segment(const uint32_t* __restrict__ p, int count, bool first, bool last, int h0,
+                                               int tail, Acc& acc, int lane) {
+    for (int i0 = 0; i0 < count; i0 += 32 * kUnroll) {
+        uint32_t v[kUnroll][V];
+        int lo[kUnroll], hi[kUnroll];
+        const bool interior = (i0 > 0 || !first || V == 1) && i0 + 32 * kUnroll <= count - (last ? 1 : 0);
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+            const int idx = i0 + 32 * u + lane;
+            const bool ok = idx < count;
+            lo[u] = (first && idx == 0) ? h0 : 0;
+            hi[u] = ok ? ((last && idx == count - 1) ? tail : V) : 0;
+            load_slot<V>(p + (int64_t)idx * V, ok, v[u]);
+        }
+        if (interior) fold<T, Acc, OPC, V, false>(acc, v, lo, hi);
+        else fold<T, Acc, OPC, V, true>(acc, v, lo, hi);
+    }
+}
+
+// Long runs (nslot >= T): a task is at most two contiguous segments (the end of
+// run j0 and the start of run j0+1).
+template <typename T, class Acc, int OPC, int V>
+__device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
+                                            Acc& acc, int lane, int w) {
+    int64_t t = t0 + w;
+    if (t >= t1) return;
+    const int T_ = d.T, h0 = d.h0;
+    const int64_t nslot = d.nslot, G = d.G;
+    const int tail = (int)(d.h0 + d.L - (int64_t)V * (nslot - 1));
+    int64_t j0 = (t * T_) / nslot;
+    int64_t rem = t * T_ - j0 * nslot;
+    const int64_t step = (int64_t)kWarps * T_;
+    for (; t < t1; t += kWarps) {
+        const int64_t left = G - t * T_;
+        const int n = left < T_ ? (int)left : T_;
+        const int64_t in_run = nslot - rem;
+        const int c1 = in_run < n ? (int)in_run : n;
+        stream_segment<T, Acc, OPC, V>(cube + run_addr(d, j0) + rem * V, c1, rem == 0, rem + c1 == nslot, h0, tail,
+                                       acc, lane);
+        if (c1 < n) stream_segment<T, Acc, OPC, V>(cube + run_addr(d, j0 + 1), n - c1, true, false, h0, tail, acc, lane);
+        rem += step;
         if (rem >= nslot) {
-            const int64_t dj = nslot < (1ll << 30) ? (int64_t)fdiv((uint32_t)rem, d.fnslot) : (rem >= nslot ? 1 : 0);
+            const int64_t dj = nslot < (1ll << 20) ? (int64_t)fdiv((uint32_t)rem, d.fnslot) : 1;
             j0 += dj;
             rem -= dj * nslot;
         }
     }
+}
+
+template <typename T, class Acc, int OPC, int V>
+__device__ __forceinline__ void stream_tasks(const T* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
+                                             Acc& acc, int lane, int w) {
+    const uint32_t* c = reinterpret_cast<const uint32_t*>(cube);
+    if (d.nslot < d.T) stream_short<T, Acc, OPC, V>(c, d, t0, t1, acc, lane, w);
+    else stream_long<T, Acc, OPC, V>(c, d, t0, t1, acc, lane, w);
 }
 
 // ------------------------------------------------------------------ plan
@@ -425,7 +487,7 @@ __global__ void __launch_bounds__(kPlanThreads) plan_kernel(Geo geo, int64_t nq,
 // ------------------------------------------------------------------ reduce (the hot loop)
 
 template <typename T, class Acc>
-__global__ void __launch_bounds__(kThreads, 4) reduce_kernel(const T* __restrict__ cube, int64_t nq,
+__global__ void __launch_bounds__(kThreads, kMinBlocks) reduce_kernel(const T* __restrict__ cube, int64_t nq,
                                                              const QDesc* __restrict__ desc,
                                                              const int64_t* __restrict__ item_start,
                                                              unsigned long long* counter, int32_t* done,
