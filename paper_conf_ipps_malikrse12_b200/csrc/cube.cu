@@ -25,7 +25,7 @@ constexpr int kMaxDims = 8;
 constexpr int kMaxRunDims = 7;
 constexpr int kWarps = 8;                   // warps per reduce block
 constexpr int kThreads = kWarps * 32;
-constexpr int kTaskSlots = 256;             // slots per warp task (a task spans <= 31 runs)
+constexpr int kTaskSlots = 2048;            // max slots per warp task (32 KiB of 16-B slots)
 constexpr int kUnroll = 4;                  // independent loads in flight per lane
 #ifndef OLAP_MIN_BLOCKS
 #define OLAP_MIN_BLOCKS 3
@@ -121,14 +121,15 @@ struct AccI {
     int32_t mn, mx;
     __device__ void init() { s = 0ull; mn = INT_MAX; mx = INT_MIN; }
     template <int OPC>
-    __device__ __forceinline__ void add(uint32_t bits, bool valid) {
+    __device__ __forceinline__ void add(uint32_t bits) {
         const int32_t v = (int32_t)bits;
-        if (OPC == OPC_SUM) {
-            const int32_t x = valid ? v : 0;
-            asm("mad.wide.s32 %0, %1, 1, %0;" : "+l"(s) : "r"(x));  // s += sext(x): one IMAD.WIDE
-        }
-        if (OPC == OPC_MIN) mn = min(mn, valid ? v : INT_MAX);
-        if (OPC == OPC_MAX) mx = max(mx, valid ? v : INT_MIN);
+        if (OPC == OPC_SUM) asm("mad.wide.s32 %0, %1, 1, %0;" : "+l"(s) : "r"(v));  // s += sext(v): one IMAD.WIDE
+        if (OPC == OPC_MIN) mn = min(mn, v);
+        if (OPC == OPC_MAX) mx = max(mx, v);
+    }
+    template <int OPC>
+    __device__ __forceinline__ void add_if(uint32_t bits, uint32_t valid) {
+        if (valid) add<OPC>(bits);
     }
     __device__ __forceinline__ long long sum_bits() const { return (long long)s; }
     __device__ __forceinline__ int32_t code_max() const { return mx; }
@@ -140,11 +141,15 @@ struct AccF {
     float mn, mx;
     __device__ void init() { s = 0.0; mn = __int_as_float(0x7f800000); mx = __int_as_float(0xff800000); }
     template <int OPC>
-    __device__ __forceinline__ void add(uint32_t bits, bool valid) {
+    __device__ __forceinline__ void add(uint32_t bits) {
         const float v = __uint_as_float(bits);
-        if (OPC == OPC_SUM) s += (double)(valid ? v : 0.0f);
-        if (OPC == OPC_MIN) mn = fminf(mn, valid ? v : __int_as_float(0x7f800000));
-        if (OPC == OPC_MAX) mx = fmaxf(mx, valid ? v : __int_as_float(0xff800000));
+        if (OPC == OPC_SUM) s += (double)v;
+        if (OPC == OPC_MIN) mn = fminf(mn, v);
+        if (OPC == OPC_MAX) mx = fmaxf(mx, v);
+    }
+    template <int OPC>
+    __device__ __forceinline__ void add_if(uint32_t bits, uint32_t valid) {
+        if (valid) add<OPC>(bits);
     }
     __device__ __forceinline__ long long sum_bits() const { return __double_as_longlong(s); }
     __device__ __forceinline__ int32_t code_max() const { return f32_code(mx); }
@@ -206,15 +211,17 @@ __device__ __forceinline__ int64_t find_query(const int64_t* __restrict__ item_s
     return lo + (31 - __clz(m));
 }
 
-// Load kUnroll slots (V cells each) and fold them into the accumulator.  Masks:
-// cells [lo, hi) of a slot are the box's; the rest of the slot is skipped.
-template <typename T, class Acc, int OPC, int V, bool MASKED>
-__device__ __forceinline__ void fold(Acc& acc, const uint32_t (&v)[kUnroll][V], const int (&lo)[kUnroll],
-                                     const int (&hi)[kUnroll]) {
+// Fold kUnroll slots (V cells each) into the accumulator.  m[u] bit k set <=> cell k
+// of slot u belongs to the box (masked cells are skipped through predication).
+template <class Acc, int OPC, int V, bool MASKED>
+__device__ __forceinline__ void fold(Acc& acc, const uint32_t (&v)[kUnroll][V], const uint32_t (&m)[kUnroll]) {
 #pragma unroll
     for (int u = 0; u < kUnroll; ++u)
 #pragma unroll
-        for (int k = 0; k < V; ++k) acc.template add<OPC>(v[u][k], MASKED ? (k >= lo[u] && k < hi[u]) : true);
+        for (int k = 0; k < V; ++k) {
+            if (MASKED) acc.template add_if<OPC>(v[u][k], (m[u] >> k) & 1u);
+            else acc.template add<OPC>(v[u][k]);
+        }
 }
 
 template <int V>
@@ -231,16 +238,28 @@ __device__ __forceinline__ void load_slot(const uint32_t* p, bool ok, uint32_t (
     }
 }
 
+// Masks of a run's first and last slot (bit k = cell k is in the box).
+template <int V>
+__device__ __forceinline__ void slot_masks(const QDesc& d, uint32_t& fm, uint32_t& lm) {
+    const uint32_t full = (1u << V) - 1u;
+    const int tail = (int)(d.h0 + d.L - (int64_t)V * (d.nslot - 1));  // cells of the last slot in the run
+    fm = full & ~((1u << d.h0) - 1u);
+    lm = (1u << tail) - 1u;
+    if (d.nslot == 1) fm &= lm, lm = fm;
+}
+
 // Short runs (nslot < T): a task spans <= 31 runs.  Lane i holds the first-slot
 // address of run j0+i; slot g of the task is run j = (rem+g)/nslot, slot s of it;
 // all index math is 32-bit, the run address comes from a shuffle.
-template <typename T, class Acc, int OPC, int V>
+template <class Acc, int OPC, int V>
 __device__ __forceinline__ void stream_short(const uint32_t* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
                                              Acc& acc, int lane, int w) {
     int64_t t = t0 + w;
     if (t >= t1) return;
-    const int T_ = d.T, nslot = (int)d.nslot, h0 = d.h0;
-    const int tail = (int)(d.h0 + d.L - (int64_t)V * (nslot - 1));  // valid cells of a run's last slot
+    const int T_ = d.T, nslot = (int)d.nslot;
+    uint32_t fm, lm;
+    slot_masks<V>(d, fm, lm);
+    const uint32_t full = (1u << V) - 1u;
     const FastDiv fn = d.fnslot;
     const int64_t G = d.G, R = d.R;
     int64_t j0 = (t * T_) / nslot;
@@ -252,20 +271,19 @@ __device__ __forceinline__ void stream_short(const uint32_t* __restrict__ cube, 
         const int64_t ra = (j0 + lane < R) ? run_addr(d, j0 + lane) : 0;
         for (int i0 = 0; i0 < n; i0 += 32 * kUnroll) {
             uint32_t v[kUnroll][V];
-            int lo[kUnroll], hi[kUnroll];
+            uint32_t m[kUnroll];
 #pragma unroll
             for (int u = 0; u < kUnroll; ++u) {
                 const int idx = i0 + 32 * u + lane;
                 const bool ok = idx < n;
-                const uint32_t gr = (uint32_t)(rem + (ok ? idx : 0));
+                const uint32_t gr = (uint32_t)(rem + idx);
                 const int j = (int)fdiv(gr, fn);
                 const int s = (int)gr - j * nslot;
-                const int64_t a = __shfl_sync(0xffffffffu, ra, j) + (int64_t)s * V;
-                lo[u] = s == 0 ? h0 : 0;
-                hi[u] = ok ? (s == nslot - 1 ? tail : V) : 0;
+                const int64_t a = __shfl_sync(0xffffffffu, ra, j & 31) + (int64_t)s * V;
+                m[u] = ok ? ((s == 0 ? fm : full) & (s == nslot - 1 ? lm : full)) : 0u;
                 load_slot<V>(cube + a, ok, v[u]);
             }
-            fold<T, Acc, OPC, V, true>(acc, v, lo, hi);
+            fold<Acc, OPC, V, true>(acc, v, m);
         }
         rem += step;
         const int dj = (int)fdiv((uint32_t)rem, fn);
@@ -275,38 +293,41 @@ __device__ __forceinline__ void stream_short(const uint32_t* __restrict__ cube, 
 }
 
 // Stream slots [0, count) of one run segment starting at slot address p (cells).
-// first: slot 0 is the run's first slot (mask h0 leading cells); last: slot
-// count-1 is the run's last slot (keep `tail` cells).  Interior steps skip masking.
-template <typename T, class Acc, int OPC, int V>
-__device__ __forceinline__ void stream_segment(const uint32_t* __restrict__ p, int count, bool first, bool last, int h0,
-                                               int tail, Acc& acc, int lane) {
+// fmask / lmask: masks of slot 0 and slot count-1 (full when not a run edge).
+// Steps with no edge slot skip masking entirely.
+template <class Acc, int OPC, int V>
+__device__ __forceinline__ void stream_segment(const uint32_t* __restrict__ p, int count, uint32_t fmask,
+                                               uint32_t lmask, Acc& acc, int lane) {
+    const uint32_t full = (1u << V) - 1u;
     for (int i0 = 0; i0 < count; i0 += 32 * kUnroll) {
         uint32_t v[kUnroll][V];
-        int lo[kUnroll], hi[kUnroll];
-        const bool interior = (i0 > 0 || !first || V == 1) && i0 + 32 * kUnroll <= count - (last ? 1 : 0);
+        uint32_t m[kUnroll];
+        const bool interior = (i0 > 0 || fmask == full) && (i0 + 32 * kUnroll < count || lmask == full) &&
+                              i0 + 32 * kUnroll <= count;
 #pragma unroll
         for (int u = 0; u < kUnroll; ++u) {
             const int idx = i0 + 32 * u + lane;
             const bool ok = idx < count;
-            lo[u] = (first && idx == 0) ? h0 : 0;
-            hi[u] = ok ? ((last && idx == count - 1) ? tail : V) : 0;
+            m[u] = ok ? ((idx == 0 ? fmask : full) & (idx == count - 1 ? lmask : full)) : 0u;
             load_slot<V>(p + (int64_t)idx * V, ok, v[u]);
         }
-        if (interior) fold<T, Acc, OPC, V, false>(acc, v, lo, hi);
-        else fold<T, Acc, OPC, V, true>(acc, v, lo, hi);
+        if (interior) fold<Acc, OPC, V, false>(acc, v, m);
+        else fold<Acc, OPC, V, true>(acc, v, m);
     }
 }
 
 // Long runs (nslot >= T): a task is at most two contiguous segments (the end of
 // run j0 and the start of run j0+1).
-template <typename T, class Acc, int OPC, int V>
+template <class Acc, int OPC, int V>
 __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
                                             Acc& acc, int lane, int w) {
     int64_t t = t0 + w;
     if (t >= t1) return;
-    const int T_ = d.T, h0 = d.h0;
+    const int T_ = d.T;
     const int64_t nslot = d.nslot, G = d.G;
-    const int tail = (int)(d.h0 + d.L - (int64_t)V * (nslot - 1));
+    uint32_t fm, lm;
+    slot_masks<V>(d, fm, lm);
+    const uint32_t full = (1u << V) - 1u;
     int64_t j0 = (t * T_) / nslot;
     int64_t rem = t * T_ - j0 * nslot;
     const int64_t step = (int64_t)kWarps * T_;
@@ -315,9 +336,9 @@ __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, c
         const int n = left < T_ ? (int)left : T_;
         const int64_t in_run = nslot - rem;
         const int c1 = in_run < n ? (int)in_run : n;
-        stream_segment<T, Acc, OPC, V>(cube + run_addr(d, j0) + rem * V, c1, rem == 0, rem + c1 == nslot, h0, tail,
-                                       acc, lane);
-        if (c1 < n) stream_segment<T, Acc, OPC, V>(cube + run_addr(d, j0 + 1), n - c1, true, false, h0, tail, acc, lane);
+        stream_segment<Acc, OPC, V>(cube + run_addr(d, j0) + rem * V, c1, rem == 0 ? fm : full,
+                                    rem + c1 == nslot ? lm : full, acc, lane);
+        if (c1 < n) stream_segment<Acc, OPC, V>(cube + run_addr(d, j0 + 1), n - c1, fm, full, acc, lane);
         rem += step;
         if (rem >= nslot) {
             const int64_t dj = nslot < (1ll << 20) ? (int64_t)fdiv((uint32_t)rem, d.fnslot) : 1;
@@ -331,8 +352,8 @@ template <typename T, class Acc, int OPC, int V>
 __device__ __forceinline__ void stream_tasks(const T* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
                                              Acc& acc, int lane, int w) {
     const uint32_t* c = reinterpret_cast<const uint32_t*>(cube);
-    if (d.nslot < d.T) stream_short<T, Acc, OPC, V>(c, d, t0, t1, acc, lane, w);
-    else stream_long<T, Acc, OPC, V>(c, d, t0, t1, acc, lane, w);
+    if (d.nslot < d.T) stream_short<Acc, OPC, V>(c, d, t0, t1, acc, lane, w);
+    else stream_long<Acc, OPC, V>(c, d, t0, t1, acc, lane, w);
 }
 
 // ------------------------------------------------------------------ plan
@@ -385,7 +406,11 @@ __device__ void build_desc(const Geo& g, const olap_range* r, int32_t op, QDesc&
     d.base_al = base - d.h0;
     d.nslot = (d.h0 + d.L + d.V - 1) / d.V;
     d.G = R * d.nslot;
-    d.T = d.nslot < 9 ? (int32_t)(32 * d.nslot) : kTaskSlots;
+    // task: 32 whole runs when runs are tiny; else <= 30 runs' worth of slots (so a task
+    // spans <= 31 runs, one per lane), at most kTaskSlots; long runs: kTaskSlots
+    if (d.nslot < 9) d.T = (int32_t)(32 * d.nslot);
+    else if (d.nslot < kTaskSlots) d.T = (int32_t)(((30 * d.nslot) & ~31ll) < kTaskSlots ? ((30 * d.nslot) & ~31ll) : kTaskSlots);
+    else d.T = kTaskSlots;
     d.tasks = (d.G + d.T - 1) / d.T;
     d.fnslot = dev_fastdiv(d.nslot < (1ll << 31) ? (uint32_t)d.nslot : 1u);
     d.opc = (op == OLAP_MIN) ? OPC_MIN : (op == OLAP_MAX) ? OPC_MAX : OPC_SUM;
