@@ -23,6 +23,8 @@ __all__ = ["Cube", "Dict", "OlapError", "translate", "shard_local_rows", "combin
            "RESULT_EMPTY", "RESULT_INVALID", "EXPORTS"]
 
 LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libolap_b200.so")
+if os.environ.get("OLAP_LIB"):          # development only: A/B a differently-tuned build of the same sources
+    LIB_PATH = os.path.abspath(os.environ["OLAP_LIB"])
 
 INT32, FLOAT32 = 1, 2
 SUM, COUNT, MIN, MAX, AVG = 0, 1, 2, 3, 4

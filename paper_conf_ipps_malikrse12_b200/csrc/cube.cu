@@ -26,9 +26,12 @@ constexpr int kMaxRunDims = 7;
 constexpr int kWarps = 8;                   // warps per reduce block
 constexpr int kThreads = kWarps * 32;
 constexpr int kTaskSlots = 2048;            // max slots per warp task (32 KiB of 16-B slots)
-constexpr int kUnroll = 4;                  // independent loads in flight per lane
+#ifndef OLAP_UNROLL
+#define OLAP_UNROLL 4
+#endif
+constexpr int kUnroll = OLAP_UNROLL;        // independent loads in flight per lane
 #ifndef OLAP_MIN_BLOCKS
-#define OLAP_MIN_BLOCKS 3
+#define OLAP_MIN_BLOCKS 4
 #endif
 constexpr int kMinBlocks = OLAP_MIN_BLOCKS;  // resident reduce blocks per SM the register budget targets
 constexpr int64_t kItemCells = 262144;      // minimum item: 1 MiB of 4-byte cells
