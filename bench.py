@@ -212,10 +212,16 @@ def main():
     import paper_conf_ipps_malikrse12_b200 as olap
     from paper_conf_ipps_malikrse12_b200.dist import exchange_partials
 
+    # one rank per GPU; OLAP_DIST_BACKEND=gloo lets ranks share a device to dry-run the N>1 path
+    backend = os.environ.get("OLAP_DIST_BACKEND", "nccl")
+    local = local % max(torch.cuda.device_count(), 1) if backend != "nccl" else local
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     ext, cfg = workload(args.workload, world)
     nq = cfg["nq"]
     dtype = cfg["dtype"]
