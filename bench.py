@@ -53,6 +53,17 @@ def measured_peaks():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+DESC = {
+    "C1": "4-D int32 32^4 (4 MiB, L2-resident: GB/s is L2, not HBM), 1,000 random boxes, uniform ops",
+    "C2a": "6-D float32 (16,16,16,16,16,256) 1 GiB; phi log-uniform [1e-4,1], l_d=max(1,round(n_d*phi^(1/6))); "
+           "ops SUM/MIN/MAX/AVG/COUNT 40/20/20/10/10",
+    "C2b": "6-D float32 (16,16,32,32,32,32) 1 GiB (128-B rows: short-run stress); phi log-uniform [1e-4,1]; same ops",
+    "C3": "3-D float32 (2048,2048,2048) 32 GiB; phi log-uniform [1e-5,1]; same ops",
+    "C5": "3-D float32 (1024,4096,8192) 128 GiB per GPU (1 TiB at 8 GPUs); small boxes 4 KiB..4 MiB log-uniform; "
+          "batches of 65,536",
+}
+
+
 def workload(name: str, world: int):
     cfg = synth.CONFIGS[name]
     ext = list(cfg["extents"])
@@ -121,7 +132,10 @@ def cpu_baseline(name, ext_global, cfg, seed, target_s=12.0, max_queries=None):
     sample (the first n queries of the first batch, stopping after ~target_s)."""
     import oracle
     ext = cfg["extents"]  # a one-GPU cube; the oracle evaluates the global cube semantics on it
-    cells = _host_cells(tuple(ext), np.dtype(cfg["dtype"]).str, cfg["seed"])
+    ncells = int(np.prod(ext))
+    dt = np.dtype(cfg["dtype"])
+    # materialise the cube on the host when it is small; else the oracle recomputes cells procedurally
+    cells = _host_cells(tuple(ext), dt.str, cfg["seed"]) if ncells * 4 <= (2 << 30) else None
     b, o = synth.config_queries(name, nq=cfg["nq"], seed=seed, extents=ext)
     threads = oracle.max_threads()
     done, cells_read, t_used = 0, 0, 0.0
@@ -131,7 +145,10 @@ def cpu_baseline(name, ext_global, cfg, seed, target_s=12.0, max_queries=None):
         if max_queries is not None and done >= max_queries:
             break
         bb, oo = b[done:done + chunk], o[done:done + chunk]
-        oracle.query(ext, bb, oo, cells, nthreads=threads)
+        if cells is not None:
+            oracle.query(ext, bb, oo, cells, nthreads=threads)
+        else:
+            oracle.query(ext, bb, oo, dtype=dt, gen=oracle.GEN_UNIFORM, seed=cfg["seed"], nthreads=threads)
         vol = np.prod(bb[:, :, 1] - bb[:, :, 0] + 1, axis=1)
         cells_read += int(vol[oo != synth.COUNT].sum())
         done += len(bb)
@@ -140,7 +157,8 @@ def cpu_baseline(name, ext_global, cfg, seed, target_s=12.0, max_queries=None):
         "value": done / t_used, "unit": "queries/s", "cores": threads, "kind": "oracle",
         "gbs": cells_read * 4 / t_used / 1e9,
         "sample": f"first {done} queries of a {name} batch on the 1-GPU cube {tuple(ext)}, "
-                  f"{cells_read * 4 / 2**30:.1f} GiB read, {t_used:.1f} s, OpenMP over queries",
+                  f"{cells_read * 4 / 2**30:.1f} GiB read, {t_used:.1f} s, OpenMP over queries"
+                  + ("" if cells is not None else ", cells recomputed by the oracle's generator"),
         "host": host_info(),
     }
 
@@ -179,7 +197,8 @@ def run_reference(args, rank, world):
     line = {
         "impl": "reference", "metric": METRIC, "value": q, "unit": "queries/s", "n_gpus": world,
         "steps": steps, "warmup": warm, "ms_per_step": 1000.0 / q * cfg["nq"], "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "scaling": "weak", "vs_baseline": None, "dtype": "i32" if cfg["dtype"] == np.int32 else "f32",
+        "data": "synthetic",
         "config": {"workload": args.workload, "extents": list(ext), "batch": cfg["nq"],
                    "note": "oracle on a bounded sample per step; ms_per_step extrapolated to a full batch"},
         "gbs": gbs,
@@ -197,7 +216,7 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="C2a", choices=["C2a", "C2b", "C3", "C1"])
+    ap.add_argument("--workload", default="C2a", choices=["C2a", "C2b", "C3", "C1", "C5"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
     args = ap.parse_args()
@@ -312,12 +331,15 @@ def main():
         line = {
             "metric": METRIC, "value": qps, "unit": "queries/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "scaling": "weak", "vs_baseline": None, "dtype": "i32" if dtype == np.int32 else "f32",
+            "data": "synthetic",
             "config": {"workload": args.workload, "extents": list(ext), "cube_gib_per_gpu":
                        cube.info()[1] * 4 / 2**30, "batch": nq,
-                       "queries": "phi log-uniform [1e-4,1], l_d=max(1,round(n_d*phi^(1/6))); ops 40/20/20/10/10",
-                       "l2": "no flush: inputs > L2 (1 GiB cube/GPU, ~0.4 TiB read per step)",
-                       "accumulation": "f32 cells, f64 SUM", "parallelism": f"shard{world}" if world > 1 else "1gpu"},
+                       "queries": DESC[args.workload],
+                       "l2": ("no flush: C1's 4 MiB cube is L2-resident by design (flagged)" if args.workload == "C1"
+                              else "no flush: cube > L2 (126 MB) and every step reads >> L2"),
+                       "accumulation": "int32 cells, int64 SUM" if dtype == np.int32 else "f32 cells, f64 SUM",
+                       "parallelism": f"shard{world}" if world > 1 else "1gpu"},
             "gbs": gbs_total, "frac_of_nominal_8tbs": gbs_total / world / NOMINAL_HBM_GBS,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "kernel": "reduce_kernel",

@@ -333,3 +333,39 @@ def test_c4_tpcds_pipeline():
     ref_s, ref_c = oracle.factscan(ids, qty, boxes)
     assert np.array_equal(sums["i"], ref_s)
     assert np.array_equal(cnts["i"], ref_c)
+
+
+def _sampled_full_size(name, n_small, n_random, max_cells, affine_params):
+    cfg = synth.CONFIGS[name]
+    ext = cfg["extents"]
+    c = olap.Cube(ext, cfg["dtype"])
+    try:
+        c.fill(olap.GEN_UNIFORM, cfg["seed"])
+        boxes, ops = synth.config_queries(name)
+        gpu = c.query(boxes, ops)
+        vol = np.prod(boxes[:, :, 1] - boxes[:, :, 0] + 1, axis=1)
+        rng = np.random.default_rng(1)
+        cand = np.nonzero(vol <= max_cells)[0]
+        idx = np.unique(np.concatenate([np.argsort(vol)[:n_small], rng.choice(cand, min(n_random, len(cand)),
+                                                                                replace=False)]))
+        ref = oracle.query(ext, boxes[idx], ops[idx], dtype=cfg["dtype"], gen=oracle.GEN_UNIFORM, seed=cfg["seed"],
+                           nthreads=oracle.max_threads())
+        compare(gpu[idx], ref, ops[idx], cfg["dtype"])
+        # integer-valued affine fill: float results bit-exact on a sample incl. large boxes
+        c.fill(olap.GEN_AFFINE, 0, affine_params)
+        gpu = c.query(boxes, ops)
+        ref = oracle.query(ext, boxes[idx], ops[idx], dtype=cfg["dtype"], gen=oracle.GEN_AFFINE,
+                           params=affine_params, nthreads=oracle.max_threads())
+        compare(gpu[idx], ref, ops[idx], cfg["dtype"], exact_float=True)
+    finally:
+        c.close()
+
+
+def test_c3_full_size_sampled():
+    """C3: 32 GiB float32 cube (2048^3), 4,096-query batch; sampled oracle parity."""
+    _sampled_full_size("C3", 12, 12, 150_000_000, np.array([1, 1, 2, 3], float))
+
+
+def test_c5_slice_full_size_sampled():
+    """C5 per-GPU slice: 128 GiB float32 cube (1024,4096,8192), 65,536 small boxes; sampled parity."""
+    _sampled_full_size("C5", 50, 400, 2_000_000, np.array([2, 1, 1, 1], float))
