@@ -114,6 +114,17 @@ int olap_cube_fill(olap_cube* c, int generator, uint64_t seed, const double* par
 
 int olap_cube_destroy(olap_cube* c);
 
+/* Build step ("the GPU performs ... building the cube from relational
+ * tables stored in GPU memory"): add nrows fact rows into the cells they
+ * map to.  d_ids[d*nrows + r] is row r's member id in dimension d (DEVICE, int32, inside
+ * [0, n_d)); d_values (DEVICE, nrows cells of the cube's dtype) or NULL to add 1 per
+ * row (a fact-count cube).  Rows whose dim-0 id is not owned by this shard are skipped.
+ * Cells are NOT cleared first (olap_cube_fill with params {0,...} or load zeros).
+ * int32 adds are exact (atomic, order-free); float32 adds are atomic in arrival order.
+ * Asynchronous on `stream`. */
+int olap_cube_add_facts_device(olap_cube* c, int64_t nrows, const int32_t* d_ids, const void* d_values,
+                               void* stream);
+
 /* ---------------------------------------------------------------- queries */
 
 /* Whole path on HOST buffers: validate, copy ranges (nq*ndims, query-major) and
@@ -191,6 +202,33 @@ int olap_dict_translate_device(const olap_dict* const* dicts, int ndicts,
  * GPU; HOST buffers.  A range [s1, s2] maps to ids [lower(s1), upper(s2) - 1]. */
 int olap_dict_bound(const olap_dict* d, const char* bytes, const int64_t* offsets, int64_t n,
                     int upper, int32_t* out);
+
+/* Text conditions -> Eq. 1 ranges (PAPER.md:252-256 with readings R11/R13).  One
+ * condition per (query, dimension), kinds[q*ndims + d]:
+ *   OLAP_COND_ALL    whole dimension [0, n_d - 1]; consumes no key
+ *   OLAP_COND_EQ     one key s: [id, id] with id = dicts[d][s]; a missing key gives an
+ *                    empty box [1, 0] and is counted in *n_missing
+ *   OLAP_COND_RANGE  two keys s1, s2: [lower_bound(s1), upper_bound(s2) - 1] (ids are
+ *                    sorted ranks, so this is every member with s1 <= member <= s2;
+ *                    empty when no member lies in between)
+ *   OLAP_COND_IDS    numeric condition: ranges_in[q*ndims + d] copied as given
+ * Keys are consumed in (q, d) order from bytes/offsets (nkeys keys).  dicts[d] may
+ * be NULL for a dimension that only uses ALL/IDS; a text dimension's extent must be
+ * its dictionary's size.  HOST buffers; translation runs on the dictionaries' GPU. */
+typedef enum { OLAP_COND_ALL = 0, OLAP_COND_EQ = 1, OLAP_COND_RANGE = 2, OLAP_COND_IDS = 3 } olap_cond_kind;
+
+int olap_text_ranges(const olap_dict* const* dicts, int ndims, const int64_t* extents, int64_t nq,
+                     const int32_t* kinds, const olap_range* ranges_in, const char* bytes,
+                     const int64_t* offsets, int64_t nkeys, olap_range* ranges_out, int64_t* n_missing);
+
+/* Same on DEVICE buffers, asynchronous on `stream`: d_first_key[q*ndims + d] is the
+ * index of the condition's first key (any value for ALL/IDS); d_ranges_in may be NULL
+ * when no IDS condition is present; d_n_missing (device int64, optional) is incremented.
+ * `extents` is a HOST array. */
+int olap_text_ranges_device(const olap_dict* const* dicts, int ndims, const int64_t* extents, int64_t nq,
+                            const int32_t* d_kinds, const int64_t* d_first_key,
+                            const olap_range* d_ranges_in, const char* d_bytes, const int64_t* d_offsets,
+                            int64_t nkeys, olap_range* d_ranges_out, int64_t* d_n_missing, void* stream);
 
 /* Inverse: bytes of member `id` (pointer valid until the dict is destroyed). */
 int olap_dict_lookup(const olap_dict* d, int32_t id, const char** bytes, int64_t* len);

@@ -20,7 +20,8 @@ import numpy as np
 __all__ = ["Cube", "Dict", "OlapError", "translate", "shard_local_rows", "combine_partials_device",
            "finalize_device", "translate_device", "RESULT_DTYPE", "lib", "LIB_PATH",
            "INT32", "FLOAT32", "SUM", "COUNT", "MIN", "MAX", "AVG", "GEN_UNIFORM", "GEN_AFFINE",
-           "RESULT_EMPTY", "RESULT_INVALID", "EXPORTS"]
+           "RESULT_EMPTY", "RESULT_INVALID", "EXPORTS", "text_ranges", "text_ranges_device",
+           "COND_ALL", "COND_EQ", "COND_RANGE", "COND_IDS"]
 
 LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libolap_b200.so")
 if os.environ.get("OLAP_LIB"):          # development only: A/B a differently-tuned build of the same sources
@@ -30,6 +31,7 @@ INT32, FLOAT32 = 1, 2
 SUM, COUNT, MIN, MAX, AVG = 0, 1, 2, 3, 4
 GEN_UNIFORM, GEN_AFFINE = 1, 2
 RESULT_EMPTY, RESULT_INVALID = 1, 2
+COND_ALL, COND_EQ, COND_RANGE, COND_IDS = 0, 1, 2, 3
 
 OK, E_INVALID, E_RANGE, E_NOMEM, E_CUDA, E_STATE, E_UNSUPPORTED = 0, -1, -2, -3, -4, -6, -7
 
@@ -63,6 +65,9 @@ EXPORTS = {
     "olap_dict_translate_device": (_int, [_p, _int, _p, _p, _p, _i64, _p, _p, _p]),
     "olap_dict_bound": (_int, [_p, _p, _i64p, _i64, _int, _p]),
     "olap_dict_lookup": (_int, [_p, ctypes.c_int32, ctypes.POINTER(ctypes.c_char_p), _i64p]),
+    "olap_text_ranges": (_int, [_p, _int, _i64p, _i64, _p, _p, _p, _i64p, _i64, _p, _i64p]),
+    "olap_text_ranges_device": (_int, [_p, _int, _i64p, _i64, _p, _p, _p, _p, _p, _i64, _p, _p, _p]),
+    "olap_cube_add_facts_device": (_int, [_p, _i64, _p, _p, _p]),
     "olap_dict_destroy": (_int, [_p]),
     "olap_last_error": (ctypes.c_char_p, []),
     "olap_version": (ctypes.c_char_p, []),
@@ -212,6 +217,12 @@ class Cube:
         _check(lib.olap_query_partials_device(self._h, nq, _ptr(d_ranges), _ptr(d_ops), _ptr(d_sum), _ptr(d_ext),
                                               _stream(stream)), "olap_query_partials_device")
 
+    def add_facts_device(self, d_ids, d_values=None, nrows: int | None = None, stream=None):
+        """Scatter-add fact rows into their cells (d_ids: (ndims, nrows) int32 device tensor)."""
+        nrows = d_ids.shape[-1] if nrows is None else nrows
+        _check(lib.olap_cube_add_facts_device(self._h, nrows, _ptr(d_ids), _ptr(d_values), _stream(stream)),
+               "olap_cube_add_facts_device")
+
     def profile(self, enable: bool = True):
         _check(lib.olap_cube_profile(self._h, 1 if enable else 0), "olap_cube_profile")
 
@@ -334,3 +345,50 @@ def translate_device(dicts, d_dict_of_key, d_bytes, d_offsets, n: int, d_ids, d_
     _check(lib.olap_dict_translate_device(_dict_array(dicts), len(dicts), _ptr(d_dict_of_key), _ptr(d_bytes),
                                           _ptr(d_offsets), n, _ptr(d_ids), _ptr(d_n_missing), _stream(stream)),
            "olap_dict_translate_device")
+
+
+def _dict_or_null_array(dicts):
+    return (ctypes.c_void_p * len(dicts))(*[(d.handle.value if d is not None else None) for d in dicts])
+
+
+def text_ranges(dicts, extents, conditions, ranges_in=None):
+    """Text conditions -> ranges (olap_text_ranges).
+
+    dicts: one Dict (or None) per dimension; conditions: nq lists of ndims entries, each
+    None (whole dimension), a str/bytes key (equality), a (s1, s2) tuple (string range),
+    or an int pair [lo, hi] given as ('ids', lo, hi).  Returns (ranges (nq, ndims, 2), n_missing)."""
+    nd = len(dicts)
+    kinds, keys = [], []
+    rin = np.zeros((len(conditions), nd, 2), dtype=np.int64)
+    for qi, cond in enumerate(conditions):
+        for d in range(nd):
+            c = cond[d]
+            if c is None:
+                kinds.append(COND_ALL)
+            elif isinstance(c, tuple) and len(c) == 3 and c[0] == "ids":
+                kinds.append(COND_IDS)
+                rin[qi, d] = (c[1], c[2])
+            elif isinstance(c, tuple):
+                kinds.append(COND_RANGE)
+                keys += [c[0], c[1]]
+            else:
+                kinds.append(COND_EQ)
+                keys.append(c)
+    k = np.ascontiguousarray(kinds, dtype=np.int32)
+    buf, offs = _pack(keys)
+    ext, extp = _i64arr(extents)
+    out = np.zeros((len(conditions), nd, 2), dtype=np.int64)
+    miss = ctypes.c_int64()
+    _check(lib.olap_text_ranges(_dict_or_null_array(dicts), nd, extp, len(conditions), k.ctypes.data, rin.ctypes.data,
+                                buf.ctypes.data, offs.ctypes.data_as(_i64p), len(offs) - 1, out.ctypes.data,
+                                ctypes.byref(miss)), "olap_text_ranges")
+    return out, miss.value
+
+
+def text_ranges_device(dicts, extents, nq: int, d_kinds, d_first_key, d_ranges_in, d_bytes, d_offsets, nkeys: int,
+                       d_ranges_out, d_n_missing=None, stream=None):
+    ext, extp = _i64arr(extents)
+    _check(lib.olap_text_ranges_device(_dict_or_null_array(dicts), len(ext), extp, nq, _ptr(d_kinds),
+                                       _ptr(d_first_key), _ptr(d_ranges_in), _ptr(d_bytes), _ptr(d_offsets), nkeys,
+                                       _ptr(d_ranges_out), _ptr(d_n_missing), _stream(stream)),
+           "olap_text_ranges_device")

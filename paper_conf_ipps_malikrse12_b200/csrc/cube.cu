@@ -732,6 +732,27 @@ __global__ void fill_kernel(T* cells, Geo geo, int64_t row_cells, int gen, uint6
     }
 }
 
+// ------------------------------------------------------------------ build from facts (NEXT #2)
+
+template <typename T>
+__global__ void add_facts_kernel(T* cells, Geo geo, int64_t nrows, const int32_t* __restrict__ ids,
+                                 const T* __restrict__ vals) {
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < nrows; r += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t x0 = ids[r];
+        if (x0 < 0 || x0 >= geo.n[0]) continue;
+        if (geo.G > 1 && (x0 / geo.b) % geo.G != geo.g) continue;  // row owned by another shard
+        int64_t idx = shard_local_of(x0, geo.G, geo.b) * geo.stride[0];
+        bool ok = true;
+        for (int d = 1; d < geo.nd; ++d) {
+            const int64_t x = ids[(int64_t)d * nrows + r];
+            ok = ok && x >= 0 && x < geo.n[d];
+            idx += x * geo.stride[d];
+        }
+        if (!ok) continue;
+        atomicAdd(cells + idx, vals ? vals[r] : (T)1);
+    }
+}
+
 }  // namespace olap
 
 // ====================================================================== host runtime
@@ -1068,6 +1089,29 @@ int olap_cube_fill(olap_cube* c, int generator, uint64_t seed, const double* par
                                                         generator, seed, fp);
     OLAP_CUDA_TRY(cudaGetLastError());
     OLAP_CUDA_TRY(cudaStreamSynchronize(c->stream));
+    return OLAP_OK;
+}
+
+int olap_cube_add_facts_device(olap_cube* c, int64_t nrows, const int32_t* d_ids, const void* d_values, void* stream) {
+    clear_error();
+    int rc = check_cube(c);
+    if (rc) return rc;
+    if (nrows < 0) return set_error(OLAP_E_INVALID, "nrows < 0");
+    if (nrows == 0) return OLAP_OK;
+    if (!d_ids) return set_error(OLAP_E_INVALID, "d_ids is NULL");
+    std::lock_guard<std::mutex> lk(c->mu);
+    DeviceGuard dg(c->device);
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    OLAP_CUDA_TRY(cudaStreamWaitEvent(st, c->ws_done, 0));
+    const int grid = (int)std::min<int64_t>((nrows + 255) / 256, (int64_t)c->num_sms * 16);
+    if (c->dtype == OLAP_INT32)
+        add_facts_kernel<int32_t><<<grid, 256, 0, st>>>(static_cast<int32_t*>(c->d_cells), make_geo(c), nrows, d_ids,
+                                                        static_cast<const int32_t*>(d_values));
+    else
+        add_facts_kernel<float><<<grid, 256, 0, st>>>(static_cast<float*>(c->d_cells), make_geo(c), nrows, d_ids,
+                                                      static_cast<const float*>(d_values));
+    OLAP_CUDA_TRY(cudaGetLastError());
+    OLAP_CUDA_TRY(cudaEventRecord(c->ws_done, st));
     return OLAP_OK;
 }
 

@@ -279,58 +279,136 @@ def test_dict_stress_1e6():
     assert np.array_equal(ids, od.translate(probes))
 
 
+def _expected_range(od, cond, n):
+    """Reading R11/R13 applied to the oracle dictionary's answers."""
+    if cond is None:
+        return (0, n - 1), 0
+    if isinstance(cond, tuple):
+        return (od.bound(cond[0]), od.bound(cond[1], upper=True) - 1), 0
+    i = int(od.translate([cond])[0])
+    return ((i, i), 0) if i >= 0 else ((1, 0), 1)
+
+
+def test_text_ranges_parity():
+    members = synth.tpcds_members()
+    cols = ["ca_state", "i_class", "s_store_id", "d_date"]
+    dg = [olap.Dict(members[c]) for c in cols]
+    do = [oracle.Dict(members[c]) for c in cols]
+    ext = [len(members[c]) for c in cols]
+    rng = np.random.default_rng(9)
+    conds = []
+    for _ in range(3000):
+        q = []
+        for di, c in enumerate(cols):
+            m = members[c]
+            r = rng.random()
+            if r < 0.3:
+                q.append(None)
+            elif r < 0.65:
+                k = m[rng.integers(0, len(m))]
+                q.append(k if rng.random() < 0.9 else k + "~")
+            else:
+                a, b = sorted(rng.integers(0, len(m), size=2))
+                s1, s2 = m[a], m[b]
+                if rng.random() < 0.3:
+                    s1 = s1[:-1]          # endpoint not a member
+                if rng.random() < 0.3:
+                    s2 = s2 + "zz"
+                if rng.random() < 0.05:
+                    s1, s2 = s2, s1       # reversed -> empty
+                q.append((s1, s2))
+        conds.append(q)
+    got, miss = olap.text_ranges(dg, ext, conds)
+    want = np.zeros_like(got)
+    wmiss = 0
+    for qi, q in enumerate(conds):
+        for di in range(4):
+            (lo, hi), m = _expected_range(do[di], q[di], ext[di])
+            want[qi, di] = (lo, hi)
+            wmiss += m
+    assert np.array_equal(got, want)
+    assert miss == wmiss
+    # mixed numeric (IDS) dimension and a dimension without a dictionary
+    got2, _ = olap.text_ranges([dg[0], None], [ext[0], 10], [["CA", ("ids", 2, 5)], [None, None]])
+    assert got2.tolist() == [[[int(do[0].translate(["CA"])[0])] * 2, [2, 5]], [[0, ext[0] - 1], [0, 9]]]
+    with pytest.raises(olap.OlapError):
+        olap.text_ranges([dg[0], None], [ext[0], 10], [["CA", "x"]])   # text on a dim without dictionary
+
+
+@pytest.mark.parametrize("dtype", [np.int32, np.float32])
+@pytest.mark.parametrize("shard", [None, (3, 1, 2)])
+def test_add_facts_builds_cube(dtype, shard):
+    ext = (13, 7, 11)
+    rng = np.random.default_rng(2)
+    nrows = 50_000
+    ids = np.stack([rng.integers(0, n, size=nrows) for n in ext]).astype(np.int32)
+    vals = rng.integers(-1000, 1000, size=nrows).astype(dtype)
+    ref = np.zeros(ext, np.int64)
+    np.add.at(ref, tuple(ids), vals.astype(np.int64))
+    refn = np.zeros(ext, np.int64)
+    np.add.at(refn, tuple(ids), 1)
+    G = 1 if shard is None else shard[0]
+    for cube_ref, v in ((ref, vals), (refn, None)):
+        c = olap.Cube(ext, dtype, shard=shard)
+        c.fill(olap.GEN_AFFINE, 0, np.zeros(4))
+        c.add_facts_device(torch.from_numpy(ids).cuda(), None if v is None else torch.from_numpy(v).cuda())
+        torch.cuda.synchronize()
+        # every cell through 1-cell SUM queries (partials of this shard; non-owned rows are identity)
+        boxes = np.array([[[x, x], [y, y], [z, z]] for x in range(ext[0]) for y in range(ext[1])
+                          for z in range(ext[2])])
+        nq = len(boxes)
+        s = torch.empty(nq, dtype=torch.int64, device="cuda")
+        e = torch.empty(2 * nq, dtype=torch.int32, device="cuda")
+        c.partials_device(torch.from_numpy(boxes).cuda(), torch.full((nq,), olap.SUM, dtype=torch.int32,
+                                                                   device="cuda"), s, e)
+        got = s.cpu().numpy()
+        if dtype == np.float32:
+            got = got.view(np.float64)
+        owned = np.array([((x // shard[2]) % G == shard[1]) if shard else True for x, _, _ in
+                          (b[:, 0] for b in boxes)])
+        want = cube_ref.reshape(-1).astype(np.float64 if dtype == np.float32 else np.int64)
+        assert np.array_equal(got[owned], want[owned])
+        assert not got[~owned].any()
+
+
 def test_c4_tpcds_pipeline():
-    """C4 end to end: string predicates -> GPU translation (4 dictionaries) -> cube queries
-    on cubes built from the fact rows == the oracle's fact scan over the raw rows."""
+    """C4 end to end: fact rows -> GPU cube build (quantity, count) -> string predicates ->
+    GPU translation into ranges (4 dictionaries) -> cube queries, equal to the oracle's fact
+    scan over the raw rows (SUM of quantity, fact COUNT)."""
     members = synth.tpcds_members()
     cols = ["ca_state", "i_class", "s_store_id", "d_date"]   # layout: date innermost (DESIGN.md)
     nrows = 400_000
     facts, qty, cents = synth.tpcds_facts(nrows, members)
-    dg = {c: olap.Dict(members[c]) for c in cols}
+    dg = [olap.Dict(members[c]) for c in cols]
     do = {c: oracle.Dict(members[c]) for c in cols}
-    # fact rows -> ids (GPU translation of the raw strings, checked against the oracle)
+    # fact rows -> ids (GPU translation of the raw strings, checked against the oracle on a sample)
     ids = []
-    for c in cols:
+    for di, c in enumerate(cols):
         strs = [members[c][i] for i in facts[c][:20000]]
-        g, _ = dg[c].translate(strs)
+        g, _ = dg[di].translate(strs)
         assert np.array_equal(g, do[c].translate(strs))
         ids.append(do[c].translate([members[c][i] for i in range(len(members[c]))])[facts[c]])
     ids = np.stack(ids).astype(np.int32)
     ext = tuple(len(members[c]) for c in cols)
-    cube_q = np.zeros(ext, np.int64)
-    np.add.at(cube_q, tuple(ids), qty)
-    cube_n = np.zeros(ext, np.int64)
-    np.add.at(cube_n, tuple(ids), 1)
+    d_ids = torch.from_numpy(ids).cuda()
     cq = olap.Cube(ext, np.int32)
-    cq.load(cube_q.astype(np.int32))
+    cq.fill(olap.GEN_AFFINE, 0, np.zeros(5))
+    cq.add_facts_device(d_ids, torch.from_numpy(qty).cuda())
     cn = olap.Cube(ext, np.int32)
-    cn.load(cube_n.astype(np.int32))
+    cn.fill(olap.GEN_AFFINE, 0, np.zeros(5))
+    cn.add_facts_device(d_ids)
+    torch.cuda.synchronize()
     queries = synth.tpcds_queries(300, members)
-    keys, which = [], []
-    for q in queries:
-        for c in cols:
-            if c == "d_date":
-                keys += [q[c][0], q[c][1]]
-                which += [cols.index(c)] * 2
-            elif c in q:
-                keys.append(q[c])
-                which.append(cols.index(c))
-    tid, _ = olap.translate([dg[c] for c in cols], np.array(which, np.int32), keys)
-    boxes = np.zeros((len(queries), 4, 2), np.int64)
-    k = 0
-    for qi, q in enumerate(queries):
-        for di, c in enumerate(cols):
-            if c == "d_date":
-                boxes[qi, di] = (tid[k], tid[k + 1])
-                k += 2
-            elif c in q:
-                boxes[qi, di] = (tid[k], tid[k]) if tid[k] >= 0 else (1, 0)   # miss -> empty box
-                k += 1
-            else:
-                boxes[qi, di] = (0, ext[di] - 1)
+    conds = [[q.get(c) if c != "d_date" else q[c] for c in cols] for q in queries]
+    boxes, _ = olap.text_ranges(dg, ext, conds)
     sums = cq.query(boxes, np.full(len(boxes), olap.SUM, np.int32))
     cnts = cn.query(boxes, np.full(len(boxes), olap.SUM, np.int32))
-    ref_s, ref_c = oracle.factscan(ids, qty, boxes)
+    # the oracle path: its own dictionaries on the raw strings, then a scan over the fact rows
+    ob = np.zeros_like(boxes)
+    for qi, cond in enumerate(conds):
+        for di, c in enumerate(cols):
+            ob[qi, di] = _expected_range(do[c], cond[di], ext[di])[0]
+    ref_s, ref_c = oracle.factscan(ids, qty, ob)
     assert np.array_equal(sums["i"], ref_s)
     assert np.array_equal(cnts["i"], ref_c)
 
