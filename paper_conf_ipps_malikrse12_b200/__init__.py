@@ -20,7 +20,7 @@ import numpy as np
 __all__ = ["Cube", "Dict", "OlapError", "translate", "shard_local_rows", "combine_partials_device",
            "finalize_device", "translate_device", "RESULT_DTYPE", "lib", "LIB_PATH",
            "INT32", "FLOAT32", "SUM", "COUNT", "MIN", "MAX", "AVG", "GEN_UNIFORM", "GEN_AFFINE",
-           "RESULT_EMPTY", "RESULT_INVALID", "EXPORTS", "text_ranges", "text_ranges_device",
+           "RESULT_EMPTY", "RESULT_INVALID", "EXPORTS", "text_ranges", "text_ranges_device", "pack_text_conditions",
            "COND_ALL", "COND_EQ", "COND_RANGE", "COND_IDS"]
 
 LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libolap_b200.so")
@@ -351,6 +351,33 @@ def _dict_or_null_array(dicts):
     return (ctypes.c_void_p * len(dicts))(*[(d.handle.value if d is not None else None) for d in dicts])
 
 
+def pack_text_conditions(conditions, nd: int):
+    """Marshal per-(query, dimension) text conditions into the C-ABI arrays:
+    kinds (nq*nd int32), first_key (nq*nd int64), ranges_in (nq, nd, 2), key blob, key offsets."""
+    kinds = np.zeros(len(conditions) * nd, dtype=np.int32)
+    first = np.zeros(len(conditions) * nd, dtype=np.int64)
+    rin = np.zeros((len(conditions), nd, 2), dtype=np.int64)
+    keys = []
+    for qi, cond in enumerate(conditions):
+        for d in range(nd):
+            c = cond[d]
+            i = qi * nd + d
+            first[i] = len(keys)
+            if c is None:
+                kinds[i] = COND_ALL
+            elif isinstance(c, tuple) and len(c) == 3 and c[0] == "ids":
+                kinds[i] = COND_IDS
+                rin[qi, d] = (c[1], c[2])
+            elif isinstance(c, tuple):
+                kinds[i] = COND_RANGE
+                keys += [c[0], c[1]]
+            else:
+                kinds[i] = COND_EQ
+                keys.append(c)
+    buf, offs = _pack(keys)
+    return kinds, first, rin, buf, offs
+
+
 def text_ranges(dicts, extents, conditions, ranges_in=None):
     """Text conditions -> ranges (olap_text_ranges).
 
@@ -358,24 +385,7 @@ def text_ranges(dicts, extents, conditions, ranges_in=None):
     None (whole dimension), a str/bytes key (equality), a (s1, s2) tuple (string range),
     or an int pair [lo, hi] given as ('ids', lo, hi).  Returns (ranges (nq, ndims, 2), n_missing)."""
     nd = len(dicts)
-    kinds, keys = [], []
-    rin = np.zeros((len(conditions), nd, 2), dtype=np.int64)
-    for qi, cond in enumerate(conditions):
-        for d in range(nd):
-            c = cond[d]
-            if c is None:
-                kinds.append(COND_ALL)
-            elif isinstance(c, tuple) and len(c) == 3 and c[0] == "ids":
-                kinds.append(COND_IDS)
-                rin[qi, d] = (c[1], c[2])
-            elif isinstance(c, tuple):
-                kinds.append(COND_RANGE)
-                keys += [c[0], c[1]]
-            else:
-                kinds.append(COND_EQ)
-                keys.append(c)
-    k = np.ascontiguousarray(kinds, dtype=np.int32)
-    buf, offs = _pack(keys)
+    k, _first, rin, buf, offs = pack_text_conditions(conditions, nd)
     ext, extp = _i64arr(extents)
     out = np.zeros((len(conditions), nd, 2), dtype=np.int64)
     miss = ctypes.c_int64()

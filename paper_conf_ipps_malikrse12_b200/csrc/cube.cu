@@ -70,8 +70,11 @@ struct Geo {
     int nd, dtype;
     int64_t G, g, b;
     int64_t n[kMaxDims];       // global extents
-    int64_t stride[kMaxDims];  // local strides (cells)
+    int64_t stride[kMaxDims];  // local strides (cells; the innermost pitch may be padded)
     int64_t local_rows;
+    int64_t pitch;             // cells per innermost row in HBM (n[nd-1] rounded up to 4 when padded)
+    int64_t lrow;              // logical (unpadded) cells per dim-0 row
+    int padded;                // pitch != n[nd-1]: runs never merge across innermost rows
 };
 
 struct Extents {
@@ -386,7 +389,8 @@ __device__ void build_desc(const Geo& g, const olap_range* r, int32_t op, QDesc&
     int64_t ell[kMaxDims];
     for (int k = 0; k < g.nd; ++k) ell[k] = hi[k] - lo[k] + 1;
     int ks = g.nd - 1;  // split dim: innermost dim not fully covered (dims after it merge into runs)
-    while (ks > 0 && ell[ks] == g.n[ks]) --ks;
+    if (!g.padded)      // padding cells sit between innermost rows: such runs must not merge
+        while (ks > 0 && ell[ks] == g.n[ks]) --ks;
     d.L = ell[ks] * g.stride[ks];
     int64_t R = 1, base = 0;
     for (int k = 0; k < g.nd; ++k) base += lo[k] * g.stride[k];
@@ -708,10 +712,17 @@ struct FillParams {
 template <typename T>
 __global__ void fill_kernel(T* cells, Geo geo, int64_t row_cells, int gen, uint64_t seed, FillParams fp) {
     const int64_t n = geo.local_rows * row_cells;
+    const int64_t ninner = geo.n[geo.nd - 1];
     for (int64_t li = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; li < n; li += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t lr = li / row_cells, off = li - lr * row_cells;
+        const int64_t lr = li / row_cells, poff = li - lr * row_cells;
+        const int64_t rest = geo.nd > 1 ? poff / geo.pitch : 0, xin = poff - rest * geo.pitch;
+        if (xin >= ninner) {  // padding cell: never part of a box
+            cells[li] = (T)0;
+            continue;
+        }
+        const int64_t off = rest * ninner + xin;  // logical offset inside the dim-0 row
         const int64_t gr = shard_global_of(lr, geo.G, geo.g, geo.b);
-        const int64_t gi = gr * row_cells + off;
+        const int64_t gi = gr * geo.lrow + off;
         if (gen == OLAP_GEN_UNIFORM) {
             const uint64_t z = splitmix64_at(seed, (uint64_t)gi);
             if (sizeof(T) == 4 && geo.dtype == OLAP_INT32)
@@ -763,7 +774,8 @@ struct olap_cube {
     int nd = 0, dtype = 0, device = 0;
     int64_t n[kMaxDims] = {};
     olap_shard sh{1, 0, 1};
-    int64_t local_rows = 0, row_cells = 0, local_cells = 0;
+    int64_t local_rows = 0, row_cells = 0, local_cells = 0;  // row_cells / local_cells include padding
+    int64_t pitch = 0, lrow_cells = 0;                       // innermost pitch; logical cells per dim-0 row
     int64_t stride[kMaxDims] = {};
     void* d_cells = nullptr;
 
@@ -822,6 +834,9 @@ Geo make_geo(const olap_cube* c) {
         g.stride[k] = c->stride[k];
     }
     g.local_rows = c->local_rows;
+    g.pitch = c->pitch;
+    g.lrow = c->lrow_cells;
+    g.padded = c->pitch != c->n[c->nd - 1];
     return g;
 }
 
@@ -976,9 +991,14 @@ int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_sh
     c->device = device;
     c->sh = sh;
     for (int k = 0; k < ndims; ++k) c->n[k] = extents[k];
+    // innermost pitch padded to a multiple of 4 cells (16 B) when needed so that every
+    // innermost row starts 16-B aligned for the vector path
+    c->pitch = (ndims > 1 && (c->n[ndims - 1] & 3)) ? ((c->n[ndims - 1] + 3) & ~3ll) : c->n[ndims - 1];
     c->stride[ndims - 1] = 1;
-    for (int k = ndims - 2; k >= 0; --k) c->stride[k] = c->stride[k + 1] * c->n[k + 1];
-    c->row_cells = c->stride[0];
+    for (int k = ndims - 2; k >= 0; --k) c->stride[k] = c->stride[k + 1] * (k == ndims - 2 ? c->pitch : c->n[k + 1]);
+    c->row_cells = ndims > 1 ? c->stride[0] : 1;
+    c->lrow_cells = 1;
+    for (int k = 1; k < ndims; ++k) c->lrow_cells *= c->n[k];
     c->local_rows = shard_rows(c->n[0], sh.nshards, sh.shard, sh.block);
     c->local_cells = c->local_rows * c->row_cells;
     int rc = OLAP_OK;
@@ -991,6 +1011,7 @@ int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_sh
         delete c;
         return rc;
     }
+    if (c->pitch != c->n[ndims - 1]) cudaMemset(c->d_cells, 0, c->local_cells * 4);
     if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess ||
         cudaEventCreateWithFlags(&c->ws_done, cudaEventDisableTiming) != cudaSuccess ||
         cudaMalloc(&c->d_counter, 2 * sizeof(unsigned long long)) != cudaSuccess ||
@@ -1033,7 +1054,9 @@ int olap_cube_load_rows(olap_cube* c, int64_t row_lo, int64_t row_hi, const void
     std::lock_guard<std::mutex> lk(c->mu);
     DeviceGuard dg(c->device);
     OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
-    const int64_t rb = c->row_cells * 4;
+    const int64_t rb = c->row_cells * 4, lrb = c->lrow_cells * 4;  // device (padded) / host row bytes
+    const int64_t nin = c->n[c->nd - 1];
+    const bool padded = c->pitch != nin;
     const char* src = static_cast<const char*>(cells);
     char* dst = static_cast<char*>(c->d_cells);
     const int64_t G = c->sh.nshards, g = c->sh.shard, b = c->sh.block;
@@ -1042,17 +1065,17 @@ int olap_cube_load_rows(olap_cube* c, int64_t row_lo, int64_t row_hi, const void
         // run of consecutive owned rows starting at r (or skip the unowned ones)
         const int64_t blk_end = (r / b + 1) * b;
         const int64_t end = std::min(blk_end, row_hi);
-        if ((r / b) % G == g) {
+        const int64_t stop = G == 1 ? row_hi : end;  // unsharded: the whole remainder is owned and contiguous
+        if (G == 1 || (r / b) % G == g) {
             const int64_t lr = shard_local_of(r, G, b);
-            OLAP_CUDA_TRY(cudaMemcpy(dst + lr * rb, src + (r - row_lo) * rb, (end - r) * rb, cudaMemcpyHostToDevice));
-        }
-        r = end;
-        if (G == 1) {  // whole remainder is owned and contiguous
-            if (r < row_hi)
-                OLAP_CUDA_TRY(cudaMemcpy(dst + r * rb, src + (r - row_lo) * rb, (row_hi - r) * rb,
+            if (!padded)
+                OLAP_CUDA_TRY(cudaMemcpy(dst + lr * rb, src + (r - row_lo) * lrb, (stop - r) * rb,
                                          cudaMemcpyHostToDevice));
-            break;
+            else  // innermost rows of nin cells land on a pitch of c->pitch cells
+                OLAP_CUDA_TRY(cudaMemcpy2D(dst + lr * rb, c->pitch * 4, src + (r - row_lo) * lrb, nin * 4, nin * 4,
+                                           (stop - r) * (c->lrow_cells / nin), cudaMemcpyHostToDevice));
         }
+        r = stop;
     }
     return OLAP_OK;
 }
@@ -1061,9 +1084,9 @@ int olap_cube_load(olap_cube* c, const void* cells, int64_t ncells) {
     clear_error();
     int rc = check_cube(c);
     if (rc) return rc;
-    if (ncells != c->n[0] * c->row_cells)
+    if (ncells != c->n[0] * c->lrow_cells)
         return set_error(OLAP_E_INVALID, "olap_cube_load: ncells %lld != %lld", (long long)ncells,
-                         (long long)(c->n[0] * c->row_cells));
+                         (long long)(c->n[0] * c->lrow_cells));
     return olap_cube_load_rows(c, 0, c->n[0], cells);
 }
 
