@@ -121,41 +121,35 @@ __device__ __forceinline__ FastDiv dev_fastdiv(uint32_t d) {
 
 // Per-lane accumulators.  int32 cells: SUM in uint64 (wraparound, reading R7),
 // MIN/MAX in int32.  float32 cells: SUM in double (reading R8), MIN/MAX in float.
-// add<OPC>(bits, valid): invalid (masked) cells contribute the op's identity.
+// add<OPC>(bits, mk): mk is an all-ones / all-zero mask of the cell; a masked cell
+// contributes the op's identity through one LOP3 on the raw bits (0 -> +0.0 / 0 for
+// SUM, +inf / INT_MAX for MIN, -inf / INT_MIN for MAX), so no select on the result.
 struct AccI {
     unsigned long long s;
     int32_t mn, mx;
     __device__ void init() { s = 0ull; mn = INT_MAX; mx = INT_MIN; }
     template <int OPC>
-    __device__ __forceinline__ void add(uint32_t bits) {
-        const int32_t v = (int32_t)bits;
-        if (OPC == OPC_SUM) asm("mad.wide.s32 %0, %1, 1, %0;" : "+l"(s) : "r"(v));  // s += sext(v): one IMAD.WIDE
-        if (OPC == OPC_MIN) mn = min(mn, v);
-        if (OPC == OPC_MAX) mx = max(mx, v);
-    }
-    template <int OPC>
-    __device__ __forceinline__ void add_if(uint32_t bits, uint32_t valid) {
-        if (valid) add<OPC>(bits);
+    __device__ __forceinline__ void add(uint32_t bits, uint32_t mk) {
+        if (OPC == OPC_SUM) {
+            const int32_t v = (int32_t)(bits & mk);
+            asm("mad.wide.s32 %0, %1, 1, %0;" : "+l"(s) : "r"(v));  // s += sext(v): one IMAD.WIDE
+        }
+        if (OPC == OPC_MIN) mn = min(mn, (int32_t)((bits & mk) | (0x7fffffffu & ~mk)));
+        if (OPC == OPC_MAX) mx = max(mx, (int32_t)((bits & mk) | (0x80000000u & ~mk)));
     }
     __device__ __forceinline__ long long sum_bits() const { return (long long)s; }
     __device__ __forceinline__ int32_t code_max() const { return mx; }
     __device__ __forceinline__ int32_t code_min() const { return mn; }
-    __device__ __forceinline__ bool has_max() const { return mx != INT_MIN; }
 };
 struct AccF {
     double s;
     float mn, mx;
     __device__ void init() { s = 0.0; mn = __int_as_float(0x7f800000); mx = __int_as_float(0xff800000); }
     template <int OPC>
-    __device__ __forceinline__ void add(uint32_t bits) {
-        const float v = __uint_as_float(bits);
-        if (OPC == OPC_SUM) s += (double)v;
-        if (OPC == OPC_MIN) mn = fminf(mn, v);
-        if (OPC == OPC_MAX) mx = fmaxf(mx, v);
-    }
-    template <int OPC>
-    __device__ __forceinline__ void add_if(uint32_t bits, uint32_t valid) {
-        if (valid) add<OPC>(bits);
+    __device__ __forceinline__ void add(uint32_t bits, uint32_t mk) {
+        if (OPC == OPC_SUM) s += (double)__uint_as_float(bits & mk);
+        if (OPC == OPC_MIN) mn = fminf(mn, __uint_as_float((bits & mk) | (0x7f800000u & ~mk)));
+        if (OPC == OPC_MAX) mx = fmaxf(mx, __uint_as_float((bits & mk) | (0xff800000u & ~mk)));
     }
     __device__ __forceinline__ long long sum_bits() const { return __double_as_longlong(s); }
     __device__ __forceinline__ int32_t code_max() const { return f32_code(mx); }
@@ -175,28 +169,35 @@ template <> struct SumOps<AccF> {
 };
 
 // First slot of run r: base_al + sum_e digit_e(r) * rs[e].  32-bit fast-division
-// chain when r < 2^31 (the common case), 64-bit divisions otherwise.
-__device__ __noinline__ int64_t run_addr(const QDesc& d, int64_t r) {
+// chain when r < 2^31 (the common case), 64-bit divisions otherwise.  The digit loop is
+// deliberately not unrolled: the radices stay in shared memory instead of ~30 registers.
+__device__ __noinline__ int64_t run_addr_wide(const QDesc& d, int64_t r) {  // r >= 2^31: rare
     int64_t a = d.base_al;
-    if (r < (1ll << 31)) {
-        uint32_t x = (uint32_t)r;
-#pragma unroll
-        for (int e = 0; e < kMaxRunDims; ++e) {
-            if (e < d.nrd) {
-                const uint32_t q = fdiv(x, d.frl[e]);
-                a += (int64_t)(x - q * d.frl[e].d) * d.rs[e];
-                x = q;
-            }
-        }
-    } else {
-        for (int e = 0; e < d.nrd; ++e) {
-            const int64_t l = d.frl[e].d, q = r / l;
-            a += (r - q * l) * d.rs[e];
-            r = q;
-        }
+    for (int e = 0; e < d.nrd; ++e) {
+        const int64_t l = d.frl[e].d, q = r / l;
+        a += (r - q * l) * d.rs[e];
+        r = q;
     }
     return a;
 }
+
+__device__ __forceinline__ int64_t run_addr(const QDesc& d, int64_t r) {
+    if (r >= (1ll << 31)) return run_addr_wide(d, r);
+    int64_t a = d.base_al;
+    const int nrd = d.nrd;
+    uint32_t x = (uint32_t)r;
+#pragma unroll 1
+    for (int e = 0; e < nrd; ++e) {
+        const FastDiv f = d.frl[e];
+        const uint32_t q = fdiv(x, f);
+        a += (int64_t)(x - q * f.d) * d.rs[e];
+        x = q;
+    }
+    return a;
+}
+
+// 64-bit quotient kept out of line (one per warp per item): no caller-saved spills in the loops
+__device__ __noinline__ int64_t div64(int64_t a, int64_t b) { return a / b; }
 
 // Largest q in [0,nq) with item_start[q] <= item (32-ary warp search).
 __device__ __forceinline__ int64_t find_query(const int64_t* __restrict__ item_start, int64_t nq, int64_t item,
@@ -217,41 +218,36 @@ __device__ __forceinline__ int64_t find_query(const int64_t* __restrict__ item_s
     return lo + (31 - __clz(m));
 }
 
-// Fold kUnroll slots (V cells each) into the accumulator.  m[u] bit k set <=> cell k
-// of slot u belongs to the box (masked cells are skipped through predication).
-template <class Acc, int OPC, int V, bool MASKED>
-__device__ __forceinline__ void fold(Acc& acc, const uint32_t (&v)[kUnroll][V], const uint32_t (&m)[kUnroll]) {
-#pragma unroll
-    for (int u = 0; u < kUnroll; ++u)
-#pragma unroll
-        for (int k = 0; k < V; ++k) {
-            if (MASKED) acc.template add_if<OPC>(v[u][k], (m[u] >> k) & 1u);
-            else acc.template add<OPC>(v[u][k]);
-        }
+// Slot masks are byte-mask words: byte k = 0xFF when cell k of the slot is in the box.
+// Cell k's 32-bit mask is byte k replicated (one PRMT).
+__device__ __forceinline__ uint32_t cell_mask(uint32_t w, int k) {
+    return __byte_perm(w, 0u, 0x1111u * (uint32_t)k);
+}
+__host__ __device__ __forceinline__ uint32_t byte_mask_word(uint32_t bits4) {
+    uint32_t w = 0;
+    for (int k = 0; k < 4; ++k)
+        if (bits4 >> k & 1u) w |= 0xFFu << (8 * k);
+    return w;
 }
 
+template <class Acc, int OPC, int V>
+__device__ __forceinline__ void fold_slot(Acc& acc, const uint32_t (&v)[4], uint32_t w) {
+#pragma unroll
+    for (int k = 0; k < V; ++k) acc.template add<OPC>(v[k], V == 4 ? cell_mask(w, k) : w);
+}
+
+// Byte-mask words of a run's first slot, last slot, and both (single-slot runs).
 template <int V>
-__device__ __forceinline__ void load_slot(const uint32_t* p, bool ok, uint32_t (&dst)[V]) {
-    if constexpr (V == 4) {
-        uint4 x = make_uint4(0u, 0u, 0u, 0u);
-        if (ok) x = ld_stream4(p);
-        dst[0] = x.x;
-        dst[1] = x.y;
-        dst[2] = x.z;
-        dst[3] = x.w;
-    } else {
-        dst[0] = ok ? ld_stream1(p) : 0u;
+__device__ __forceinline__ void slot_masks(const QDesc& d, uint32_t& wf, uint32_t& wl, uint32_t& wb) {
+    if (V == 1) {
+        wf = wl = wb = 0xFFFFFFFFu;
+        return;
     }
-}
-
-// Masks of a run's first and last slot (bit k = cell k is in the box).
-template <int V>
-__device__ __forceinline__ void slot_masks(const QDesc& d, uint32_t& fm, uint32_t& lm) {
-    const uint32_t full = (1u << V) - 1u;
-    const int tail = (int)(d.h0 + d.L - (int64_t)V * (d.nslot - 1));  // cells of the last slot in the run
-    fm = full & ~((1u << d.h0) - 1u);
-    lm = (1u << tail) - 1u;
-    if (d.nslot == 1) fm &= lm, lm = fm;
+    const int tail = (int)(d.h0 + d.L - 4 * (d.nslot - 1));  // cells of the last slot in the run
+    const uint32_t fm = 0xFu & ~((1u << d.h0) - 1u), lm = (1u << tail) - 1u;
+    wf = byte_mask_word(fm);
+    wl = byte_mask_word(lm);
+    wb = byte_mask_word(fm & lm);
 }
 
 // Short runs (nslot < T): a task spans <= 31 runs.  Lane i holds the first-slot
@@ -262,13 +258,12 @@ __device__ __forceinline__ void stream_short(const uint32_t* __restrict__ cube, 
                                              Acc& acc, int lane, int w) {
     int64_t t = t0 + w;
     if (t >= t1) return;
-    const int T_ = d.T, nslot = (int)d.nslot;
-    uint32_t fm, lm;
-    slot_masks<V>(d, fm, lm);
-    const uint32_t full = (1u << V) - 1u;
+    const int T_ = d.T, nslot = (int)d.nslot, last = nslot - 1;
+    uint32_t wf, wl, wb;
+    slot_masks<V>(d, wf, wl, wb);
     const FastDiv fn = d.fnslot;
     const int64_t G = d.G, R = d.R;
-    int64_t j0 = (t * T_) / nslot;
+    int64_t j0 = div64(t * T_, nslot);
     int rem = (int)(t * T_ - j0 * nslot);
     const int step = kWarps * T_;
     for (; t < t1; t += kWarps) {
@@ -276,20 +271,33 @@ __device__ __forceinline__ void stream_short(const uint32_t* __restrict__ cube, 
         const int n = left < T_ ? (int)left : T_;
         const int64_t ra = (j0 + lane < R) ? run_addr(d, j0 + lane) : 0;
         for (int i0 = 0; i0 < n; i0 += 32 * kUnroll) {
-            uint32_t v[kUnroll][V];
+            uint32_t v[kUnroll][4];
             uint32_t m[kUnroll];
 #pragma unroll
             for (int u = 0; u < kUnroll; ++u) {
-                const int idx = i0 + 32 * u + lane;
-                const bool ok = idx < n;
+                // out-of-range lanes re-read the task's last slot (same sectors, no extra traffic)
+                // with an all-zero mask: every load is unconditional, no state carried across steps
+                const int idx0 = i0 + 32 * u + lane;
+                const bool ok = idx0 < n;
+                const int idx = ok ? idx0 : n - 1;
                 const uint32_t gr = (uint32_t)(rem + idx);
                 const int j = (int)fdiv(gr, fn);
                 const int s = (int)gr - j * nslot;
                 const int64_t a = __shfl_sync(0xffffffffu, ra, j & 31) + (int64_t)s * V;
-                m[u] = ok ? ((s == 0 ? fm : full) & (s == nslot - 1 ? lm : full)) : 0u;
-                load_slot<V>(cube + a, ok, v[u]);
+                const uint32_t wm = s == 0 ? (s == last ? wb : wf) : (s == last ? wl : 0xFFFFFFFFu);
+                m[u] = ok ? wm : 0u;
+                if constexpr (V == 4) {
+                    const uint4 x = ld_stream4(cube + a);
+                    v[u][0] = x.x;
+                    v[u][1] = x.y;
+                    v[u][2] = x.z;
+                    v[u][3] = x.w;
+                } else {
+                    v[u][0] = ld_stream1(cube + a);
+                }
             }
-            fold<Acc, OPC, V, true>(acc, v, m);
+#pragma unroll
+            for (int u = 0; u < kUnroll; ++u) fold_slot<Acc, OPC, V>(acc, v[u], m[u]);
         }
         rem += step;
         const int dj = (int)fdiv((uint32_t)rem, fn);
@@ -299,26 +307,40 @@ __device__ __forceinline__ void stream_short(const uint32_t* __restrict__ cube, 
 }
 
 // Stream slots [0, count) of one run segment starting at slot address p (cells).
-// fmask / lmask: masks of slot 0 and slot count-1 (full when not a run edge).
-// Steps with no edge slot skip masking entirely.
+// wfirst / wlast: byte-mask words of slot 0 and slot count-1 (all ones when not a run
+// edge; wboth when one slot is both).  Steps with no edge slot skip masking entirely.
 template <class Acc, int OPC, int V>
-__device__ __forceinline__ void stream_segment(const uint32_t* __restrict__ p, int count, uint32_t fmask,
-                                               uint32_t lmask, Acc& acc, int lane) {
-    const uint32_t full = (1u << V) - 1u;
+__device__ __forceinline__ void stream_segment(const uint32_t* __restrict__ p, int count, uint32_t wfirst,
+                                               uint32_t wlast, uint32_t wboth, Acc& acc, int lane) {
     for (int i0 = 0; i0 < count; i0 += 32 * kUnroll) {
-        uint32_t v[kUnroll][V];
+        uint32_t v[kUnroll][4];
         uint32_t m[kUnroll];
-        const bool interior = (i0 > 0 || fmask == full) && (i0 + 32 * kUnroll < count || lmask == full) &&
+        const bool interior = (i0 > 0 || wfirst == 0xFFFFFFFFu) && (i0 + 32 * kUnroll < count || wlast == 0xFFFFFFFFu) &&
                               i0 + 32 * kUnroll <= count;
 #pragma unroll
         for (int u = 0; u < kUnroll; ++u) {
-            const int idx = i0 + 32 * u + lane;
-            const bool ok = idx < count;
-            m[u] = ok ? ((idx == 0 ? fmask : full) & (idx == count - 1 ? lmask : full)) : 0u;
-            load_slot<V>(p + (int64_t)idx * V, ok, v[u]);
+            const int idx0 = i0 + 32 * u + lane;
+            const bool ok = idx0 < count;
+            const int idx = ok ? idx0 : count - 1;  // re-read the last slot, masked out
+            const uint32_t wm = idx == 0 ? (idx == count - 1 ? wboth : wfirst) : (idx == count - 1 ? wlast : 0xFFFFFFFFu);
+            m[u] = ok ? wm : 0u;
+            if constexpr (V == 4) {
+                const uint4 x = ld_stream4(p + (int64_t)idx * 4);
+                v[u][0] = x.x;
+                v[u][1] = x.y;
+                v[u][2] = x.z;
+                v[u][3] = x.w;
+            } else {
+                v[u][0] = ld_stream1(p + idx);
+            }
         }
-        if (interior) fold<Acc, OPC, V, false>(acc, v, m);
-        else fold<Acc, OPC, V, true>(acc, v, m);
+        if (interior) {
+#pragma unroll
+            for (int u = 0; u < kUnroll; ++u) fold_slot<Acc, OPC, V>(acc, v[u], 0xFFFFFFFFu);
+        } else {
+#pragma unroll
+            for (int u = 0; u < kUnroll; ++u) fold_slot<Acc, OPC, V>(acc, v[u], m[u]);
+        }
     }
 }
 
@@ -331,10 +353,10 @@ __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, c
     if (t >= t1) return;
     const int T_ = d.T;
     const int64_t nslot = d.nslot, G = d.G;
-    uint32_t fm, lm;
-    slot_masks<V>(d, fm, lm);
-    const uint32_t full = (1u << V) - 1u;
-    int64_t j0 = (t * T_) / nslot;
+    uint32_t wf, wl, wb;
+    slot_masks<V>(d, wf, wl, wb);
+    const uint32_t full = 0xFFFFFFFFu;
+    int64_t j0 = div64(t * T_, nslot);
     int64_t rem = t * T_ - j0 * nslot;
     const int64_t step = (int64_t)kWarps * T_;
     for (; t < t1; t += kWarps) {
@@ -342,9 +364,10 @@ __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, c
         const int n = left < T_ ? (int)left : T_;
         const int64_t in_run = nslot - rem;
         const int c1 = in_run < n ? (int)in_run : n;
-        stream_segment<Acc, OPC, V>(cube + run_addr(d, j0) + rem * V, c1, rem == 0 ? fm : full,
-                                    rem + c1 == nslot ? lm : full, acc, lane);
-        if (c1 < n) stream_segment<Acc, OPC, V>(cube + run_addr(d, j0 + 1), n - c1, fm, full, acc, lane);
+        const bool first = rem == 0, lastin = rem + c1 == nslot;
+        stream_segment<Acc, OPC, V>(cube + run_addr(d, j0) + rem * V, c1, first ? wf : full, lastin ? wl : full,
+                                    first && lastin ? wb : (first ? wf : wl), acc, lane);
+        if (c1 < n) stream_segment<Acc, OPC, V>(cube + run_addr(d, j0 + 1), n - c1, wf, full, wf, acc, lane);
         rem += step;
         if (rem >= nslot) {
             const int64_t dj = nslot < (1ll << 20) ? (int64_t)fdiv((uint32_t)rem, d.fnslot) : 1;
