@@ -41,7 +41,11 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     lib = out or LIB
     if not force and not defines and out is None and not stale():
         return LIB
-    bdir = BUILD if not defines else BUILD + "_" + "_".join(d.replace("=", "") for d in defines)
+    if defines:
+        import hashlib
+        bdir = BUILD + "_" + hashlib.sha1("|".join(defines).encode()).hexdigest()[:10]
+    else:
+        bdir = BUILD
     os.makedirs(bdir, exist_ok=True)
     extra = (["-Xptxas", "-v"] if verbose else []) + [f"-D{d}" for d in defines]
 

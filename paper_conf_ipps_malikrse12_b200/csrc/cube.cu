@@ -83,16 +83,22 @@ struct Extents {
 
 // ------------------------------------------------------------------ device helpers
 
+#ifndef OLAP_LD4
+#define OLAP_LD4 "ld.global.nc.L1::no_allocate.v4.u32"
+#endif
+#ifndef OLAP_LD1
+#define OLAP_LD1 "ld.global.nc.L1::no_allocate.u32"
+#endif
 __device__ __forceinline__ uint4 ld_stream4(const void* p) {
     uint4 r;
-    asm("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+    asm(OLAP_LD4 " {%0,%1,%2,%3}, [%4];"
         : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
         : "l"(p));
     return r;
 }
 __device__ __forceinline__ uint32_t ld_stream1(const void* p) {
     uint32_t r;
-    asm("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
+    asm(OLAP_LD1 " %0, [%1];" : "=r"(r) : "l"(p));
     return r;
 }
 
@@ -468,19 +474,20 @@ __device__ V block_sum(V v, V* sh) {
     return t;
 }
 
-// One block: descriptors, adaptive item size, exclusive scan of item counts.
-__global__ void __launch_bounds__(kPlanThreads) plan_kernel(Geo geo, int64_t nq, const olap_range* __restrict__ ranges,
+constexpr int kDescThreads = 256;
+
+// Grid-wide, one thread per query: descriptor, identity partials for queries that read
+// no cell, per-query (tasks, cells per task) for the scan, batch totals (atomics on
+// integers: order-free, deterministic).
+__global__ void __launch_bounds__(kDescThreads) desc_kernel(Geo geo, int64_t nq, const olap_range* __restrict__ ranges,
                                                             const int32_t* __restrict__ ops, QDesc* desc,
-                                                            int64_t* item_start, int32_t* done,
-                                                            unsigned long long* counter, int64_t* psum,
-                                                            int32_t* pext, int64_t items_cap,
-                                                            unsigned long long* bytes_acc) {
+                                                            int64_t* q_tasks, int32_t* q_tv, int32_t* done,
+                                                            int64_t* psum, int32_t* pext,
+                                                            unsigned long long* totals) {
     __shared__ int64_t sh[32];
-    const int tid = threadIdx.x;
-    const int64_t per = (nq + kPlanThreads - 1) / kPlanThreads;
-    const int64_t q0 = min(nq, (int64_t)tid * per), q1 = min(nq, q0 + per);
-    int64_t my_cells = 0, my_slot_cells = 0;
-    for (int64_t q = q0; q < q1; ++q) {
+    const int64_t q = blockIdx.x * (int64_t)kDescThreads + threadIdx.x;
+    int64_t cells = 0, slot_cells = 0;
+    if (q < nq) {
         QDesc d;
         build_desc(geo, ranges + q * geo.nd, ops[q], d);
         desc[q] = d;
@@ -489,28 +496,48 @@ __global__ void __launch_bounds__(kPlanThreads) plan_kernel(Geo geo, int64_t nq,
             psum[q] = 0;
             pext[2 * q] = INT_MIN;
             pext[2 * q + 1] = INT_MIN;
+            q_tasks[q] = 0;
+            q_tv[q] = 1;
         } else {
-            my_cells += d.vlocal;
-            my_slot_cells += d.G * d.V;
+            cells = d.vlocal;
+            slot_cells = d.G * d.V;
+            q_tasks[q] = d.tasks;
+            q_tv[q] = d.T * d.V;
         }
     }
-    const int64_t total_cells = block_sum<int64_t>(my_cells, sh);
-    const int64_t total_slot_cells = block_sum<int64_t>(my_slot_cells, sh);
+    cells = block_sum<int64_t>(cells, sh);
+    slot_cells = block_sum<int64_t>(slot_cells, sh);
+    if (threadIdx.x == 0) {
+        if (cells) atomicAdd(totals + 0, (unsigned long long)cells);
+        if (slot_cells) atomicAdd(totals + 1, (unsigned long long)slot_cells);
+    }
+}
+
+// One block: adaptive item size, tasks-per-item per query, exclusive scan of item counts.
+__global__ void __launch_bounds__(kPlanThreads) scan_kernel(int64_t nq, QDesc* desc, const int64_t* __restrict__ q_tasks,
+                                                            const int32_t* __restrict__ q_tv, int64_t* item_start,
+                                                            unsigned long long* counter, int64_t items_cap,
+                                                            const unsigned long long* totals,
+                                                            unsigned long long* bytes_acc) {
+    const int tid = threadIdx.x;
+    const int64_t total_cells = (int64_t)totals[0], total_slot_cells = (int64_t)totals[1];
     // item size: >= 1 MiB, and large enough that sum_q items_q <= items_cap:
     // items_q <= tasks_q/tpi_q + 1 <= 2*G_q*V_q/teff + 2 (tpi_q*T_q*V_q >= teff/2)
     const int64_t cap_left = items_cap - 2 * nq;
     int64_t teff = (4 * total_slot_cells + cap_left - 1) / cap_left;
     if (teff < kItemCells) teff = kItemCells;
+    const int64_t per = (nq + kPlanThreads - 1) / kPlanThreads;
+    const int64_t q0 = min(nq, (int64_t)tid * per), q1 = min(nq, q0 + per);
     int64_t my_items = 0;
     for (int64_t q = q0; q < q1; ++q) {
-        QDesc& d = desc[q];
+        const int64_t tasks = q_tasks[q];
         int64_t items = 0;
-        if (d.opc != OPC_NONE) {
-            int64_t tpi = teff / ((int64_t)d.T * d.V);
+        if (tasks) {
+            int64_t tpi = teff / q_tv[q];
             if (tpi < 1) tpi = 1;
             if (tpi > (1ll << 30)) tpi = (1ll << 30);
-            d.tpi = (int32_t)tpi;
-            items = (d.tasks + tpi - 1) / tpi;
+            desc[q].tpi = (int32_t)tpi;
+            items = (tasks + tpi - 1) / tpi;
         }
         item_start[q] = items;
         my_items += items;
@@ -811,7 +838,9 @@ struct olap_cube {
     QDesc* d_desc = nullptr;
     int64_t* d_item_start = nullptr;
     int32_t* d_done = nullptr;
-    unsigned long long* d_counter = nullptr;  // [0] item counter, [1] algorithmic bytes
+    int64_t* d_qtasks = nullptr;              // per query: tasks (planning scratch)
+    int32_t* d_qtv = nullptr;                 // per query: cells per task (planning scratch)
+    unsigned long long* d_counter = nullptr;  // [0] item counter, [1] algorithmic bytes, [2..3] batch totals
     long long* d_item_sum = nullptr;
     int32_t* d_item_ext = nullptr;
     // host-path staging
@@ -867,6 +896,10 @@ void free_ws(olap_cube* c) {
     cudaFree(c->d_desc);
     cudaFree(c->d_item_start);
     cudaFree(c->d_done);
+    cudaFree(c->d_qtasks);
+    cudaFree(c->d_qtv);
+    c->d_qtasks = nullptr;
+    c->d_qtv = nullptr;
     cudaFree(c->d_item_sum);
     cudaFree(c->d_item_ext);
     c->d_desc = nullptr;
@@ -886,6 +919,8 @@ int ensure_ws(olap_cube* c, int64_t nq) {
     OLAP_CUDA_TRY(cudaMalloc(&c->d_desc, sizeof(QDesc) * cap));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_item_start, sizeof(int64_t) * (cap + 1)));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_done, sizeof(int32_t) * cap));
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_qtasks, sizeof(int64_t) * cap));
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_qtv, sizeof(int32_t) * cap));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_item_sum, sizeof(long long) * items));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_item_ext, sizeof(int32_t) * 2 * items));
     c->nq_cap = cap;
@@ -927,8 +962,12 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
     int rc = ensure_ws(c, nq);
     if (rc) return rc;
     OLAP_CUDA_TRY(cudaStreamWaitEvent(st, c->ws_done, 0));
-    plan_kernel<<<1, kPlanThreads, 0, st>>>(make_geo(c), nq, d_ranges, d_ops, c->d_desc, c->d_item_start, c->d_done,
-                                            c->d_counter, d_psum, d_pext, c->items_cap, c->d_counter + 1);
+    OLAP_CUDA_TRY(cudaMemsetAsync(c->d_counter + 2, 0, 2 * sizeof(unsigned long long), st));
+    desc_kernel<<<(int)((nq + kDescThreads - 1) / kDescThreads), kDescThreads, 0, st>>>(
+        make_geo(c), nq, d_ranges, d_ops, c->d_desc, c->d_qtasks, c->d_qtv, c->d_done, d_psum, d_pext, c->d_counter + 2);
+    OLAP_CUDA_TRY(cudaGetLastError());
+    scan_kernel<<<1, kPlanThreads, 0, st>>>(nq, c->d_desc, c->d_qtasks, c->d_qtv, c->d_item_start, c->d_counter,
+                                            c->items_cap, c->d_counter + 2, c->d_counter + 1);
     OLAP_CUDA_TRY(cudaGetLastError());
     const int grid = c->num_sms * c->blocks_per_sm;
     cudaEvent_t e0 = nullptr, e1 = nullptr;
@@ -1037,8 +1076,8 @@ int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_sh
     if (c->pitch != c->n[ndims - 1]) cudaMemset(c->d_cells, 0, c->local_cells * 4);
     if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess ||
         cudaEventCreateWithFlags(&c->ws_done, cudaEventDisableTiming) != cudaSuccess ||
-        cudaMalloc(&c->d_counter, 2 * sizeof(unsigned long long)) != cudaSuccess ||
-        cudaMemset(c->d_counter, 0, 2 * sizeof(unsigned long long)) != cudaSuccess) {
+        cudaMalloc(&c->d_counter, 4 * sizeof(unsigned long long)) != cudaSuccess ||
+        cudaMemset(c->d_counter, 0, 4 * sizeof(unsigned long long)) != cudaSuccess) {
         rc = set_error(OLAP_E_CUDA, "stream/event/counter setup failed");
         olap_cube_destroy(c);
         return rc;
@@ -1054,6 +1093,7 @@ int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_sh
         if (v > 0 && v < bps) bps = v;
     }
     c->blocks_per_sm = std::max(bps, 1);
+
     *out = c;
     return OLAP_OK;
 }
