@@ -25,7 +25,8 @@ constexpr int kMaxDims = 8;
 constexpr int kMaxRunDims = 7;
 constexpr int kWarps = 8;                   // warps per reduce block
 constexpr int kThreads = kWarps * 32;
-constexpr int kTaskSlots = 2048;            // max slots per warp task (32 KiB of 16-B slots)
+constexpr int kTaskSlots = 2048;            // slots per warp task (long path), slot budget of a short task
+constexpr int kShortMaxSlots = 512;         // runs of at most this many slots: short path (<= 31 runs per task)
 #ifndef OLAP_UNROLL
 #define OLAP_UNROLL 4
 #endif
@@ -56,12 +57,13 @@ struct QDesc {
     int64_t G;        // slots in the box
     int64_t tasks;    // ceil(G / T)
     int64_t vlocal;   // cells of the box on this shard (R * L)
-    int32_t T;        // slots per task
+    int32_t T;        // short path: runs per task (<= 31); long path: slots per task
     int32_t tpi;      // tasks per item
     int32_t h0;       // masked leading cells of each run's first slot
-    int32_t V;        // cells per slot (4 or 1)
-    int32_t opc, nrd, op, pad;
-    FastDiv fnslot;   // / nslot (valid when nslot < 2^31)
+    int32_t V;        // cells per slot (8, 4 or 1)
+    int32_t opc, nrd, op, shortp;  // shortp: runs of <= kShortMaxSlots slots take the short path
+    FastDiv fnslot;   // / nslot (long path; valid when nslot < 2^31)
+    FastDiv fni;      // / (nslot - 2), the interior slots of a run (short path)
     FastDiv frl[kMaxRunDims];
     int64_t rs[kMaxRunDims];
 };
@@ -95,6 +97,14 @@ __device__ __forceinline__ uint4 ld_stream4(const void* p) {
         : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
         : "l"(p));
     return r;
+}
+#ifndef OLAP_LD8
+#define OLAP_LD8 "ld.global.nc.L1::no_allocate.v8.u32"
+#endif
+__device__ __forceinline__ void ld_stream8(const void* p, uint32_t (&r)[8]) {  // LDG.256 (sm_100)
+    asm(OLAP_LD8 " {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7])
+        : "l"(p));
 }
 __device__ __forceinline__ uint32_t ld_stream1(const void* p) {
     uint32_t r;
@@ -224,134 +234,159 @@ __device__ __forceinline__ int64_t find_query(const int64_t* __restrict__ item_s
     return lo + (31 - __clz(m));
 }
 
-// Slot masks are byte-mask words: byte k = 0xFF when cell k of the slot is in the box.
-// Cell k's 32-bit mask is byte k replicated (one PRMT).
-__device__ __forceinline__ uint32_t cell_mask(uint32_t w, int k) {
-    return __byte_perm(w, 0u, 0x1111u * (uint32_t)k);
+// Slot masks are byte-mask words: byte k = 0xFF when cell k of the slot is in the box
+// (8 bytes for 8-cell slots).  Cell k's 32-bit mask is byte k replicated (one PRMT).
+template <int V>
+__device__ __forceinline__ uint32_t cell_mask(uint64_t w, int k) {
+    if (V == 1) return (uint32_t)w;
+    return __byte_perm(k < 4 ? (uint32_t)w : (uint32_t)(w >> 32), 0u, 0x1111u * (uint32_t)(k & 3));
 }
-__host__ __device__ __forceinline__ uint32_t byte_mask_word(uint32_t bits4) {
-    uint32_t w = 0;
-    for (int k = 0; k < 4; ++k)
-        if (bits4 >> k & 1u) w |= 0xFFu << (8 * k);
+__device__ __forceinline__ uint64_t byte_mask_word(uint32_t bits8) {
+    uint64_t w = 0;
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+        if (bits8 >> k & 1u) w |= 0xFFull << (8 * k);
     return w;
 }
 
+template <int V>
+__device__ __forceinline__ void load_slot(const uint32_t* p, uint32_t (&v)[V]) {
+    if constexpr (V == 8) {
+        ld_stream8(p, v);
+    } else if constexpr (V == 4) {
+        const uint4 x = ld_stream4(p);
+        v[0] = x.x;
+        v[1] = x.y;
+        v[2] = x.z;
+        v[3] = x.w;
+    } else {
+        v[0] = ld_stream1(p);
+    }
+}
+
 template <class Acc, int OPC, int V>
-__device__ __forceinline__ void fold_slot(Acc& acc, const uint32_t (&v)[4], uint32_t w) {
+__device__ __forceinline__ void fold_slot(Acc& acc, const uint32_t (&v)[V], uint64_t w) {
 #pragma unroll
-    for (int k = 0; k < V; ++k) acc.template add<OPC>(v[k], V == 4 ? cell_mask(w, k) : w);
+    for (int k = 0; k < V; ++k) acc.template add<OPC>(v[k], cell_mask<V>(w, k));
+}
+template <class Acc, int OPC, int V>
+__device__ __forceinline__ void fold_full(Acc& acc, const uint32_t (&v)[V]) {
+#pragma unroll
+    for (int k = 0; k < V; ++k) acc.template add<OPC>(v[k], 0xFFFFFFFFu);
 }
 
 // Byte-mask words of a run's first slot, last slot, and both (single-slot runs).
 template <int V>
-__device__ __forceinline__ void slot_masks(const QDesc& d, uint32_t& wf, uint32_t& wl, uint32_t& wb) {
+__device__ __forceinline__ void slot_masks(const QDesc& d, uint64_t& wf, uint64_t& wl, uint64_t& wb) {
     if (V == 1) {
-        wf = wl = wb = 0xFFFFFFFFu;
+        wf = wl = wb = ~0ull;
         return;
     }
-    const int tail = (int)(d.h0 + d.L - 4 * (d.nslot - 1));  // cells of the last slot in the run
-    const uint32_t fm = 0xFu & ~((1u << d.h0) - 1u), lm = (1u << tail) - 1u;
+    const int tail = (int)(d.h0 + d.L - (int64_t)V * (d.nslot - 1));  // cells of the last slot in the run
+    const uint32_t full = (1u << V) - 1u;
+    const uint32_t fm = full & ~((1u << d.h0) - 1u), lm = (1u << tail) - 1u;
     wf = byte_mask_word(fm);
     wl = byte_mask_word(lm);
     wb = byte_mask_word(fm & lm);
 }
 
-// Short runs (nslot < T): a task spans <= 31 runs.  Lane i holds the first-slot
-// address of run j0+i; slot g of the task is run j = (rem+g)/nslot, slot s of it;
-// all index math is 32-bit, the run address comes from a shuffle.
+constexpr int unroll_for(int V) { return V == 8 ? 2 : 4; }  // 64 B (or 16 B) of loads in flight per lane
+
+// Short runs (nslot <= kShortMaxSlots): a task is up to 31 whole runs.  Lane i holds
+// the first-slot address of run r0+i.  The interior slots of all the task's runs
+// (slots 1..nslot-2) are flattened and streamed WITHOUT masks: slot g is run
+// j = g / (nslot-2) (fast division), slot 1 + g % (nslot-2), address via a shuffle.
+// The two edge slots of every run go through a short masked pass.
 template <class Acc, int OPC, int V>
 __device__ __forceinline__ void stream_short(const uint32_t* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
                                              Acc& acc, int lane, int w) {
+    constexpr int U = unroll_for(V);
     int64_t t = t0 + w;
     if (t >= t1) return;
-    const int T_ = d.T, nslot = (int)d.nslot, last = nslot - 1;
-    uint32_t wf, wl, wb;
+    const int rpt = d.T, nslot = (int)d.nslot;
+    const int ni = nslot >= 2 ? nslot - 2 : 0, ne = nslot >= 2 ? 2 : 1;
+    uint64_t wf, wl, wb;
     slot_masks<V>(d, wf, wl, wb);
-    const FastDiv fn = d.fnslot;
-    const int64_t G = d.G, R = d.R;
-    int64_t j0 = div64(t * T_, nslot);
-    int rem = (int)(t * T_ - j0 * nslot);
-    const int step = kWarps * T_;
+    const FastDiv fni = d.fni;
+    const int64_t R = d.R;
     for (; t < t1; t += kWarps) {
-        const int64_t left = G - t * T_;
-        const int n = left < T_ ? (int)left : T_;
-        const int64_t ra = (j0 + lane < R) ? run_addr(d, j0 + lane) : 0;
-        for (int i0 = 0; i0 < n; i0 += 32 * kUnroll) {
-            uint32_t v[kUnroll][4];
-            uint32_t m[kUnroll];
+        const int64_t r0 = t * rpt;
+        const int nr = (int)min((int64_t)rpt, R - r0);
+        const int64_t ra = lane < nr ? run_addr(d, r0 + lane) : 0;
+        const int nint = nr * ni;
+        for (int i0 = 0; i0 < nint; i0 += 32 * U) {
+            uint32_t v[U][V];
+            bool ok[U];
 #pragma unroll
-            for (int u = 0; u < kUnroll; ++u) {
-                // out-of-range lanes re-read the task's last slot (same sectors, no extra traffic)
-                // with an all-zero mask: every load is unconditional, no state carried across steps
+            for (int u = 0; u < U; ++u) {
                 const int idx0 = i0 + 32 * u + lane;
-                const bool ok = idx0 < n;
-                const int idx = ok ? idx0 : n - 1;
-                const uint32_t gr = (uint32_t)(rem + idx);
-                const int j = (int)fdiv(gr, fn);
-                const int s = (int)gr - j * nslot;
-                const int64_t a = __shfl_sync(0xffffffffu, ra, j & 31) + (int64_t)s * V;
-                const uint32_t wm = s == 0 ? (s == last ? wb : wf) : (s == last ? wl : 0xFFFFFFFFu);
-                m[u] = ok ? wm : 0u;
-                if constexpr (V == 4) {
-                    const uint4 x = ld_stream4(cube + a);
-                    v[u][0] = x.x;
-                    v[u][1] = x.y;
-                    v[u][2] = x.z;
-                    v[u][3] = x.w;
-                } else {
-                    v[u][0] = ld_stream1(cube + a);
-                }
+                ok[u] = idx0 < nint;
+                const int idx = ok[u] ? idx0 : nint - 1;  // re-read a valid slot, then drop it
+                const int j = (int)fdiv((uint32_t)idx, fni);
+                const int sl = 1 + idx - j * ni;
+                load_slot<V>(cube + __shfl_sync(0xffffffffu, ra, j & 31) + (int64_t)sl * V, v[u]);
+            }
+            if (i0 + 32 * U <= nint) {
+#pragma unroll
+                for (int u = 0; u < U; ++u) fold_full<Acc, OPC, V>(acc, v[u]);
+            } else {
+#pragma unroll
+                for (int u = 0; u < U; ++u) fold_slot<Acc, OPC, V>(acc, v[u], ok[u] ? ~0ull : 0ull);
+            }
+        }
+        const int nedge = nr * ne;
+        for (int i0 = 0; i0 < nedge; i0 += 32 * U) {
+            uint32_t v[U][V];
+            uint64_t m[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const int idx0 = i0 + 32 * u + lane;
+                const bool ok = idx0 < nedge;
+                const int idx = ok ? idx0 : nedge - 1;
+                const int j = ne == 2 ? idx >> 1 : idx;
+                const bool tailside = ne == 2 && (idx & 1);
+                const int sl = tailside ? nslot - 1 : 0;
+                m[u] = ok ? (nslot == 1 ? wb : (tailside ? wl : wf)) : 0ull;
+                load_slot<V>(cube + __shfl_sync(0xffffffffu, ra, j & 31) + (int64_t)sl * V, v[u]);
             }
 #pragma unroll
-            for (int u = 0; u < kUnroll; ++u) fold_slot<Acc, OPC, V>(acc, v[u], m[u]);
+            for (int u = 0; u < U; ++u) fold_slot<Acc, OPC, V>(acc, v[u], m[u]);
         }
-        rem += step;
-        const int dj = (int)fdiv((uint32_t)rem, fn);
-        j0 += dj;
-        rem -= dj * nslot;
     }
 }
 
 // Stream slots [0, count) of one run segment starting at slot address p (cells).
-// wfirst / wlast: byte-mask words of slot 0 and slot count-1 (all ones when not a run
-// edge; wboth when one slot is both).  Steps with no edge slot skip masking entirely.
+// wfirst / wlast: masks of slot 0 and slot count-1 (all ones when not a run edge;
+// wboth when one slot is both).  Steps with no edge slot skip masking entirely.
 template <class Acc, int OPC, int V>
-__device__ __forceinline__ void stream_segment(const uint32_t* __restrict__ p, int count, uint32_t wfirst,
-                                               uint32_t wlast, uint32_t wboth, Acc& acc, int lane) {
-    for (int i0 = 0; i0 < count; i0 += 32 * kUnroll) {
-        uint32_t v[kUnroll][4];
-        uint32_t m[kUnroll];
-        const bool interior = (i0 > 0 || wfirst == 0xFFFFFFFFu) && (i0 + 32 * kUnroll < count || wlast == 0xFFFFFFFFu) &&
-                              i0 + 32 * kUnroll <= count;
+__device__ __forceinline__ void stream_segment(const uint32_t* __restrict__ p, int count, uint64_t wfirst,
+                                               uint64_t wlast, uint64_t wboth, Acc& acc, int lane) {
+    constexpr int U = unroll_for(V);
+    for (int i0 = 0; i0 < count; i0 += 32 * U) {
+        uint32_t v[U][V];
+        uint64_t m[U];
+        const bool interior = (i0 > 0 || wfirst == ~0ull) && (i0 + 32 * U < count || wlast == ~0ull) &&
+                              i0 + 32 * U <= count;
 #pragma unroll
-        for (int u = 0; u < kUnroll; ++u) {
+        for (int u = 0; u < U; ++u) {
             const int idx0 = i0 + 32 * u + lane;
             const bool ok = idx0 < count;
             const int idx = ok ? idx0 : count - 1;  // re-read the last slot, masked out
-            const uint32_t wm = idx == 0 ? (idx == count - 1 ? wboth : wfirst) : (idx == count - 1 ? wlast : 0xFFFFFFFFu);
-            m[u] = ok ? wm : 0u;
-            if constexpr (V == 4) {
-                const uint4 x = ld_stream4(p + (int64_t)idx * 4);
-                v[u][0] = x.x;
-                v[u][1] = x.y;
-                v[u][2] = x.z;
-                v[u][3] = x.w;
-            } else {
-                v[u][0] = ld_stream1(p + idx);
-            }
+            m[u] = ok ? (idx == 0 ? (idx == count - 1 ? wboth : wfirst) : (idx == count - 1 ? wlast : ~0ull)) : 0ull;
+            load_slot<V>(p + (int64_t)idx * V, v[u]);
         }
         if (interior) {
 #pragma unroll
-            for (int u = 0; u < kUnroll; ++u) fold_slot<Acc, OPC, V>(acc, v[u], 0xFFFFFFFFu);
+            for (int u = 0; u < U; ++u) fold_full<Acc, OPC, V>(acc, v[u]);
         } else {
 #pragma unroll
-            for (int u = 0; u < kUnroll; ++u) fold_slot<Acc, OPC, V>(acc, v[u], m[u]);
+            for (int u = 0; u < U; ++u) fold_slot<Acc, OPC, V>(acc, v[u], m[u]);
         }
     }
 }
 
-// Long runs (nslot >= T): a task is at most two contiguous segments (the end of
-// run j0 and the start of run j0+1).
+// Long runs (nslot > kShortMaxSlots): a task is kTaskSlots slots, at most two
+// contiguous segments (the end of run j0 and the start of run j0+1).
 template <class Acc, int OPC, int V>
 __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
                                             Acc& acc, int lane, int w) {
@@ -359,9 +394,8 @@ __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, c
     if (t >= t1) return;
     const int T_ = d.T;
     const int64_t nslot = d.nslot, G = d.G;
-    uint32_t wf, wl, wb;
+    uint64_t wf, wl, wb;
     slot_masks<V>(d, wf, wl, wb);
-    const uint32_t full = 0xFFFFFFFFu;
     int64_t j0 = div64(t * T_, nslot);
     int64_t rem = t * T_ - j0 * nslot;
     const int64_t step = (int64_t)kWarps * T_;
@@ -371,9 +405,9 @@ __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, c
         const int64_t in_run = nslot - rem;
         const int c1 = in_run < n ? (int)in_run : n;
         const bool first = rem == 0, lastin = rem + c1 == nslot;
-        stream_segment<Acc, OPC, V>(cube + run_addr(d, j0) + rem * V, c1, first ? wf : full, lastin ? wl : full,
+        stream_segment<Acc, OPC, V>(cube + run_addr(d, j0) + rem * V, c1, first ? wf : ~0ull, lastin ? wl : ~0ull,
                                     first && lastin ? wb : (first ? wf : wl), acc, lane);
-        if (c1 < n) stream_segment<Acc, OPC, V>(cube + run_addr(d, j0 + 1), n - c1, wf, full, wf, acc, lane);
+        if (c1 < n) stream_segment<Acc, OPC, V>(cube + run_addr(d, j0 + 1), n - c1, wf, ~0ull, wf, acc, lane);
         rem += step;
         if (rem >= nslot) {
             const int64_t dj = nslot < (1ll << 20) ? (int64_t)fdiv((uint32_t)rem, d.fnslot) : 1;
@@ -387,7 +421,7 @@ template <typename T, class Acc, int OPC, int V>
 __device__ __forceinline__ void stream_tasks(const T* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
                                              Acc& acc, int lane, int w) {
     const uint32_t* c = reinterpret_cast<const uint32_t*>(cube);
-    if (d.nslot < d.T) stream_short<Acc, OPC, V>(c, d, t0, t1, acc, lane, w);
+    if (d.shortp) stream_short<Acc, OPC, V>(c, d, t0, t1, acc, lane, w);
     else stream_long<Acc, OPC, V>(c, d, t0, t1, acc, lane, w);
 }
 
@@ -424,31 +458,41 @@ __device__ void build_desc(const Geo& g, const olap_range* r, int32_t op, QDesc&
     int64_t R = 1, base = 0;
     for (int k = 0; k < g.nd; ++k) base += lo[k] * g.stride[k];
     int nrd = 0;
-    bool aligned = true;
+    bool a8 = true, a4 = true;
     for (int k = ks - 1; k >= 0; --k) {
         R *= ell[k];
         if (ell[k] > 1) {
             d.frl[nrd] = dev_fastdiv((uint32_t)ell[k]);
             d.rs[nrd] = g.stride[k];
-            if (g.stride[k] & 3) aligned = false;
+            if (g.stride[k] & 7) a8 = false;
+            if (g.stride[k] & 3) a4 = false;
             ++nrd;
         }
     }
     d.nrd = nrd;
     d.R = R;
     d.vlocal = R * d.L;
-    d.V = aligned ? 4 : 1;
-    d.h0 = aligned ? (int32_t)(base & 3) : 0;
+    // widest slot such that every run starts at the same offset inside its slot
+    d.V = a8 ? 8 : (a4 ? 4 : 1);
+    d.h0 = (int32_t)(base & (d.V - 1));
     d.base_al = base - d.h0;
     d.nslot = (d.h0 + d.L + d.V - 1) / d.V;
     d.G = R * d.nslot;
-    // task: 32 whole runs when runs are tiny; else <= 30 runs' worth of slots (so a task
-    // spans <= 31 runs, one per lane), at most kTaskSlots; long runs: kTaskSlots
-    if (d.nslot < 9) d.T = (int32_t)(32 * d.nslot);
-    else if (d.nslot < kTaskSlots) d.T = (int32_t)(((30 * d.nslot) & ~31ll) < kTaskSlots ? ((30 * d.nslot) & ~31ll) : kTaskSlots);
-    else d.T = kTaskSlots;
-    d.tasks = (d.G + d.T - 1) / d.T;
-    d.fnslot = dev_fastdiv(d.nslot < (1ll << 31) ? (uint32_t)d.nslot : 1u);
+    if (d.nslot <= kShortMaxSlots) {  // short path: tasks of whole runs, <= 31 per task
+        d.shortp = 1;
+        int64_t rpt = kTaskSlots / d.nslot;
+        rpt = rpt < 1 ? 1 : (rpt > 31 ? 31 : rpt);
+        d.T = (int32_t)rpt;
+        d.tasks = (R + rpt - 1) / rpt;
+        d.fni = dev_fastdiv(d.nslot > 2 ? (uint32_t)(d.nslot - 2) : 1u);
+        d.fnslot = dev_fastdiv(1u);
+    } else {
+        d.shortp = 0;
+        d.T = d.nslot < kTaskSlots ? (int32_t)d.nslot : kTaskSlots;  // T <= nslot: a task spans <= 2 runs
+        d.tasks = (d.G + d.T - 1) / d.T;
+        d.fnslot = dev_fastdiv(d.nslot < (1ll << 31) ? (uint32_t)d.nslot : 1u);
+        d.fni = dev_fastdiv(1u);
+    }
     d.opc = (op == OLAP_MIN) ? OPC_MIN : (op == OLAP_MAX) ? OPC_MAX : OPC_SUM;
 }
 
@@ -502,7 +546,7 @@ __global__ void __launch_bounds__(kDescThreads) desc_kernel(Geo geo, int64_t nq,
             cells = d.vlocal;
             slot_cells = d.G * d.V;
             q_tasks[q] = d.tasks;
-            q_tv[q] = d.T * d.V;
+            q_tv[q] = d.shortp ? (int32_t)(d.T * d.nslot * d.V) : d.T * d.V;  // cells per task
         }
     }
     cells = block_sum<int64_t>(cells, sh);
@@ -591,9 +635,14 @@ __global__ void bucket_kernel(int64_t nq, const QDesc* __restrict__ desc, const 
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
         const int64_t q = find_query_thread(item_start, nq, i);
         const QDesc& d = desc[q];
-        const int64_t g = (i - __ldg(item_start + q)) * (int64_t)d.tpi * d.T;  // first slot of the item
-        const int64_t j = g / d.nslot;
-        const int64_t addr = run_addr(d, j) + (g - j * d.nslot) * d.V;
+        const int64_t t0 = (i - __ldg(item_start + q)) * (int64_t)d.tpi;  // first task of the item
+        int64_t addr;
+        if (d.shortp) {
+            addr = run_addr(d, t0 * d.T);
+        } else {
+            const int64_t g = t0 * d.T, j = g / d.nslot;
+            addr = run_addr(d, j) + (g - j * d.nslot) * d.V;
+        }
         int64_t b = addr >> shift;
         if (b >= kMaxBuckets) b = kMaxBuckets - 1;
         bucket[i] = (int32_t)b;
@@ -669,7 +718,11 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) reduce_kernel(const T* _
         Acc acc;
         acc.init();
         const int opc = sd.opc;
-        if (sd.V == 4) {
+        if (sd.V == 8) {
+            if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 8>(cube, sd, t0, t1, acc, lane, w);
+            else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 8>(cube, sd, t0, t1, acc, lane, w);
+            else stream_tasks<T, Acc, OPC_MAX, 8>(cube, sd, t0, t1, acc, lane, w);
+        } else if (sd.V == 4) {
             if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 4>(cube, sd, t0, t1, acc, lane, w);
             else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 4>(cube, sd, t0, t1, acc, lane, w);
             else stream_tasks<T, Acc, OPC_MAX, 4>(cube, sd, t0, t1, acc, lane, w);
@@ -1142,7 +1195,10 @@ int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_sh
     for (int k = 0; k < ndims; ++k) c->n[k] = extents[k];
     // innermost pitch padded to a multiple of 4 cells (16 B) when needed so that every
     // innermost row starts 16-B aligned for the vector path
-    c->pitch = (ndims > 1 && (c->n[ndims - 1] & 3)) ? ((c->n[ndims - 1] + 3) & ~3ll) : c->n[ndims - 1];
+    // (8 cells = 32 B for LDG.256 slots when the extent is >= 32, so padding stays <= 22%)
+    c->pitch = c->n[ndims - 1];
+    if (ndims > 1 && c->pitch >= 32 && (c->pitch & 7)) c->pitch = (c->pitch + 7) & ~7ll;
+    else if (ndims > 1 && (c->pitch & 3)) c->pitch = (c->pitch + 3) & ~3ll;
     c->stride[ndims - 1] = 1;
     for (int k = ndims - 2; k >= 0; --k) c->stride[k] = c->stride[k + 1] * (k == ndims - 2 ? c->pitch : c->n[k + 1]);
     c->row_cells = ndims > 1 ? c->stride[0] : 1;
@@ -1151,7 +1207,7 @@ int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_sh
     c->local_rows = shard_rows(c->n[0], sh.nshards, sh.shard, sh.block);
     c->local_cells = c->local_rows * c->row_cells;
     int rc = OLAP_OK;
-    // +64 B: a run's last 16-B slot may extend up to 3 cells past the final cell (masked)
+    // +64 B: a run's last 32-B slot may extend up to 7 cells past the final cell (masked)
     cudaError_t e = cudaMalloc(&c->d_cells, std::max<int64_t>(c->local_cells, 1) * 4 + 64);
     if (e != cudaSuccess) {
         rc = set_error(e == cudaErrorMemoryAllocation ? OLAP_E_NOMEM : OLAP_E_CUDA, "cudaMalloc of %lld cells: %s",
