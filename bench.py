@@ -457,7 +457,12 @@ def main():
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "kernel": "reduce_kernel",
                          "peak_source": peak_src,
-                         "reduce_share_of_step": reduce_ms / elapsed_ms if elapsed_ms else None},
+                         "algorithmic_bytes_per_launch": alg_bytes / max(launches, 1),
+                         "reduce_share_of_step": reduce_ms / elapsed_ms if elapsed_ms else None,
+                         "note": ("achieved = algorithmic bytes (sum of V_q*4 over non-COUNT queries, Eq. 3) / "
+                                  "reduce-kernel time; frac > 1 is L2 reuse: items are scheduled in cube-address "
+                                  "order so queries overlapping in the cube read it from L2 (traffic = DRAM "
+                                  "bytes per launch from ncu, profiles/traffic.json)")},
             "gpu_launches": int(args.steps * 3),
             "clocks": clk,
             "e2e": e2e,

@@ -70,6 +70,12 @@ SHAPES = [
     ((1, 1, 37), "extent-1 dims"),
     ((64, 129, 7), "odd inner extents"),
     ((17, 4099), "piece boundaries (2048-cell pieces) + tail"),
+    ((5, 3, 40), "inner 40: 32-B slots, short runs"),
+    ((9, 36), "inner 36: pitch padded to 40 (32-B slots)"),
+    ((7, 12), "inner 12: 16-B slots"),
+    ((6, 4096), "runs of 512/513 slots: short/long switch"),
+    ((3, 5, 8), "runs of 1-2 slots: edge pass only"),
+    ((2, 9, 16384), "long runs over several 2048-slot tasks"),
 ]
 
 
