@@ -385,6 +385,8 @@ def main():
         dist.barrier()
     torch.cuda.synchronize()
     cube.profile(True)
+    k0, l2_order = cube.stats()
+    f0 = olap.lib.olap_finalize_launches()
     clocks = Clocks(local)
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
@@ -397,6 +399,7 @@ def main():
     torch.cuda.synchronize()
     elapsed_ms = e0.elapsed_time(e1)
     clk = clocks.stop()
+    gpu_launches = cube.stats()[0] - k0 + olap.lib.olap_finalize_launches() - f0
     reduce_ms, launches, alg_bytes = cube.profile_read()
     cube.profile(False)
     t = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev)
@@ -463,7 +466,7 @@ def main():
                                   "reduce-kernel time; frac > 1 is L2 reuse: items are scheduled in cube-address "
                                   "order so queries overlapping in the cube read it from L2 (traffic = DRAM "
                                   "bytes per launch from ncu, profiles/traffic.json)")},
-            "gpu_launches": int(args.steps * 3),
+            "gpu_launches": int(gpu_launches), "l2_order": l2_order,
             "clocks": clk,
             "e2e": e2e,
             "cpu_baseline": cpu,

@@ -170,6 +170,13 @@ int olap_shard_local_rows(int64_t n0, const olap_shard* shard, int64_t lo, int64
 int olap_cube_profile(olap_cube* c, int enable);
 int olap_cube_profile_read(olap_cube* c, double* reduce_ms, int64_t* launches, int64_t* bytes);
 
+/* Kernels this cube has launched so far (plan, order, reduce; fill and fact build
+ * included) and whether the L2-aware item order is active (cubes > 64 MiB). */
+int olap_cube_stats(const olap_cube* c, int64_t* kernel_launches, int* l2_order);
+
+/* Number of finalize kernels launched by this process (not bound to a cube). */
+int64_t olap_finalize_launches(void);
+
 /* ---------------------------------------------------------------- dictionaries */
 
 /* Build one text column's dictionary from n keys (key i = bytes[offsets[i],

@@ -69,6 +69,8 @@ EXPORTS = {
     "olap_text_ranges_device": (_int, [_p, _int, _i64p, _i64, _p, _p, _p, _p, _p, _i64, _p, _p, _p]),
     "olap_cube_add_facts_device": (_int, [_p, _i64, _p, _p, _p]),
     "olap_dict_destroy": (_int, [_p]),
+    "olap_cube_stats": (_int, [_p, _i64p, ctypes.POINTER(_int)]),
+    "olap_finalize_launches": (_i64, []),
     "olap_last_error": (ctypes.c_char_p, []),
     "olap_version": (ctypes.c_char_p, []),
 }
@@ -231,6 +233,12 @@ class Cube:
         _check(lib.olap_cube_profile_read(self._h, ctypes.byref(ms), ctypes.byref(n), ctypes.byref(b)),
                "olap_cube_profile_read")
         return ms.value, n.value, b.value
+
+    def stats(self):
+        """(kernel launches so far, L2-aware order active)"""
+        n, o = ctypes.c_int64(), ctypes.c_int()
+        _check(lib.olap_cube_stats(self._h, ctypes.byref(n), ctypes.byref(o)), "olap_cube_stats")
+        return n.value, bool(o.value)
 
     def close(self):
         if getattr(self, "_h", None):

@@ -13,6 +13,7 @@
 #include <climits>
 #include <cstdlib>
 #include <cstring>
+#include <atomic>
 #include <mutex>
 #include <new>
 #include <vector>
@@ -975,10 +976,13 @@ struct olap_cube {
     std::vector<cudaEvent_t> ev;
     size_t ev_used = 0;
     int64_t launches = 0;
+    int64_t kernel_launches = 0;  // every kernel this cube launched (all entry points)
     unsigned long long bytes_base = 0;
 };
 
 namespace {
+
+std::atomic<int64_t> g_finalize_launches{0};  // finalize is not bound to a cube (multi-GPU path)
 
 struct DeviceGuard {
     int prev = -1;
@@ -1099,7 +1103,9 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
                                             c->items_cap, c->d_counter + 2, c->d_counter + 1);
     OLAP_CUDA_TRY(cudaGetLastError());
     const int32_t* order = nullptr;
+    c->kernel_launches += 3;  // desc, scan, reduce
     if (c->order_shift >= 0) {
+        c->kernel_launches += 3;
         OLAP_CUDA_TRY(cudaMemsetAsync(c->d_bcount, 0, sizeof(unsigned int) * kMaxBuckets, st));
         bucket_kernel<<<c->num_sms * 8, 256, 0, st>>>(nq, c->d_desc, c->d_item_start, c->order_shift, c->d_bucket,
                                                        c->d_bcount);
@@ -1145,6 +1151,7 @@ int launch_finalize(int nd, const int64_t* ext, int dtype, int64_t nq, const ola
     std::memset(&e, 0, sizeof(e));
     for (int k = 0; k < nd; ++k) e.n[k] = ext[k];
     const int grid = (int)std::min<int64_t>((nq + 255) / 256, 4096);
+    g_finalize_launches.fetch_add(1);
     finalize_kernel<<<grid, 256, 0, st>>>(nd, e, dtype, nq, d_ranges, d_ops, d_psum, d_pext, d_results);
     OLAP_CUDA_TRY(cudaGetLastError());
     return OLAP_OK;
@@ -1316,6 +1323,7 @@ int olap_cube_fill(olap_cube* c, int generator, uint64_t seed, const double* par
     if (params)
         for (int k = 0; k <= c->nd; ++k) fp.c[k] = params[k];
     const int grid = c->num_sms * 8;
+    ++c->kernel_launches;
     if (c->dtype == OLAP_INT32)
         fill_kernel<int32_t><<<grid, 256, 0, c->stream>>>(static_cast<int32_t*>(c->d_cells), make_geo(c), c->row_cells,
                                                           generator, seed, fp);
@@ -1339,6 +1347,7 @@ int olap_cube_add_facts_device(olap_cube* c, int64_t nrows, const int32_t* d_ids
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     OLAP_CUDA_TRY(cudaStreamWaitEvent(st, c->ws_done, 0));
     const int grid = (int)std::min<int64_t>((nrows + 255) / 256, (int64_t)c->num_sms * 16);
+    ++c->kernel_launches;
     if (c->dtype == OLAP_INT32)
         add_facts_kernel<int32_t><<<grid, 256, 0, st>>>(static_cast<int32_t*>(c->d_cells), make_geo(c), nrows, d_ids,
                                                         static_cast<const int32_t*>(d_values));
@@ -1497,6 +1506,16 @@ int olap_shard_local_rows(int64_t n0, const olap_shard* s, int64_t lo, int64_t h
     }
     return OLAP_OK;
 }
+
+int olap_cube_stats(const olap_cube* c, int64_t* kernel_launches, int* l2_order) {
+    clear_error();
+    if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    if (kernel_launches) *kernel_launches = c->kernel_launches;
+    if (l2_order) *l2_order = c->order_shift >= 0 ? 1 : 0;
+    return OLAP_OK;
+}
+
+int64_t olap_finalize_launches(void) { return g_finalize_launches.load(); }
 
 int olap_cube_profile(olap_cube* c, int enable) {
     clear_error();
