@@ -10,6 +10,7 @@ Functions (all cite the passage they follow in oracle.cpp):
   query()      Eq. 1 / Eq. 3 / PAPER.md:25 — odometer sub-cube aggregation.
   Dict         PAPER.md:252-256 — one std::map dictionary per text column.
   factscan()   PAPER.md:206-208 — filtered aggregation over a fact table.
+  tablescan()  Eq. 11-12, PAPER.md:206-216 — the paper's GPU query Q_D over a column store.
   fill()       the counter-based cell generator (independent re-implementation).
 
 Parity of every function is pinned in tests/test_oracle_*.py against brute
@@ -82,6 +83,10 @@ def lib():
         L.oracle_factscan.argtypes = [ctypes.c_int64, ctypes.c_int, ctypes.c_void_p, ctypes.c_int,
                                       ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p,
                                       ctypes.c_void_p, ctypes.c_void_p]
+        L.oracle_tablescan.restype = ctypes.c_int
+        L.oracle_tablescan.argtypes = [ctypes.c_int64, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64,
+                                       ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                       ctypes.c_void_p, ctypes.c_int]
         _lib = L
     return _lib
 
@@ -217,3 +222,34 @@ def factscan(dims, data, ranges):
     if data.dtype == np.float32:
         s = s.view(np.float64)
     return s, c
+
+
+COND_DTYPE = np.dtype([("col", "<i4"), ("pad", "<i4"), ("lo", "<i8"), ("hi", "<i8")])
+
+
+def tablescan(columns, queries, nthreads: int = 1):
+    """Q_D (Eq. 11) over a column-store fact table.
+
+    columns: list of 1-D int32 / float32 arrays (equal length).  queries: list of
+    (conds, data_col, op) with conds a list of (col, lo, hi).  Returns RESULT_DTYPE array."""
+    cols = [np.ascontiguousarray(c) for c in columns]
+    nrows = len(cols[0])
+    ptrs = (ctypes.c_void_p * len(cols))(*[c.ctypes.data for c in cols])
+    dts = np.array([_dtype_code(c.dtype) for c in cols], dtype=np.int32)
+    off = np.zeros(len(queries) + 1, dtype=np.int64)
+    flat = []
+    for i, (conds, _dc, _op) in enumerate(queries):
+        flat += list(conds)
+        off[i + 1] = len(flat)
+    ca = np.zeros(max(len(flat), 1), dtype=COND_DTYPE)
+    for k, (c, lo, hi) in enumerate(flat):
+        ca[k] = (c, 0, lo, hi)
+    dcol = np.array([q[1] for q in queries], dtype=np.int32)
+    ops = np.array([q[2] for q in queries], dtype=np.int32)
+    out = np.zeros(len(queries), dtype=RESULT_DTYPE)
+    rc = lib().oracle_tablescan(nrows, len(cols), ctypes.cast(ptrs, ctypes.c_void_p), dts.ctypes.data, len(queries),
+                                off.ctypes.data, ca.ctypes.data, dcol.ctypes.data, ops.ctypes.data, out.ctypes.data,
+                                nthreads)
+    if rc:
+        raise ValueError("oracle_tablescan: invalid arguments")
+    return out

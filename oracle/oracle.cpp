@@ -17,6 +17,9 @@
  *                       Plain odometer over the box in row-major order.  PAPER.md:109-112, Fig. 2 :151
  *   oracle_dict_*     — one text-to-integer dictionary per text column  PAPER.md:252-256 (§III-F)
  *                       as std::map<std::string,int32_t>; id = rank in byte order (reading R11).
+ *   oracle_tablescan  — the paper's GPU query Q_D over a column-store fact table
+ *                       (Eq. 11-12): conditions on dimension
+ *                       columns, aggregate of one data column, COUNT = matching rows.
  *   oracle_factscan   — filtered aggregation over a fact table of translated
  *                       (integer) dimension columns and one data column  PAPER.md:206-208 (§III-E)
  *                       used as an independent path to the cube answer for SUM.
@@ -334,6 +337,86 @@ int oracle_factscan(int64_t nrows, int nd, const int32_t* dims, int dtype, const
         if (dtype == ORC_INT32) out_sum[q] = (int64_t)su;
         else std::memcpy(&out_sum[q], &sf, sizeof(double));
         out_count[q] = cnt;
+    }
+    return 0;
+}
+
+/*
+ * Fact-table query Q_D (Eq. 11; §III-E): the table
+ * is a set of columns ("all columns of the table one after another"), dimension columns
+ * hold integer member ids (one column per dimension x level), data columns hold the
+ * measures.  Query q has conditions conds[cond_off[q] .. cond_off[q+1]) — each a column
+ * and an inclusive range [f, t] on its ids — a data column and an aggregate op.  A row
+ * matches when it satisfies every condition; the answer aggregates the data column over
+ * matching rows.  COUNT counts matching rows (facts).  AVG = SUM / COUNT.  No matching
+ * row: flags = 1 (EMPTY), i = d = 0.  Accumulation as oracle_query (readings R7/R8).
+ * cols[c] points to nrows 4-byte values; dtypes[c] is ORC_INT32 or ORC_FLOAT32.
+ */
+struct TCond { int32_t col; int32_t pad; int64_t lo, hi; };
+
+int oracle_tablescan(int64_t nrows, int ncols, const void* const* cols, const int32_t* dtypes, int64_t nq,
+                     const int64_t* cond_off, const void* conds_v, const int32_t* data_cols, const int32_t* ops,
+                     void* results, int nthreads) {
+    const TCond* conds = static_cast<const TCond*>(conds_v);
+    Result* out = static_cast<Result*>(results);
+    for (int64_t q = 0; q < nq; ++q) {
+        if (data_cols[q] < 0 || data_cols[q] >= ncols || ops[q] < ORC_SUM || ops[q] > ORC_AVG) return -1;
+        for (int64_t k = cond_off[q]; k < cond_off[q + 1]; ++k)
+            if (conds[k].col < 0 || conds[k].col >= ncols || dtypes[conds[k].col] != ORC_INT32) return -1;
+    }
+#ifdef _OPENMP
+#pragma omp parallel for schedule(dynamic, 1) num_threads(nthreads > 1 ? nthreads : 1)
+#endif
+    for (int64_t q = 0; q < nq; ++q) {
+        const int dc = data_cols[q];
+        const bool fl = dtypes[dc] == ORC_FLOAT32;
+        uint64_t su = 0;
+        double sf = 0.0;
+        int64_t cnt = 0;
+        int32_t mn_i = INT32_MAX, mx_i = INT32_MIN;
+        float mn_f = 0.f, mx_f = 0.f;
+        for (int64_t r = 0; r < nrows; ++r) {
+            bool hit = true;
+            for (int64_t k = cond_off[q]; k < cond_off[q + 1] && hit; ++k) {
+                const int64_t v = static_cast<const int32_t*>(cols[conds[k].col])[r];
+                hit = conds[k].lo <= v && v <= conds[k].hi;
+            }
+            if (!hit) continue;
+            if (fl) {
+                const float v = static_cast<const float*>(cols[dc])[r];
+                sf += (double)v;
+                if (cnt == 0) { mn_f = v; mx_f = v; }
+                if (v < mn_f) mn_f = v;
+                if (mx_f < v) mx_f = v;
+            } else {
+                const int32_t v = static_cast<const int32_t*>(cols[dc])[r];
+                su += (uint64_t)(int64_t)v;
+                if (v < mn_i) mn_i = v;
+                if (mx_i < v) mx_i = v;
+            }
+            ++cnt;
+        }
+        Result res;
+        std::memset(&res, 0, sizeof(res));
+        if (cnt == 0) {
+            res.flags = 1;
+        } else {
+            const int op = ops[q];
+            if (op == ORC_COUNT) res.i = cnt;
+            else if (!fl) {
+                const int64_t sum = (int64_t)su;
+                if (op == ORC_SUM) res.i = sum;
+                else if (op == ORC_MIN) res.i = mn_i;
+                else if (op == ORC_MAX) res.i = mx_i;
+                else res.d = (double)sum / (double)cnt;
+            } else {
+                if (op == ORC_SUM) res.d = sf;
+                else if (op == ORC_MIN) res.d = (double)mn_f;
+                else if (op == ORC_MAX) res.d = (double)mx_f;
+                else res.d = sf / (double)cnt;
+            }
+        }
+        out[q] = res;
     }
     return 0;
 }
