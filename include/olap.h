@@ -242,6 +242,45 @@ int olap_dict_lookup(const olap_dict* d, int32_t id, const char** bytes, int64_t
 
 int olap_dict_destroy(olap_dict* d);
 
+/* ---------------------------------------------------------------- fact tables */
+
+/* The paper's GPU data structure (§III-E): a fact
+ * table of nrows rows held in GPU memory as one 1-D array of columns "one after
+ * another".  Dimension columns hold int32 member ids (one column per dimension x
+ * level, e.g. translated text); data columns hold int32 or float32
+ * measures.  At most 16 columns. */
+typedef struct olap_table olap_table;
+
+/* One condition C_L(f, t, l_K) of a query Q_D (Eq. 11): column `col`
+ * (an int32 dimension column) and an inclusive id range [lo, hi]; lo > hi matches
+ * nothing. */
+typedef struct { int32_t col; int32_t _pad; int64_t lo, hi; } olap_cond;
+
+int olap_table_create(int64_t nrows, int ncols, const int32_t* col_dtypes, int device, olap_table** out);
+
+/* Copy column `col` (nrows 4-byte values, HOST buffer). */
+int olap_table_load_column(olap_table* t, int col, const void* values);
+
+/* Device pointer of column `col` (nrows 4-byte values), e.g. to fill it on the device. */
+int olap_table_column_device(olap_table* t, int col, void** d_ptr);
+
+/* Answer nq queries Q_D on HOST buffers.  Query q has conditions
+ * conds[cond_offsets[q] .. cond_offsets[q+1]) (at most 16; cond_offsets[0] = 0), data
+ * column data_cols[q] and op ops[q].  A row matches when it satisfies every condition
+ * (PAPER.md:208); the result aggregates the data column over matching rows: COUNT =
+ * matching rows (facts), SUM (int64 wraparound / fp64), MIN, MAX, AVG = SUM / COUNT.
+ * No matching row: OLAP_RESULT_EMPTY.  One shared scan answers the whole batch. */
+int olap_table_query_batch(olap_table* t, int64_t nq, const int64_t* cond_offsets, const olap_cond* conds,
+                           const int32_t* data_cols, const int32_t* ops, olap_result* results);
+
+/* Same on DEVICE buffers, asynchronous on `stream`; malformed queries are flagged
+ * OLAP_RESULT_INVALID. */
+int olap_table_query_batch_device(olap_table* t, int64_t nq, const int64_t* d_cond_offsets,
+                                  const olap_cond* d_conds, const int32_t* d_data_cols, const int32_t* d_ops,
+                                  olap_result* d_results, void* stream);
+
+int olap_table_destroy(olap_table* t);
+
 /* ---------------------------------------------------------------- misc */
 
 const char* olap_last_error(void); /* thread-local; valid until the next olap_* call */

@@ -21,7 +21,7 @@ __all__ = ["Cube", "Dict", "OlapError", "translate", "shard_local_rows", "combin
            "finalize_device", "translate_device", "RESULT_DTYPE", "lib", "LIB_PATH",
            "INT32", "FLOAT32", "SUM", "COUNT", "MIN", "MAX", "AVG", "GEN_UNIFORM", "GEN_AFFINE",
            "RESULT_EMPTY", "RESULT_INVALID", "EXPORTS", "text_ranges", "text_ranges_device", "pack_text_conditions",
-           "COND_ALL", "COND_EQ", "COND_RANGE", "COND_IDS"]
+           "COND_ALL", "COND_EQ", "COND_RANGE", "COND_IDS", "Table", "COND_DTYPE"]
 
 LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libolap_b200.so")
 if os.environ.get("OLAP_LIB"):          # development only: A/B a differently-tuned build of the same sources
@@ -70,6 +70,12 @@ EXPORTS = {
     "olap_cube_add_facts_device": (_int, [_p, _i64, _p, _p, _p]),
     "olap_dict_destroy": (_int, [_p]),
     "olap_cube_stats": (_int, [_p, _i64p, ctypes.POINTER(_int)]),
+    "olap_table_create": (_int, [_i64, _int, _p, _int, ctypes.POINTER(_p)]),
+    "olap_table_load_column": (_int, [_p, _int, _p]),
+    "olap_table_column_device": (_int, [_p, _int, ctypes.POINTER(_p)]),
+    "olap_table_query_batch": (_int, [_p, _i64, _p, _p, _p, _p, _p]),
+    "olap_table_query_batch_device": (_int, [_p, _i64, _p, _p, _p, _p, _p, _p]),
+    "olap_table_destroy": (_int, [_p]),
     "olap_finalize_launches": (_i64, []),
     "olap_last_error": (ctypes.c_char_p, []),
     "olap_version": (ctypes.c_char_p, []),
@@ -410,3 +416,70 @@ def text_ranges_device(dicts, extents, nq: int, d_kinds, d_first_key, d_ranges_i
                                        _ptr(d_first_key), _ptr(d_ranges_in), _ptr(d_bytes), _ptr(d_offsets), nkeys,
                                        _ptr(d_ranges_out), _ptr(d_n_missing), _stream(stream)),
            "olap_text_ranges_device")
+
+
+# olap_cond: {int32 col; int32 _pad; int64 lo, hi}
+COND_DTYPE = np.dtype([("col", "<i4"), ("pad", "<i4"), ("lo", "<i8"), ("hi", "<i8")])
+
+
+def pack_table_queries(queries):
+    """queries: list of (conds, data_col, op), conds a list of (col, lo, hi) ->
+    (cond_offsets int64[nq+1], conds COND_DTYPE[], data_cols int32[nq], ops int32[nq])."""
+    off = np.zeros(len(queries) + 1, dtype=np.int64)
+    flat = []
+    for i, (conds, _dc, _op) in enumerate(queries):
+        flat += list(conds)
+        off[i + 1] = len(flat)
+    ca = np.zeros(max(len(flat), 1), dtype=COND_DTYPE)
+    for k, (c, lo, hi) in enumerate(flat):
+        ca[k] = (c, 0, lo, hi)
+    dcol = np.array([q[1] for q in queries], dtype=np.int32)
+    ops = np.array([q[2] for q in queries], dtype=np.int32)
+    return off, ca, dcol, ops
+
+
+class Table:
+    """A column-store fact table in GPU memory (the paper's GPU data structure)."""
+
+    def __init__(self, nrows: int, dtypes, device: int = 0):
+        self.nrows = int(nrows)
+        self.dtypes = [_dtype_code(d) for d in dtypes]
+        dt = np.array(self.dtypes, dtype=np.int32)
+        h = ctypes.c_void_p()
+        _check(lib.olap_table_create(self.nrows, len(dt), dt.ctypes.data, device, ctypes.byref(h)),
+               "olap_table_create")
+        self._h = h
+        self.device = device
+
+    def load_column(self, col: int, values: np.ndarray):
+        v = np.ascontiguousarray(values, dtype=np.int32 if self.dtypes[col] == INT32 else np.float32)
+        if v.size != self.nrows:
+            raise ValueError("column length != nrows")
+        _check(lib.olap_table_load_column(self._h, col, v.ctypes.data), "olap_table_load_column")
+
+    def column_device(self, col: int) -> int:
+        p = ctypes.c_void_p()
+        _check(lib.olap_table_column_device(self._h, col, ctypes.byref(p)), "olap_table_column_device")
+        return p.value
+
+    def query(self, queries) -> np.ndarray:
+        off, ca, dcol, ops = pack_table_queries(queries)
+        out = np.zeros(len(queries), dtype=RESULT_DTYPE)
+        _check(lib.olap_table_query_batch(self._h, len(queries), off.ctypes.data, ca.ctypes.data, dcol.ctypes.data,
+                                          ops.ctypes.data, out.ctypes.data), "olap_table_query_batch")
+        return out
+
+    def query_device(self, nq: int, d_off, d_conds, d_dcol, d_ops, d_results, stream=None):
+        _check(lib.olap_table_query_batch_device(self._h, nq, _ptr(d_off), _ptr(d_conds), _ptr(d_dcol), _ptr(d_ops),
+                                                 _ptr(d_results), _stream(stream)), "olap_table_query_batch_device")
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib.olap_table_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

@@ -1,0 +1,491 @@
+// table.cu — the paper's own GPU path: queries Q_D (Eq. 11,
+// PAPER.md:210-216) over a column-store fact table held in GPU memory ("a 1D array
+// memory structure ... placing all columns of the table one after another",
+// PAPER.md:206).  A query is a set of conditions C_L(f, t, l_K) — one column (dimension
+// L at level K) and an inclusive id range — plus a data column and an aggregate op; a
+// row contributes when it satisfies every condition.
+//
+// The paper ran one query per SM partition and read each referenced column whole per
+// query (Eq. 12: bytes = rows x C_QD x 4).  B200 design: a SHARED scan — one persistent
+// launch per batch streams every column once, tile by tile, into shared memory, and
+// every warp evaluates its share of the batch's queries on the staged tile (each
+// condition one unsigned range compare).  Per-(block, query) partials are folded in
+// fixed block order by a second kernel, so results are deterministic.
+#include <algorithm>
+#include <climits>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <vector>
+
+#include "common.cuh"
+
+namespace olap {
+
+constexpr int kMaxTableCols = 16;
+constexpr int kMaxConds = 16;
+constexpr int kTileRows = 1024;
+constexpr int kScanWarps = 8;
+constexpr int kScanThreads = kScanWarps * 32;
+
+// Condition in the kernel's form: row value v passes iff (uint32)(v - lo) <= span.
+struct TCond {
+    int32_t col;
+    uint32_t lo;
+    uint32_t span;
+};
+
+struct TQuery {
+    int32_t ncond;
+    int32_t data_col;
+    int32_t op;
+    int32_t flags;  // OLAP_RESULT_INVALID / impossible (some condition empty)
+    TCond c[kMaxConds];
+};
+
+struct TPartial {  // per (block, query)
+    long long sum;     // int64 wraparound sum or double bits
+    int64_t count;     // matching rows
+    int32_t code_max;  // order-preserving code of MAX (INT_MIN = none)
+    int32_t code_min;  // ~code of MIN           (INT_MIN = none)
+};
+
+struct TableCols {
+    const uint32_t* col[kMaxTableCols];
+    int32_t dtype[kMaxTableCols];
+};
+
+__device__ __forceinline__ int32_t tf32_code(float f) {
+    const int32_t b = __float_as_int(f);
+    return b ^ ((b >> 31) & 0x7fffffff);
+}
+__device__ __forceinline__ float tf32_decode(int32_t c) { return __int_as_float(c ^ ((c >> 31) & 0x7fffffff)); }
+
+// conditions -> TQuery (one thread per query)
+__global__ void table_prep_kernel(int64_t nq, int ncols, TableCols tc, const int64_t* __restrict__ off,
+                                  const olap_cond* __restrict__ conds, const int32_t* __restrict__ data_cols,
+                                  const int32_t* __restrict__ ops, TQuery* __restrict__ qs) {
+    const int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (q >= nq) return;
+    TQuery t;
+    t.flags = 0;
+    t.op = ops[q];
+    t.data_col = data_cols[q];
+    const int64_t a = off[q], b = off[q + 1];
+    t.ncond = (int32_t)(b - a);
+    if (t.op < OLAP_SUM || t.op > OLAP_AVG || t.data_col < 0 || t.data_col >= ncols || b < a || b - a > kMaxConds)
+        t.flags = OLAP_RESULT_INVALID;
+    bool impossible = false;
+    for (int64_t k = a; k < b && !t.flags; ++k) {
+        const olap_cond c = conds[k];
+        if (c.col < 0 || c.col >= ncols || tc.dtype[c.col] != OLAP_INT32) {
+            t.flags = OLAP_RESULT_INVALID;
+            break;
+        }
+        const int64_t lo = c.lo < INT_MIN ? (int64_t)INT_MIN : c.lo;
+        const int64_t hi = c.hi > INT_MAX ? (int64_t)INT_MAX : c.hi;
+        TCond& d = t.c[k - a];
+        d.col = c.col;
+        if (lo > hi) {
+            impossible = true;
+            d.lo = 0;
+            d.span = 0;
+        } else {
+            d.lo = (uint32_t)(int32_t)lo;
+            d.span = (uint32_t)(hi - lo);
+        }
+    }
+    if (impossible && !t.flags) t.ncond = -1;  // no row can match
+    qs[q] = t;
+}
+
+// One query on one staged tile.  Lane l owns rows l, l+32, ..., l+992: every condition
+// is loaded once per tile (uniform) and evaluated into a 32-bit pass mask (bit i = row
+// l + 32 i); COUNT is a popcount, and only matching rows touch the data column.
+template <bool FLOAT_DATA>
+__device__ __forceinline__ void scan_query_tile(const uint32_t* __restrict__ smem, int rows, const TQuery& tq, int lane,
+                                                long long& s, int64_t& cnt, int32_t& cmx, int32_t& cmn) {
+    static_assert(kTileRows == 1024, "one 32-bit pass mask per lane");
+    uint32_t pass = rows >= kTileRows ? 0xFFFFFFFFu : 0u;
+    if (rows < kTileRows)
+        for (int i = 0; i < 32; ++i)
+            if (lane + 32 * i < rows) pass |= 1u << i;
+    const int nc = tq.ncond;
+    for (int k = 0; k < nc && pass; ++k) {
+        const TCond c = tq.c[k];
+        const uint32_t* col = smem + c.col * kTileRows + lane;
+        uint32_t m = 0;
+#pragma unroll
+        for (int i = 0; i < 32; ++i) m |= (uint32_t)((col[32 * i] - c.lo) <= c.span) << i;
+        pass &= m;
+    }
+    int32_t n = __popc(pass);
+    const bool need_data = tq.op != OLAP_COUNT;
+    const uint32_t* data = smem + tq.data_col * kTileRows + lane;
+    unsigned long long si = 0ull;
+    double sf = 0.0;
+    float fmn = __int_as_float(0x7f800000), fmx = __int_as_float(0xff800000);
+    int32_t imn = INT_MAX, imx = INT_MIN;
+    uint32_t bits_left = need_data ? pass : 0u;
+    while (bits_left) {
+        const int i = __ffs(bits_left) - 1;
+        bits_left &= bits_left - 1;
+        const uint32_t bits = data[32 * i];
+        if (FLOAT_DATA) {
+            const float v = __uint_as_float(bits);
+            sf += (double)v;
+            fmn = fminf(fmn, v);
+            fmx = fmaxf(fmx, v);
+        } else {
+            const int32_t v = (int32_t)bits;
+            si += (unsigned long long)(long long)v;
+            imn = min(imn, v);
+            imx = max(imx, v);
+        }
+    }
+    // warp reduction in fixed order
+    long long sb = FLOAT_DATA ? __double_as_longlong(sf) : (long long)si;
+    int32_t mx = FLOAT_DATA ? tf32_code(fmx) : imx, mn = ~(FLOAT_DATA ? tf32_code(fmn) : imn);
+    if (n == 0) mx = mn = INT_MIN;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        const long long so = __shfl_xor_sync(0xffffffffu, sb, o);
+        sb = FLOAT_DATA ? __double_as_longlong(__longlong_as_double(sb) + __longlong_as_double(so))
+                        : (long long)((unsigned long long)sb + (unsigned long long)so);
+        n += __shfl_xor_sync(0xffffffffu, n, o);
+    }
+    mx = __reduce_max_sync(0xffffffffu, mx);
+    mn = __reduce_max_sync(0xffffffffu, mn);
+    s = FLOAT_DATA ? __double_as_longlong(__longlong_as_double(s) + __longlong_as_double(sb))
+                   : (long long)((unsigned long long)s + (unsigned long long)sb);
+    cnt += n;
+    cmx = max(cmx, mx);
+    cmn = max(cmn, mn);
+}
+
+// The shared scan.  Block b stages tiles b, b+G, ... (all columns) into shared memory;
+// warp w evaluates queries w, w+8, ... on every staged tile.
+__global__ void __launch_bounds__(kScanThreads) table_scan_kernel(TableCols tc, int ncols, int64_t nrows, int64_t nq,
+                                                                  const TQuery* __restrict__ qs,
+                                                                  TPartial* __restrict__ part) {
+    extern __shared__ uint32_t smem[];  // ncols x kTileRows
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t ntiles = (nrows + kTileRows - 1) / kTileRows;
+    TPartial* mine = part + (int64_t)blockIdx.x * nq;
+    for (int64_t q = threadIdx.x; q < nq; q += kScanThreads) {
+        TPartial p;
+        p.sum = 0;
+        p.count = 0;
+        p.code_max = INT_MIN;
+        p.code_min = INT_MIN;
+        mine[q] = p;
+    }
+    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        const int64_t r0 = t * kTileRows;
+        const int rows = (int)min((int64_t)kTileRows, nrows - r0);
+        __syncthreads();  // previous tile fully consumed
+        for (int c = 0; c < ncols; ++c) {
+            const uint32_t* src = tc.col[c] + r0;
+            uint32_t* dst = smem + c * kTileRows;
+            for (int r = threadIdx.x; r < rows; r += kScanThreads) dst[r] = __ldg(src + r);
+        }
+        __syncthreads();
+        for (int64_t q = w; q < nq; q += kScanWarps) {
+            const TQuery& tq = qs[q];
+            if (tq.flags || tq.ncond < 0) continue;
+            TPartial p = mine[q];  // warp w owns these partials: no race
+            long long s = p.sum;
+            int64_t cnt = p.count;
+            int32_t cmx = p.code_max, cmn = p.code_min;
+            if (tc.dtype[tq.data_col] == OLAP_FLOAT32) scan_query_tile<true>(smem, rows, tq, lane, s, cnt, cmx, cmn);
+            else scan_query_tile<false>(smem, rows, tq, lane, s, cnt, cmx, cmn);
+            if (lane == 0) {
+                p.sum = s;
+                p.count = cnt;
+                p.code_max = cmx;
+                p.code_min = cmn;
+                mine[q] = p;
+            }
+        }
+    }
+}
+
+// fold per-block partials in block order -> results
+__global__ void table_final_kernel(TableCols tc, int64_t nq, int nblocks, const TQuery* __restrict__ qs,
+                                   const TPartial* __restrict__ part, olap_result* __restrict__ out) {
+    const int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (q >= nq) return;
+    const TQuery& tq = qs[q];
+    olap_result r;
+    r.i = 0;
+    r.d = 0.0;
+    r.flags = 0;
+    r._pad = 0;
+    if (tq.flags) {
+        r.flags = OLAP_RESULT_INVALID;
+        out[q] = r;
+        return;
+    }
+    const bool fl = tc.dtype[tq.data_col] == OLAP_FLOAT32;
+    long long s = 0;
+    int64_t cnt = 0;
+    int32_t cmx = INT_MIN, cmn = INT_MIN;
+    if (tq.ncond >= 0) {
+        for (int b = 0; b < nblocks; ++b) {
+            const TPartial p = part[(int64_t)b * nq + q];
+            s = fl ? __double_as_longlong(__longlong_as_double(s) + __longlong_as_double(p.sum))
+                   : (long long)((unsigned long long)s + (unsigned long long)p.sum);
+            cnt += p.count;
+            cmx = max(cmx, p.code_max);
+            cmn = max(cmn, p.code_min);
+        }
+    }
+    if (cnt == 0) {
+        r.flags = OLAP_RESULT_EMPTY;
+    } else if (tq.op == OLAP_COUNT) {
+        r.i = cnt;
+    } else if (!fl) {
+        if (tq.op == OLAP_SUM) r.i = s;
+        else if (tq.op == OLAP_MIN) r.i = ~cmn;
+        else if (tq.op == OLAP_MAX) r.i = cmx;
+        else r.d = (double)s / (double)cnt;
+    } else {
+        const double ds = __longlong_as_double(s);
+        if (tq.op == OLAP_SUM) r.d = ds;
+        else if (tq.op == OLAP_MIN) r.d = (double)tf32_decode(~cmn);
+        else if (tq.op == OLAP_MAX) r.d = (double)tf32_decode(cmx);
+        else r.d = ds / (double)cnt;
+    }
+    out[q] = r;
+}
+
+}  // namespace olap
+
+using namespace olap;
+
+struct olap_table {
+    int device = 0;
+    int64_t nrows = 0;
+    int ncols = 0;
+    int32_t dtype[kMaxTableCols] = {};
+    void* d_data = nullptr;      // all columns one after another, 256-B aligned
+    int64_t col_stride = 0;      // cells between column starts
+    std::mutex mu;
+    cudaStream_t stream = nullptr;
+    int num_sms = 0, blocks = 0;
+    int64_t nq_cap = 0;
+    TQuery* d_qs = nullptr;
+    TPartial* d_part = nullptr;
+    olap_cond* d_conds = nullptr;
+    int64_t conds_cap = 0;
+    int64_t* d_off = nullptr;
+    int32_t* d_dcol = nullptr;
+    int32_t* d_ops = nullptr;
+    olap_result* d_res = nullptr;
+    int64_t launches = 0;
+};
+
+namespace {
+
+struct TDevGuard {
+    int prev = -1;
+    explicit TDevGuard(int dev) {
+        if (cudaGetDevice(&prev) == cudaSuccess) cudaSetDevice(dev);
+    }
+    ~TDevGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
+TableCols cols_of(const olap_table* t) {
+    TableCols tc;
+    std::memset(&tc, 0, sizeof(tc));
+    for (int c = 0; c < t->ncols; ++c) {
+        tc.col[c] = static_cast<const uint32_t*>(t->d_data) + c * t->col_stride;
+        tc.dtype[c] = t->dtype[c];
+    }
+    return tc;
+}
+
+void free_tws(olap_table* t) {
+    cudaFree(t->d_qs);
+    cudaFree(t->d_part);
+    cudaFree(t->d_off);
+    cudaFree(t->d_dcol);
+    cudaFree(t->d_ops);
+    cudaFree(t->d_res);
+    t->d_qs = nullptr;
+    t->d_part = nullptr;
+    t->d_off = nullptr;
+    t->d_dcol = nullptr;
+    t->d_ops = nullptr;
+    t->d_res = nullptr;
+    t->nq_cap = 0;
+}
+
+int ensure_tws(olap_table* t, int64_t nq, int64_t nconds) {
+    if (nq > t->nq_cap) {
+        OLAP_CUDA_TRY(cudaStreamSynchronize(t->stream));
+        free_tws(t);
+        const int64_t cap = std::max<int64_t>(nq, 256);
+        OLAP_CUDA_TRY(cudaMalloc(&t->d_qs, sizeof(TQuery) * cap));
+        OLAP_CUDA_TRY(cudaMalloc(&t->d_part, sizeof(TPartial) * cap * t->blocks));
+        OLAP_CUDA_TRY(cudaMalloc(&t->d_off, sizeof(int64_t) * (cap + 1)));
+        OLAP_CUDA_TRY(cudaMalloc(&t->d_dcol, sizeof(int32_t) * cap));
+        OLAP_CUDA_TRY(cudaMalloc(&t->d_ops, sizeof(int32_t) * cap));
+        OLAP_CUDA_TRY(cudaMalloc(&t->d_res, sizeof(olap_result) * cap));
+        t->nq_cap = cap;
+    }
+    if (nconds > t->conds_cap) {
+        OLAP_CUDA_TRY(cudaStreamSynchronize(t->stream));
+        cudaFree(t->d_conds);
+        t->d_conds = nullptr;
+        const int64_t cap = std::max<int64_t>(nconds, 1024);
+        OLAP_CUDA_TRY(cudaMalloc(&t->d_conds, sizeof(olap_cond) * cap));
+        t->conds_cap = cap;
+    }
+    return OLAP_OK;
+}
+
+int launch_scan(olap_table* t, int64_t nq, const int64_t* d_off, const olap_cond* d_conds, const int32_t* d_dcol,
+                const int32_t* d_ops, olap_result* d_res, cudaStream_t st) {
+    const TableCols tc = cols_of(t);
+    table_prep_kernel<<<(int)((nq + 255) / 256), 256, 0, st>>>(nq, t->ncols, tc, d_off, d_conds, d_dcol, d_ops, t->d_qs);
+    const size_t smem = sizeof(uint32_t) * kTileRows * t->ncols;
+    table_scan_kernel<<<t->blocks, kScanThreads, smem, st>>>(tc, t->ncols, t->nrows, nq, t->d_qs, t->d_part);
+    table_final_kernel<<<(int)((nq + 255) / 256), 256, 0, st>>>(tc, nq, t->blocks, t->d_qs, t->d_part, d_res);
+    OLAP_CUDA_TRY(cudaGetLastError());
+    t->launches += 3;
+    return OLAP_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int olap_table_create(int64_t nrows, int ncols, const int32_t* dtypes, int device, olap_table** out) {
+    clear_error();
+    if (!out || !dtypes) return set_error(OLAP_E_INVALID, "olap_table_create: NULL argument");
+    if (nrows < 1) return set_error(OLAP_E_INVALID, "nrows < 1");
+    if (ncols < 1 || ncols > kMaxTableCols) return set_error(OLAP_E_INVALID, "ncols %d not in [1,16]", ncols);
+    for (int c = 0; c < ncols; ++c)
+        if (dtypes[c] != OLAP_INT32 && dtypes[c] != OLAP_FLOAT32)
+            return set_error(OLAP_E_INVALID, "column %d: bad dtype %d", c, dtypes[c]);
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
+        return set_error(OLAP_E_CUDA, "no CUDA device available (the library has no CPU fallback)");
+    if (device < 0 || device >= ndev) return set_error(OLAP_E_INVALID, "device %d not in [0,%d)", device, ndev);
+    TDevGuard g(device);
+    olap_table* t = new (std::nothrow) olap_table();
+    if (!t) return set_error(OLAP_E_NOMEM, "host allocation failed");
+    t->device = device;
+    t->nrows = nrows;
+    t->ncols = ncols;
+    for (int c = 0; c < ncols; ++c) t->dtype[c] = dtypes[c];
+    t->col_stride = (nrows + 63) & ~63ll;  // 256-B aligned column starts
+    cudaError_t e = cudaMalloc(&t->d_data, sizeof(uint32_t) * t->col_stride * ncols);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        delete t;
+        return set_error(e == cudaErrorMemoryAllocation ? OLAP_E_NOMEM : OLAP_E_CUDA, "table allocation: %s",
+                         cudaGetErrorString(e));
+    }
+    cudaStreamCreateWithFlags(&t->stream, cudaStreamNonBlocking);
+    cudaDeviceGetAttribute(&t->num_sms, cudaDevAttrMultiProcessorCount, device);
+    const size_t smem = sizeof(uint32_t) * kTileRows * ncols;
+    if (smem > 48 * 1024)
+        cudaFuncSetAttribute(table_scan_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int bps = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, table_scan_kernel, kScanThreads, smem);
+    t->blocks = t->num_sms * std::max(bps, 1);
+    *out = t;
+    return OLAP_OK;
+}
+
+int olap_table_load_column(olap_table* t, int col, const void* values) {
+    clear_error();
+    if (!t || !values) return set_error(OLAP_E_INVALID, "NULL argument");
+    if (col < 0 || col >= t->ncols) return set_error(OLAP_E_INVALID, "column %d not in [0,%d)", col, t->ncols);
+    std::lock_guard<std::mutex> lk(t->mu);
+    TDevGuard g(t->device);
+    OLAP_CUDA_TRY(cudaMemcpy(static_cast<uint32_t*>(t->d_data) + col * t->col_stride, values,
+                             sizeof(uint32_t) * t->nrows, cudaMemcpyHostToDevice));
+    return OLAP_OK;
+}
+
+int olap_table_column_device(olap_table* t, int col, void** d_ptr) {
+    clear_error();
+    if (!t || !d_ptr) return set_error(OLAP_E_INVALID, "NULL argument");
+    if (col < 0 || col >= t->ncols) return set_error(OLAP_E_INVALID, "column %d not in [0,%d)", col, t->ncols);
+    *d_ptr = static_cast<uint32_t*>(t->d_data) + col * t->col_stride;
+    return OLAP_OK;
+}
+
+int olap_table_query_batch_device(olap_table* t, int64_t nq, const int64_t* d_cond_offsets, const olap_cond* d_conds,
+                                  const int32_t* d_data_cols, const int32_t* d_ops, olap_result* d_results,
+                                  void* stream) {
+    clear_error();
+    if (!t) return set_error(OLAP_E_INVALID, "table handle is NULL");
+    if (nq < 0) return set_error(OLAP_E_INVALID, "nq < 0");
+    if (nq == 0) return OLAP_OK;
+    if (!d_cond_offsets || !d_data_cols || !d_ops || !d_results) return set_error(OLAP_E_INVALID, "NULL device buffer");
+    std::lock_guard<std::mutex> lk(t->mu);
+    TDevGuard g(t->device);
+    int rc = ensure_tws(t, nq, 0);
+    if (rc) return rc;
+    return launch_scan(t, nq, d_cond_offsets, d_conds, d_data_cols, d_ops, d_results, static_cast<cudaStream_t>(stream));
+}
+
+int olap_table_query_batch(olap_table* t, int64_t nq, const int64_t* cond_offsets, const olap_cond* conds,
+                           const int32_t* data_cols, const int32_t* ops, olap_result* results) {
+    clear_error();
+    if (!t) return set_error(OLAP_E_INVALID, "table handle is NULL");
+    if (nq < 0) return set_error(OLAP_E_INVALID, "nq < 0");
+    if (nq == 0) return OLAP_OK;
+    if (!cond_offsets || !data_cols || !ops || !results) return set_error(OLAP_E_INVALID, "NULL buffer");
+    if (cond_offsets[0] != 0) return set_error(OLAP_E_INVALID, "cond_offsets[0] must be 0");
+    for (int64_t q = 0; q < nq; ++q) {
+        const int64_t n = cond_offsets[q + 1] - cond_offsets[q];
+        if (n < 0 || n > kMaxConds)
+            return set_error(OLAP_E_INVALID, "query %lld: %lld conditions (max 16)", (long long)q, (long long)n);
+        if (ops[q] < OLAP_SUM || ops[q] > OLAP_AVG)
+            return set_error(OLAP_E_INVALID, "query %lld: unknown op %d", (long long)q, ops[q]);
+        if (data_cols[q] < 0 || data_cols[q] >= t->ncols)
+            return set_error(OLAP_E_INVALID, "query %lld: data column %d", (long long)q, data_cols[q]);
+        for (int64_t k = cond_offsets[q]; k < cond_offsets[q + 1]; ++k)
+            if (conds[k].col < 0 || conds[k].col >= t->ncols || t->dtype[conds[k].col] != OLAP_INT32)
+                return set_error(OLAP_E_INVALID, "query %lld: condition on column %d (must be an int32 column)",
+                                 (long long)q, conds[k].col);
+    }
+    const int64_t nconds = cond_offsets[nq];
+    std::lock_guard<std::mutex> lk(t->mu);
+    TDevGuard g(t->device);
+    int rc = ensure_tws(t, nq, nconds);
+    if (rc) return rc;
+    cudaStream_t st = t->stream;
+    OLAP_CUDA_TRY(cudaMemcpyAsync(t->d_off, cond_offsets, sizeof(int64_t) * (nq + 1), cudaMemcpyHostToDevice, st));
+    if (nconds)
+        OLAP_CUDA_TRY(cudaMemcpyAsync(t->d_conds, conds, sizeof(olap_cond) * nconds, cudaMemcpyHostToDevice, st));
+    OLAP_CUDA_TRY(cudaMemcpyAsync(t->d_dcol, data_cols, sizeof(int32_t) * nq, cudaMemcpyHostToDevice, st));
+    OLAP_CUDA_TRY(cudaMemcpyAsync(t->d_ops, ops, sizeof(int32_t) * nq, cudaMemcpyHostToDevice, st));
+    rc = launch_scan(t, nq, t->d_off, t->d_conds, t->d_dcol, t->d_ops, t->d_res, st);
+    if (rc) return rc;
+    OLAP_CUDA_TRY(cudaMemcpyAsync(results, t->d_res, sizeof(olap_result) * nq, cudaMemcpyDeviceToHost, st));
+    OLAP_CUDA_TRY(cudaStreamSynchronize(st));
+    return OLAP_OK;
+}
+
+int olap_table_destroy(olap_table* t) {
+    clear_error();
+    if (!t) return OLAP_OK;
+    TDevGuard g(t->device);
+    if (t->stream) cudaStreamSynchronize(t->stream);
+    free_tws(t);
+    cudaFree(t->d_conds);
+    cudaFree(t->d_data);
+    if (t->stream) cudaStreamDestroy(t->stream);
+    delete t;
+    return OLAP_OK;
+}
+
+}  // extern "C"

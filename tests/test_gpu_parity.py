@@ -453,3 +453,50 @@ def test_c3_full_size_sampled():
 def test_c5_slice_full_size_sampled():
     """C5 per-GPU slice: 128 GiB float32 cube (1024,4096,8192), 65,536 small boxes; sampled parity."""
     _sampled_full_size("C5", 50, 400, 2_000_000, np.array([2, 1, 1, 1], float))
+
+
+# ------------------------------------------------------------------ fact tables (NEXT #1)
+
+def _table_cols(nrows, rng):
+    dims = [rng.integers(0, n, size=nrows).astype(np.int32) for n in (40, 7, 13, 5)]
+    qty = rng.integers(-50, 100, size=nrows).astype(np.int32)
+    paid = rng.random(nrows).astype(np.float32)
+    return dims + [qty, paid]
+
+
+def _table_queries(rng, nq):
+    qs = []
+    for _ in range(nq):
+        conds = []
+        for c, n in enumerate((40, 7, 13, 5)):
+            if rng.random() < 0.6:
+                a, b = sorted(rng.integers(-2, n + 2, size=2))
+                if rng.random() < 0.05:
+                    a, b = b + 1, a
+                conds.append((c, int(a), int(b)))
+        qs.append((conds, int(rng.integers(4, 6)), int(rng.integers(0, 5))))
+    return qs
+
+
+@pytest.mark.parametrize("nrows", [1, 1000, 1024, 5000, 300_001])
+def test_table_scan_parity(nrows):
+    """Q_D over a column store (Eq. 11-12): GPU shared scan vs oracle.tablescan."""
+    rng = np.random.default_rng(nrows)
+    cols = _table_cols(nrows, rng)
+    t = olap.Table(nrows, [c.dtype for c in cols])
+    for i, c in enumerate(cols):
+        t.load_column(i, c)
+    qs = _table_queries(rng, 500)
+    qs.append(([], 4, olap.SUM))                          # no condition: whole column
+    qs.append(([(0, 10, 10), (0, 11, 11)], 5, olap.AVG))  # contradictory -> empty
+    got = t.query(qs)
+    ref = oracle.tablescan(cols, qs, nthreads=oracle.max_threads())
+    ops = np.array([q[2] for q in qs], np.int32)
+    isf = np.array([cols[q[1]].dtype == np.float32 for q in qs])
+    assert np.array_equal(got["flags"], ref["flags"]) and np.array_equal(got["i"], ref["i"])
+    ex = ~isf | (ops == olap.MIN) | (ops == olap.MAX) | (ops == olap.COUNT)
+    assert np.array_equal(got["d"][ex], ref["d"][ex])
+    tol = 1e-6 * np.abs(ref["d"]) + 1e-300
+    assert (np.abs(got["d"] - ref["d"]) <= tol).all()
+    with pytest.raises(olap.OlapError):
+        t.query([([(5, 0, 1)], 4, olap.SUM)])             # condition on a float column
