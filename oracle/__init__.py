@@ -10,6 +10,7 @@ Functions (all cite the passage they follow in oracle.cpp):
   query()      Eq. 1 / Eq. 3 / PAPER.md:25 — odometer sub-cube aggregation.
   Dict         PAPER.md:252-256 — one std::map dictionary per text column.
   factscan()   PAPER.md:206-208 — filtered aggregation over a fact table.
+  rollup(), convert_range()  PAPER.md:103-136, Fig. 1, Eq. 1-2 — multi-resolution cube set.
   tablescan()  Eq. 11-12, PAPER.md:206-216 — the paper's GPU query Q_D over a column store.
   fill()       the counter-based cell generator (independent re-implementation).
 
@@ -87,6 +88,13 @@ def lib():
         L.oracle_tablescan.argtypes = [ctypes.c_int64, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64,
                                        ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
                                        ctypes.c_void_p, ctypes.c_int]
+        L.oracle_rollup.restype = ctypes.c_int
+        L.oracle_rollup.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int,
+                                    ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int, ctypes.c_void_p,
+                                    ctypes.c_void_p, ctypes.c_int]
+        L.oracle_convert_range.restype = ctypes.c_int
+        L.oracle_convert_range.argtypes = [ctypes.c_int, ctypes.c_int64, ctypes.c_void_p, ctypes.c_int, ctypes.c_int,
+                                           ctypes.c_int64, ctypes.c_int64, c_i64p, c_i64p]
         _lib = L
     return _lib
 
@@ -253,3 +261,36 @@ def tablescan(columns, queries, nthreads: int = 1):
     if rc:
         raise ValueError("oracle_tablescan: invalid arguments")
     return out
+
+
+def _levels_ptrs(level_ids):
+    """level_ids: list over dims of lists over levels of int32 arrays (finest-member -> level id)."""
+    arrs = [np.ascontiguousarray(a, dtype=np.int32) for dim in level_ids for a in dim]
+    ptrs = (ctypes.c_void_p * len(arrs))(*[a.ctypes.data for a in arrs])
+    return arrs, ptrs
+
+
+def rollup(level_ids, fine, rf, rc, op=SUM):
+    """Aggregate the level-rf cube `fine` (ndarray, shape = level-rf extents) to level rc."""
+    nd, L = len(level_ids), len(level_ids[0])
+    n_fin = np.array([len(level_ids[d][-1]) for d in range(nd)], dtype=np.int64)
+    arrs, ptrs = _levels_ptrs(level_ids)
+    ext_f = np.array(fine.shape, dtype=np.int64)
+    ext_c = np.array([int(level_ids[d][rc].max()) + 1 for d in range(nd)], dtype=np.int64)
+    f = np.ascontiguousarray(fine)
+    out = np.empty(tuple(ext_c), dtype=f.dtype)
+    rc_ = lib().oracle_rollup(nd, L, n_fin.ctypes.data, ctypes.cast(ptrs, ctypes.c_void_p), _dtype_code(f.dtype), rf,
+                              ext_f.ctypes.data, f.ctypes.data, rc, ext_c.ctypes.data, out.ctypes.data, op)
+    if rc_:
+        raise ValueError("oracle_rollup failed")
+    return out
+
+
+def convert_range(ids_of_dim, r, R, f, t):
+    """[f, t] at level r -> [lo, hi] at level R (lo > hi if empty)."""
+    arrs = [np.ascontiguousarray(a, dtype=np.int32) for a in ids_of_dim]
+    ptrs = (ctypes.c_void_p * len(arrs))(*[a.ctypes.data for a in arrs])
+    lo, hi = ctypes.c_int64(), ctypes.c_int64()
+    lib().oracle_convert_range(len(arrs), len(arrs[-1]), ctypes.cast(ptrs, ctypes.c_void_p), r, R, f, t,
+                               ctypes.byref(lo), ctypes.byref(hi))
+    return lo.value, hi.value

@@ -20,6 +20,10 @@
  *   oracle_tablescan  — the paper's GPU query Q_D over a column-store fact table
  *                       (Eq. 11-12): conditions on dimension
  *                       columns, aggregate of one data column, COUNT = matching rows.
+ *   oracle_rollup / oracle_convert_range — the multi-resolution cube set
+ *                       (Fig. 1, Eq. 1-2): coarse cells
+ *                       aggregate the fine cells mapping to them; a level-r range in
+ *                       level-R members.
  *   oracle_factscan   — filtered aggregation over a fact table of translated
  *                       (integer) dimension columns and one data column  PAPER.md:206-208 (§III-E)
  *                       used as an independent path to the cube answer for SUM.
@@ -35,6 +39,7 @@
  *
  * Parity pins for every function live in tests/test_oracle_*.py (-m "not gpu").
  */
+#include <climits>
 #include <cstdint>
 #include <cstring>
 #include <map>
@@ -418,6 +423,73 @@ int oracle_tablescan(int64_t nrows, int ncols, const void* const* cols, const in
         }
         out[q] = res;
     }
+    return 0;
+}
+
+/*
+ * Multi-resolution cube set (Fig. 1, Eq. 1-2).  Dimension d
+ * has levels 0 (coarsest) .. L-1 (finest); level_ids[d*L + r][x] is the level-r member
+ * of finest member x.
+ *
+ * oracle_rollup: the cell of a cube at level rc is the aggregate (op: SUM, MIN or MAX)
+ * of every cell of the level-rf cube (rf > rc) whose members map to it.  Plain loop over
+ * the fine cells; int32 SUM wraps mod 2^32 into the int32 cell, float32 SUM accumulates
+ * in double and rounds once to float32.  fine/coarse: row-major host arrays.
+ */
+int oracle_rollup(int nd, int L, const int64_t* n_finest, const int32_t* const* level_ids, int dtype,
+                  int rf, const int64_t* ext_f, const void* fine, int rc, const int64_t* ext_c, void* coarse, int op) {
+    (void)L;
+    int64_t nf = 1, ncc = 1;
+    for (int d = 0; d < nd; ++d) { nf *= ext_f[d]; ncc *= ext_c[d]; }
+    // member map level rf -> level rc per dimension, through any finest member
+    std::vector<std::vector<int64_t>> up(nd);
+    for (int d = 0; d < nd; ++d) {
+        up[d].assign(ext_f[d], -1);
+        for (int64_t x = 0; x < n_finest[d]; ++x)
+            up[d][level_ids[d * L + rf][x]] = level_ids[d * L + rc][x];
+    }
+    std::vector<double> accf(ncc, 0.0);
+    std::vector<int64_t> acci(ncc, 0);
+    std::vector<char> seen(ncc, 0);
+    std::vector<int64_t> x(nd, 0);
+    for (int64_t i = 0; i < nf; ++i) {
+        int64_t rem = i, ci = 0, mul = 1;
+        for (int d = nd - 1; d >= 0; --d) { x[d] = rem % ext_f[d]; rem /= ext_f[d]; }
+        for (int d = nd - 1; d >= 0; --d) { ci += up[d][x[d]] * mul; mul *= ext_c[d]; }
+        if (dtype == ORC_INT32) {
+            const int64_t v = static_cast<const int32_t*>(fine)[i];
+            if (op == ORC_SUM) acci[ci] += v;
+            else if (!seen[ci] || (op == ORC_MIN ? v < acci[ci] : v > acci[ci])) acci[ci] = v;
+        } else {
+            const double v = static_cast<const float*>(fine)[i];
+            if (op == ORC_SUM) accf[ci] += v;
+            else if (!seen[ci] || (op == ORC_MIN ? v < accf[ci] : v > accf[ci])) accf[ci] = v;
+        }
+        seen[ci] = 1;
+    }
+    for (int64_t c = 0; c < ncc; ++c) {
+        if (dtype == ORC_INT32) static_cast<int32_t*>(coarse)[c] = (int32_t)(uint32_t)(uint64_t)acci[c];
+        else static_cast<float*>(coarse)[c] = (float)accf[c];
+    }
+    return 0;
+}
+
+/* Eq. 1 condition [f, t] given at level r, expressed at level R >= r: every level-R member
+ * whose level-r ancestor lies in [f, t] (scan of the finest members). */
+int oracle_convert_range(int L, int64_t n_finest, const int32_t* const* ids_of_dim, int r, int R, int64_t f,
+                         int64_t t, int64_t* out_lo, int64_t* out_hi) {
+    (void)L;
+    int64_t lo = INT64_MAX, hi = INT64_MIN;
+    for (int64_t x = 0; x < n_finest; ++x) {
+        const int64_t a = ids_of_dim[r][x];
+        if (a < f || a > t) continue;
+        const int64_t b = ids_of_dim[R][x];
+        if (b < lo) lo = b;
+        if (b > hi) hi = b;
+    }
+    if (lo > hi) { lo = 1; hi = 0; }
+    *out_lo = lo;
+    *out_hi = hi;
     return 0;
 }
 

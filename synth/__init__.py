@@ -227,3 +227,30 @@ def random_keys(n: int, seed: int, min_len: int = 1, max_len: int = 24, alphabet
     offs = np.zeros(n + 1, dtype=np.int64)
     offs[1:] = np.cumsum(lens)
     return [blob[offs[i]:offs[i + 1]] for i in range(n)]
+
+
+# ---------------------------------------------------------------- multi-resolution hierarchies (NEXT #3)
+
+def date_hierarchy():
+    """d_date members 1998-01-01 .. 2002-12-31 at levels year (0), month (1), day (2):
+    finest-member -> level-id arrays (ids are ranks in time order)."""
+    import datetime as _dt
+    d0 = _dt.date(1998, 1, 1)
+    days = [d0 + _dt.timedelta(days=i) for i in range(1826)]
+    year = np.array([d.year - 1998 for d in days], dtype=np.int32)
+    month = np.array([(d.year - 1998) * 12 + d.month - 1 for d in days], dtype=np.int32)
+    return [year, month, np.arange(1826, dtype=np.int32)]
+
+
+def random_hierarchy(n_finest: int, levels: int, rng: np.random.Generator):
+    """A monotone hierarchy: level L-1 is the identity; each coarser level groups
+    consecutive members of the next finer level into random-size blocks."""
+    ids = [np.arange(n_finest, dtype=np.int32)]
+    for _ in range(levels - 1):
+        prev = ids[0]
+        n_prev = int(prev.max()) + 1
+        cuts = np.sort(rng.choice(np.arange(1, n_prev), size=max(0, min(n_prev - 1, n_prev // 3)), replace=False)) \
+            if n_prev > 1 else np.zeros(0, dtype=np.int64)
+        group = np.searchsorted(cuts, np.arange(n_prev), side="right").astype(np.int32)
+        ids.insert(0, group[prev])
+    return ids
