@@ -281,6 +281,48 @@ int olap_table_query_batch_device(olap_table* t, int64_t nq, const int64_t* d_co
 
 int olap_table_destroy(olap_table* t);
 
+/* ---------------------------------------------------------------- multi-resolution cube set */
+
+/* Resolution hierarchy (Fig. 1: "years (low resolution), months, days,
+ * hours (high resolution)"): levels 0 (coarsest) .. nlevels-1 (finest) for every
+ * dimension.  level_ids[d*nlevels + r] points to n_finest[d] int32: the level-r member of
+ * each finest member of dimension d; ids start at 0 and step by 0 or 1 (every coarse
+ * member is a contiguous block), the finest level is the identity, and a member never
+ * splits a member of a coarser level.  A dimension without a hierarchy passes the
+ * identity at every level.  HOST buffers, copied. */
+typedef struct olap_hier olap_hier;
+int olap_hier_create(int ndims, int nlevels, const int64_t* n_finest, const int32_t* const* level_ids,
+                     olap_hier** out);
+int olap_hier_extents(const olap_hier* h, int level, int64_t* extents /* ndims */);
+
+/* Conditions of Eq. 1 given at their own resolution r (levels[q*ndims + d]) expressed at
+ * level `target` >= r: [f, t] -> [first target member in f, last target member in t].
+ * Empty stays empty; out of bounds -> OLAP_E_RANGE.  HOST buffers. */
+int olap_hier_convert(const olap_hier* h, int64_t nq, const olap_range* ranges, const int32_t* levels,
+                      int target, olap_range* out);
+
+/* Pre-calculate a coarser cube: coarse cell = SUM (or MIN / MAX) of the
+ * fine cells mapping to it, computed on the GPU (int32 SUM wraps into int32 cells,
+ * float32 SUM accumulates in fp64 and rounds once).  Both cubes unsharded, on one device,
+ * with extents equal to their levels' member counts.  Synchronous. */
+int olap_cube_rollup(const olap_hier* h, const olap_cube* fine, int fine_level, olap_cube* coarse,
+                     int coarse_level, int op);
+int olap_hier_destroy(olap_hier* h);
+
+/* A set of cubes at different resolutions sharing one hierarchy (cubes are borrowed,
+ * not owned).  olap_cubeset_query routes every query by Eq. 2:
+ * R = max_i r_i; the cube of resolution R answers it, its conditions converted to level
+ * R.  SUM, which roll-up preserves, may also use the lowest-resolution finer cube.  A
+ * query no cube can answer gets OLAP_RESULT_INVALID (answer it from the fact table,
+ * olap_table_*, as the paper does on the GPU).  level_used[q] (optional) = cube level,
+ * or -1.  HOST buffers. */
+typedef struct olap_cubeset olap_cubeset;
+int olap_cubeset_create(const olap_hier* h, olap_cubeset** out);
+int olap_cubeset_add(olap_cubeset* s, int level, olap_cube* c);
+int olap_cubeset_query(olap_cubeset* s, int64_t nq, const olap_range* ranges, const int32_t* levels,
+                       const int32_t* ops, olap_result* results, int32_t* level_used);
+int olap_cubeset_destroy(olap_cubeset* s);
+
 /* ---------------------------------------------------------------- misc */
 
 const char* olap_last_error(void); /* thread-local; valid until the next olap_* call */

@@ -21,7 +21,7 @@ __all__ = ["Cube", "Dict", "OlapError", "translate", "shard_local_rows", "combin
            "finalize_device", "translate_device", "RESULT_DTYPE", "lib", "LIB_PATH",
            "INT32", "FLOAT32", "SUM", "COUNT", "MIN", "MAX", "AVG", "GEN_UNIFORM", "GEN_AFFINE",
            "RESULT_EMPTY", "RESULT_INVALID", "EXPORTS", "text_ranges", "text_ranges_device", "pack_text_conditions",
-           "COND_ALL", "COND_EQ", "COND_RANGE", "COND_IDS", "Table", "COND_DTYPE"]
+           "COND_ALL", "COND_EQ", "COND_RANGE", "COND_IDS", "Table", "COND_DTYPE", "Hierarchy", "CubeSet"]
 
 LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libolap_b200.so")
 if os.environ.get("OLAP_LIB"):          # development only: A/B a differently-tuned build of the same sources
@@ -76,6 +76,15 @@ EXPORTS = {
     "olap_table_query_batch": (_int, [_p, _i64, _p, _p, _p, _p, _p]),
     "olap_table_query_batch_device": (_int, [_p, _i64, _p, _p, _p, _p, _p, _p]),
     "olap_table_destroy": (_int, [_p]),
+    "olap_hier_create": (_int, [_int, _int, _p, _p, ctypes.POINTER(_p)]),
+    "olap_hier_extents": (_int, [_p, _int, _p]),
+    "olap_hier_convert": (_int, [_p, _i64, _p, _p, _int, _p]),
+    "olap_cube_rollup": (_int, [_p, _p, _int, _p, _int, _int]),
+    "olap_hier_destroy": (_int, [_p]),
+    "olap_cubeset_create": (_int, [_p, ctypes.POINTER(_p)]),
+    "olap_cubeset_add": (_int, [_p, _int, _p]),
+    "olap_cubeset_query": (_int, [_p, _i64, _p, _p, _p, _p, _p]),
+    "olap_cubeset_destroy": (_int, [_p]),
     "olap_finalize_launches": (_i64, []),
     "olap_last_error": (ctypes.c_char_p, []),
     "olap_version": (ctypes.c_char_p, []),
@@ -476,6 +485,91 @@ class Table:
     def close(self):
         if getattr(self, "_h", None):
             lib.olap_table_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class Hierarchy:
+    """Resolution levels per dimension (Fig. 1).
+
+    level_ids: list over dimensions of lists over levels (coarsest first) of int32 arrays
+    mapping each finest member to its level-r member."""
+
+    def __init__(self, level_ids):
+        self.nd, self.L = len(level_ids), len(level_ids[0])
+        self._arrs = [np.ascontiguousarray(a, dtype=np.int32) for dim in level_ids for a in dim]
+        ptrs = (ctypes.c_void_p * len(self._arrs))(*[a.ctypes.data for a in self._arrs])
+        nf = np.array([len(level_ids[d][-1]) for d in range(self.nd)], dtype=np.int64)
+        h = ctypes.c_void_p()
+        _check(lib.olap_hier_create(self.nd, self.L, nf.ctypes.data, ctypes.cast(ptrs, ctypes.c_void_p),
+                                    ctypes.byref(h)), "olap_hier_create")
+        self._h = h
+
+    @property
+    def handle(self):
+        return self._h
+
+    def extents(self, level: int):
+        e = np.zeros(self.nd, dtype=np.int64)
+        _check(lib.olap_hier_extents(self._h, level, e.ctypes.data), "olap_hier_extents")
+        return tuple(int(v) for v in e)
+
+    def convert(self, ranges, levels, target: int):
+        r = np.ascontiguousarray(ranges, dtype=np.int64).reshape(-1, self.nd, 2)
+        lv = np.ascontiguousarray(levels, dtype=np.int32).reshape(-1, self.nd)
+        out = np.zeros_like(r)
+        _check(lib.olap_hier_convert(self._h, r.shape[0], r.ctypes.data, lv.ctypes.data, target, out.ctypes.data),
+               "olap_hier_convert")
+        return out
+
+    def rollup(self, fine: "Cube", fine_level: int, coarse: "Cube", coarse_level: int, op: int = SUM):
+        _check(lib.olap_cube_rollup(self._h, fine.handle, fine_level, coarse.handle, coarse_level, op),
+               "olap_cube_rollup")
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib.olap_hier_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class CubeSet:
+    """Cubes at several resolutions; queries routed by Eq. 2."""
+
+    def __init__(self, hier: Hierarchy):
+        self.hier = hier
+        self._cubes = {}
+        h = ctypes.c_void_p()
+        _check(lib.olap_cubeset_create(hier.handle, ctypes.byref(h)), "olap_cubeset_create")
+        self._h = h
+
+    def add(self, level: int, cube: "Cube"):
+        _check(lib.olap_cubeset_add(self._h, level, cube.handle), "olap_cubeset_add")
+        self._cubes[level] = cube   # keep alive (the set borrows it)
+
+    def query(self, ranges, levels, ops):
+        r = np.ascontiguousarray(ranges, dtype=np.int64).reshape(-1, self.hier.nd, 2)
+        lv = np.ascontiguousarray(levels, dtype=np.int32).reshape(-1, self.hier.nd)
+        o = np.ascontiguousarray(ops, dtype=np.int32).reshape(-1)
+        out = np.zeros(len(o), dtype=RESULT_DTYPE)
+        used = np.zeros(len(o), dtype=np.int32)
+        _check(lib.olap_cubeset_query(self._h, len(o), r.ctypes.data, lv.ctypes.data, o.ctypes.data, out.ctypes.data,
+                                      used.ctypes.data), "olap_cubeset_query")
+        return out, used
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib.olap_cubeset_destroy(self._h)
             self._h = None
 
     def __del__(self):

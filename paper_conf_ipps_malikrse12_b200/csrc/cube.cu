@@ -1165,6 +1165,18 @@ int check_cube(const olap_cube* c) {
 
 }  // namespace
 
+namespace olap {
+// geometry for other translation units (hier.cu): dims, extents, dtype, inner pitch, shards
+int cube_geometry(const olap_cube* c, int* nd, int64_t* n, int* dtype, int64_t* pitch, int64_t* nshards) {
+    *nd = c->nd;
+    for (int k = 0; k < c->nd; ++k) n[k] = c->n[k];
+    *dtype = c->dtype;
+    *pitch = c->pitch;
+    *nshards = c->sh.nshards;
+    return OLAP_OK;
+}
+}  // namespace olap
+
 extern "C" {
 
 int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_shard* shard, int device,

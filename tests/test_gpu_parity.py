@@ -500,3 +500,76 @@ def test_table_scan_parity(nrows):
     assert (np.abs(got["d"] - ref["d"]) <= tol).all()
     with pytest.raises(olap.OlapError):
         t.query([([(5, 0, 1)], 4, olap.SUM)])             # condition on a float column
+
+
+# ------------------------------------------------------------------ multi-resolution cube set (NEXT #3)
+
+def _hier(rng):
+    return [synth.date_hierarchy(), synth.random_hierarchy(37, 3, rng), synth.random_hierarchy(50, 3, rng)]
+
+
+@pytest.mark.parametrize("dtype", [np.int32, np.float32])
+def test_rollup_parity(dtype):
+    rng = np.random.default_rng(31)
+    ids = _hier(rng)
+    h = olap.Hierarchy(ids)
+    fine_ext = h.extents(2)
+    cells = (rng.integers(-1000, 1000, size=fine_ext) if dtype == np.int32 else
+             rng.random(fine_ext)).astype(dtype)
+    fine = olap.Cube(fine_ext, dtype)
+    fine.load(cells)
+    for rc in (0, 1):
+        for op in (olap.SUM, olap.MIN, olap.MAX):
+            ce = h.extents(rc)
+            coarse = olap.Cube(ce, dtype)
+            h.rollup(fine, 2, coarse, rc, op)
+            want = oracle.rollup(ids, cells, 2, rc, op)
+            # read every coarse cell back through 1-cell MAX queries
+            boxes = np.stack(np.meshgrid(*[np.arange(n) for n in ce], indexing="ij"), -1).reshape(-1, 3)
+            boxes = np.repeat(boxes[:, :, None], 2, axis=2)
+            r = coarse.query(boxes, np.full(len(boxes), olap.MAX, np.int32))
+            got = r["i"].astype(np.int32) if dtype == np.int32 else r["d"].astype(np.float32)
+            assert np.array_equal(got, want.ravel()), (rc, op)
+
+
+def test_cubeset_routing_eq2():
+    rng = np.random.default_rng(32)
+    ids = _hier(rng)
+    h = olap.Hierarchy(ids)
+    cells = rng.integers(0, 1000, size=h.extents(2)).astype(np.int32)
+    cubes = {2: olap.Cube(h.extents(2), np.int32)}
+    cubes[2].load(cells)
+    cubes[0] = olap.Cube(h.extents(0), np.int32)
+    h.rollup(cubes[2], 2, cubes[0], 0, olap.SUM)
+    cs = olap.CubeSet(h)
+    cs.add(2, cubes[2])
+    cs.add(0, cubes[0])                     # level 1 deliberately missing
+    nq = 600
+    levels = rng.integers(0, 3, size=(nq, 3)).astype(np.int32)
+    ranges = np.zeros((nq, 3, 2), np.int64)
+    for q in range(nq):
+        for d in range(3):
+            n = int(ids[d][levels[q, d]].max()) + 1
+            ranges[q, d] = sorted(rng.integers(0, n, size=2))
+    ops = synth.ops_uniform(nq, rng)
+    got, used = cs.query(ranges, levels, ops)
+    R = levels.max(axis=1)
+    coarse_cells = oracle.rollup(ids, cells, 2, 0)
+    for q in range(nq):
+        if R[q] == 1 and ops[q] != olap.SUM:
+            assert used[q] == -1 and got["flags"][q] == olap.RESULT_INVALID
+            continue
+        tgt = R[q] if R[q] != 1 else 2             # SUM at level 1 falls through to the finest cube
+        assert used[q] == tgt
+        box = np.array([oracle.convert_range(ids[d], int(levels[q, d]), int(tgt), *ranges[q, d]) for d in range(3)])
+        src = cells if tgt == 2 else coarse_cells
+        ref = oracle.query(src.shape, box[None], ops[q:q + 1], src.ravel())
+        assert got[q:q + 1].tobytes() == ref.tobytes(), q
+    # SUM is the same at every resolution that can answer it (roll-up preserves sums)
+    ext0 = h.extents(0)
+    r0 = np.stack([np.sort(rng.integers(0, n, size=(nq, 2)), axis=1) for n in ext0], axis=1)
+    sums, used0 = cs.query(r0, np.zeros_like(levels), np.full(nq, olap.SUM, np.int32))
+    assert (used0 == 0).all()
+    fine_box = h.convert(r0, np.zeros_like(levels), 2)
+    direct = cubes[2].query(fine_box, np.full(nq, olap.SUM, np.int32))
+    assert np.array_equal(sums["i"], direct["i"])

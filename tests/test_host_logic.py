@@ -94,3 +94,42 @@ def test_dict_hash_host_matches_definition():
         assert olap.lib.olap_selftest_hash(key, len(key)) == _ref_hash(key)
     # zero padding must not collide keys of different lengths
     assert olap.lib.olap_selftest_hash(b"ab", 2) != olap.lib.olap_selftest_hash(b"ab\0", 3)
+
+
+def test_hier_convert_matches_oracle():
+    """olap_hier_convert (host code in the product library) vs oracle.convert_range."""
+    import oracle
+    import synth
+    rng = np.random.default_rng(21)
+    hier_ids = [synth.date_hierarchy(), synth.random_hierarchy(50, 3, rng), [np.zeros(7, np.int32),
+                                                                             np.zeros(7, np.int32),
+                                                                             np.arange(7, dtype=np.int32)]]
+    h = olap.Hierarchy(hier_ids)
+    assert h.extents(2) == (1826, 50, 7) and h.extents(0)[0] == 5
+    for target in (1, 2):
+        ranges, levels = [], []
+        for _ in range(200):
+            q, lq = [], []
+            for d in range(3):
+                r = int(rng.integers(0, target + 1))
+                n = int(hier_ids[d][r].max()) + 1
+                a, b = sorted(rng.integers(0, n, size=2))
+                if rng.random() < 0.05:
+                    a, b = b + 1, a
+                q.append((int(a), int(b)))
+                lq.append(r)
+            ranges.append(q)
+            levels.append(lq)
+        got = h.convert(ranges, levels, target)
+        for qi in range(200):
+            for d in range(3):
+                want = oracle.convert_range(hier_ids[d], levels[qi][d], target, *ranges[qi][d])
+                g = tuple(got[qi, d])
+                if want[0] > want[1]:
+                    assert g[0] > g[1]
+                else:
+                    assert g == want
+    with pytest.raises(olap.OlapError):
+        olap.Hierarchy([[np.array([0, 2, 2], np.int32), np.arange(3, dtype=np.int32)]])   # gap in ids
+    with pytest.raises(olap.OlapError):
+        h.convert([[(0, 9), (0, 1), (0, 1)]], [[0, 0, 0]], 2)                              # year 9 does not exist
