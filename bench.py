@@ -414,13 +414,104 @@ def run_table(args, rank, world):
     return 0
 
 
+def run_resolution(args, rank, world):
+    """R: the multi-resolution cube set (Eq. 2).  The C4
+    quantity cube at day resolution (52,100,128,1826) is rolled up on the GPU to month (60)
+    and year (5) resolution.  Each step is a batch of 10,000 queries whose date condition is
+    given in years, months or days (1/3 each) with 0-3 equality predicates; olap_cubeset_query
+    answers each from the cube of its resolution R = max r_i (Eq. 2).  The same batch answered
+    entirely on the day cube is reported beside it (`day_cube_only`)."""
+    import torch
+
+    import paper_conf_ipps_malikrse12_b200 as olap
+
+    if world > 1:
+        raise SystemExit("R is a single-GPU workload")
+    torch.cuda.set_device(0)
+    members = synth.tpcds_members()
+    cols = ["ca_state", "i_class", "s_store_id", "d_date"]
+    card = [len(members[c]) for c in cols]
+    ident = lambda n: np.arange(n, dtype=np.int32)
+    levels = [[ident(card[i])] * 3 for i in range(3)] + [synth.date_hierarchy()]
+    h = olap.Hierarchy(levels)
+    nrows = 1 << 26
+    facts, qty, _ = synth.tpcds_facts(nrows, members)
+    dicts = [olap.Dict(members[c]) for c in cols]
+    ids = np.stack([dicts[i].translate(members[c])[0][facts[c]] for i, c in enumerate(cols)]).astype(np.int32)
+    day = olap.Cube(h.extents(2), np.int32)
+    day.fill(olap.GEN_AFFINE, 0, np.zeros(5))
+    day.add_facts_device(torch.from_numpy(ids).cuda(), torch.from_numpy(qty).cuda())
+    torch.cuda.synchronize()
+    cubes = {2: day}
+    tb = time.perf_counter()
+    for lvl in (1, 0):
+        cubes[lvl] = olap.Cube(h.extents(lvl), np.int32)
+        h.rollup(day, 2, cubes[lvl], lvl, olap.SUM)
+    rollup_s = time.perf_counter() - tb
+    cs = olap.CubeSet(h)
+    for lvl, c in cubes.items():
+        cs.add(lvl, c)
+    nq = 10_000
+    rng = np.random.default_rng(synth.SEED_BASE + 11)
+    steps, warm = args.steps, args.warmup
+    batches_ = []
+    for _ in range(warm + steps):
+        lv = np.zeros((nq, 4), np.int32)
+        rr = np.zeros((nq, 4, 2), np.int64)
+        ops = rng.choice(np.array([olap.SUM, olap.MIN, olap.MAX, olap.AVG, olap.COUNT], np.int32), size=nq)
+        for q in range(nq):
+            r = int(rng.integers(0, 3))
+            n = len(np.unique(levels[3][r]))
+            lv[q, :] = 0
+            lv[q, 3] = r
+            rr[q, 3] = sorted(rng.integers(0, n, size=2))
+            for d in range(3):
+                if rng.random() < 0.5:
+                    v = int(rng.integers(0, card[d]))
+                    rr[q, d] = (v, v)
+                else:
+                    rr[q, d] = (0, card[d] - 1)
+        batches_.append((rr, lv, ops))
+    for k in range(warm):
+        cs.query(*batches_[k])
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    used_hist = np.zeros(3, np.int64)
+    for k in range(warm, warm + steps):
+        _, used = cs.query(*batches_[k])
+        used_hist += np.bincount(used[used >= 0], minlength=3)
+    routed_s = time.perf_counter() - t0
+    # the same queries answered on the day cube only (conditions converted to days)
+    conv = [(h.convert(b[0], b[1], 2), b[2]) for b in batches_]
+    for k in range(warm):
+        day.query(*conv[k])
+    t0 = time.perf_counter()
+    for k in range(warm, warm + steps):
+        day.query(*conv[k])
+    day_s = time.perf_counter() - t0
+    line = {
+        "metric": METRIC, "value": nq * steps / routed_s, "unit": "queries/s", "n_gpus": 1, "steps": steps,
+        "warmup": warm, "ms_per_step": routed_s / steps * 1e3, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "i32", "data": "synthetic",
+        "config": {"workload": "R", "levels": {"year": h.extents(0), "month": h.extents(1), "day": h.extents(2)},
+                   "batch": nq, "queries": "date condition in years / months / days (1/3 each) + 0-3 equality "
+                   "predicates, random op; host-buffer API timed end to end",
+                   "rollup_s": rollup_s, "queries_per_level_used": used_hist.tolist()},
+        "day_cube_only": {"value": nq * steps / day_s, "unit": "queries/s"},
+        "e2e": {"value": nq * steps / routed_s, "unit": "queries/s", "api": "olap_cubeset_query (host buffers)"},
+        "cpu_baseline": None, "roofline": None, "gpu_launches": None,
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="C2a", choices=["C2a", "C2b", "C3", "C1", "C4", "C5", "T"])
+    ap.add_argument("--workload", default="C2a", choices=["C2a", "C2b", "C3", "C1", "C4", "C5", "T", "R"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
     args = ap.parse_args()
@@ -432,6 +523,8 @@ def main():
         return run_c4(args, rank, world)
     if args.workload == "T":
         return run_table(args, rank, world)
+    if args.workload == "R":
+        return run_resolution(args, rank, world)
 
     import torch
     import torch.distributed as dist
