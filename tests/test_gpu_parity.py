@@ -160,14 +160,18 @@ def test_c2_full_size_sampled():
     compare(gpu[idx2], ref2, ops[idx2], np.float32, exact_float=True)
 
 
-def test_determinism_float_sums():
-    ext = (16, 16, 16, 16, 16, 16)
+@pytest.mark.parametrize("ext", [(16, 16, 16, 16, 16, 16), (16, 16, 16, 16, 16, 48)])
+def test_determinism_float_sums(ext):
+    """Float sums are bit-stable run to run, with and without the L2-aware item order
+    (the 192 MiB cube takes it): blocks pick items up in a different order every run,
+    but partials are folded in item order."""
     c = olap.Cube(ext, np.float32)
     c.fill(olap.GEN_UNIFORM, 99)
-    boxes, ops = synth.config_queries("C2a", nq=512, extents=ext)
+    assert c.stats()[1] == (int(np.prod(ext)) * 4 > (64 << 20))
+    boxes, ops = synth.config_queries("C2a", nq=2048, extents=ext)
     a = c.query(boxes, ops)
-    b = c.query(boxes, ops)
-    assert a.tobytes() == b.tobytes()
+    for _ in range(3):
+        assert c.query(boxes, ops).tobytes() == a.tobytes()
 
 
 def test_empty_invalid_and_errors():
