@@ -1043,7 +1043,11 @@ int ensure_ws(olap_cube* c, int64_t nq) {
     OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
     free_ws(c);
     int64_t cap = std::max<int64_t>(nq, 1024);
-    int64_t items = std::max<int64_t>(1ll << 20, 4 * cap);
+    // item partial capacity: >= 2^20 and 4 per query, and for big cubes enough that items stay a
+    // few MiB (the L2-aware order needs the ~600 in-flight items to fit in L2): one per 4 KiB of
+    // cube, <= 2^24 (a batch reads the cube ~10^2-10^3 times over at C3-like overlap)
+    const int64_t by_size = std::min<int64_t>(1ll << 24, (c->local_cells * 4) >> 12);
+    int64_t items = std::max<int64_t>(std::max<int64_t>(1ll << 20, 4 * cap), by_size);
     OLAP_CUDA_TRY(cudaMalloc(&c->d_desc, sizeof(QDesc) * cap));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_item_start, sizeof(int64_t) * (cap + 1)));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_done, sizeof(int32_t) * cap));
