@@ -618,9 +618,34 @@ def main():
         e2e = {"value": nq * args.e2e_steps / e2e_s, "unit": "queries/s",
                "h2d_bytes_per_step": int(nq * nd * 16 + nq * 4), "d2h_bytes_per_step": int(nq * 24),
                "api": "olap_query_batch (host buffers; pinned staging inside the library)"}
-    elif world > 1:
-        e2e = {"value": None, "unit": "queries/s", "h2d_bytes_per_step": int(nq * nd * 16 + nq * 4),
-               "d2h_bytes_per_step": int(nq * 24), "note": "host-buffer e2e measured at N=1 only"}
+    elif world > 1 and args.e2e_steps > 0:
+        # host arrays in, host results out, through the sharded path on every rank:
+        # pinned H2D -> shard partials -> NCCL exchange -> finalize -> D2H (timed max over ranks)
+        pin_r = torch.empty((nq, nd, 2), dtype=torch.int64).pin_memory()
+        pin_o = torch.empty(nq, dtype=torch.int32).pin_memory()
+        pin_res = torch.empty(nq * olap.RESULT_DTYPE.itemsize, dtype=torch.uint8).pin_memory()
+        d_r = torch.empty((nq, nd, 2), dtype=torch.int64, device=dev)
+        d_o = torch.empty(nq, dtype=torch.int32, device=dev)
+        dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for k in range(args.e2e_steps):
+            b, o = host_batches[args.warmup + (k % args.steps)]
+            pin_r.numpy()[...] = b
+            pin_o.numpy()[...] = o
+            with torch.cuda.stream(stream):
+                d_r.copy_(pin_r, non_blocking=True)
+                d_o.copy_(pin_o, non_blocking=True)
+                cube.partials_device(d_r, d_o, psum, pext, nq=nq, stream=stream)
+                exchange_partials(psum, pext, cube.dtype_code)
+                olap.finalize_device(ext, cube.dtype_code, nq, d_r, d_o, psum, pext, res, stream=stream)
+                pin_res.copy_(res, non_blocking=True)
+            stream.synchronize()
+        e2e_t = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
+        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+        e2e = {"value": nq * args.e2e_steps / float(e2e_t.item()), "unit": "queries/s",
+               "h2d_bytes_per_step": int(nq * nd * 16 + nq * 4), "d2h_bytes_per_step": int(nq * 24),
+               "api": "ShardedCube path: H2D, olap_query_partials_device, NCCL all-reduce, olap_finalize_device, D2H"}
 
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
