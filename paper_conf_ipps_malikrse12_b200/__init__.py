@@ -20,7 +20,7 @@ import numpy as np
 __all__ = ["Cube", "Dict", "OlapError", "translate", "shard_local_rows", "combine_partials_device",
            "finalize_device", "translate_device", "RESULT_DTYPE", "lib", "LIB_PATH",
            "INT32", "FLOAT32", "SUM", "COUNT", "MIN", "MAX", "AVG", "GEN_UNIFORM", "GEN_AFFINE",
-           "RESULT_EMPTY", "RESULT_INVALID", "EXPORTS", "text_ranges", "text_ranges_device", "pack_text_conditions",
+           "RESULT_EMPTY", "RESULT_INVALID", "EXPORTS", "text_ranges", "text_ranges_device", "pack_text_conditions", "text_ranges_packed",
            "COND_ALL", "COND_EQ", "COND_RANGE", "COND_IDS", "Table", "COND_DTYPE", "Hierarchy", "CubeSet"]
 
 LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libolap_b200.so")
@@ -399,6 +399,17 @@ def pack_text_conditions(conditions, nd: int):
                 keys.append(c)
     buf, offs = _pack(keys)
     return kinds, first, rin, buf, offs
+
+
+def text_ranges_packed(dicts, extents, nq: int, kinds, rin, buf, offs):
+    """olap_text_ranges on conditions already in the C-ABI layout (see pack_text_conditions)."""
+    ext, extp = _i64arr(extents)
+    out = np.zeros((nq, len(dicts), 2), dtype=np.int64)
+    miss = ctypes.c_int64()
+    _check(lib.olap_text_ranges(_dict_or_null_array(dicts), len(dicts), extp, nq, kinds.ctypes.data, rin.ctypes.data,
+                                buf.ctypes.data, offs.ctypes.data_as(_i64p), len(offs) - 1, out.ctypes.data,
+                                ctypes.byref(miss)), "olap_text_ranges")
+    return out, miss.value
 
 
 def text_ranges(dicts, extents, conditions, ranges_in=None):
