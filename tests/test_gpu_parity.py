@@ -577,3 +577,72 @@ def test_cubeset_routing_eq2():
     fine_box = h.convert(r0, np.zeros_like(levels), 2)
     direct = cubes[2].query(fine_box, np.full(nq, olap.SUM, np.int32))
     assert np.array_equal(sums["i"], direct["i"])
+
+
+# ------------------------------------------------------------------ robustness
+
+def test_out_of_memory_is_an_error_not_a_crash():
+    # 2^40 float32 cells = 4 TiB: cudaMalloc fails -> OLAP_E_NOMEM, and the device stays usable
+    with pytest.raises(olap.OlapError) as ei:
+        olap.Cube((1 << 10, 1 << 10, 1 << 20), np.float32)
+    assert ei.value.status == olap.E_NOMEM
+    c = olap.Cube((4, 4), np.int32)
+    c.load(np.arange(16, dtype=np.int32))
+    assert c.query(np.array([[[0, 3], [0, 3]]]), [olap.SUM])["i"][0] == 120
+
+
+def test_concurrent_queries_one_cube():
+    """Several host threads query one cube at once: calls serialize on the cube's mutex
+    and its workspace event; every thread gets its own correct answers."""
+    import threading
+    ext = (16, 16, 16, 16, 16, 48)   # > 64 MiB: the L2-ordered path
+    c = olap.Cube(ext, np.float32)
+    c.fill(olap.GEN_UNIFORM, 5)
+    batches = [synth.config_queries("C2a", nq=256, seed=900 + i, extents=ext) for i in range(6)]
+    want = [c.query(b, o) for b, o in batches]
+    got = [None] * 6
+
+    def run(i):
+        for _ in range(3):
+            got[i] = c.query(*batches[i])
+
+    th = [threading.Thread(target=run, args=(i,)) for i in range(6)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    for i in range(6):
+        assert got[i].tobytes() == want[i].tobytes()
+
+
+def test_dict_stress_1e7():
+    """SURVEY §8(a) a2 stress size: 10^7 keys (16-byte ids), translated on the GPU."""
+    rng = np.random.default_rng(77)
+    ids = rng.integers(0, 1 << 62, size=10_000_000, dtype=np.int64)
+    keys = [b"%016x" % int(v) for v in ids[:2_000_000]]   # 16-char keys; the host build sorts them
+    keys += [bytes(8) + int(v).to_bytes(8, "little") for v in ids[2_000_000:]]
+    d = olap.Dict(keys)
+    assert len(d) == len(set(keys))
+    probe_idx = rng.integers(0, len(keys), size=200_000)
+    probes = [keys[i] for i in probe_idx] + [b"%016x" % int(v) + b"!" for v in ids[:10_000]]
+    got, miss = d.translate(probes)
+    assert miss == 10_000
+    # ids are ranks in byte order: check against a sorted copy of the distinct keys
+    s = sorted(set(keys))
+    for k in range(0, 200_000, 997):
+        assert s[got[k]] == probes[k]
+    assert (got[200_000:] == -1).all()
+
+
+def test_translate_device_counts_misses_on_device():
+    d = olap.Dict(["a", "bb", "ccc"])
+    keys = [b"a", b"x", b"ccc", b"bb", b""]
+    buf = np.frombuffer(b"".join(keys), np.uint8).copy()
+    offs = np.concatenate([[0], np.cumsum([len(k) for k in keys])]).astype(np.int64)
+    dbuf = torch.from_numpy(buf).cuda()
+    doff = torch.from_numpy(offs).cuda()
+    ids = torch.empty(len(keys), dtype=torch.int32, device="cuda")
+    miss = torch.zeros(1, dtype=torch.int64, device="cuda")
+    olap.translate_device([d], None, dbuf, doff, len(keys), ids, miss)
+    torch.cuda.synchronize()
+    assert ids.cpu().tolist() == [0, -1, 2, 1, -1] and int(miss.item()) == 2
