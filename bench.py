@@ -527,6 +527,7 @@ def main():
     ap.add_argument("--workload", default="C2a", choices=["C2a", "C2b", "C3", "C1", "C4", "C5", "T", "R"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--graph", action="store_true", help="replay each step as a captured CUDA graph (N=1)")
     args = ap.parse_args()
 
     rank, world, local = env_int("RANK", 0), env_int("WORLD_SIZE", 1), env_int("LOCAL_RANK", 0)
@@ -582,6 +583,19 @@ def main():
         for k in range(args.warmup):
             step(k)
     stream.synchronize()
+    graphs = None
+    if args.graph and world == 1:
+        # one CUDA graph per batch (plan, order, reduce, finalize), captured after the warm-up sized the workspace
+        graphs = []
+        for k in range(args.warmup + args.steps):
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=stream):
+                cube.query_device(d_batches[k][0], d_batches[k][1], res, nq=nq, stream=torch.cuda.current_stream())
+            graphs.append(g)
+        torch.cuda.synchronize()
+
+        def step(k):  # noqa: F811
+            graphs[k].replay()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()

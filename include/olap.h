@@ -135,7 +135,10 @@ int olap_query_batch(olap_cube* c, int64_t nq, const olap_range* ranges, const i
 
 /* Same path on DEVICE buffers, asynchronous on `stream` (cudaStream_t, NULL =
  * legacy default stream).  Invalid queries are flagged OLAP_RESULT_INVALID in
- * their result instead of failing the batch.  Unsharded cubes only. */
+ * their result instead of failing the batch.  Unsharded cubes only.  The call can be
+ * captured into a CUDA graph (and olap_query_partials_device likewise) after one
+ * uncaptured call with at least nq queries has sized the cube's workspace; a replayed
+ * graph must not overlap another batch on the same cube. */
 int olap_query_batch_device(olap_cube* c, int64_t nq, const olap_range* d_ranges,
                             const int32_t* d_ops, olap_result* d_results, void* stream);
 

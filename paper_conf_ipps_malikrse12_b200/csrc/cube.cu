@@ -567,14 +567,18 @@ __global__ void __launch_bounds__(kPlanThreads) scan_kernel(int64_t nq, QDesc* d
                                                             const int32_t* __restrict__ q_tv, int64_t* item_start,
                                                             unsigned long long* counter, int64_t items_cap,
                                                             const unsigned long long* totals,
-                                                            unsigned long long* bytes_acc) {
+                                                            unsigned long long* bytes_acc, int grid) {
     const int tid = threadIdx.x;
     const int64_t total_cells = (int64_t)totals[0], total_slot_cells = (int64_t)totals[1];
-    // item size: >= 1 MiB, and large enough that sum_q items_q <= items_cap:
+    // item size: 1 MiB, smaller for small batches so that there are >= 4 items per resident
+    // block (latency), and large enough that sum_q items_q <= items_cap:
     // items_q <= tasks_q/tpi_q + 1 <= 2*G_q*V_q/teff + 2 (tpi_q*T_q*V_q >= teff/2)
     const int64_t cap_left = items_cap - 2 * nq;
-    int64_t teff = (4 * total_slot_cells + cap_left - 1) / cap_left;
-    if (teff < kItemCells) teff = kItemCells;
+    int64_t teff = total_slot_cells / (4ll * grid);
+    if (teff > kItemCells) teff = kItemCells;
+    const int64_t teff_cap = (4 * total_slot_cells + cap_left - 1) / cap_left;
+    if (teff < teff_cap) teff = teff_cap;
+    if (teff < 1) teff = 1;
     const int64_t per = (nq + kPlanThreads - 1) / kPlanThreads;
     const int64_t q0 = min(nq, (int64_t)tid * per), q1 = min(nq, q0 + per);
     int64_t my_items = 0;
@@ -1098,17 +1102,30 @@ int ensure_stage(olap_cube* c, int64_t nq) {
 }
 
 // plan + reduce for nq queries already on the device; writes partials
+bool capturing(cudaStream_t st) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    return cudaStreamIsCapturing(st, &cs) == cudaSuccess && cs == cudaStreamCaptureStatusActive;
+}
+
+// plan + reduce for nq queries already on the device; writes partials.  Capturable into a
+// CUDA graph once the workspace has grown to nq (a warm-up call outside capture): inside a
+// capture the cross-stream workspace event and the profiling events are left out.
 int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int32_t* d_ops, int64_t* d_psum,
                  int32_t* d_pext, cudaStream_t st) {
+    const bool cap = capturing(st);
+    if (cap && nq > c->nq_cap)
+        return set_error(OLAP_E_STATE, "stream capture: run one batch of %lld queries outside capture first "
+                         "(the workspace cannot grow inside a CUDA graph)", (long long)nq);
     int rc = ensure_ws(c, nq);
     if (rc) return rc;
-    OLAP_CUDA_TRY(cudaStreamWaitEvent(st, c->ws_done, 0));
+    if (!cap) OLAP_CUDA_TRY(cudaStreamWaitEvent(st, c->ws_done, 0));
     OLAP_CUDA_TRY(cudaMemsetAsync(c->d_counter + 2, 0, 2 * sizeof(unsigned long long), st));
     desc_kernel<<<(int)((nq + kDescThreads - 1) / kDescThreads), kDescThreads, 0, st>>>(
         make_geo(c), nq, d_ranges, d_ops, c->d_desc, c->d_qtasks, c->d_qtv, c->d_done, d_psum, d_pext, c->d_counter + 2);
     OLAP_CUDA_TRY(cudaGetLastError());
     scan_kernel<<<1, kPlanThreads, 0, st>>>(nq, c->d_desc, c->d_qtasks, c->d_qtv, c->d_item_start, c->d_counter,
-                                            c->items_cap, c->d_counter + 2, c->d_counter + 1);
+                                            c->items_cap, c->d_counter + 2, c->d_counter + 1,
+                                            c->num_sms * c->blocks_per_sm);
     OLAP_CUDA_TRY(cudaGetLastError());
     const int32_t* order = nullptr;
     c->kernel_launches += 3;  // desc, scan, reduce
@@ -1125,7 +1142,8 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
     }
     const int grid = c->num_sms * c->blocks_per_sm;
     cudaEvent_t e0 = nullptr, e1 = nullptr;
-    if (c->prof) {
+    const bool prof = c->prof && !cap;
+    if (prof) {
         while (c->ev.size() < c->ev_used + 2) {
             cudaEvent_t e;
             OLAP_CUDA_TRY(cudaEventCreate(&e));
@@ -1145,11 +1163,11 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
             static_cast<const float*>(c->d_cells), nq, c->d_desc, c->d_item_start, c->d_counter, c->d_done,
             c->d_item_sum, c->d_item_ext, d_psum, d_pext, order);
     OLAP_CUDA_TRY(cudaGetLastError());
-    if (c->prof) {
+    if (prof) {
         OLAP_CUDA_TRY(cudaEventRecord(e1, st));
         ++c->launches;
     }
-    OLAP_CUDA_TRY(cudaEventRecord(c->ws_done, st));
+    if (!cap) OLAP_CUDA_TRY(cudaEventRecord(c->ws_done, st));
     return OLAP_OK;
 }
 
@@ -1474,13 +1492,17 @@ int olap_query_batch_device(olap_cube* c, int64_t nq, const olap_range* d_ranges
     std::lock_guard<std::mutex> lk(c->mu);
     DeviceGuard dg(c->device);
     cudaStream_t st = static_cast<cudaStream_t>(stream);
+    const bool cap = capturing(st);
+    if (cap && nq > c->stage_cap)
+        return set_error(OLAP_E_STATE, "stream capture: run one batch of %lld queries outside capture first",
+                         (long long)nq);
     rc = ensure_stage(c, nq);
     if (rc) return rc;
     rc = run_partials(c, nq, d_ranges, d_ops, c->d_psum, c->d_pext, st);
     if (rc) return rc;
     rc = launch_finalize(c->nd, c->n, c->dtype, nq, d_ranges, d_ops, c->d_psum, c->d_pext, d_results, st);
     if (rc) return rc;
-    OLAP_CUDA_TRY(cudaEventRecord(c->ws_done, st));
+    if (!cap) OLAP_CUDA_TRY(cudaEventRecord(c->ws_done, st));
     return OLAP_OK;
 }
 
