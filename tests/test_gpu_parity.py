@@ -677,3 +677,36 @@ def test_cuda_graph_capture_replay():
             with torch.cuda.graph(g2, stream=st):
                 c.query_device(big, torch.cat([do] * 8), torch.zeros(4096 * 24, dtype=torch.uint8, device="cuda"),
                                stream=torch.cuda.current_stream())
+
+
+@pytest.mark.parametrize("ext", [(9, 40, 33), (5, 7, 1000), (3, 3, 3, 64)])
+def test_full_range_int32_cells(ext):
+    """int32 cells over the whole int32 range: SUM through mad.wide (sign extension, int64),
+    MIN/MAX at the extremes, AVG = SUM/V — bit-exact vs the oracle."""
+    rng = np.random.default_rng(int(np.prod(ext)))
+    n = int(np.prod(ext))
+    cells = rng.integers(-(2 ** 31), 2 ** 31, size=n, dtype=np.int64).astype(np.int32)
+    cells[:3] = [-(2 ** 31), 2 ** 31 - 1, 0]
+    c = olap.Cube(ext, np.int32)
+    c.load(cells)
+    boxes = np.concatenate([synth.random_boxes(ext, 300, rng), np.array([[[0, e - 1] for e in ext]])])
+    for op in range(5):
+        ops = np.full(len(boxes), op, np.int32)
+        compare(c.query(boxes, ops), oracle.query(ext, boxes, ops, cells), ops, np.int32)
+
+
+def test_text_ranges_device_matches_host():
+    members = synth.tpcds_members()
+    cols = ["ca_state", "i_class", "s_store_id", "d_date"]
+    dg = [olap.Dict(members[c]) for c in cols]
+    ext = [len(members[c]) for c in cols]
+    qs = synth.tpcds_queries(2000, members, seed=123)
+    conds = [[q.get(c) if c != "d_date" else q[c] for c in cols] for q in qs]
+    want, wmiss = olap.text_ranges(dg, ext, conds)
+    kinds, first, rin, buf, offs = olap.pack_text_conditions(conds, 4)
+    out = torch.empty((len(conds), 4, 2), dtype=torch.int64, device="cuda")
+    miss = torch.zeros(1, dtype=torch.int64, device="cuda")
+    olap.text_ranges_device(dg, ext, len(conds), torch.from_numpy(kinds).cuda(), torch.from_numpy(first).cuda(), None,
+                            torch.from_numpy(buf.copy()).cuda(), torch.from_numpy(offs).cuda(), len(offs) - 1, out, miss)
+    torch.cuda.synchronize()
+    assert np.array_equal(out.cpu().numpy(), want) and int(miss.item()) == wmiss
