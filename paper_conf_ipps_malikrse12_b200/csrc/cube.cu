@@ -86,10 +86,10 @@ struct Extents {
 
 // ------------------------------------------------------------------ device helpers
 
-// Cube loads go through L1 (ld.global.nc, L1-allocating): with the L2-aware item order the
-// blocks resident on one SM often work on overlapping regions of different queries, and the
-// L1 (up to ~256 KB per SM; the reduce kernel asks for the maximum L1 carveout) catches
-// those re-reads.  Measured +9-10% over L1::no_allocate on C2a/C3/C4 (profiles/).
+// Cube loads use ld.global.nc (L1-allocating).  Measured +9-10% over L1::no_allocate on
+// C2a/C3/C4 once the data is L2-resident (profiles/sweep_r01_load_flavor.txt) although the
+// L1 hit rate stays ~2% (ncu): the no_allocate variant costs more L1TEX pipeline
+// throughput (80% vs 73% at the same work), which is what bounds the L2-served kernel.
 #ifndef OLAP_LD4
 #define OLAP_LD4 "ld.global.nc.v4.u32"
 #endif
