@@ -295,7 +295,10 @@ __device__ __forceinline__ void slot_masks(const QDesc& d, uint64_t& wf, uint64_
     wb = byte_mask_word(fm & lm);
 }
 
-constexpr int unroll_for(int V) { return V == 8 ? 2 : 4; }  // 64 B (or 16 B) of loads in flight per lane
+#ifndef OLAP_U8
+#define OLAP_U8 3
+#endif
+constexpr int unroll_for(int V) { return V == 8 ? OLAP_U8 : 4; }  // 32-B slots: OLAP_U8 x 32 B in flight per lane
 
 // Short runs (nslot <= kShortMaxSlots): a task is up to 31 whole runs.  Lane i holds
 // the first-slot address of run r0+i.  The interior slots of all the task's runs
