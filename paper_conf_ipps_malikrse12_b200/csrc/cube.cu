@@ -35,7 +35,11 @@ constexpr int kUnroll = OLAP_UNROLL;        // independent loads in flight per l
 #ifndef OLAP_MIN_BLOCKS
 #define OLAP_MIN_BLOCKS 4
 #endif
-constexpr int kMinBlocks = OLAP_MIN_BLOCKS;  // resident reduce blocks per SM the register budget targets
+constexpr int kMinBlocks = OLAP_MIN_BLOCKS;
+#ifndef OLAP_WARP_ITEMS
+#define OLAP_WARP_ITEMS 0
+#endif
+constexpr bool kWarpItems = OLAP_WARP_ITEMS != 0;  // warp-granular items (reduce_kernel_w) vs block items  // resident reduce blocks per SM the register budget targets
 constexpr int64_t kItemCells = 262144;      // minimum item: 1 MiB of 4-byte cells
 constexpr int64_t kMaxExtent = (1ll << 30); // per-dimension limit (32-bit digit arithmetic)
 constexpr int64_t kMaxCells = (1ll << 42);
@@ -295,20 +299,23 @@ __device__ __forceinline__ void slot_masks(const QDesc& d, uint64_t& wf, uint64_
     wb = byte_mask_word(fm & lm);
 }
 
+// loads in flight per lane: 32-B slots take 3 LDG.256 (long-run segments, and short runs of >= 16
+// slots) or 2 (runs of < 16 slots, where a third mostly re-reads masked slots); 16-B / 4-B slots 4.
+// Measured (profiles/sweep_r01_unroll.txt): C2a/C3/C4 gain 1-6% from the third load, C2b (runs of
+// 1-5 slots) loses 20% with it.
 #ifndef OLAP_U8
 #define OLAP_U8 3
 #endif
-constexpr int unroll_for(int V) { return V == 8 ? OLAP_U8 : 4; }  // 32-B slots: OLAP_U8 x 32 B in flight per lane
+constexpr int unroll_for(int V) { return V == 8 ? OLAP_U8 : 4; }
 
 // Short runs (nslot <= kShortMaxSlots): a task is up to 31 whole runs.  Lane i holds
 // the first-slot address of run r0+i.  The interior slots of all the task's runs
 // (slots 1..nslot-2) are flattened and streamed WITHOUT masks: slot g is run
 // j = g / (nslot-2) (fast division), slot 1 + g % (nslot-2), address via a shuffle.
 // The two edge slots of every run go through a short masked pass.
-template <class Acc, int OPC, int V>
+template <class Acc, int OPC, int V, int U>
 __device__ __forceinline__ void stream_short(const uint32_t* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
-                                             Acc& acc, int lane, int w) {
-    constexpr int U = unroll_for(V);
+                                             Acc& acc, int lane, int w, int ws) {
     int64_t t = t0 + w;
     if (t >= t1) return;
     const int rpt = d.T, nslot = (int)d.nslot;
@@ -317,7 +324,7 @@ __device__ __forceinline__ void stream_short(const uint32_t* __restrict__ cube, 
     slot_masks<V>(d, wf, wl, wb);
     const FastDiv fni = d.fni;
     const int64_t R = d.R;
-    for (; t < t1; t += kWarps) {
+    for (; t < t1; t += ws) {
         const int64_t r0 = t * rpt;
         const int nr = (int)min((int64_t)rpt, R - r0);
         const int64_t ra = lane < nr ? run_addr(d, r0 + lane) : 0;
@@ -397,7 +404,7 @@ __device__ __forceinline__ void stream_segment(const uint32_t* __restrict__ p, i
 // contiguous segments (the end of run j0 and the start of run j0+1).
 template <class Acc, int OPC, int V>
 __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
-                                            Acc& acc, int lane, int w) {
+                                            Acc& acc, int lane, int w, int ws) {
     int64_t t = t0 + w;
     if (t >= t1) return;
     const int T_ = d.T;
@@ -406,8 +413,8 @@ __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, c
     slot_masks<V>(d, wf, wl, wb);
     int64_t j0 = div64(t * T_, nslot);
     int64_t rem = t * T_ - j0 * nslot;
-    const int64_t step = (int64_t)kWarps * T_;
-    for (; t < t1; t += kWarps) {
+    const int64_t step = (int64_t)ws * T_;
+    for (; t < t1; t += ws) {
         const int64_t left = G - t * T_;
         const int n = left < T_ ? (int)left : T_;
         const int64_t in_run = nslot - rem;
@@ -425,12 +432,16 @@ __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, c
     }
 }
 
+// Tasks t0+w, t0+w+ws, ... < t1 of one query's item (ws warps share the item).
 template <typename T, class Acc, int OPC, int V>
 __device__ __forceinline__ void stream_tasks(const T* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
-                                             Acc& acc, int lane, int w) {
+                                             Acc& acc, int lane, int w, int ws = kWarps) {
     const uint32_t* c = reinterpret_cast<const uint32_t*>(cube);
-    if (d.shortp) stream_short<Acc, OPC, V>(c, d, t0, t1, acc, lane, w);
-    else stream_long<Acc, OPC, V>(c, d, t0, t1, acc, lane, w);
+    if (d.shortp) {
+        if (V == 8 && d.nslot < 16) stream_short<Acc, OPC, V, 2>(c, d, t0, t1, acc, lane, w, ws);
+        else stream_short<Acc, OPC, V, unroll_for(V)>(c, d, t0, t1, acc, lane, w, ws);
+    }
+    else stream_long<Acc, OPC, V>(c, d, t0, t1, acc, lane, w, ws);
 }
 
 // ------------------------------------------------------------------ plan
@@ -577,8 +588,10 @@ __global__ void __launch_bounds__(kPlanThreads) scan_kernel(int64_t nq, QDesc* d
     // block (latency), and large enough that sum_q items_q <= items_cap:
     // items_q <= tasks_q/tpi_q + 1 <= 2*G_q*V_q/teff + 2 (tpi_q*T_q*V_q >= teff/2)
     const int64_t cap_left = items_cap - 2 * nq;
-    int64_t teff = total_slot_cells / (4ll * grid);
-    if (teff > kItemCells) teff = kItemCells;
+    const int64_t workers = kWarpItems ? 8ll * grid : (int64_t)grid;
+    const int64_t target = kWarpItems ? kItemCells / 4 : kItemCells;
+    int64_t teff = total_slot_cells / (4ll * workers);
+    if (teff > target) teff = target;
     const int64_t teff_cap = (4 * total_slot_cells + cap_left - 1) / cap_left;
     if (teff < teff_cap) teff = teff_cap;
     if (teff < 1) teff = 1;
@@ -687,6 +700,101 @@ __global__ void scatter_kernel(int64_t nq, const int64_t* __restrict__ item_star
 
 // ------------------------------------------------------------------ reduce (the hot loop)
 
+// op-class x slot-width dispatch of one item's tasks
+template <typename T, class Acc>
+__device__ __forceinline__ void stream_item(const T* __restrict__ cube, const QDesc& sd, int64_t t0, int64_t t1, Acc& acc,
+                                            int lane, int w, int ws) {
+    const int opc = sd.opc;
+    if (sd.V == 8) {
+        if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 8>(cube, sd, t0, t1, acc, lane, w, ws);
+        else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 8>(cube, sd, t0, t1, acc, lane, w, ws);
+        else stream_tasks<T, Acc, OPC_MAX, 8>(cube, sd, t0, t1, acc, lane, w, ws);
+    } else if (sd.V == 4) {
+        if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 4>(cube, sd, t0, t1, acc, lane, w, ws);
+        else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 4>(cube, sd, t0, t1, acc, lane, w, ws);
+        else stream_tasks<T, Acc, OPC_MAX, 4>(cube, sd, t0, t1, acc, lane, w, ws);
+    } else {
+        if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 1>(cube, sd, t0, t1, acc, lane, w, ws);
+        else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 1>(cube, sd, t0, t1, acc, lane, w, ws);
+        else stream_tasks<T, Acc, OPC_MAX, 1>(cube, sd, t0, t1, acc, lane, w, ws);
+    }
+}
+
+// Warp-granular variant: every warp pops its own item, streams all of its tasks, and the
+// last warp to finish a query folds its item partials — no block barriers at all.
+template <typename T, class Acc>
+__global__ void __launch_bounds__(kThreads, kMinBlocks) reduce_kernel_w(const T* __restrict__ cube, int64_t nq,
+                                                               const QDesc* __restrict__ desc,
+                                                               const int64_t* __restrict__ item_start,
+                                                               unsigned long long* counter, int32_t* done,
+                                                               long long* item_sum, int32_t* item_ext, int64_t* psum,
+                                                               int32_t* pext, const int32_t* __restrict__ order) {
+    __shared__ QDesc sdw[kWarps];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    QDesc& sd = sdw[w];
+    const int64_t total = __ldg(item_start + nq);
+    for (;;) {
+        long long item = 0;
+        if (lane == 0) {
+            const int64_t slot = (int64_t)atomicAdd(counter, 1ull);
+            item = (order && slot < total) ? (long long)__ldg(order + slot) : (long long)slot;
+        }
+        item = __shfl_sync(0xffffffffu, item, 0);
+        if (item >= total) break;
+        const int64_t q = find_query(item_start, nq, item, lane);
+        {
+            const int* src = reinterpret_cast<const int*>(desc + q);
+            int* dst = reinterpret_cast<int*>(&sd);
+            for (int i = lane; i < (int)(sizeof(QDesc) / 4); i += 32) dst[i] = __ldg(src + i);
+        }
+        __syncwarp();
+        const int64_t first_item = __ldg(item_start + q);
+        const int64_t t0 = (item - first_item) * (int64_t)sd.tpi;
+        const int64_t t1 = min(sd.tasks, t0 + (int64_t)sd.tpi);
+        Acc acc;
+        acc.init();
+        const int opc = sd.opc;
+        stream_item<T, Acc>(cube, sd, t0, t1, acc, lane, 0, 1);
+        long long s = acc.sum_bits();
+        int32_t cmx = opc == OPC_MAX ? acc.code_max() : INT_MIN, cmn = opc == OPC_MIN ? ~acc.code_min() : INT_MIN;
+#pragma unroll
+        for (int o = 16; o; o >>= 1) s = SumOps<Acc>::add(s, __shfl_xor_sync(0xffffffffu, s, o));
+        cmx = __reduce_max_sync(0xffffffffu, cmx);
+        cmn = __reduce_max_sync(0xffffffffu, cmn);
+        const int64_t nitems = (sd.tasks + sd.tpi - 1) / sd.tpi;
+        int last = 0;
+        if (lane == 0) {
+            item_sum[item] = s;
+            item_ext[2 * item] = cmx;
+            item_ext[2 * item + 1] = cmn;
+            __threadfence();
+            last = atomicAdd(done + q, 1) == (int)nitems - 1;
+        }
+        last = __shfl_sync(0xffffffffu, last, 0);
+        if (last) {  // fold the query's item partials in fixed order
+            __threadfence();
+            long long ts = 0;
+            int32_t tmx = INT_MIN, tmn = INT_MIN;
+            for (int64_t i = lane; i < nitems; i += 32) {
+                const int64_t it = first_item + i;
+                ts = SumOps<Acc>::add(ts, __ldcg(item_sum + it));
+                tmx = max(tmx, __ldcg(item_ext + 2 * it));
+                tmn = max(tmn, __ldcg(item_ext + 2 * it + 1));
+            }
+#pragma unroll
+            for (int o = 16; o; o >>= 1) ts = SumOps<Acc>::add(ts, __shfl_xor_sync(0xffffffffu, ts, o));
+            tmx = __reduce_max_sync(0xffffffffu, tmx);
+            tmn = __reduce_max_sync(0xffffffffu, tmn);
+            if (lane == 0) {
+                psum[q] = ts;
+                pext[2 * q] = tmx;
+                pext[2 * q + 1] = tmn;
+            }
+        }
+        __syncwarp();
+    }
+}
+
 template <typename T, class Acc>
 __global__ void __launch_bounds__(kThreads, kMinBlocks) reduce_kernel(const T* __restrict__ cube, int64_t nq,
                                                              const QDesc* __restrict__ desc,
@@ -730,19 +838,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) reduce_kernel(const T* _
         Acc acc;
         acc.init();
         const int opc = sd.opc;
-        if (sd.V == 8) {
-            if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 8>(cube, sd, t0, t1, acc, lane, w);
-            else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 8>(cube, sd, t0, t1, acc, lane, w);
-            else stream_tasks<T, Acc, OPC_MAX, 8>(cube, sd, t0, t1, acc, lane, w);
-        } else if (sd.V == 4) {
-            if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 4>(cube, sd, t0, t1, acc, lane, w);
-            else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 4>(cube, sd, t0, t1, acc, lane, w);
-            else stream_tasks<T, Acc, OPC_MAX, 4>(cube, sd, t0, t1, acc, lane, w);
-        } else {
-            if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 1>(cube, sd, t0, t1, acc, lane, w);
-            else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 1>(cube, sd, t0, t1, acc, lane, w);
-            else stream_tasks<T, Acc, OPC_MAX, 1>(cube, sd, t0, t1, acc, lane, w);
-        }
+        stream_item<T, Acc>(cube, sd, t0, t1, acc, lane, w, kWarps);
 
         // warp -> block -> item partial (fixed order: deterministic)
         long long s = acc.sum_bits();
@@ -1058,7 +1154,7 @@ int ensure_ws(olap_cube* c, int64_t nq) {
     // few MiB (the L2-aware order needs the ~600 in-flight items to fit in L2): one per 4 KiB of
     // cube, <= 2^24 (a batch reads the cube ~10^2-10^3 times over at C3-like overlap)
     const int64_t by_size = std::min<int64_t>(1ll << 24, (c->local_cells * 4) >> 12);
-    int64_t items = std::max<int64_t>(std::max<int64_t>(1ll << 20, 4 * cap), by_size);
+    int64_t items = std::max<int64_t>(std::max<int64_t>(kWarpItems ? (1ll << 22) : (1ll << 20), 4 * cap), by_size);
     OLAP_CUDA_TRY(cudaMalloc(&c->d_desc, sizeof(QDesc) * cap));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_item_start, sizeof(int64_t) * (cap + 1)));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_done, sizeof(int32_t) * cap));
@@ -1157,7 +1253,16 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
         c->ev_used += 2;
         OLAP_CUDA_TRY(cudaEventRecord(e0, st));
     }
-    if (c->dtype == OLAP_INT32)
+    if (kWarpItems) {
+        if (c->dtype == OLAP_INT32)
+            reduce_kernel_w<int32_t, AccI><<<grid, kThreads, 0, st>>>(
+                static_cast<const int32_t*>(c->d_cells), nq, c->d_desc, c->d_item_start, c->d_counter, c->d_done,
+                c->d_item_sum, c->d_item_ext, d_psum, d_pext, order);
+        else
+            reduce_kernel_w<float, AccF><<<grid, kThreads, 0, st>>>(
+                static_cast<const float*>(c->d_cells), nq, c->d_desc, c->d_item_start, c->d_counter, c->d_done,
+                c->d_item_sum, c->d_item_ext, d_psum, d_pext, order);
+    } else if (c->dtype == OLAP_INT32)
         reduce_kernel<int32_t, AccI><<<grid, kThreads, 0, st>>>(
             static_cast<const int32_t*>(c->d_cells), nq, c->d_desc, c->d_item_start, c->d_counter, c->d_done,
             c->d_item_sum, c->d_item_ext, d_psum, d_pext, order);
@@ -1279,7 +1384,12 @@ int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_sh
                          cudaSharedmemCarveoutMaxL1);
     cudaFuncSetAttribute(reduce_kernel<float, AccF>, cudaFuncAttributePreferredSharedMemoryCarveout,
                          cudaSharedmemCarveoutMaxL1);
-    if (dtype == OLAP_INT32)
+    if (kWarpItems) {
+        if (dtype == OLAP_INT32)
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, reduce_kernel_w<int32_t, AccI>, kThreads, 0);
+        else
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, reduce_kernel_w<float, AccF>, kThreads, 0);
+    } else if (dtype == OLAP_INT32)
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, reduce_kernel<int32_t, AccI>, kThreads, 0);
     else
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, reduce_kernel<float, AccF>, kThreads, 0);
