@@ -528,6 +528,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--graph", action="store_true", help="replay each step as a captured CUDA graph (N=1)")
+    ap.add_argument("--batch", type=int, default=0, help="queries per batch (default: the config's)")
     args = ap.parse_args()
 
     rank, world, local = env_int("RANK", 0), env_int("WORLD_SIZE", 1), env_int("LOCAL_RANK", 0)
@@ -557,7 +558,7 @@ def main():
         else:
             dist.init_process_group(backend)
     ext, cfg = workload(args.workload, world)
-    nq = cfg["nq"]
+    nq = args.batch or cfg["nq"]
     dtype = cfg["dtype"]
     nd = len(ext)
     cube = olap.Cube(ext, dtype, shard=(world, rank, 1) if world > 1 else None, device=local)
