@@ -13,10 +13,12 @@ Functions (all cite the passage they follow in oracle.cpp):
   rollup(), convert_range()  PAPER.md:103-136, Fig. 1, Eq. 1-2 — multi-resolution cube set.
   tablescan()  Eq. 11-12, PAPER.md:206-216 — the paper's GPU query Q_D over a column store.
   fill()       the counter-based cell generator (independent re-implementation).
+  sched.Fig10  Fig. 10 / Eq. 4-18 — the CPU/GPU scheduling algorithm,
+               plain Python (oracle/sched.py), for the dispatcher.
 
 Parity of every function is pinned in tests/test_oracle_*.py against brute
 force (numpy slicing), an independent summed-area-table algorithm, the affine
-closed form, a hand-worked example and invariants; none is "parity unpinned".
+closed form, hand-worked examples (tests/golden/) and invariants; none is "parity unpinned".
 """
 from __future__ import annotations
 
