@@ -284,6 +284,78 @@ int olap_table_query_batch_device(olap_table* t, int64_t nq, const int64_t* d_co
 
 int olap_table_destroy(olap_table* t);
 
+/* A GPU partition for fact-table queries (Fig. 7: the paper
+ * splits its C2070 into partitions of 1, 2 and 4 SMs so several queries are answered
+ * concurrently, each by one partition).  A partition launches the scan on at most
+ * sm_count SMs' worth of blocks (sm_count x resident blocks per SM; sm_count <= 0 or
+ * above the device's SM count = every SM) with its own workspace, so partitions of one
+ * table may run concurrently on different streams.  Every scan reads only the columns
+ * the batch references: its conditions' columns plus, unless every query is COUNT,
+ * their data columns (Eq. 12). */
+typedef struct olap_table_part olap_table_part;
+int olap_table_part_create(olap_table* t, int sm_count, olap_table_part** out);
+int olap_table_part_sms(const olap_table_part* p, int* sm_count, int* blocks);
+
+/* olap_table_query_batch_device on the partition. */
+int olap_table_part_query_device(olap_table_part* p, int64_t nq, const int64_t* d_cond_offsets,
+                                 const olap_cond* d_conds, const int32_t* d_data_cols, const int32_t* d_ops,
+                                 olap_result* d_results, void* stream);
+
+/* Queries given as boxes over dimension columns, e.g. olap_text_ranges output: query q's
+ * condition on dimension d is column dim_cols[d] in d_boxes[q*ndims + d] (inclusive); a
+ * range covering all of [0, extents[d]) is no condition and reads no column (Eq. 12); an
+ * empty range matches nothing.  dim_cols and extents are HOST arrays of ndims <= 16. */
+int olap_table_part_query_boxes_device(olap_table_part* p, int64_t nq, int ndims, const int32_t* dim_cols,
+                                       const int64_t* extents, const olap_range* d_boxes,
+                                       const int32_t* d_data_cols, const int32_t* d_ops, olap_result* d_results,
+                                       void* stream);
+int olap_table_part_destroy(olap_table_part* p);
+
+/* ---------------------------------------------------------------- dispatcher (NEXT #4) */
+
+/* The paper's scheduling algorithm, Fig. 10 (§III-G), host code.
+ * Every query Q gets a deadline T_D = T_O + T_C.  Fig. 10 estimates Q's response time on
+ * every partition, then picks one:
+ *   - a cube partition that meets T_D and beats the fastest table partition;
+ *   - otherwise the slowest table partition that meets T_D;
+ *   - otherwise the partition that answers first.
+ * The partition's queue time T_Q is then advanced.  olap_sched_complete applies the
+ * paper's correction: real minus estimated processing time is added to
+ * the queue's T_Q.
+ *
+ * Performance function of a partition, Eq. 4, generalised:
+ *     T(x) = a1 * x^p1 + b1   if x < x_split        (range A)
+ *            a2 * x^p2 + b2   otherwise             (range B, reading R25)
+ * Eq. 7 / Eq. 10 (CPU cube model, x = SC_size in MB) and Eq. 14-15 (GPU table model,
+ * x = C_QD / C_TOTAL) are instances, and so is the B200 roofline T = bytes / BW + t0
+ * (DESIGN.md §8(f)). */
+typedef struct { double x_split, a1, p1, b1, a2, p2, b2; } olap_perf_fn;
+typedef enum { OLAP_PART_CUBE = 0, OLAP_PART_TABLE = 1 } olap_part_kind;
+/* CUBE partitions play the paper's CPU OLAP partition (answers from pre-computed cubes,
+ * x = cube_mb), TABLE partitions its GPU partitions (fact-table scan, x = col_frac).
+ * Partitions are listed in the order Fig. 10's FOR loop visits them (slow -> fast).
+ * needs_translation: the partition's queries pass through the translation queue first
+ * (the paper: GPU partitions only). */
+typedef struct { int32_t kind; int32_t needs_translation; olap_perf_fn perf; } olap_sched_partition;
+/* t_arrival = T_O (s); cube_mb = SC_size (Eq. 3) in MB of the cube that answers Q, < 0 if
+ * none can; col_frac = C_QD / C_TOTAL (Eq. 12-13), < 0 if no table can; t_trans = T_TRANS
+ * (Eq. 18) in s, 0 when Q has no text parameter. */
+typedef struct { double t_arrival, cube_mb, col_frac, t_trans; } olap_sched_query;
+/* partition = chosen index (-1: no partition can answer Q); translated = Q goes through the
+ * translation queue; t_response = estimated T_R; t_deadline = T_D; t_est = estimated
+ * processing time on the chosen partition (pass it back to olap_sched_complete). */
+typedef struct { int32_t partition, translated; double t_response, t_deadline, t_est; } olap_sched_decision;
+typedef struct olap_sched olap_sched;
+
+/* nparts in [1, 64]; t_c = T_C > 0 (s), +inf allowed. */
+int olap_sched_create(int nparts, const olap_sched_partition* parts, double t_c, olap_sched** out);
+/* Schedule n queries in order (online: each sees the queue state the previous left). */
+int olap_sched_submit(olap_sched* s, int64_t n, const olap_sched_query* qs, olap_sched_decision* out);
+int olap_sched_complete(olap_sched* s, int partition, double t_est, double t_real);
+/* t_q[0..nparts-1] = T_Q of every partition, t_q[nparts] = T_Q|TRANS. */
+int olap_sched_queues(const olap_sched* s, double* t_q);
+int olap_sched_destroy(olap_sched* s);
+
 /* ---------------------------------------------------------------- multi-resolution cube set */
 
 /* Resolution hierarchy (Fig. 1: "years (low resolution), months, days,

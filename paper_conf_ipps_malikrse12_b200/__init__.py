@@ -21,7 +21,9 @@ __all__ = ["Cube", "Dict", "OlapError", "translate", "shard_local_rows", "combin
            "finalize_device", "translate_device", "RESULT_DTYPE", "lib", "LIB_PATH",
            "INT32", "FLOAT32", "SUM", "COUNT", "MIN", "MAX", "AVG", "GEN_UNIFORM", "GEN_AFFINE",
            "RESULT_EMPTY", "RESULT_INVALID", "EXPORTS", "text_ranges", "text_ranges_device", "pack_text_conditions", "text_ranges_packed",
-           "COND_ALL", "COND_EQ", "COND_RANGE", "COND_IDS", "Table", "COND_DTYPE", "Hierarchy", "CubeSet"]
+           "COND_ALL", "COND_EQ", "COND_RANGE", "COND_IDS", "Table", "COND_DTYPE", "Hierarchy", "CubeSet",
+           "TablePart", "Scheduler", "PART_CUBE", "PART_TABLE", "SCHED_PART_DTYPE", "SCHED_QUERY_DTYPE",
+           "SCHED_DECISION_DTYPE", "perf_fn"]
 
 LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libolap_b200.so")
 if os.environ.get("OLAP_LIB"):          # development only: A/B a differently-tuned build of the same sources
@@ -34,6 +36,15 @@ RESULT_EMPTY, RESULT_INVALID = 1, 2
 COND_ALL, COND_EQ, COND_RANGE, COND_IDS = 0, 1, 2, 3
 
 OK, E_INVALID, E_RANGE, E_NOMEM, E_CUDA, E_STATE, E_UNSUPPORTED = 0, -1, -2, -3, -4, -6, -7
+
+PART_CUBE, PART_TABLE = 0, 1
+
+# olap_sched_partition / olap_sched_query / olap_sched_decision (include/olap.h, dispatcher)
+_PERF = [("x_split", "<f8"), ("a1", "<f8"), ("p1", "<f8"), ("b1", "<f8"), ("a2", "<f8"), ("p2", "<f8"), ("b2", "<f8")]
+SCHED_PART_DTYPE = np.dtype([("kind", "<i4"), ("needs_translation", "<i4")] + _PERF)
+SCHED_QUERY_DTYPE = np.dtype([("t_arrival", "<f8"), ("cube_mb", "<f8"), ("col_frac", "<f8"), ("t_trans", "<f8")])
+SCHED_DECISION_DTYPE = np.dtype([("partition", "<i4"), ("translated", "<i4"), ("t_response", "<f8"),
+                                 ("t_deadline", "<f8"), ("t_est", "<f8")])
 
 # olap_result: {int64 i; double d; uint32 flags; uint32 _pad}
 RESULT_DTYPE = np.dtype([("i", "<i8"), ("d", "<f8"), ("flags", "<u4"), ("pad", "<u4")])
@@ -76,6 +87,16 @@ EXPORTS = {
     "olap_table_query_batch": (_int, [_p, _i64, _p, _p, _p, _p, _p]),
     "olap_table_query_batch_device": (_int, [_p, _i64, _p, _p, _p, _p, _p, _p]),
     "olap_table_destroy": (_int, [_p]),
+    "olap_table_part_create": (_int, [_p, _int, ctypes.POINTER(_p)]),
+    "olap_table_part_sms": (_int, [_p, ctypes.POINTER(_int), ctypes.POINTER(_int)]),
+    "olap_table_part_query_device": (_int, [_p, _i64, _p, _p, _p, _p, _p, _p]),
+    "olap_table_part_query_boxes_device": (_int, [_p, _i64, _int, _p, _p, _p, _p, _p, _p, _p]),
+    "olap_table_part_destroy": (_int, [_p]),
+    "olap_sched_create": (_int, [_int, _p, ctypes.c_double, ctypes.POINTER(_p)]),
+    "olap_sched_submit": (_int, [_p, _i64, _p, _p]),
+    "olap_sched_complete": (_int, [_p, _int, ctypes.c_double, ctypes.c_double]),
+    "olap_sched_queues": (_int, [_p, _p]),
+    "olap_sched_destroy": (_int, [_p]),
     "olap_hier_create": (_int, [_int, _int, _p, _p, ctypes.POINTER(_p)]),
     "olap_hier_extents": (_int, [_p, _int, _p]),
     "olap_hier_convert": (_int, [_p, _i64, _p, _p, _int, _p]),
@@ -496,6 +517,92 @@ class Table:
     def close(self):
         if getattr(self, "_h", None):
             lib.olap_table_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class TablePart:
+    """A GPU partition of `sm_count` SMs for fact-table queries (Fig. 7)."""
+
+    def __init__(self, table: "Table", sm_count: int = 0):
+        h = ctypes.c_void_p()
+        _check(lib.olap_table_part_create(table._h, int(sm_count), ctypes.byref(h)), "olap_table_part_create")
+        self._h = h
+        self.table = table  # keeps the table alive
+        sm, bl = _int(), _int()
+        _check(lib.olap_table_part_sms(h, ctypes.byref(sm), ctypes.byref(bl)), "olap_table_part_sms")
+        self.sm_count, self.blocks = sm.value, bl.value
+
+    def query_device(self, nq: int, d_off, d_conds, d_dcol, d_ops, d_results, stream=None):
+        _check(lib.olap_table_part_query_device(self._h, nq, _ptr(d_off), _ptr(d_conds), _ptr(d_dcol), _ptr(d_ops),
+                                                _ptr(d_results), _stream(stream)), "olap_table_part_query_device")
+
+    def query_boxes_device(self, nq: int, dim_cols, extents, d_boxes, d_dcol, d_ops, d_results, stream=None):
+        dc = np.ascontiguousarray(dim_cols, dtype=np.int32)
+        ex = np.ascontiguousarray(extents, dtype=np.int64)
+        _check(lib.olap_table_part_query_boxes_device(self._h, nq, len(dc), dc.ctypes.data, ex.ctypes.data,
+                                                      _ptr(d_boxes), _ptr(d_dcol), _ptr(d_ops), _ptr(d_results),
+                                                      _stream(stream)), "olap_table_part_query_boxes_device")
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib.olap_table_part_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def perf_fn(a1, p1=1.0, b1=0.0, x_split=float("inf"), a2=0.0, p2=1.0, b2=0.0):
+    """Eq. 4 performance function: a1*x^p1 + b1 below x_split, a2*x^p2 + b2 from it on."""
+    return (x_split, a1, p1, b1, a2, p2, b2)
+
+
+class Scheduler:
+    """Fig. 10's dispatcher in the library (host code).
+
+    partitions: [(kind PART_CUBE / PART_TABLE, needs_translation, perf_fn(...))] in FOR-loop
+    order (slow -> fast); t_c: T_C in seconds."""
+
+    def __init__(self, partitions, t_c: float):
+        arr = np.zeros(len(partitions), dtype=SCHED_PART_DTYPE)
+        for i, (kind, needs, fn) in enumerate(partitions):
+            arr[i]["kind"], arr[i]["needs_translation"] = kind, int(bool(needs))
+            for k, v in zip(("x_split", "a1", "p1", "b1", "a2", "p2", "b2"), fn):
+                arr[i][k] = v
+        h = ctypes.c_void_p()
+        _check(lib.olap_sched_create(len(arr), arr.ctypes.data, float(t_c), ctypes.byref(h)), "olap_sched_create")
+        self._h = h
+        self.nparts = len(arr)
+
+    def submit(self, queries) -> np.ndarray:
+        """queries: SCHED_QUERY_DTYPE array or [(t_arrival, cube_mb, col_frac, t_trans)]."""
+        q = queries if isinstance(queries, np.ndarray) and queries.dtype == SCHED_QUERY_DTYPE else \
+            np.array([tuple(map(float, x)) for x in queries], dtype=SCHED_QUERY_DTYPE)
+        q = np.ascontiguousarray(q)
+        out = np.zeros(len(q), dtype=SCHED_DECISION_DTYPE)
+        _check(lib.olap_sched_submit(self._h, len(q), q.ctypes.data, out.ctypes.data), "olap_sched_submit")
+        return out
+
+    def complete(self, partition: int, t_est: float, t_real: float):
+        _check(lib.olap_sched_complete(self._h, int(partition), float(t_est), float(t_real)), "olap_sched_complete")
+
+    def queues(self):
+        out = np.zeros(self.nparts + 1, dtype=np.float64)
+        _check(lib.olap_sched_queues(self._h, out.ctypes.data), "olap_sched_queues")
+        return out
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib.olap_sched_destroy(self._h)
             self._h = None
 
     def __del__(self):

@@ -22,7 +22,7 @@ FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-I", INCLUDE,
 
 
 def sources():
-    return sorted(glob.glob(os.path.join(CSRC, "*.cu")))
+    return sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cpp")))
 
 
 def _deps():
@@ -37,7 +37,7 @@ def stale() -> bool:
 
 
 def build(force: bool = False, verbose: bool = False, defines=(), out: str | None = None) -> str:
-    """Compile csrc/*.cu -> libolap_b200.so (or `out`, with extra -D defines, for tuning sweeps)."""
+    """Compile csrc/*.cu + csrc/*.cpp -> libolap_b200.so (or `out`, with extra -D defines, for tuning sweeps)."""
     lib = out or LIB
     if not force and not defines and out is None and not stale():
         return LIB

@@ -61,10 +61,22 @@ __device__ __forceinline__ int32_t tf32_code(float f) {
 }
 __device__ __forceinline__ float tf32_decode(int32_t c) { return __int_as_float(c ^ ((c >> 31) & 0x7fffffff)); }
 
+// Columns the batch reads (Eq. 12): every condition's column, and the
+// data column unless the query is COUNT.  A query that cannot match reads nothing.
+// Called by every thread of a query-per-thread kernel (the trailing threads of the last
+// block return early, so the OR is a plain atomic, not a warp-collective one).
+__device__ __forceinline__ void note_columns(const TQuery& t, uint32_t* colmask) {
+    if (t.flags || t.ncond < 0) return;
+    uint32_t m = t.op != OLAP_COUNT ? 1u << t.data_col : 0u;
+    for (int k = 0; k < t.ncond; ++k) m |= 1u << t.c[k].col;
+    if (m) atomicOr(colmask, m);
+}
+
 // conditions -> TQuery (one thread per query)
 __global__ void table_prep_kernel(int64_t nq, int ncols, TableCols tc, const int64_t* __restrict__ off,
                                   const olap_cond* __restrict__ conds, const int32_t* __restrict__ data_cols,
-                                  const int32_t* __restrict__ ops, TQuery* __restrict__ qs) {
+                                  const int32_t* __restrict__ ops, TQuery* __restrict__ qs,
+                                  uint32_t* __restrict__ colmask) {
     const int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (q >= nq) return;
     TQuery t;
@@ -97,6 +109,47 @@ __global__ void table_prep_kernel(int64_t nq, int ncols, TableCols tc, const int
     }
     if (impossible && !t.flags) t.ncond = -1;  // no row can match
     qs[q] = t;
+    note_columns(t, colmask);
+}
+
+// Column-map of box queries: dimension d is column col[d] with members [0, extent[d]).
+struct BoxMap {
+    int32_t ndims;
+    int32_t col[kMaxConds];
+    int64_t extent[kMaxConds];
+};
+
+// boxes -> TQuery: a range covering the whole dimension is no condition (reads no column).
+__global__ void table_prep_boxes_kernel(int64_t nq, int ncols, TableCols tc, BoxMap bm,
+                                        const olap_range* __restrict__ boxes, const int32_t* __restrict__ data_cols,
+                                        const int32_t* __restrict__ ops, TQuery* __restrict__ qs,
+                                        uint32_t* __restrict__ colmask) {
+    const int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (q >= nq) return;
+    TQuery t;
+    t.flags = 0;
+    t.op = ops[q];
+    t.data_col = data_cols[q];
+    t.ncond = 0;
+    if (t.op < OLAP_SUM || t.op > OLAP_AVG || t.data_col < 0 || t.data_col >= ncols) t.flags = OLAP_RESULT_INVALID;
+    bool impossible = false;
+    for (int d = 0; d < bm.ndims && !t.flags; ++d) {
+        const olap_range r = boxes[q * bm.ndims + d];
+        if (r.lo > r.hi) {
+            impossible = true;
+            continue;
+        }
+        if (r.lo <= 0 && r.hi >= bm.extent[d] - 1) continue;  // the whole dimension: no condition
+        const int64_t lo = r.lo < INT_MIN ? (int64_t)INT_MIN : r.lo;
+        const int64_t hi = r.hi > INT_MAX ? (int64_t)INT_MAX : r.hi;
+        TCond& c = t.c[t.ncond++];
+        c.col = bm.col[d];
+        c.lo = (uint32_t)(int32_t)lo;
+        c.span = (uint32_t)(hi - lo);
+    }
+    if (impossible && !t.flags) t.ncond = -1;
+    qs[q] = t;
+    note_columns(t, colmask);
 }
 
 // One query on one staged tile.  Lane l owns rows l, l+32, ..., l+992: every condition
@@ -167,8 +220,10 @@ __device__ __forceinline__ void scan_query_tile(const uint32_t* __restrict__ sme
 // warp w evaluates queries w, w+8, ... on every staged tile.
 __global__ void __launch_bounds__(kScanThreads) table_scan_kernel(TableCols tc, int ncols, int64_t nrows, int64_t nq,
                                                                   const TQuery* __restrict__ qs,
-                                                                  TPartial* __restrict__ part) {
-    extern __shared__ uint32_t smem[];  // ncols x kTileRows
+                                                                  TPartial* __restrict__ part,
+                                                                  const uint32_t* __restrict__ colmask) {
+    extern __shared__ uint32_t smem[];  // ncols x kTileRows (only the batch's columns are staged)
+    const uint32_t used = *colmask;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int64_t ntiles = (nrows + kTileRows - 1) / kTileRows;
     TPartial* mine = part + (int64_t)blockIdx.x * nq;
@@ -185,9 +240,15 @@ __global__ void __launch_bounds__(kScanThreads) table_scan_kernel(TableCols tc, 
         const int rows = (int)min((int64_t)kTileRows, nrows - r0);
         __syncthreads();  // previous tile fully consumed
         for (int c = 0; c < ncols; ++c) {
+            if (!((used >> c) & 1u)) continue;
             const uint32_t* src = tc.col[c] + r0;
             uint32_t* dst = smem + c * kTileRows;
-            for (int r = threadIdx.x; r < rows; r += kScanThreads) dst[r] = __ldg(src + r);
+            if (rows == kTileRows) {  // column starts are 256-B aligned: one 16-B load per thread
+                static_assert(kTileRows == 4 * kScanThreads, "one uint4 per thread per column");
+                reinterpret_cast<uint4*>(dst)[threadIdx.x] = __ldg(reinterpret_cast<const uint4*>(src) + threadIdx.x);
+            } else {
+                for (int r = threadIdx.x; r < rows; r += kScanThreads) dst[r] = __ldg(src + r);
+            }
         }
         __syncthreads();
         for (int64_t q = w; q < nq; q += kScanWarps) {
@@ -263,6 +324,18 @@ __global__ void table_final_kernel(TableCols tc, int64_t nq, int nblocks, const 
 
 using namespace olap;
 
+// Launch workspace: per-query descriptors and per-(block, query) partials.  The table's
+// own calls use one; every partition (olap_table_part) has its own, so partitions run
+// concurrently.
+struct TWork {
+    int sm_count = 0, blocks = 0;
+    int64_t nq_cap = 0;
+    TQuery* d_qs = nullptr;
+    TPartial* d_part = nullptr;
+    uint32_t* d_colmask = nullptr;
+    std::mutex mu;
+};
+
 struct olap_table {
     int device = 0;
     int64_t nrows = 0;
@@ -270,19 +343,23 @@ struct olap_table {
     int32_t dtype[kMaxTableCols] = {};
     void* d_data = nullptr;      // all columns one after another, 256-B aligned
     int64_t col_stride = 0;      // cells between column starts
-    std::mutex mu;
+    std::mutex mu;               // host staging buffers below
     cudaStream_t stream = nullptr;
-    int num_sms = 0, blocks = 0;
-    int64_t nq_cap = 0;
-    TQuery* d_qs = nullptr;
-    TPartial* d_part = nullptr;
+    int num_sms = 0, blocks_per_sm = 0;
+    TWork work;
+    olap_result* d_res = nullptr;
+    int64_t res_cap = 0;
     olap_cond* d_conds = nullptr;
     int64_t conds_cap = 0;
     int64_t* d_off = nullptr;
     int32_t* d_dcol = nullptr;
     int32_t* d_ops = nullptr;
-    olap_result* d_res = nullptr;
     int64_t launches = 0;
+};
+
+struct olap_table_part {
+    olap_table* t = nullptr;
+    TWork work;
 };
 
 namespace {
@@ -307,39 +384,63 @@ TableCols cols_of(const olap_table* t) {
     return tc;
 }
 
-void free_tws(olap_table* t) {
-    cudaFree(t->d_qs);
-    cudaFree(t->d_part);
-    cudaFree(t->d_off);
-    cudaFree(t->d_dcol);
-    cudaFree(t->d_ops);
-    cudaFree(t->d_res);
-    t->d_qs = nullptr;
-    t->d_part = nullptr;
-    t->d_off = nullptr;
-    t->d_dcol = nullptr;
-    t->d_ops = nullptr;
-    t->d_res = nullptr;
-    t->nq_cap = 0;
+void free_work(TWork& w) {
+    cudaFree(w.d_qs);
+    cudaFree(w.d_part);
+    cudaFree(w.d_colmask);
+    w.d_qs = nullptr;
+    w.d_part = nullptr;
+    w.d_colmask = nullptr;
+    w.nq_cap = 0;
 }
 
-int ensure_tws(olap_table* t, int64_t nq, int64_t nconds) {
-    if (nq > t->nq_cap) {
-        OLAP_CUDA_TRY(cudaStreamSynchronize(t->stream));
-        free_tws(t);
+void init_work(const olap_table* t, TWork& w, int sm_count) {
+    w.sm_count = (sm_count <= 0 || sm_count > t->num_sms) ? t->num_sms : sm_count;
+    w.blocks = w.sm_count * std::max(t->blocks_per_sm, 1);
+}
+
+// (re)size a workspace; `st` is the stream its previous launches were queued on
+int ensure_work(TWork& w, int64_t nq, cudaStream_t st) {
+    if (!w.d_colmask) OLAP_CUDA_TRY(cudaMalloc(&w.d_colmask, sizeof(uint32_t)));
+    if (nq > w.nq_cap) {
+        OLAP_CUDA_TRY(cudaStreamSynchronize(st));
+        cudaFree(w.d_qs);
+        cudaFree(w.d_part);
+        w.d_qs = nullptr;
+        w.d_part = nullptr;
+        w.nq_cap = 0;
         const int64_t cap = std::max<int64_t>(nq, 256);
-        OLAP_CUDA_TRY(cudaMalloc(&t->d_qs, sizeof(TQuery) * cap));
-        OLAP_CUDA_TRY(cudaMalloc(&t->d_part, sizeof(TPartial) * cap * t->blocks));
+        OLAP_CUDA_TRY(cudaMalloc(&w.d_qs, sizeof(TQuery) * cap));
+        OLAP_CUDA_TRY(cudaMalloc(&w.d_part, sizeof(TPartial) * cap * w.blocks));
+        w.nq_cap = cap;
+    }
+    return OLAP_OK;
+}
+
+int ensure_staging(olap_table* t, int64_t nq, int64_t nconds) {
+    if (nq > t->res_cap) {
+        OLAP_CUDA_TRY(cudaStreamSynchronize(t->stream));
+        cudaFree(t->d_off);
+        cudaFree(t->d_dcol);
+        cudaFree(t->d_ops);
+        cudaFree(t->d_res);
+        t->d_off = nullptr;
+        t->d_dcol = nullptr;
+        t->d_ops = nullptr;
+        t->d_res = nullptr;
+        t->res_cap = 0;
+        const int64_t cap = std::max<int64_t>(nq, 256);
         OLAP_CUDA_TRY(cudaMalloc(&t->d_off, sizeof(int64_t) * (cap + 1)));
         OLAP_CUDA_TRY(cudaMalloc(&t->d_dcol, sizeof(int32_t) * cap));
         OLAP_CUDA_TRY(cudaMalloc(&t->d_ops, sizeof(int32_t) * cap));
         OLAP_CUDA_TRY(cudaMalloc(&t->d_res, sizeof(olap_result) * cap));
-        t->nq_cap = cap;
+        t->res_cap = cap;
     }
     if (nconds > t->conds_cap) {
         OLAP_CUDA_TRY(cudaStreamSynchronize(t->stream));
         cudaFree(t->d_conds);
         t->d_conds = nullptr;
+        t->conds_cap = 0;
         const int64_t cap = std::max<int64_t>(nconds, 1024);
         OLAP_CUDA_TRY(cudaMalloc(&t->d_conds, sizeof(olap_cond) * cap));
         t->conds_cap = cap;
@@ -347,16 +448,33 @@ int ensure_tws(olap_table* t, int64_t nq, int64_t nconds) {
     return OLAP_OK;
 }
 
-int launch_scan(olap_table* t, int64_t nq, const int64_t* d_off, const olap_cond* d_conds, const int32_t* d_dcol,
-                const int32_t* d_ops, olap_result* d_res, cudaStream_t st) {
+// scan + fold, after a prep kernel has written w.d_qs and w.d_colmask on `st`
+int launch_scan_fold(olap_table* t, TWork& w, int64_t nq, olap_result* d_res, cudaStream_t st) {
     const TableCols tc = cols_of(t);
-    table_prep_kernel<<<(int)((nq + 255) / 256), 256, 0, st>>>(nq, t->ncols, tc, d_off, d_conds, d_dcol, d_ops, t->d_qs);
     const size_t smem = sizeof(uint32_t) * kTileRows * t->ncols;
-    table_scan_kernel<<<t->blocks, kScanThreads, smem, st>>>(tc, t->ncols, t->nrows, nq, t->d_qs, t->d_part);
-    table_final_kernel<<<(int)((nq + 255) / 256), 256, 0, st>>>(tc, nq, t->blocks, t->d_qs, t->d_part, d_res);
+    table_scan_kernel<<<w.blocks, kScanThreads, smem, st>>>(tc, t->ncols, t->nrows, nq, w.d_qs, w.d_part, w.d_colmask);
+    table_final_kernel<<<(int)((nq + 255) / 256), 256, 0, st>>>(tc, nq, w.blocks, w.d_qs, w.d_part, d_res);
     OLAP_CUDA_TRY(cudaGetLastError());
-    t->launches += 3;
+    __atomic_fetch_add(&t->launches, 3, __ATOMIC_RELAXED);
     return OLAP_OK;
+}
+
+int launch_scan(olap_table* t, TWork& w, int64_t nq, const int64_t* d_off, const olap_cond* d_conds,
+                const int32_t* d_dcol, const int32_t* d_ops, olap_result* d_res, cudaStream_t st) {
+    const TableCols tc = cols_of(t);
+    OLAP_CUDA_TRY(cudaMemsetAsync(w.d_colmask, 0, sizeof(uint32_t), st));
+    table_prep_kernel<<<(int)((nq + 255) / 256), 256, 0, st>>>(nq, t->ncols, tc, d_off, d_conds, d_dcol, d_ops,
+                                                               w.d_qs, w.d_colmask);
+    return launch_scan_fold(t, w, nq, d_res, st);
+}
+
+int launch_scan_boxes(olap_table* t, TWork& w, int64_t nq, const BoxMap& bm, const olap_range* d_boxes,
+                      const int32_t* d_dcol, const int32_t* d_ops, olap_result* d_res, cudaStream_t st) {
+    const TableCols tc = cols_of(t);
+    OLAP_CUDA_TRY(cudaMemsetAsync(w.d_colmask, 0, sizeof(uint32_t), st));
+    table_prep_boxes_kernel<<<(int)((nq + 255) / 256), 256, 0, st>>>(nq, t->ncols, tc, bm, d_boxes, d_dcol, d_ops,
+                                                                     w.d_qs, w.d_colmask);
+    return launch_scan_fold(t, w, nq, d_res, st);
 }
 
 }  // namespace
@@ -397,7 +515,8 @@ int olap_table_create(int64_t nrows, int ncols, const int32_t* dtypes, int devic
         cudaFuncSetAttribute(table_scan_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     int bps = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, table_scan_kernel, kScanThreads, smem);
-    t->blocks = t->num_sms * std::max(bps, 1);
+    t->blocks_per_sm = std::max(bps, 1);
+    init_work(t, t->work, 0);
     *out = t;
     return OLAP_OK;
 }
@@ -429,11 +548,12 @@ int olap_table_query_batch_device(olap_table* t, int64_t nq, const int64_t* d_co
     if (nq < 0) return set_error(OLAP_E_INVALID, "nq < 0");
     if (nq == 0) return OLAP_OK;
     if (!d_cond_offsets || !d_data_cols || !d_ops || !d_results) return set_error(OLAP_E_INVALID, "NULL device buffer");
-    std::lock_guard<std::mutex> lk(t->mu);
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    std::lock_guard<std::mutex> lk(t->work.mu);
     TDevGuard g(t->device);
-    int rc = ensure_tws(t, nq, 0);
+    int rc = ensure_work(t->work, nq, st);
     if (rc) return rc;
-    return launch_scan(t, nq, d_cond_offsets, d_conds, d_data_cols, d_ops, d_results, static_cast<cudaStream_t>(stream));
+    return launch_scan(t, t->work, nq, d_cond_offsets, d_conds, d_data_cols, d_ops, d_results, st);
 }
 
 int olap_table_query_batch(olap_table* t, int64_t nq, const int64_t* cond_offsets, const olap_cond* conds,
@@ -459,16 +579,19 @@ int olap_table_query_batch(olap_table* t, int64_t nq, const int64_t* cond_offset
     }
     const int64_t nconds = cond_offsets[nq];
     std::lock_guard<std::mutex> lk(t->mu);
+    std::lock_guard<std::mutex> lw(t->work.mu);
     TDevGuard g(t->device);
-    int rc = ensure_tws(t, nq, nconds);
-    if (rc) return rc;
     cudaStream_t st = t->stream;
+    int rc = ensure_staging(t, nq, nconds);
+    if (rc) return rc;
+    rc = ensure_work(t->work, nq, st);
+    if (rc) return rc;
     OLAP_CUDA_TRY(cudaMemcpyAsync(t->d_off, cond_offsets, sizeof(int64_t) * (nq + 1), cudaMemcpyHostToDevice, st));
     if (nconds)
         OLAP_CUDA_TRY(cudaMemcpyAsync(t->d_conds, conds, sizeof(olap_cond) * nconds, cudaMemcpyHostToDevice, st));
     OLAP_CUDA_TRY(cudaMemcpyAsync(t->d_dcol, data_cols, sizeof(int32_t) * nq, cudaMemcpyHostToDevice, st));
     OLAP_CUDA_TRY(cudaMemcpyAsync(t->d_ops, ops, sizeof(int32_t) * nq, cudaMemcpyHostToDevice, st));
-    rc = launch_scan(t, nq, t->d_off, t->d_conds, t->d_dcol, t->d_ops, t->d_res, st);
+    rc = launch_scan(t, t->work, nq, t->d_off, t->d_conds, t->d_dcol, t->d_ops, t->d_res, st);
     if (rc) return rc;
     OLAP_CUDA_TRY(cudaMemcpyAsync(results, t->d_res, sizeof(olap_result) * nq, cudaMemcpyDeviceToHost, st));
     OLAP_CUDA_TRY(cudaStreamSynchronize(st));
@@ -479,12 +602,91 @@ int olap_table_destroy(olap_table* t) {
     clear_error();
     if (!t) return OLAP_OK;
     TDevGuard g(t->device);
-    if (t->stream) cudaStreamSynchronize(t->stream);
-    free_tws(t);
+    cudaDeviceSynchronize();  // the table's and its partitions' launches (any stream)
+    free_work(t->work);
+    cudaFree(t->d_off);
+    cudaFree(t->d_dcol);
+    cudaFree(t->d_ops);
+    cudaFree(t->d_res);
     cudaFree(t->d_conds);
     cudaFree(t->d_data);
     if (t->stream) cudaStreamDestroy(t->stream);
     delete t;
+    return OLAP_OK;
+}
+
+int olap_table_part_create(olap_table* t, int sm_count, olap_table_part** out) {
+    clear_error();
+    if (!t || !out) return set_error(OLAP_E_INVALID, "NULL argument");
+    olap_table_part* p = new (std::nothrow) olap_table_part();
+    if (!p) return set_error(OLAP_E_NOMEM, "host allocation failed");
+    p->t = t;
+    init_work(t, p->work, sm_count);
+    *out = p;
+    return OLAP_OK;
+}
+
+int olap_table_part_sms(const olap_table_part* p, int* sm_count, int* blocks) {
+    clear_error();
+    if (!p) return set_error(OLAP_E_INVALID, "NULL argument");
+    if (sm_count) *sm_count = p->work.sm_count;
+    if (blocks) *blocks = p->work.blocks;
+    return OLAP_OK;
+}
+
+int olap_table_part_query_device(olap_table_part* p, int64_t nq, const int64_t* d_cond_offsets,
+                                 const olap_cond* d_conds, const int32_t* d_data_cols, const int32_t* d_ops,
+                                 olap_result* d_results, void* stream) {
+    clear_error();
+    if (!p) return set_error(OLAP_E_INVALID, "partition handle is NULL");
+    if (nq < 0) return set_error(OLAP_E_INVALID, "nq < 0");
+    if (nq == 0) return OLAP_OK;
+    if (!d_cond_offsets || !d_data_cols || !d_ops || !d_results) return set_error(OLAP_E_INVALID, "NULL device buffer");
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    std::lock_guard<std::mutex> lk(p->work.mu);
+    TDevGuard g(p->t->device);
+    int rc = ensure_work(p->work, nq, st);
+    if (rc) return rc;
+    return launch_scan(p->t, p->work, nq, d_cond_offsets, d_conds, d_data_cols, d_ops, d_results, st);
+}
+
+int olap_table_part_query_boxes_device(olap_table_part* p, int64_t nq, int ndims, const int32_t* dim_cols,
+                                       const int64_t* extents, const olap_range* d_boxes,
+                                       const int32_t* d_data_cols, const int32_t* d_ops, olap_result* d_results,
+                                       void* stream) {
+    clear_error();
+    if (!p) return set_error(OLAP_E_INVALID, "partition handle is NULL");
+    if (nq < 0) return set_error(OLAP_E_INVALID, "nq < 0");
+    if (nq == 0) return OLAP_OK;
+    if (ndims < 1 || ndims > kMaxConds) return set_error(OLAP_E_INVALID, "ndims %d not in [1,16]", ndims);
+    if (!dim_cols || !extents || !d_boxes || !d_data_cols || !d_ops || !d_results)
+        return set_error(OLAP_E_INVALID, "NULL buffer");
+    olap_table* t = p->t;
+    BoxMap bm;
+    std::memset(&bm, 0, sizeof(bm));
+    bm.ndims = ndims;
+    for (int d = 0; d < ndims; ++d) {
+        if (dim_cols[d] < 0 || dim_cols[d] >= t->ncols || t->dtype[dim_cols[d]] != OLAP_INT32)
+            return set_error(OLAP_E_INVALID, "dimension %d: column %d is not an int32 column", d, dim_cols[d]);
+        if (extents[d] < 1) return set_error(OLAP_E_INVALID, "dimension %d: extent < 1", d);
+        bm.col[d] = dim_cols[d];
+        bm.extent[d] = extents[d];
+    }
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    std::lock_guard<std::mutex> lk(p->work.mu);
+    TDevGuard g(t->device);
+    int rc = ensure_work(p->work, nq, st);
+    if (rc) return rc;
+    return launch_scan_boxes(t, p->work, nq, bm, d_boxes, d_data_cols, d_ops, d_results, st);
+}
+
+int olap_table_part_destroy(olap_table_part* p) {
+    clear_error();
+    if (!p) return OLAP_OK;
+    TDevGuard g(p->t->device);
+    cudaDeviceSynchronize();
+    free_work(p->work);
+    delete p;
     return OLAP_OK;
 }
 
