@@ -710,3 +710,114 @@ def test_text_ranges_device_matches_host():
                             torch.from_numpy(buf.copy()).cuda(), torch.from_numpy(offs).cuda(), len(offs) - 1, out, miss)
     torch.cuda.synchronize()
     assert np.array_equal(out.cpu().numpy(), want) and int(miss.item()) == wmiss
+
+
+# ------------------------------------------------------------------ fact-table partitions (NEXT #4, Fig. 7)
+
+def _check_table(got, ref, cols, qs):
+    ops = np.array([q[2] for q in qs], np.int32)
+    isf = np.array([cols[q[1]].dtype == np.float32 for q in qs])
+    assert np.array_equal(got["flags"], ref["flags"]) and np.array_equal(got["i"], ref["i"])
+    ex = ~isf | (ops == olap.MIN) | (ops == olap.MAX) | (ops == olap.COUNT)
+    assert np.array_equal(got["d"][ex], ref["d"][ex])
+    tol = 1e-6 * np.abs(ref["d"]) + 1e-300
+    assert (np.abs(got["d"] - ref["d"]) <= tol).all()
+
+
+def _dev_table_queries(qs):
+    off, ca, dcol, ops = olap.pack_table_queries(qs)
+    return [torch.from_numpy(a.view(np.uint8) if a.dtype.names else a).cuda() for a in (off, ca, dcol, ops)]
+
+
+@pytest.mark.parametrize("sm_count", [1, 2, 4, 37, 0])
+def test_table_partition_parity(sm_count):
+    """A partition of 1/2/4 SMs (the paper's Fig. 7 sizes), an odd count and the whole GPU:
+    same answers as the oracle, grid bounded by the partition."""
+    nrows = 200_003
+    rng = np.random.default_rng(sm_count + 100)
+    cols = _table_cols(nrows, rng)
+    t = olap.Table(nrows, [c.dtype for c in cols])
+    for i, c in enumerate(cols):
+        t.load_column(i, c)
+    p = olap.TablePart(t, sm_count)
+    nsm = torch.cuda.get_device_properties(0).multi_processor_count
+    assert p.sm_count == (sm_count if 0 < sm_count <= nsm else nsm)
+    assert 1 <= p.blocks and p.blocks % p.sm_count == 0
+    qs = _table_queries(rng, 300)
+    qs.append(([], 5, olap.SUM))
+    qs.append(([(1, 3, 3), (1, 4, 4)], 4, olap.MIN))        # contradictory -> empty
+    qs.append(([(0, 0, 39)], 1, olap.COUNT))                 # every query COUNT-free columns mix
+    d = _dev_table_queries(qs)
+    res = torch.empty(len(qs) * olap.RESULT_DTYPE.itemsize, dtype=torch.uint8, device="cuda")
+    p.query_device(len(qs), *d, res)
+    torch.cuda.synchronize()
+    got = res.cpu().numpy().view(olap.RESULT_DTYPE)
+    _check_table(got, oracle.tablescan(cols, qs, nthreads=oracle.max_threads()), cols, qs)
+
+
+def test_table_partitions_concurrent_streams():
+    """Six partitions of 1/1/2/2/4/4 SMs (Fig. 7) on one table, each on its own stream,
+    launched back to back: every batch equals the oracle (own workspaces, no sharing)."""
+    nrows = 100_000
+    rng = np.random.default_rng(7)
+    cols = _table_cols(nrows, rng)
+    t = olap.Table(nrows, [c.dtype for c in cols])
+    for i, c in enumerate(cols):
+        t.load_column(i, c)
+    parts = [olap.TablePart(t, s) for s in (1, 1, 2, 2, 4, 4)]
+    streams = [torch.cuda.Stream() for _ in parts]
+    batches, outs = [], []
+    for p, s in zip(parts, streams):
+        qs = _table_queries(rng, int(rng.integers(1, 120)))
+        d = _dev_table_queries(qs)
+        res = torch.empty(len(qs) * olap.RESULT_DTYPE.itemsize, dtype=torch.uint8, device="cuda")
+        torch.cuda.current_stream().synchronize()
+        with torch.cuda.stream(s):
+            p.query_device(len(qs), *d, res, stream=s)
+        batches.append((qs, d))
+        outs.append(res)
+    torch.cuda.synchronize()
+    for (qs, _d), res in zip(batches, outs):
+        got = res.cpu().numpy().view(olap.RESULT_DTYPE)
+        _check_table(got, oracle.tablescan(cols, qs, nthreads=oracle.max_threads()), cols, qs)
+
+
+def test_table_partition_boxes():
+    """Box-form queries over dimension columns (e.g. olap_text_ranges output): a full-range
+    dimension is no condition, an empty range matches nothing; equal to the oracle on the
+    equivalent condition lists."""
+    nrows = 150_001
+    rng = np.random.default_rng(3)
+    cols = _table_cols(nrows, rng)
+    ext = (40, 7, 13, 5)
+    t = olap.Table(nrows, [c.dtype for c in cols])
+    for i, c in enumerate(cols):
+        t.load_column(i, c)
+    p = olap.TablePart(t, 4)
+    nq = 400
+    lo = np.zeros((nq, 4), np.int64)
+    hi = np.zeros((nq, 4), np.int64)
+    for q in range(nq):
+        for d, n in enumerate(ext):
+            r = rng.random()
+            if r < 0.4:
+                lo[q, d], hi[q, d] = 0, n - 1                     # full: no condition
+            elif r < 0.45:
+                lo[q, d], hi[q, d] = 1, 0                         # empty
+            else:
+                a, b = sorted(rng.integers(0, n, size=2))
+                lo[q, d], hi[q, d] = a, b
+    dcol = rng.integers(4, 6, size=nq).astype(np.int32)
+    ops = rng.integers(0, 5, size=nq).astype(np.int32)
+    flat = np.stack([lo, hi], axis=-1).reshape(-1)                # olap_range {lo, hi} query-major
+    qs = []
+    for q in range(nq):
+        conds = [(d, int(lo[q, d]), int(hi[q, d])) for d in range(4)
+                 if not (lo[q, d] == 0 and hi[q, d] == ext[d] - 1)]
+        qs.append((conds, int(dcol[q]), int(ops[q])))
+    res = torch.empty(nq * olap.RESULT_DTYPE.itemsize, dtype=torch.uint8, device="cuda")
+    p.query_boxes_device(nq, [0, 1, 2, 3], ext, torch.from_numpy(flat).cuda(), torch.from_numpy(dcol).cuda(),
+                         torch.from_numpy(ops).cuda(), res)
+    torch.cuda.synchronize()
+    got = res.cpu().numpy().view(olap.RESULT_DTYPE)
+    _check_table(got, oracle.tablescan(cols, qs, nthreads=oracle.max_threads()), cols, qs)
