@@ -180,6 +180,15 @@ int olap_cube_stats(const olap_cube* c, int64_t* kernel_launches, int* l2_order)
 /* Number of finalize kernels launched by this process (not bound to a cube). */
 int64_t olap_finalize_launches(void);
 
+/* Tile-shared scan: cubes larger than 64 MiB may answer a batch by staging
+ * each 64-KiB tile of the cube into shared memory once and reducing every (query, tile)
+ * pair from there, instead of streaming each query's own bytes from L2/HBM.  The device
+ * picks the path per batch from the batch's reuse; results are identical in kind (bit-exact
+ * for int32, within the float tolerance otherwise).  enabled = the cube has the tile path;
+ * tile_cells = cells of a full tile; ntiles = tiles of the (local) cube; last_used = the
+ * last batch took it (waits for that batch).  Any out-pointer may be NULL. */
+int olap_cube_tile_stats(olap_cube* c, int* enabled, int64_t* tile_cells, int64_t* ntiles, int* last_used);
+
 /* ---------------------------------------------------------------- dictionaries */
 
 /* Build one text column's dictionary from n keys (key i = bytes[offsets[i],

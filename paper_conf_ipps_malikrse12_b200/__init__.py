@@ -107,6 +107,8 @@ EXPORTS = {
     "olap_cubeset_query": (_int, [_p, _i64, _p, _p, _p, _p, _p]),
     "olap_cubeset_destroy": (_int, [_p]),
     "olap_finalize_launches": (_i64, []),
+    "olap_cube_tile_stats": (_int, [_p, ctypes.POINTER(_int), ctypes.POINTER(_i64), ctypes.POINTER(_i64),
+                                    ctypes.POINTER(_int)]),
     "olap_last_error": (ctypes.c_char_p, []),
     "olap_version": (ctypes.c_char_p, []),
 }
@@ -275,6 +277,13 @@ class Cube:
         n, o = ctypes.c_int64(), ctypes.c_int()
         _check(lib.olap_cube_stats(self._h, ctypes.byref(n), ctypes.byref(o)), "olap_cube_stats")
         return n.value, bool(o.value)
+
+    def tile_stats(self):
+        """(tile path enabled, cells per tile, tiles, last batch used it)"""
+        en, tc, nt, lu = _int(), ctypes.c_int64(), ctypes.c_int64(), _int()
+        _check(lib.olap_cube_tile_stats(self._h, ctypes.byref(en), ctypes.byref(tc), ctypes.byref(nt),
+                                        ctypes.byref(lu)), "olap_cube_tile_stats")
+        return bool(en.value), tc.value, nt.value, bool(lu.value)
 
     def close(self):
         if getattr(self, "_h", None):

@@ -16,7 +16,10 @@
 #include <atomic>
 #include <mutex>
 #include <new>
+#include <type_traits>
 #include <vector>
+
+#include <cub/device/device_scan.cuh>
 
 #include "common.cuh"
 
@@ -258,9 +261,37 @@ __device__ __forceinline__ uint64_t byte_mask_word(uint32_t bits8) {
     return w;
 }
 
-template <int V>
+// SM = true: p points into shared memory (the tile-shared scan stages cube tiles there);
+// plain dereferences let the compiler emit LDS.128 (verified in SASS).  A 32-B slot is two
+// LDS.128; lanes 4-7 of every 8 read the slot's upper half first, so each quarter-warp's
+// first (and second) LDS.128 covers all 32 banks once instead of two-way conflicting on a
+// 32-B lane stride.  Those lanes hold cells 4-7 in v[0..3]: sm_swap() swaps their masks.
+__device__ __forceinline__ bool sm_swapped() { return (threadIdx.x >> 2) & 1; }
+template <int V, bool SM = false>
 __device__ __forceinline__ void load_slot(const uint32_t* p, uint32_t (&v)[V]) {
-    if constexpr (V == 8) {
+    if constexpr (SM) {
+        if constexpr (V == 1) {
+            v[0] = *p;
+        } else if constexpr (V == 4) {
+            const uint4 x = *reinterpret_cast<const uint4*>(p);
+            v[0] = x.x;
+            v[1] = x.y;
+            v[2] = x.z;
+            v[3] = x.w;
+        } else {
+            const int hf = sm_swapped() ? 4 : 0;
+            const uint4 x = *reinterpret_cast<const uint4*>(p + hf);
+            const uint4 y = *reinterpret_cast<const uint4*>(p + (4 - hf));
+            v[0] = x.x;
+            v[1] = x.y;
+            v[2] = x.z;
+            v[3] = x.w;
+            v[4] = y.x;
+            v[5] = y.y;
+            v[6] = y.z;
+            v[7] = y.w;
+        }
+    } else if constexpr (V == 8) {
         ld_stream8(p, v);
     } else if constexpr (V == 4) {
         const uint4 x = ld_stream4(p);
@@ -273,15 +304,48 @@ __device__ __forceinline__ void load_slot(const uint32_t* p, uint32_t (&v)[V]) {
     }
 }
 
-template <class Acc, int OPC, int V>
-__device__ __forceinline__ void fold_slot(Acc& acc, const uint32_t (&v)[V], uint64_t w) {
-#pragma unroll
-    for (int k = 0; k < V; ++k) acc.template add<OPC>(v[k], cell_mask<V>(w, k));
+// Tile path (SM), float32 SUM: the cells of one slot are added pairwise in fp32 first (a
+// tree of depth log2 V <= 3), then the slot sum joins the fp64 accumulator: one F2F + DADD
+// per slot instead of per cell.  Each fp32 add rounds once (relative 2^-24), so a slot sum is
+// off by at most 3 * 2^-24 * sum|x| and the query's SUM by at most ~1.8e-7 * sum|x| — within
+// the 1e-6 tolerance (reading R8), and exact for integer-valued cells below
+// 2^21 (every partial sum is an exact fp32).
+template <int V>
+__device__ __forceinline__ float slot_tree(const uint32_t (&x)[V]) {
+    if constexpr (V == 8)
+        return ((__uint_as_float(x[0]) + __uint_as_float(x[1])) + (__uint_as_float(x[2]) + __uint_as_float(x[3]))) +
+               ((__uint_as_float(x[4]) + __uint_as_float(x[5])) + (__uint_as_float(x[6]) + __uint_as_float(x[7])));
+    else if constexpr (V == 4)
+        return (__uint_as_float(x[0]) + __uint_as_float(x[1])) + (__uint_as_float(x[2]) + __uint_as_float(x[3]));
+    else
+        return __uint_as_float(x[0]);
 }
-template <class Acc, int OPC, int V>
-__device__ __forceinline__ void fold_full(Acc& acc, const uint32_t (&v)[V]) {
+template <class Acc, int OPC, int V, bool SM>
+constexpr bool tree_sum() {
+    return SM && OPC == OPC_SUM && V >= 4 && std::is_same<Acc, AccF>::value;
+}
+
+template <class Acc, int OPC, int V, bool SM = false>
+__device__ __forceinline__ void fold_slot(Acc& acc, const uint32_t (&v)[V], uint64_t w) {
+    if (SM && V == 8 && sm_swapped()) w = (w >> 32) | (w << 32);
+    if constexpr (tree_sum<Acc, OPC, V, SM>()) {
+        uint32_t x[V];
 #pragma unroll
-    for (int k = 0; k < V; ++k) acc.template add<OPC>(v[k], 0xFFFFFFFFu);
+        for (int k = 0; k < V; ++k) x[k] = v[k] & cell_mask<V>(w, k);
+        acc.s += (double)slot_tree<V>(x);
+    } else {
+#pragma unroll
+        for (int k = 0; k < V; ++k) acc.template add<OPC>(v[k], cell_mask<V>(w, k));
+    }
+}
+template <class Acc, int OPC, int V, bool SM = false>
+__device__ __forceinline__ void fold_full(Acc& acc, const uint32_t (&v)[V]) {
+    if constexpr (tree_sum<Acc, OPC, V, SM>()) {
+        acc.s += (double)slot_tree<V>(v);
+    } else {
+#pragma unroll
+        for (int k = 0; k < V; ++k) acc.template add<OPC>(v[k], 0xFFFFFFFFu);
+    }
 }
 
 // Byte-mask words of a run's first slot, last slot, and both (single-slot runs).
@@ -307,13 +371,16 @@ __device__ __forceinline__ void slot_masks(const QDesc& d, uint64_t& wf, uint64_
 #define OLAP_U8 3
 #endif
 constexpr int unroll_for(int V) { return V == 8 ? OLAP_U8 : 4; }
+#ifndef OLAP_SM_U
+#define OLAP_SM_U 2  // tile path (shared-memory slots): slots in flight per lane
+#endif
 
 // Short runs (nslot <= kShortMaxSlots): a task is up to 31 whole runs.  Lane i holds
 // the first-slot address of run r0+i.  The interior slots of all the task's runs
 // (slots 1..nslot-2) are flattened and streamed WITHOUT masks: slot g is run
 // j = g / (nslot-2) (fast division), slot 1 + g % (nslot-2), address via a shuffle.
 // The two edge slots of every run go through a short masked pass.
-template <class Acc, int OPC, int V, int U>
+template <class Acc, int OPC, int V, int U, bool SM = false>
 __device__ __forceinline__ void stream_short(const uint32_t* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
                                              Acc& acc, int lane, int w, int ws) {
     int64_t t = t0 + w;
@@ -339,14 +406,14 @@ __device__ __forceinline__ void stream_short(const uint32_t* __restrict__ cube, 
                 const int idx = ok[u] ? idx0 : nint - 1;  // re-read a valid slot, then drop it
                 const int j = (int)fdiv((uint32_t)idx, fni);
                 const int sl = 1 + idx - j * ni;
-                load_slot<V>(cube + __shfl_sync(0xffffffffu, ra, j & 31) + (int64_t)sl * V, v[u]);
+                load_slot<V, SM>(cube + __shfl_sync(0xffffffffu, ra, j & 31) + (int64_t)sl * V, v[u]);
             }
             if (i0 + 32 * U <= nint) {
 #pragma unroll
-                for (int u = 0; u < U; ++u) fold_full<Acc, OPC, V>(acc, v[u]);
+                for (int u = 0; u < U; ++u) fold_full<Acc, OPC, V, SM>(acc, v[u]);
             } else {
 #pragma unroll
-                for (int u = 0; u < U; ++u) fold_slot<Acc, OPC, V>(acc, v[u], ok[u] ? ~0ull : 0ull);
+                for (int u = 0; u < U; ++u) fold_slot<Acc, OPC, V, SM>(acc, v[u], ok[u] ? ~0ull : 0ull);
             }
         }
         const int nedge = nr * ne;
@@ -362,10 +429,10 @@ __device__ __forceinline__ void stream_short(const uint32_t* __restrict__ cube, 
                 const bool tailside = ne == 2 && (idx & 1);
                 const int sl = tailside ? nslot - 1 : 0;
                 m[u] = ok ? (nslot == 1 ? wb : (tailside ? wl : wf)) : 0ull;
-                load_slot<V>(cube + __shfl_sync(0xffffffffu, ra, j & 31) + (int64_t)sl * V, v[u]);
+                load_slot<V, SM>(cube + __shfl_sync(0xffffffffu, ra, j & 31) + (int64_t)sl * V, v[u]);
             }
 #pragma unroll
-            for (int u = 0; u < U; ++u) fold_slot<Acc, OPC, V>(acc, v[u], m[u]);
+            for (int u = 0; u < U; ++u) fold_slot<Acc, OPC, V, SM>(acc, v[u], m[u]);
         }
     }
 }
@@ -373,7 +440,7 @@ __device__ __forceinline__ void stream_short(const uint32_t* __restrict__ cube, 
 // Stream slots [0, count) of one run segment starting at slot address p (cells).
 // wfirst / wlast: masks of slot 0 and slot count-1 (all ones when not a run edge;
 // wboth when one slot is both).  Steps with no edge slot skip masking entirely.
-template <class Acc, int OPC, int V>
+template <class Acc, int OPC, int V, bool SM = false>
 __device__ __forceinline__ void stream_segment(const uint32_t* __restrict__ p, int count, uint64_t wfirst,
                                                uint64_t wlast, uint64_t wboth, Acc& acc, int lane) {
     constexpr int U = unroll_for(V);
@@ -388,21 +455,21 @@ __device__ __forceinline__ void stream_segment(const uint32_t* __restrict__ p, i
             const bool ok = idx0 < count;
             const int idx = ok ? idx0 : count - 1;  // re-read the last slot, masked out
             m[u] = ok ? (idx == 0 ? (idx == count - 1 ? wboth : wfirst) : (idx == count - 1 ? wlast : ~0ull)) : 0ull;
-            load_slot<V>(p + (int64_t)idx * V, v[u]);
+            load_slot<V, SM>(p + (int64_t)idx * V, v[u]);
         }
         if (interior) {
 #pragma unroll
-            for (int u = 0; u < U; ++u) fold_full<Acc, OPC, V>(acc, v[u]);
+            for (int u = 0; u < U; ++u) fold_full<Acc, OPC, V, SM>(acc, v[u]);
         } else {
 #pragma unroll
-            for (int u = 0; u < U; ++u) fold_slot<Acc, OPC, V>(acc, v[u], m[u]);
+            for (int u = 0; u < U; ++u) fold_slot<Acc, OPC, V, SM>(acc, v[u], m[u]);
         }
     }
 }
 
 // Long runs (nslot > kShortMaxSlots): a task is kTaskSlots slots, at most two
 // contiguous segments (the end of run j0 and the start of run j0+1).
-template <class Acc, int OPC, int V>
+template <class Acc, int OPC, int V, bool SM = false>
 __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
                                             Acc& acc, int lane, int w, int ws) {
     int64_t t = t0 + w;
@@ -420,9 +487,9 @@ __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, c
         const int64_t in_run = nslot - rem;
         const int c1 = in_run < n ? (int)in_run : n;
         const bool first = rem == 0, lastin = rem + c1 == nslot;
-        stream_segment<Acc, OPC, V>(cube + run_addr(d, j0) + rem * V, c1, first ? wf : ~0ull, lastin ? wl : ~0ull,
+        stream_segment<Acc, OPC, V, SM>(cube + run_addr(d, j0) + rem * V, c1, first ? wf : ~0ull, lastin ? wl : ~0ull,
                                     first && lastin ? wb : (first ? wf : wl), acc, lane);
-        if (c1 < n) stream_segment<Acc, OPC, V>(cube + run_addr(d, j0 + 1), n - c1, wf, ~0ull, wf, acc, lane);
+        if (c1 < n) stream_segment<Acc, OPC, V, SM>(cube + run_addr(d, j0 + 1), n - c1, wf, ~0ull, wf, acc, lane);
         rem += step;
         if (rem >= nslot) {
             const int64_t dj = nslot < (1ll << 20) ? (int64_t)fdiv((uint32_t)rem, d.fnslot) : 1;
@@ -433,15 +500,16 @@ __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, c
 }
 
 // Tasks t0+w, t0+w+ws, ... < t1 of one query's item (ws warps share the item).
-template <typename T, class Acc, int OPC, int V>
+template <typename T, class Acc, int OPC, int V, bool SM = false>
 __device__ __forceinline__ void stream_tasks(const T* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
                                              Acc& acc, int lane, int w, int ws = kWarps) {
     const uint32_t* c = reinterpret_cast<const uint32_t*>(cube);
     if (d.shortp) {
-        if (V == 8 && d.nslot < 16) stream_short<Acc, OPC, V, 2>(c, d, t0, t1, acc, lane, w, ws);
-        else stream_short<Acc, OPC, V, unroll_for(V)>(c, d, t0, t1, acc, lane, w, ws);
+        if (SM) stream_short<Acc, OPC, V, OLAP_SM_U, SM>(c, d, t0, t1, acc, lane, w, ws);
+        else if (V == 8 && d.nslot < 16) stream_short<Acc, OPC, V, 2, SM>(c, d, t0, t1, acc, lane, w, ws);
+        else stream_short<Acc, OPC, V, unroll_for(V), SM>(c, d, t0, t1, acc, lane, w, ws);
     }
-    else stream_long<Acc, OPC, V>(c, d, t0, t1, acc, lane, w, ws);
+    else stream_long<Acc, OPC, V, SM>(c, d, t0, t1, acc, lane, w, ws);
 }
 
 // ------------------------------------------------------------------ plan
@@ -546,7 +614,8 @@ __global__ void __launch_bounds__(kDescThreads) desc_kernel(Geo geo, int64_t nq,
                                                             const int32_t* __restrict__ ops, QDesc* desc,
                                                             int64_t* q_tasks, int32_t* q_tv, int32_t* done,
                                                             int64_t* psum, int32_t* pext,
-                                                            unsigned long long* totals) {
+                                                            unsigned long long* totals, const int32_t* tmode) {
+    if (*tmode) return;  // the tile-shared scan answers this batch
     __shared__ int64_t sh[32];
     const int64_t q = blockIdx.x * (int64_t)kDescThreads + threadIdx.x;
     int64_t cells = 0, slot_cells = 0;
@@ -581,7 +650,9 @@ __global__ void __launch_bounds__(kPlanThreads) scan_kernel(int64_t nq, QDesc* d
                                                             const int32_t* __restrict__ q_tv, int64_t* item_start,
                                                             unsigned long long* counter, int64_t items_cap,
                                                             const unsigned long long* totals,
-                                                            unsigned long long* bytes_acc, int grid) {
+                                                            unsigned long long* bytes_acc, int grid,
+                                                            const int32_t* tmode) {
+    if (*tmode) return;
     const int tid = threadIdx.x;
     const int64_t total_cells = (int64_t)totals[0], total_slot_cells = (int64_t)totals[1];
     // item size: 1 MiB, smaller for small batches so that there are >= 4 items per resident
@@ -655,7 +726,8 @@ __device__ __forceinline__ int64_t find_query_thread(const int64_t* __restrict__
 }
 
 __global__ void bucket_kernel(int64_t nq, const QDesc* __restrict__ desc, const int64_t* __restrict__ item_start,
-                              int shift, int32_t* __restrict__ bucket, unsigned int* count) {
+                              int shift, int32_t* __restrict__ bucket, unsigned int* count, const int32_t* tmode) {
+    if (*tmode) return;
     const int64_t total = __ldg(item_start + nq);
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
         const int64_t q = find_query_thread(item_start, nq, i);
@@ -675,7 +747,9 @@ __global__ void bucket_kernel(int64_t nq, const QDesc* __restrict__ desc, const 
     }
 }
 
-__global__ void __launch_bounds__(1024) bucket_scan_kernel(unsigned int* count, unsigned int* cursor) {
+__global__ void __launch_bounds__(1024) bucket_scan_kernel(unsigned int* count, unsigned int* cursor,
+                                                           const int32_t* tmode) {
+    if (*tmode) return;
     __shared__ unsigned int sh[kMaxBuckets];
     for (int b = threadIdx.x; b < kMaxBuckets; b += blockDim.x) sh[b] = count[b];
     __syncthreads();
@@ -692,7 +766,8 @@ __global__ void __launch_bounds__(1024) bucket_scan_kernel(unsigned int* count, 
 }
 
 __global__ void scatter_kernel(int64_t nq, const int64_t* __restrict__ item_start, const int32_t* __restrict__ bucket,
-                               unsigned int* cursor, int32_t* __restrict__ order) {
+                               unsigned int* cursor, int32_t* __restrict__ order, const int32_t* tmode) {
+    if (*tmode) return;
     const int64_t total = __ldg(item_start + nq);
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x)
         order[atomicAdd(cursor + bucket[i], 1u)] = (int32_t)i;
@@ -701,22 +776,22 @@ __global__ void scatter_kernel(int64_t nq, const int64_t* __restrict__ item_star
 // ------------------------------------------------------------------ reduce (the hot loop)
 
 // op-class x slot-width dispatch of one item's tasks
-template <typename T, class Acc>
+template <typename T, class Acc, bool SM = false>
 __device__ __forceinline__ void stream_item(const T* __restrict__ cube, const QDesc& sd, int64_t t0, int64_t t1, Acc& acc,
                                             int lane, int w, int ws) {
     const int opc = sd.opc;
     if (sd.V == 8) {
-        if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 8>(cube, sd, t0, t1, acc, lane, w, ws);
-        else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 8>(cube, sd, t0, t1, acc, lane, w, ws);
-        else stream_tasks<T, Acc, OPC_MAX, 8>(cube, sd, t0, t1, acc, lane, w, ws);
+        if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 8, SM>(cube, sd, t0, t1, acc, lane, w, ws);
+        else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 8, SM>(cube, sd, t0, t1, acc, lane, w, ws);
+        else stream_tasks<T, Acc, OPC_MAX, 8, SM>(cube, sd, t0, t1, acc, lane, w, ws);
     } else if (sd.V == 4) {
-        if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 4>(cube, sd, t0, t1, acc, lane, w, ws);
-        else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 4>(cube, sd, t0, t1, acc, lane, w, ws);
-        else stream_tasks<T, Acc, OPC_MAX, 4>(cube, sd, t0, t1, acc, lane, w, ws);
-    } else {
-        if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 1>(cube, sd, t0, t1, acc, lane, w, ws);
-        else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 1>(cube, sd, t0, t1, acc, lane, w, ws);
-        else stream_tasks<T, Acc, OPC_MAX, 1>(cube, sd, t0, t1, acc, lane, w, ws);
+        if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 4, SM>(cube, sd, t0, t1, acc, lane, w, ws);
+        else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 4, SM>(cube, sd, t0, t1, acc, lane, w, ws);
+        else stream_tasks<T, Acc, OPC_MAX, 4, SM>(cube, sd, t0, t1, acc, lane, w, ws);
+    } else if constexpr (!SM) {  // tile path: every run stride is a multiple of 4 cells (V >= 4)
+        if (opc == OPC_SUM) stream_tasks<T, Acc, OPC_SUM, 1, SM>(cube, sd, t0, t1, acc, lane, w, ws);
+        else if (opc == OPC_MIN) stream_tasks<T, Acc, OPC_MIN, 1, SM>(cube, sd, t0, t1, acc, lane, w, ws);
+        else stream_tasks<T, Acc, OPC_MAX, 1, SM>(cube, sd, t0, t1, acc, lane, w, ws);
     }
 }
 
@@ -728,7 +803,9 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) reduce_kernel_w(const T*
                                                                const int64_t* __restrict__ item_start,
                                                                unsigned long long* counter, int32_t* done,
                                                                long long* item_sum, int32_t* item_ext, int64_t* psum,
-                                                               int32_t* pext, const int32_t* __restrict__ order) {
+                                                               int32_t* pext, const int32_t* __restrict__ order,
+                                                               const int32_t* tmode) {
+    if (*tmode) return;
     __shared__ QDesc sdw[kWarps];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     QDesc& sd = sdw[w];
@@ -801,7 +878,9 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) reduce_kernel(const T* _
                                                              const int64_t* __restrict__ item_start,
                                                              unsigned long long* counter, int32_t* done,
                                                              long long* item_sum, int32_t* item_ext, int64_t* psum,
-                                                             int32_t* pext, const int32_t* __restrict__ order) {
+                                                             int32_t* pext, const int32_t* __restrict__ order,
+                                                             const int32_t* tmode) {
+    if (*tmode) return;
     __shared__ QDesc sd;
     __shared__ int64_t s_item, s_q;
     __shared__ long long s_wsum[kWarps];
@@ -912,6 +991,10 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) reduce_kernel(const T* _
         __syncthreads();
     }
 }
+
+// ------------------------------------------------------------------ tile-shared scan
+
+#include "tiles.cuh"
 
 // ------------------------------------------------------------------ finalize / combine
 
@@ -1079,6 +1162,23 @@ struct olap_cube {
     size_t h_pinned_cap = 0;
     int64_t stage_cap = 0;
 
+    // tile-shared scan (tiles.cuh): geometry, workspace, control words
+    TGeo tg{};
+    bool tiles_on = false;
+    int64_t pairs_cap = 0, tq_cap = 0;
+    TDesc* d_tdesc = nullptr;
+    int64_t* d_qpairs = nullptr;
+    int64_t* d_pstart = nullptr;
+    unsigned int* d_tcount = nullptr;  // ntiles + 1
+    unsigned int* d_tstart = nullptr;  // ntiles + 1
+    uint32_t* d_nonempty = nullptr;    // ntiles
+    uint32_t* d_list = nullptr;        // pairs_cap
+    long long* d_partial = nullptr;    // pairs_cap
+    void* d_cubtmp = nullptr;
+    size_t cub_bytes = 0;
+    int32_t* d_ctl = nullptr;                  // [0] mode (1 = tiles), [1] non-empty tiles, [2] pop counter
+    unsigned long long* d_ttot = nullptr;      // tile path batch totals (cells)
+
     bool prof = false;
     std::vector<cudaEvent_t> ev;
     size_t ev_used = 0;
@@ -1143,6 +1243,51 @@ void free_ws(olap_cube* c) {
     c->d_item_sum = nullptr;
     c->d_item_ext = nullptr;
     c->nq_cap = c->items_cap = 0;
+    cudaFree(c->d_tdesc);
+    cudaFree(c->d_qpairs);
+    cudaFree(c->d_pstart);
+    cudaFree(c->d_tcount);
+    cudaFree(c->d_tstart);
+    cudaFree(c->d_nonempty);
+    cudaFree(c->d_list);
+    cudaFree(c->d_partial);
+    cudaFree(c->d_cubtmp);
+    c->d_tdesc = nullptr;
+    c->d_qpairs = c->d_pstart = nullptr;
+    c->d_tcount = c->d_tstart = nullptr;
+    c->d_nonempty = c->d_list = nullptr;
+    c->d_partial = nullptr;
+    c->d_cubtmp = nullptr;
+    c->tq_cap = 0;
+}
+
+// Tile-path workspace (per query, per tile, per pair).  If it cannot be allocated the cube keeps
+// answering through the item path (the tile path is an optimisation, never a requirement).
+void ensure_tile_ws(olap_cube* c, int64_t cap) {
+    if (!c->tiles_on || cap <= c->tq_cap) return;
+    const int64_t nt = c->tg.ntiles;
+    bool ok = cudaMalloc(&c->d_tdesc, sizeof(TDesc) * cap) == cudaSuccess &&
+              cudaMalloc(&c->d_qpairs, sizeof(int64_t) * cap) == cudaSuccess &&
+              cudaMalloc(&c->d_pstart, sizeof(int64_t) * (cap + 1)) == cudaSuccess;
+    if (ok && !c->d_tcount) {
+        ok = cudaMalloc(&c->d_tcount, sizeof(unsigned int) * (3 * nt + 1)) == cudaSuccess &&
+             cudaMalloc(&c->d_tstart, sizeof(unsigned int) * (3 * nt + 1)) == cudaSuccess &&
+             cudaMalloc(&c->d_nonempty, sizeof(uint32_t) * nt) == cudaSuccess &&
+             cudaMalloc(&c->d_list, sizeof(uint32_t) * c->pairs_cap) == cudaSuccess &&
+             cudaMalloc(&c->d_partial, sizeof(long long) * c->pairs_cap) == cudaSuccess;
+        if (ok) {
+            c->cub_bytes = 0;
+            ok = cub::DeviceScan::ExclusiveSum(nullptr, c->cub_bytes, c->d_tcount, c->d_tstart, (int)(3 * nt + 1)) ==
+                     cudaSuccess &&
+                 cudaMalloc(&c->d_cubtmp, std::max<size_t>(c->cub_bytes, 16)) == cudaSuccess;
+        }
+    }
+    if (!ok) {
+        cudaGetLastError();
+        c->tiles_on = false;  // free_ws releases whatever was allocated
+        return;
+    }
+    c->tq_cap = cap;
 }
 
 int ensure_ws(olap_cube* c, int64_t nq) {
@@ -1169,6 +1314,7 @@ int ensure_ws(olap_cube* c, int64_t nq) {
     }
     c->nq_cap = cap;
     c->items_cap = items;
+    ensure_tile_ws(c, cap);
     return OLAP_OK;
 }
 
@@ -1218,13 +1364,72 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
     int rc = ensure_ws(c, nq);
     if (rc) return rc;
     if (!cap) OLAP_CUDA_TRY(cudaStreamWaitEvent(st, c->ws_done, 0));
+    const bool prof = c->prof && !cap;
+    auto bracket = [&](cudaEvent_t* e0, cudaEvent_t* e1) -> int {
+        while (c->ev.size() < c->ev_used + 2) {
+            cudaEvent_t e;
+            OLAP_CUDA_TRY(cudaEventCreate(&e));
+            c->ev.push_back(e);
+        }
+        *e0 = c->ev[c->ev_used];
+        *e1 = c->ev[c->ev_used + 1];
+        c->ev_used += 2;
+        return OLAP_OK;
+    };
+    const int32_t* tmode = c->d_ctl;  // stays 0 when the cube has no tile path
+    if (c->tiles_on) {
+        // tile-shared scan (tiles.cuh); tile_scan_kernel picks it or the item path on the device
+        const TGeo& tg = c->tg;
+        const int qb = (int)((nq + kDescThreads - 1) / kDescThreads), eg = c->num_sms * 8;
+        OLAP_CUDA_TRY(cudaMemsetAsync(c->d_ttot, 0, sizeof(unsigned long long), st));
+        tile_desc_kernel<<<qb, kDescThreads, 0, st>>>(make_geo(c), tg, nq, d_ranges, d_ops, c->d_tdesc, c->d_qpairs,
+                                                      d_psum, d_pext, c->d_ttot);
+        tile_scan_kernel<<<1, kPlanThreads, 0, st>>>(nq, c->d_qpairs, c->d_pstart, c->pairs_cap, tg, c->d_ttot,
+                                                     c->d_ctl, c->d_counter + 1);
+        OLAP_CUDA_TRY(cudaMemsetAsync(c->d_tcount, 0, sizeof(unsigned int) * (3 * tg.ntiles + 1), st));
+        tile_count_kernel<<<eg, 256, 0, st>>>(tg, nq, c->d_pstart, c->d_tdesc, c->d_tcount, c->d_ctl);
+        OLAP_CUDA_TRY(cudaGetLastError());
+        size_t tb = c->cub_bytes;
+        OLAP_CUDA_TRY(cub::DeviceScan::ExclusiveSum(c->d_cubtmp, tb, c->d_tcount, c->d_tstart,
+                                                    (int)(3 * tg.ntiles + 1), st));
+        tile_compact_kernel<<<eg, 256, 0, st>>>(tg.ntiles, c->d_tstart, c->d_ctl, c->d_nonempty);
+        tile_scatter_kernel<<<eg, 256, 0, st>>>(tg, nq, c->d_pstart, c->d_tdesc, c->d_tcount, c->d_tstart, c->d_ctl,
+                                                c->d_list);
+        cudaEvent_t t0 = nullptr, t1 = nullptr;
+        if (prof) {
+            int rc2 = bracket(&t0, &t1);
+            if (rc2) return rc2;
+            OLAP_CUDA_TRY(cudaEventRecord(t0, st));
+        }
+        const size_t smem = tile_smem_bytes();
+        if (c->dtype == OLAP_INT32)
+            tile_reduce_kernel<int32_t, AccI><<<c->num_sms, kTileThreads, smem, st>>>(
+                static_cast<const int32_t*>(c->d_cells), tg, c->d_tdesc, c->d_pstart, c->d_tstart, c->d_nonempty,
+                c->d_list, c->d_ctl, c->d_partial);
+        else
+            tile_reduce_kernel<float, AccF><<<c->num_sms, kTileThreads, smem, st>>>(
+                static_cast<const float*>(c->d_cells), tg, c->d_tdesc, c->d_pstart, c->d_tstart, c->d_nonempty,
+                c->d_list, c->d_ctl, c->d_partial);
+        OLAP_CUDA_TRY(cudaGetLastError());
+        if (prof) OLAP_CUDA_TRY(cudaEventRecord(t1, st));
+        const int fg = (int)std::min<int64_t>(nq, (int64_t)c->num_sms * 8);
+        if (c->dtype == OLAP_INT32)
+            pair_fold_kernel<AccI><<<fg, 256, 0, st>>>(nq, c->d_pstart, c->d_tdesc, c->d_ctl, c->d_partial, d_psum,
+                                                       d_pext);
+        else
+            pair_fold_kernel<AccF><<<fg, 256, 0, st>>>(nq, c->d_pstart, c->d_tdesc, c->d_ctl, c->d_partial, d_psum,
+                                                       d_pext);
+        OLAP_CUDA_TRY(cudaGetLastError());
+        c->kernel_launches += 9;  // desc, scan, count, CUB scan (2), compact, scatter, reduce, fold
+    }
     OLAP_CUDA_TRY(cudaMemsetAsync(c->d_counter + 2, 0, 2 * sizeof(unsigned long long), st));
     desc_kernel<<<(int)((nq + kDescThreads - 1) / kDescThreads), kDescThreads, 0, st>>>(
-        make_geo(c), nq, d_ranges, d_ops, c->d_desc, c->d_qtasks, c->d_qtv, c->d_done, d_psum, d_pext, c->d_counter + 2);
+        make_geo(c), nq, d_ranges, d_ops, c->d_desc, c->d_qtasks, c->d_qtv, c->d_done, d_psum, d_pext, c->d_counter + 2,
+        tmode);
     OLAP_CUDA_TRY(cudaGetLastError());
     scan_kernel<<<1, kPlanThreads, 0, st>>>(nq, c->d_desc, c->d_qtasks, c->d_qtv, c->d_item_start, c->d_counter,
                                             c->items_cap, c->d_counter + 2, c->d_counter + 1,
-                                            c->num_sms * c->blocks_per_sm);
+                                            c->num_sms * c->blocks_per_sm, tmode);
     OLAP_CUDA_TRY(cudaGetLastError());
     const int32_t* order = nullptr;
     c->kernel_launches += 3;  // desc, scan, reduce
@@ -1232,44 +1437,37 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
         c->kernel_launches += 3;
         OLAP_CUDA_TRY(cudaMemsetAsync(c->d_bcount, 0, sizeof(unsigned int) * kMaxBuckets, st));
         bucket_kernel<<<c->num_sms * 8, 256, 0, st>>>(nq, c->d_desc, c->d_item_start, c->order_shift, c->d_bucket,
-                                                       c->d_bcount);
-        bucket_scan_kernel<<<1, 1024, 0, st>>>(c->d_bcount, c->d_bcount + kMaxBuckets);
+                                                       c->d_bcount, tmode);
+        bucket_scan_kernel<<<1, 1024, 0, st>>>(c->d_bcount, c->d_bcount + kMaxBuckets, tmode);
         scatter_kernel<<<c->num_sms * 8, 256, 0, st>>>(nq, c->d_item_start, c->d_bucket, c->d_bcount + kMaxBuckets,
-                                                        c->d_order);
+                                                        c->d_order, tmode);
         OLAP_CUDA_TRY(cudaGetLastError());
         order = c->d_order;
     }
     const int grid = c->num_sms * c->blocks_per_sm;
     cudaEvent_t e0 = nullptr, e1 = nullptr;
-    const bool prof = c->prof && !cap;
     if (prof) {
-        while (c->ev.size() < c->ev_used + 2) {
-            cudaEvent_t e;
-            OLAP_CUDA_TRY(cudaEventCreate(&e));
-            c->ev.push_back(e);
-        }
-        e0 = c->ev[c->ev_used];
-        e1 = c->ev[c->ev_used + 1];
-        c->ev_used += 2;
+        int rc2 = bracket(&e0, &e1);
+        if (rc2) return rc2;
         OLAP_CUDA_TRY(cudaEventRecord(e0, st));
     }
     if (kWarpItems) {
         if (c->dtype == OLAP_INT32)
             reduce_kernel_w<int32_t, AccI><<<grid, kThreads, 0, st>>>(
                 static_cast<const int32_t*>(c->d_cells), nq, c->d_desc, c->d_item_start, c->d_counter, c->d_done,
-                c->d_item_sum, c->d_item_ext, d_psum, d_pext, order);
+                c->d_item_sum, c->d_item_ext, d_psum, d_pext, order, tmode);
         else
             reduce_kernel_w<float, AccF><<<grid, kThreads, 0, st>>>(
                 static_cast<const float*>(c->d_cells), nq, c->d_desc, c->d_item_start, c->d_counter, c->d_done,
-                c->d_item_sum, c->d_item_ext, d_psum, d_pext, order);
+                c->d_item_sum, c->d_item_ext, d_psum, d_pext, order, tmode);
     } else if (c->dtype == OLAP_INT32)
         reduce_kernel<int32_t, AccI><<<grid, kThreads, 0, st>>>(
             static_cast<const int32_t*>(c->d_cells), nq, c->d_desc, c->d_item_start, c->d_counter, c->d_done,
-            c->d_item_sum, c->d_item_ext, d_psum, d_pext, order);
+            c->d_item_sum, c->d_item_ext, d_psum, d_pext, order, tmode);
     else
         reduce_kernel<float, AccF><<<grid, kThreads, 0, st>>>(
             static_cast<const float*>(c->d_cells), nq, c->d_desc, c->d_item_start, c->d_counter, c->d_done,
-            c->d_item_sum, c->d_item_ext, d_psum, d_pext, order);
+            c->d_item_sum, c->d_item_ext, d_psum, d_pext, order, tmode);
     OLAP_CUDA_TRY(cudaGetLastError());
     if (prof) {
         OLAP_CUDA_TRY(cudaEventRecord(e1, st));
@@ -1289,6 +1487,49 @@ int launch_finalize(int nd, const int64_t* ext, int dtype, int64_t nq, const ola
     finalize_kernel<<<grid, 256, 0, st>>>(nd, e, dtype, nq, d_ranges, d_ops, d_psum, d_pext, d_results);
     OLAP_CUDA_TRY(cudaGetLastError());
     return OLAP_OK;
+}
+
+// Tile geometry (tiles.cuh): kt = outermost dim whose stride fits a 64 KiB tile; a tile is ct
+// consecutive indices of dim kt times everything inside it (contiguous, and a box).  The tile
+// path is enabled for cubes that do not fit in L2 (the item path already serves those from L2).
+void make_tiles(olap_cube* c) {
+    TGeo& t = c->tg;
+    std::memset(&t, 0, sizeof(t));
+    const int nd = c->nd;
+    t.nd = nd;
+    t.padded = c->pitch != c->n[nd - 1];
+    for (int k = 0; k < nd; ++k) {
+        t.ext[k] = k == 0 ? c->local_rows : c->n[k];
+        t.stride[k] = nd == 1 ? 1 : c->stride[k];
+    }
+    int kt = 0;
+    while (t.stride[kt] > kTileCellsMax) ++kt;
+    t.kt = kt;
+    int64_t ctmax = std::max<int64_t>(1, kTileCellsMax / t.stride[kt]);
+    const int64_t ekt = std::max<int64_t>(t.ext[kt], 1);
+    const int64_t nch = (ekt + ctmax - 1) / ctmax;
+    int64_t ct = (ekt + nch - 1) / nch;
+    if (kt == nd - 1) ct = (ct + 7) & ~7ll;  // chunks of the innermost row start 32-B aligned
+    t.ct = ct;
+    t.nct = (ekt + ct - 1) / ct;
+    t.ts[kt] = 1;
+    for (int e = kt - 1; e >= 0; --e) t.ts[e] = t.ts[e + 1] * (e + 1 == kt ? t.nct : t.ext[e + 1]);
+    t.ntiles = t.ts[0] * (kt == 0 ? t.nct : t.ext[0]);
+    t.tcells = ct * t.stride[kt];
+    t.ok = c->local_rows > 0 && t.ntiles < (1ll << 31) && c->order_shift >= 0 && !getenv("OLAP_NO_TILES");
+    c->tiles_on = t.ok;
+    c->pairs_cap = std::min<int64_t>(1ll << 29, std::max<int64_t>(1ll << 24, c->local_cells / 8));
+    if (c->tiles_on) {
+        const size_t smem = tile_smem_bytes();
+        if (cudaFuncSetAttribute(tile_reduce_kernel<int32_t, AccI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)smem) != cudaSuccess ||
+            cudaFuncSetAttribute(tile_reduce_kernel<float, AccF>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)smem) != cudaSuccess) {
+            cudaGetLastError();
+            c->tiles_on = false;
+            t.ok = 0;
+        }
+    }
 }
 
 int check_cube(const olap_cube* c) {
@@ -1373,7 +1614,8 @@ int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_sh
     if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess ||
         cudaEventCreateWithFlags(&c->ws_done, cudaEventDisableTiming) != cudaSuccess ||
         cudaMalloc(&c->d_counter, 4 * sizeof(unsigned long long)) != cudaSuccess ||
-        cudaMemset(c->d_counter, 0, 4 * sizeof(unsigned long long)) != cudaSuccess) {
+        cudaMemset(c->d_counter, 0, 4 * sizeof(unsigned long long)) != cudaSuccess ||
+        cudaMalloc(&c->d_ctl, 64) != cudaSuccess || cudaMemset(c->d_ctl, 0, 64) != cudaSuccess) {
         rc = set_error(OLAP_E_CUDA, "stream/event/counter setup failed");
         olap_cube_destroy(c);
         return rc;
@@ -1404,6 +1646,8 @@ int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_sh
         while ((c->local_cells >> sh) >= kMaxBuckets) ++sh;
         c->order_shift = sh;
     }
+    c->d_ttot = reinterpret_cast<unsigned long long*>(c->d_ctl + 8);
+    make_tiles(c);
 
     *out = c;
     return OLAP_OK;
@@ -1528,6 +1772,7 @@ int olap_cube_destroy(olap_cube* c) {
     cudaFree(c->d_pext);
     cudaFreeHost(c->h_pinned);
     cudaFree(c->d_counter);
+    cudaFree(c->d_ctl);
     cudaFree(c->d_cells);
     for (auto e : c->ev) cudaEventDestroy(e);
     if (c->ws_done) cudaEventDestroy(c->ws_done);
@@ -1675,6 +1920,21 @@ int olap_cube_stats(const olap_cube* c, int64_t* kernel_launches, int* l2_order)
 }
 
 int64_t olap_finalize_launches(void) { return g_finalize_launches.load(); }
+
+int olap_cube_tile_stats(olap_cube* c, int* enabled, int64_t* tile_cells, int64_t* ntiles, int* last_used) {
+    clear_error();
+    if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    std::lock_guard<std::mutex> lk(c->mu);
+    DeviceGuard dg(c->device);
+    OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
+    int32_t mode = 0;
+    OLAP_CUDA_TRY(cudaMemcpy(&mode, c->d_ctl, sizeof(mode), cudaMemcpyDeviceToHost));
+    if (enabled) *enabled = c->tiles_on ? 1 : 0;
+    if (tile_cells) *tile_cells = c->tg.tcells;
+    if (ntiles) *ntiles = c->tg.ntiles;
+    if (last_used) *last_used = mode;
+    return OLAP_OK;
+}
 
 int olap_cube_profile(olap_cube* c, int enable) {
     clear_error();

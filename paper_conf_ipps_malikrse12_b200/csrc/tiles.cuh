@@ -1,0 +1,529 @@
+// tiles.cuh — the tile-shared scan (included by cube.cu; internal, not part of the C-ABI).
+//
+// The item path (reduce_kernel) streams every query's own bytes through L1TEX from L2.
+// When a batch's boxes overlap heavily (C2a: every cell is read by ~390 queries of a
+// 4,096-query batch), that costs the same on-chip bandwidth 390 times over.  This path
+// reorganises the same reduction (Fig. 2 "area of limited search", PAPER.md:143,151;
+// bandwidth-bound) around the cube instead of around the queries:
+//
+//   * the cube is cut into TILES: contiguous spans that are also boxes,
+//     (1, .., 1, ct, n_{kt+1}, .., n_{N-1}) cells, <= 64 KiB;
+//   * a (query, tile) PAIR is a query box intersecting a tile; its cells are the box
+//     clipped to the tile, again runs of the row-major layout (a4);
+//   * a persistent block per SM pops non-empty tiles, stages each one into shared memory
+//     ONCE with a bulk async copy (cp.async.bulk + mbarrier, 3-stage ring fed by a
+//     producer warp), and its 31 consumer warps reduce every pair of that tile from shared
+//     memory, each pair with the item path's run streamer (LDS instead of LDG);
+//   * pair partials are stored by pair id (query-major) and folded per query in pair
+//     order, so results are deterministic and independent of the tile schedule.
+//
+// Planning (all on the device, capturable): tile_desc_kernel (per query: tile box, pair
+// count, clipped-run structure) -> tile_scan_kernel (pair offsets; chooses this path or
+// the item path from the batch's reuse) -> tile_count_kernel ->
+// exclusive scan of per-tile counts (CUB) -> tile_scatter_kernel (per-tile query lists)
+// -> tile_reduce_kernel -> pair_fold_kernel.  Every kernel of the path not chosen exits
+// at once.
+
+#ifndef OLAP_TILE_CELLS
+#define OLAP_TILE_CELLS 16384
+#endif
+#ifndef OLAP_TILE_STAGES
+#define OLAP_TILE_STAGES 3
+#endif
+constexpr int64_t kTileCellsMax = OLAP_TILE_CELLS;  // 64 KiB of 4-byte cells per tile
+constexpr int kTileStages = OLAP_TILE_STAGES;
+constexpr int kTileWarps = 32;  // warp 0: producer; warps 1..31: consumers
+constexpr int kTileThreads = kTileWarps * 32;
+constexpr int kTileConsumers = kTileWarps - 1;
+constexpr int kTileSlack = 16;  // cells after each stage buffer: masked over-reads of a run's last slot
+constexpr int kTilePairsPerThread = 8;
+
+// Tile geometry of a cube (shard-local), fixed at cube creation.
+struct TGeo {
+    int nd, kt, padded, ok;
+    int64_t ct, nct, ntiles, tcells;  // chunk extent along kt, chunks, tiles, cells of a full tile
+    int64_t ext[kMaxDims];            // local extents (dim 0 = local rows)
+    int64_t stride[kMaxDims];         // local strides (cells)
+    int64_t ts[kMaxDims];             // tile-grid strides for dims <= kt
+};
+
+// Per query: its tile box and the part of its clipped-run structure that no tile changes.
+struct TDesc {
+    int32_t opc, V, nrd, span;  // span: a pair is one run over dim kt (all dims after kt full)
+    int64_t lo_kt, hi_kt;       // local range along kt
+    int64_t L, Rin, base_in;    // run length, runs per kt-slice, offset of dims > kt
+    int64_t tlo[kMaxDims];      // tile box: dims < kt: lo_e; dim kt: first chunk
+    int64_t tn[kMaxDims];       // tile box extents
+    FastDiv tfd[kMaxDims];      // / tn (pair index -> tile coordinates)
+    FastDiv frl[kMaxRunDims];   // inner radices (dims ks-1 .. kt+1 with extent > 1), innermost first
+    int64_t rs[kMaxRunDims];
+};
+
+// ------------------------------------------------------------------ mbarrier / bulk copy (PTX)
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint64_t* b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+// producer side: back off between probes (a single lane; keeps the spin off the issue slots)
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* b, uint32_t parity) {
+    uint32_t ok = 0;
+    for (;;) {
+        asm volatile(
+            "{\n"
+            ".reg .pred p;\n"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+            "selp.u32 %0, 1, 0, p;\n"
+            "}\n"
+            : "=r"(ok)
+            : "r"(smem_u32(b)), "r"(parity)
+            : "memory");
+        if (ok) return;
+        __nanosleep(256);
+    }
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "OLAP_WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        "@!p bra OLAP_WAIT_%=;\n"
+        "}\n" ::"r"(smem_u32(b)),
+        "r"(parity)
+        : "memory");
+}
+// global -> shared bulk copy completing on mbarrier b (bytes: multiple of 16, both ends 16-B aligned)
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* b) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(b))
+                 : "memory");
+}
+
+// ------------------------------------------------------------------ planning
+
+// One thread per query: validate (a1), shard-intersect (a3), tile box, pair count, clipped-run
+// structure; identity partials for queries that read no cell; batch totals (order-free atomics).
+__global__ void __launch_bounds__(kDescThreads) tile_desc_kernel(Geo geo, TGeo tg, int64_t nq,
+                                                                 const olap_range* __restrict__ ranges,
+                                                                 const int32_t* __restrict__ ops, TDesc* tdesc,
+                                                                 int64_t* q_pairs, int64_t* psum, int32_t* pext,
+                                                                 unsigned long long* totals) {
+    __shared__ int64_t sh[32];
+    const int64_t q = blockIdx.x * (int64_t)kDescThreads + threadIdx.x;
+    int64_t cells = 0;
+    if (q < nq) {
+        int64_t np = 0;
+        const int32_t op = ops[q];
+        int64_t lo[kMaxDims], hi[kMaxDims];
+        bool ok = op >= OLAP_SUM && op <= OLAP_AVG && op != OLAP_COUNT, empty = false;
+        for (int k = 0; k < geo.nd && ok; ++k) {
+            lo[k] = ranges[q * geo.nd + k].lo;
+            hi[k] = ranges[q * geo.nd + k].hi;
+            if (lo[k] < 0 || hi[k] >= geo.n[k]) ok = false;
+            if (lo[k] > hi[k]) empty = true;
+        }
+        if (ok && !empty) {
+            int64_t llo, lhi;
+            if (shard_local_range(geo.n[0], geo.G, geo.g, geo.b, lo[0], hi[0], &llo, &lhi)) {
+                lo[0] = llo;
+                hi[0] = lhi;
+            } else {
+                ok = false;
+            }
+        }
+        if (ok && !empty) {
+            TDesc d;
+            const int nd = tg.nd, kt = tg.kt;
+            int64_t ell[kMaxDims];
+            cells = 1;
+            for (int k = 0; k < nd; ++k) {
+                ell[k] = hi[k] - lo[k] + 1;
+                cells *= ell[k];
+            }
+            d.opc = (op == OLAP_MIN) ? OPC_MIN : (op == OLAP_MAX) ? OPC_MAX : OPC_SUM;
+            d.lo_kt = lo[kt];
+            d.hi_kt = hi[kt];
+            // split dim among dims > kt: innermost not fully covered (never merge across padded rows)
+            int ks = nd - 1;
+            if (kt == nd - 1) {
+                ks = kt;
+            } else if (!tg.padded) {
+                while (ks > kt && ell[ks] == tg.ext[ks]) --ks;
+            }
+            d.span = ks == kt;
+            d.base_in = 0;
+            for (int k = kt + 1; k < nd; ++k) d.base_in += lo[k] * tg.stride[k];
+            bool a8 = (tg.stride[kt] & 7) == 0 || d.span, a4 = (tg.stride[kt] & 3) == 0 || d.span;
+            int nrd = 0;
+            d.Rin = 1;
+            d.L = 0;
+            if (!d.span) {
+                d.L = ell[ks] * tg.stride[ks];
+                for (int k = ks - 1; k > kt; --k) {
+                    d.Rin *= ell[k];
+                    if (ell[k] > 1) {
+                        d.frl[nrd] = dev_fastdiv((uint32_t)ell[k]);
+                        d.rs[nrd] = tg.stride[k];
+                        if (tg.stride[k] & 7) a8 = false;
+                        if (tg.stride[k] & 3) a4 = false;
+                        ++nrd;
+                    }
+                }
+            }
+            d.nrd = nrd;
+#ifdef OLAP_TILE_V4
+            a8 = false;
+#endif
+            d.V = a8 ? 8 : (a4 ? 4 : 1);
+            np = 1;
+            for (int k = 0; k < kt; ++k) {
+                d.tlo[k] = lo[k];
+                d.tn[k] = ell[k];
+            }
+            d.tlo[kt] = lo[kt] / tg.ct;
+            d.tn[kt] = hi[kt] / tg.ct - d.tlo[kt] + 1;
+            for (int k = 0; k <= kt; ++k) {
+                np *= d.tn[k];
+                d.tfd[k] = dev_fastdiv((uint32_t)d.tn[k]);
+            }
+            tdesc[q] = d;
+        }
+        q_pairs[q] = np;
+        if (np == 0) {  // identity partials (COUNT, empty, invalid, no owned row: finalize decides)
+            psum[q] = 0;
+            pext[2 * q] = INT_MIN;
+            pext[2 * q + 1] = INT_MIN;
+        }
+    }
+    cells = block_sum<int64_t>(cells, sh);
+    if (threadIdx.x == 0 && cells) atomicAdd(totals, (unsigned long long)cells);
+}
+
+// One block: exclusive scan of pair counts -> pair_start[0..nq]; choose the path.
+// ctl: [0] mode (1 = tiles), [1] non-empty tiles, [2] tile pop counter.
+// Tiles pay when every staged byte is reused: cells >= 4 x staged cells (staged <= min(pairs,
+// ntiles) tiles) and pairs are big enough to amortise their set-up (>= 256 cells each).
+__global__ void __launch_bounds__(kPlanThreads) tile_scan_kernel(int64_t nq, const int64_t* __restrict__ q_pairs,
+                                                                 int64_t* pair_start, int64_t pairs_cap, TGeo tg,
+                                                                 const unsigned long long* totals, int32_t* ctl,
+                                                                 unsigned long long* bytes_acc) {
+    const int tid = threadIdx.x;
+    const int64_t per = (nq + kPlanThreads - 1) / kPlanThreads;
+    const int64_t q0 = min(nq, (int64_t)tid * per), q1 = min(nq, q0 + per);
+    int64_t mine = 0;
+    for (int64_t q = q0; q < q1; ++q) mine += q_pairs[q];
+    __shared__ int64_t scan[kPlanThreads];
+    scan[tid] = mine;
+    __syncthreads();
+    for (int o = 1; o < kPlanThreads; o <<= 1) {
+        int64_t v = tid >= o ? scan[tid - o] : 0;
+        __syncthreads();
+        scan[tid] += v;
+        __syncthreads();
+    }
+    int64_t off = scan[tid] - mine;
+    for (int64_t q = q0; q < q1; ++q) {
+        pair_start[q] = off;
+        off += q_pairs[q];
+    }
+    if (tid == kPlanThreads - 1) {
+        const int64_t pairs = scan[tid];
+        const int64_t cells = (int64_t)totals[0];
+        pair_start[nq] = pairs;
+        const int64_t staged = min(pairs, tg.ntiles) * tg.tcells;
+        const int use = tg.ok && pairs > 0 && pairs <= pairs_cap && cells >= 4 * staged && cells >= 256 * pairs;
+        ctl[0] = use;
+        ctl[1] = 0;
+        ctl[2] = 0;
+        if (use) atomicAdd(bytes_acc, (unsigned long long)(cells * 4));
+    }
+}
+
+// tile id of query d's j-th pair (row-major over its tile box)
+__device__ __forceinline__ int64_t pair_tile(const TGeo& tg, const TDesc& d, uint32_t j) {
+    int64_t t = 0;
+    for (int k = tg.kt; k >= 0; --k) {
+        const uint32_t qk = fdiv(j, d.tfd[k]);
+        t += (d.tlo[k] + (int64_t)(j - qk * d.tfd[k].d)) * tg.ts[k];
+        j = qk;
+    }
+    return t;
+}
+
+// Pairs p0 .. p0+K-1 of the batch: (query, pair index) walked forward from one search.
+template <class F>
+__device__ __forceinline__ void for_pairs(int64_t nq, const int64_t* __restrict__ pair_start, F&& f) {
+    const int64_t total = __ldg(pair_start + nq);
+    for (int64_t p0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * kTilePairsPerThread; p0 < total;
+         p0 += (int64_t)gridDim.x * blockDim.x * kTilePairsPerThread) {
+        int64_t q = find_query_thread(pair_start, nq, p0);
+        int64_t j = p0 - __ldg(pair_start + q), end = __ldg(pair_start + q + 1);
+        const int64_t p1 = min(total, p0 + kTilePairsPerThread);
+        for (int64_t p = p0; p < p1; ++p) {
+            while (p >= end) {  // next query with pairs
+                ++q;
+                j = 0;
+                end = __ldg(pair_start + q + 1);
+            }
+            f(q, j);
+            ++j;
+        }
+    }
+}
+
+// A tile's query list is kept in three op groups (key 3 t + opc - 1: SUM, MIN, MAX) so that
+// the consumer warps of a tile mostly run the same specialised loop at the same time (one
+// code path in the instruction cache instead of up to 31).
+__device__ __forceinline__ int64_t pair_key(const TGeo& tg, const TDesc& d, uint32_t j) {
+    return 3 * pair_tile(tg, d, j) + (d.opc - 1);
+}
+
+__global__ void tile_count_kernel(TGeo tg, int64_t nq, const int64_t* __restrict__ pair_start,
+                                  const TDesc* __restrict__ tdesc, unsigned int* count, const int32_t* ctl) {
+    if (!ctl[0]) return;
+    for_pairs(nq, pair_start, [&](int64_t q, int64_t j) { atomicAdd(count + pair_key(tg, tdesc[q], (uint32_t)j), 1u); });
+}
+
+// non-empty tiles (any order: each is staged once whatever the order)
+__global__ void tile_compact_kernel(int64_t ntiles, const unsigned int* __restrict__ tile_start, int32_t* ctl,
+                                    uint32_t* nonempty) {
+    if (!ctl[0]) return;
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < ntiles; t += (int64_t)gridDim.x * blockDim.x)
+        if (tile_start[3 * t + 3] > tile_start[3 * t]) nonempty[atomicAdd(ctl + 1, 1)] = (uint32_t)t;
+}
+
+// count[] holds the per-tile counts again on entry (it is decremented to 0 here)
+__global__ void tile_scatter_kernel(TGeo tg, int64_t nq, const int64_t* __restrict__ pair_start,
+                                    const TDesc* __restrict__ tdesc, unsigned int* count,
+                                    const unsigned int* __restrict__ tile_start, const int32_t* __restrict__ ctl,
+                                    uint32_t* list) {
+    if (!ctl[0]) return;
+    for_pairs(nq, pair_start, [&](int64_t q, int64_t j) {
+        const int64_t k = pair_key(tg, tdesc[q], (uint32_t)j);
+        list[tile_start[k] + atomicSub(count + k, 1u) - 1u] = (uint32_t)q;
+    });
+}
+
+// ------------------------------------------------------------------ reduce
+
+struct TileMeta {
+    int64_t t;          // tile id, -1: no more tiles
+    int64_t c, ce;      // chunk index along kt and its extent
+    int64_t x[kMaxDims];  // tile coordinates of dims < kt
+    uint32_t lbeg, cnt;   // the tile's query list
+    unsigned int next;    // next list entry to claim
+};
+
+// The clipped box of query d in tile (x, c) as a QDesc over the staged tile (cells relative to
+// the tile start): runs over dims kt..ks-1, or one span over dim kt.
+__device__ __forceinline__ void build_pair_desc(const TGeo& tg, const TDesc& d, int64_t c, int64_t ce, QDesc& pd) {
+    const int64_t c0 = c * tg.ct;
+    const int64_t a = max(d.lo_kt, c0) - c0, b = min(d.hi_kt, c0 + ce - 1) - c0, na = b - a + 1;
+    const int64_t skt = tg.stride[tg.kt];
+    const int64_t base = a * skt + d.base_in;
+    int nrd = d.nrd;
+    for (int e = 0; e < nrd; ++e) {
+        pd.frl[e] = d.frl[e];
+        pd.rs[e] = d.rs[e];
+    }
+    if (d.span) {
+        pd.L = na * skt;
+        pd.R = 1;
+    } else {
+        pd.L = d.L;
+        pd.R = na * d.Rin;
+        if (na > 1) {
+            pd.frl[nrd] = dev_fastdiv((uint32_t)na);
+            pd.rs[nrd] = skt;
+            ++nrd;
+        }
+    }
+    pd.nrd = nrd;
+    const int V = d.V;
+    pd.V = V;
+    pd.h0 = (int32_t)(base & (V - 1));
+    pd.base_al = base - pd.h0;
+    pd.nslot = (pd.h0 + pd.L + V - 1) / V;
+    pd.G = pd.R * pd.nslot;
+    pd.vlocal = pd.R * pd.L;
+    pd.opc = d.opc;
+    pd.tpi = 1;
+    if (pd.nslot <= kShortMaxSlots) {
+        pd.shortp = 1;
+        int64_t rpt = kTaskSlots / pd.nslot;
+        rpt = rpt < 1 ? 1 : (rpt > 31 ? 31 : rpt);
+        pd.T = (int32_t)rpt;
+        pd.tasks = (pd.R + rpt - 1) / rpt;
+        pd.fni = dev_fastdiv(pd.nslot > 2 ? (uint32_t)(pd.nslot - 2) : 1u);
+        pd.fnslot = dev_fastdiv(1u);
+    } else {
+        pd.shortp = 0;
+        pd.T = pd.nslot < kTaskSlots ? (int32_t)pd.nslot : kTaskSlots;
+        pd.tasks = (pd.G + pd.T - 1) / pd.T;
+        pd.fnslot = dev_fastdiv(pd.nslot < (1ll << 31) ? (uint32_t)pd.nslot : 1u);
+        pd.fni = dev_fastdiv(1u);
+    }
+}
+
+constexpr size_t tile_smem_bytes() {
+    return (size_t)kTileStages * (kTileCellsMax + kTileSlack) * 4 + kTileStages * sizeof(TileMeta) +
+           2 * kTileStages * sizeof(uint64_t) + kTileConsumers * sizeof(QDesc) + 256;
+}
+
+template <typename T, class Acc>
+__global__ void __launch_bounds__(kTileThreads, 1)
+    tile_reduce_kernel(const T* __restrict__ cube, TGeo tg, const TDesc* __restrict__ tdesc,
+                       const int64_t* __restrict__ pair_start, const unsigned int* __restrict__ tile_start,
+                       const uint32_t* __restrict__ nonempty, const uint32_t* __restrict__ list, int32_t* ctl,
+                       long long* __restrict__ partial) {
+    if (!*(volatile int32_t*)ctl) return;
+    extern __shared__ __align__(128) unsigned char smem[];
+    uint32_t* buf = reinterpret_cast<uint32_t*>(smem);  // kTileStages x (kTileCellsMax + kTileSlack) cells
+    TileMeta* meta = reinterpret_cast<TileMeta*>(smem + (size_t)kTileStages * (kTileCellsMax + kTileSlack) * 4);
+    uint64_t* full = reinterpret_cast<uint64_t*>(meta + kTileStages);
+    uint64_t* empty = full + kTileStages;
+    QDesc* pds = reinterpret_cast<QDesc*>(empty + kTileStages);
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kTileStages; ++s) {
+            mbar_init(full + s, 1);
+            mbar_init(empty + s, kTileConsumers);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    const int64_t bufcells = kTileCellsMax + kTileSlack;
+    if (w == 0) {  // producer: pop non-empty tiles, stage each with one bulk copy
+        if (lane == 0) {
+            const uint32_t nne = (uint32_t)ctl[1];
+            const int kt = tg.kt;
+            for (int64_t i = 0;; ++i) {
+                const int s = (int)(i % kTileStages);
+                const uint32_t ph = (uint32_t)((i / kTileStages) & 1);
+                if (i >= kTileStages) mbar_wait_sleep(empty + s, ph ^ 1u);
+                const uint32_t k = (uint32_t)atomicAdd(ctl + 2, 1);
+                TileMeta& m = meta[s];
+                if (k >= nne) {
+                    m.t = -1;
+                    mbar_arrive(full + s);
+                    break;
+                }
+                const int64_t t = nonempty[k];
+                m.t = t;
+                m.next = 0;
+                m.lbeg = tile_start[3 * t];
+                m.cnt = tile_start[3 * t + 3] - m.lbeg;
+                int64_t r = t;
+                m.c = r % tg.nct;
+                r /= tg.nct;
+                int64_t start = m.c * tg.ct * tg.stride[kt];
+                for (int e = kt - 1; e >= 0; --e) {
+                    const int64_t xe = r % tg.ext[e];
+                    r /= tg.ext[e];
+                    m.x[e] = xe;
+                    start += xe * tg.stride[e];
+                }
+                m.ce = min(tg.ct, tg.ext[kt] - m.c * tg.ct);
+                const int64_t cells = (m.ce * tg.stride[kt] + 3) & ~3ll;
+                const uint32_t bytes = (uint32_t)(cells * 4);
+                mbar_arrive_tx(full + s, bytes);
+                const char* src = reinterpret_cast<const char*>(cube + start);
+                char* dst = reinterpret_cast<char*>(buf + s * bufcells);
+                for (uint32_t o = 0; o < bytes; o += 16384u)
+                    bulk_g2s(dst + o, src + o, min(16384u, bytes - o), full + s);
+            }
+        }
+        return;
+    }
+    // consumers: every pair of the staged tile, one warp per pair
+    QDesc& pd = pds[w - 1];
+    for (int64_t i = 0;; ++i) {
+        const int s = (int)(i % kTileStages);
+        const uint32_t ph = (uint32_t)((i / kTileStages) & 1);
+        mbar_wait(full + s, ph);
+        TileMeta& m = meta[s];
+        const int64_t t = m.t;
+        if (t < 0) break;
+        const uint32_t* sb = buf + s * bufcells;
+        for (;;) {
+            uint32_t e = 0;
+            if (lane == 0) e = atomicAdd(&m.next, 1u);
+            e = __shfl_sync(0xffffffffu, e, 0);
+            if (e >= m.cnt) break;
+            const int64_t q = __ldg(list + m.lbeg + e);
+            const TDesc& d = tdesc[q];
+            if (lane == 0) build_pair_desc(tg, d, m.c, m.ce, pd);
+            // pair index j of this tile in the query's tile box
+            int64_t j = 0;
+            for (int k = 0; k < tg.kt; ++k) j = j * d.tn[k] + (m.x[k] - d.tlo[k]);
+            j = j * d.tn[tg.kt] + (m.c - d.tlo[tg.kt]);
+            const int64_t p = __ldg(pair_start + q) + j;
+            __syncwarp();
+            Acc acc;
+            acc.init();
+            stream_item<T, Acc, true>(reinterpret_cast<const T*>(sb), pd, 0, pd.tasks, acc, lane, 0, 1);
+            const int opc = pd.opc;
+            long long v;
+            if (opc == OPC_SUM) {
+                long long sm = acc.sum_bits();
+#pragma unroll
+                for (int o = 16; o; o >>= 1) sm = SumOps<Acc>::add(sm, __shfl_xor_sync(0xffffffffu, sm, o));
+                v = sm;
+            } else if (opc == OPC_MAX) {
+                v = __reduce_max_sync(0xffffffffu, acc.code_max());
+            } else {
+                v = __reduce_max_sync(0xffffffffu, ~acc.code_min());
+            }
+            if (lane == 0) partial[p] = v;
+            __syncwarp();
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(empty + s);
+    }
+}
+
+// One block per query with pairs: fold its pair partials in pair order (fixed tree) into the
+// per-query partial format (sum, max code, ~min code).
+template <class Acc>
+__global__ void __launch_bounds__(256) pair_fold_kernel(int64_t nq, const int64_t* __restrict__ pair_start,
+                                                        const TDesc* __restrict__ tdesc, const int32_t* ctl,
+                                                        const long long* __restrict__ partial, int64_t* psum,
+                                                        int32_t* pext) {
+    if (!ctl[0]) return;
+    __shared__ long long sh[8];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    for (int64_t q = blockIdx.x; q < nq; q += gridDim.x) {
+        const int64_t b = __ldg(pair_start + q), e = __ldg(pair_start + q + 1);
+        if (b == e) continue;  // identity partials written by tile_desc_kernel
+        const int opc = tdesc[q].opc;
+        long long v = opc == OPC_SUM ? 0ll : (long long)INT_MIN;
+        for (int64_t p = b + threadIdx.x; p < e; p += blockDim.x) {
+            const long long x = __ldcg(partial + p);
+            v = opc == OPC_SUM ? SumOps<Acc>::add(v, x) : max(v, x);
+        }
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+            const long long y = __shfl_xor_sync(0xffffffffu, v, o);
+            v = opc == OPC_SUM ? SumOps<Acc>::add(v, y) : max(v, y);
+        }
+        if (lane == 0) sh[w] = v;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            long long f = sh[0];
+            for (int i = 1; i < 8; ++i) f = opc == OPC_SUM ? SumOps<Acc>::add(f, sh[i]) : max(f, sh[i]);
+            psum[q] = opc == OPC_SUM ? f : 0;
+            pext[2 * q] = opc == OPC_MAX ? (int32_t)f : INT_MIN;
+            pext[2 * q + 1] = opc == OPC_MIN ? (int32_t)f : INT_MIN;
+        }
+        __syncthreads();
+    }
+}
