@@ -267,6 +267,7 @@ __device__ __forceinline__ uint64_t byte_mask_word(uint32_t bits8) {
 // first (and second) LDS.128 covers all 32 banks once instead of two-way conflicting on a
 // 32-B lane stride.  Those lanes hold cells 4-7 in v[0..3]: sm_swap() swaps their masks.
 __device__ __forceinline__ bool sm_swapped() { return (threadIdx.x >> 2) & 1; }
+__device__ __forceinline__ uint32_t smem_addr_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 template <int V, bool SM = false>
 __device__ __forceinline__ void load_slot(const uint32_t* p, uint32_t (&v)[V]) {
     if constexpr (SM) {
@@ -371,6 +372,9 @@ __device__ __forceinline__ void slot_masks(const QDesc& d, uint64_t& wf, uint64_
 #define OLAP_U8 3
 #endif
 constexpr int unroll_for(int V) { return V == 8 ? OLAP_U8 : 4; }
+#ifndef OLAP_SM_COLS
+#define OLAP_SM_COLS 1  // tile path: column mode for runs of <= 32 slots (stream_cols)
+#endif
 #ifndef OLAP_SM_U
 #define OLAP_SM_U 2  // tile path (shared-memory slots): slots in flight per lane
 #endif
@@ -500,10 +504,138 @@ __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, c
 }
 
 // Tasks t0+w, t0+w+ws, ... < t1 of one query's item (ws warps share the item).
+// Tile path, runs of <= 32 slots whose start addresses need <= 2 digits (every pair of the
+// benchmark cubes): "column mode".  Lane l owns slot s = l % nslot of run group l / nslot and
+// keeps it for the whole pair, so its mask is fixed (built once) and the warp reads
+// g = 32 / nslot whole runs per step, each as one contiguous span of shared memory (no
+// per-slot division, no shuffle, no separate edge pass).  Idle lanes read lane 0's slot
+// with an all-zero mask.  Offsets inside a staged tile fit in 32 bits.
+template <class Acc, int OPC, int V>
+__device__ __forceinline__ void fold_masked(Acc& acc, const uint32_t (&v)[V], const uint32_t (&m)[V]) {
+    if constexpr (tree_sum<Acc, OPC, V, true>()) {
+        uint32_t x[V];
+#pragma unroll
+        for (int k = 0; k < V; ++k) x[k] = v[k] & m[k];
+        acc.s += (double)slot_tree<V>(x);
+    } else {
+#pragma unroll
+        for (int k = 0; k < V; ++k) acc.template add<OPC>(v[k], m[k]);
+    }
+}
+
+__device__ __forceinline__ uint4 lds128(uint32_t a) {
+    uint4 r;
+    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "r"(a));
+    return r;
+}
+// one slot at shared byte addresses pa (cells 0-3 of v) and pb (cells 4-7; V == 8 only)
+template <int V>
+__device__ __forceinline__ void lds_slot(uint32_t pa, uint32_t pb, uint32_t (&v)[V]) {
+    const uint4 x = lds128(pa);
+    v[0] = x.x;
+    v[1] = x.y;
+    v[2] = x.z;
+    v[3] = x.w;
+    if constexpr (V == 8) {
+        const uint4 y = lds128(pb);
+        v[4] = y.x;
+        v[5] = y.y;
+        v[6] = y.z;
+        v[7] = y.w;
+    }
+}
+
+// NRD = digits of a run's start (0: one run; 1: r * rs0; 2: (r mod rad0) * rs0 + (r div rad0) * rs1).
+// The lane's run advances by g per step; its offset is updated incrementally (one carry test).
+template <class Acc, int OPC, int V, int NRD>
+__device__ __forceinline__ void stream_cols(const uint32_t* __restrict__ sb, const QDesc& d, Acc& acc, int lane) {
+    static_assert(V == 4 || V == 8, "column mode reads 16-B slots");
+    const uint32_t nslot = (uint32_t)d.nslot;
+    const uint32_t g = 32u / nslot;
+    const uint32_t grp = (uint32_t)lane / nslot;
+    const uint32_t R = (uint32_t)d.R;
+    const bool act = grp < g && grp < R;
+    const uint32_t sl = act ? (uint32_t)lane - grp * nslot : 0u;
+    uint64_t wf, wl, wb;
+    slot_masks<V>(d, wf, wl, wb);
+    uint64_t w = nslot == 1 ? wb : (sl == 0 ? wf : (sl == nslot - 1 ? wl : ~0ull));
+    if (!act) w = 0;
+    const bool swp = V == 8 && sm_swapped();
+    if (swp) w = (w >> 32) | (w << 32);
+    uint32_t m[V];
+#pragma unroll
+    for (int k = 0; k < V; ++k) m[k] = cell_mask<V>(w, k);
+    // lane byte addresses of its slot's two halves (half-swapped lanes read the upper half first)
+    const uint32_t a0 = smem_addr_u32(sb) + ((uint32_t)d.base_al + sl * V) * 4u;
+    const uint32_t pa = a0 + (swp ? 16u : 0u), pb = a0 + (swp ? 0u : 16u);
+    const uint32_t my = act ? grp : 0u;
+    uint32_t off = 0, x0 = 0, rad0 = 1, s0 = 0, dstep = 0, dcarry = 0;
+    if constexpr (NRD == 1) {
+        const uint32_t rs0 = (uint32_t)d.rs[0] * 4u;
+        off = my * rs0;
+        dstep = g * rs0;
+    } else if constexpr (NRD == 2) {
+        const FastDiv f0 = d.frl[0];
+        const uint32_t rs0 = (uint32_t)d.rs[0] * 4u, rs1 = (uint32_t)d.rs[1] * 4u;
+        rad0 = f0.d;
+        const uint32_t q = fdiv(my, f0), s1 = fdiv(g, f0);
+        x0 = my - q * rad0;
+        s0 = g - s1 * rad0;
+        off = x0 * rs0 + q * rs1;
+        dstep = s0 * rs0 + s1 * rs1;
+        dcarry = rs1 - rad0 * rs0;
+    }
+    auto step = [&]() {
+        off += dstep;
+        if constexpr (NRD == 2) {
+            x0 += s0;
+            if (x0 >= rad0) {
+                x0 -= rad0;
+                off += dcarry;
+            }
+        }
+    };
+    const uint32_t full = (R / g) * g;  // steps in which every group has a run
+    uint32_t r0 = 0;
+    for (; r0 + 2 * g <= full; r0 += 2 * g) {
+        uint32_t v0[V], v1[V];
+        lds_slot<V>(pa + off, pb + off, v0);
+        step();
+        lds_slot<V>(pa + off, pb + off, v1);
+        step();
+        fold_masked<Acc, OPC, V>(acc, v0, m);
+        fold_masked<Acc, OPC, V>(acc, v1, m);
+    }
+    if (r0 < full) {
+        uint32_t v0[V];
+        lds_slot<V>(pa + off, pb + off, v0);
+        step();
+        fold_masked<Acc, OPC, V>(acc, v0, m);
+        r0 += g;
+    }
+    if (r0 < R) {  // last, partial step: groups past the last run read run 0 and contribute identities
+        const bool ok = r0 + my < R;
+        const uint32_t okm = ok ? 0xFFFFFFFFu : 0u, o = ok ? off : 0u;
+        uint32_t v0[V], mm[V];
+        lds_slot<V>(pa + o, pb + o, v0);
+#pragma unroll
+        for (int k = 0; k < V; ++k) mm[k] = m[k] & okm;
+        fold_masked<Acc, OPC, V>(acc, v0, mm);
+    }
+}
+
 template <typename T, class Acc, int OPC, int V, bool SM = false>
 __device__ __forceinline__ void stream_tasks(const T* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
                                              Acc& acc, int lane, int w, int ws = kWarps) {
     const uint32_t* c = reinterpret_cast<const uint32_t*>(cube);
+    if constexpr (SM && V >= 4) {
+        if (OLAP_SM_COLS && d.shortp && d.nslot <= 32 && d.nrd <= 2) {
+            if (d.nrd == 2) stream_cols<Acc, OPC, V, 2>(c, d, acc, lane);
+            else if (d.nrd == 1) stream_cols<Acc, OPC, V, 1>(c, d, acc, lane);
+            else stream_cols<Acc, OPC, V, 0>(c, d, acc, lane);
+            return;
+        }
+    }
     if (d.shortp) {
         if (SM) stream_short<Acc, OPC, V, OLAP_SM_U, SM>(c, d, t0, t1, acc, lane, w, ws);
         else if (V == 8 && d.nslot < 16) stream_short<Acc, OPC, V, 2, SM>(c, d, t0, t1, acc, lane, w, ws);

@@ -25,12 +25,12 @@
 // at once.
 
 #ifndef OLAP_TILE_CELLS
-#define OLAP_TILE_CELLS 16384
+#define OLAP_TILE_CELLS 24576
 #endif
 #ifndef OLAP_TILE_STAGES
-#define OLAP_TILE_STAGES 3
+#define OLAP_TILE_STAGES 2
 #endif
-constexpr int64_t kTileCellsMax = OLAP_TILE_CELLS;  // 64 KiB of 4-byte cells per tile
+constexpr int64_t kTileCellsMax = OLAP_TILE_CELLS;  // 96 KiB of 4-byte cells per tile (2 stages: measured best)
 constexpr int kTileStages = OLAP_TILE_STAGES;
 constexpr int kTileWarps = 32;  // warp 0: producer; warps 1..31: consumers
 constexpr int kTileThreads = kTileWarps * 32;
@@ -326,50 +326,59 @@ struct TileMeta {
 // The clipped box of query d in tile (x, c) as a QDesc over the staged tile (cells relative to
 // the tile start): runs over dims kt..ks-1, or one span over dim kt.
 __device__ __forceinline__ void build_pair_desc(const TGeo& tg, const TDesc& d, int64_t c, int64_t ce, QDesc& pd) {
+    // everything inside a staged tile fits 32-bit arithmetic (offsets < kTileCellsMax); no 64-bit
+    // division on the common path (column mode needs only the innermost radix, from TDesc)
     const int64_t c0 = c * tg.ct;
-    const int64_t a = max(d.lo_kt, c0) - c0, b = min(d.hi_kt, c0 + ce - 1) - c0, na = b - a + 1;
-    const int64_t skt = tg.stride[tg.kt];
-    const int64_t base = a * skt + d.base_in;
+    const uint32_t a = (uint32_t)(max(d.lo_kt, c0) - c0), b = (uint32_t)(min(d.hi_kt, c0 + ce - 1) - c0);
+    const uint32_t na = b - a + 1;
+    const uint32_t skt = (uint32_t)tg.stride[tg.kt];
+    const uint32_t base = a * skt + (uint32_t)d.base_in;
     int nrd = d.nrd;
     for (int e = 0; e < nrd; ++e) {
         pd.frl[e] = d.frl[e];
         pd.rs[e] = d.rs[e];
     }
+    uint32_t L, R;
+    bool radix_na = false;
     if (d.span) {
-        pd.L = na * skt;
-        pd.R = 1;
+        L = na * skt;
+        R = 1;
     } else {
-        pd.L = d.L;
-        pd.R = na * d.Rin;
+        L = (uint32_t)d.L;
+        R = na * (uint32_t)d.Rin;
         if (na > 1) {
-            pd.frl[nrd] = dev_fastdiv((uint32_t)na);
+            radix_na = true;
             pd.rs[nrd] = skt;
             ++nrd;
         }
     }
     pd.nrd = nrd;
-    const int V = d.V;
-    pd.V = V;
-    pd.h0 = (int32_t)(base & (V - 1));
-    pd.base_al = base - pd.h0;
-    pd.nslot = (pd.h0 + pd.L + V - 1) / V;
-    pd.G = pd.R * pd.nslot;
-    pd.vlocal = pd.R * pd.L;
+    const uint32_t V = (uint32_t)d.V, lv = V == 8 ? 3u : (V == 4 ? 2u : 0u);
+    const uint32_t h0 = base & (V - 1), nslot = (h0 + L + V - 1) >> lv;
+    pd.V = (int32_t)V;
+    pd.h0 = (int32_t)h0;
+    pd.base_al = base - h0;
+    pd.L = L;
+    pd.R = R;
+    pd.nslot = nslot;
+    pd.G = (int64_t)R * nslot;
+    pd.vlocal = (int64_t)R * L;
     pd.opc = d.opc;
     pd.tpi = 1;
-    if (pd.nslot <= kShortMaxSlots) {
-        pd.shortp = 1;
-        int64_t rpt = kTaskSlots / pd.nslot;
+    pd.shortp = nslot <= (uint32_t)kShortMaxSlots;
+    if (OLAP_SM_COLS && pd.shortp && nslot <= 32 && nrd <= 2) return;  // column mode: nothing else needed
+    if (radix_na) pd.frl[nrd - 1] = dev_fastdiv(na);
+    if (pd.shortp) {
+        uint32_t rpt = (uint32_t)kTaskSlots / nslot;
         rpt = rpt < 1 ? 1 : (rpt > 31 ? 31 : rpt);
         pd.T = (int32_t)rpt;
-        pd.tasks = (pd.R + rpt - 1) / rpt;
-        pd.fni = dev_fastdiv(pd.nslot > 2 ? (uint32_t)(pd.nslot - 2) : 1u);
+        pd.tasks = (R + rpt - 1) / rpt;
+        pd.fni = dev_fastdiv(nslot > 2 ? nslot - 2 : 1u);
         pd.fnslot = dev_fastdiv(1u);
     } else {
-        pd.shortp = 0;
-        pd.T = pd.nslot < kTaskSlots ? (int32_t)pd.nslot : kTaskSlots;
+        pd.T = nslot < (uint32_t)kTaskSlots ? (int32_t)nslot : kTaskSlots;
         pd.tasks = (pd.G + pd.T - 1) / pd.T;
-        pd.fnslot = dev_fastdiv(pd.nslot < (1ll << 31) ? (uint32_t)pd.nslot : 1u);
+        pd.fnslot = dev_fastdiv(nslot);
         pd.fni = dev_fastdiv(1u);
     }
 }

@@ -17,8 +17,10 @@ from test_gpu_parity import compare
 
 pytestmark = pytest.mark.gpu
 
+TILE_CELLS_MAX = 24576   # tiles.cuh kTileCellsMax (96 KiB)
+
 TILE_SHAPES = [
-    ((40, 16, 16, 16, 160), "kt=2, chunks 6/6/4 (ragged), 32-B slots"),
+    ((40, 16, 20, 16, 160), "kt=2, chunks 7/7/6 (ragged), 32-B slots"),
     ((6, 3000003), "kt = innermost dim: chunks of a padded 3M-cell row"),
     ((17000003,), "1-D: chunks of the only dim"),
     ((1500, 1000, 12), "inner 12: 16-B slots, tile = one dim-0 row"),
@@ -45,7 +47,7 @@ def test_tile_path_parity(ext, why, dtype):
     c = olap.Cube(ext, dtype)
     c.fill(olap.GEN_UNIFORM, seed)
     en, tcells, ntiles, _ = c.tile_stats()
-    assert en and 0 < tcells <= 16384 and ntiles >= 1
+    assert en and 0 < tcells <= TILE_CELLS_MAX and ntiles >= 1
     rng = np.random.default_rng(seed)
     boxes, ops = _batch(ext, rng)
     got = c.query(boxes, ops)
