@@ -168,12 +168,23 @@ def _host_cells(ext, dtype_str, seed):
     return synth.uniform_cells(int(np.prod(ext)), np.dtype(dtype_str), seed)
 
 
-def _traffic(workload):
+def _traffic(workload, kernel="reduce_kernel"):
+    """DRAM read+write bytes per launch of `kernel` on `workload` from ncu (profiles/traffic.json)."""
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
         with open(tp) as f:
-            return json.load(f).get(workload)
+            v = json.load(f).get(workload)
+        if isinstance(v, dict):
+            return v.get(kernel)
+        return v if kernel == "reduce_kernel" else None
     return None
+
+
+# shared-memory bandwidth of one B200: 32 banks x 4 B per clock per SM (B300_MICROARCH.md / Blackwell guide;
+# same SM design), x 148 SMs x the measured max SM clock.  The tile path serves every per-query read from
+# shared memory, so this — not HBM — is the ceiling its kernel is measured against (DESIGN.md §6).
+def smem_peak_gbs(sm_mhz):
+    return 128 * 148 * sm_mhz * 1e6 / 1e9
 
 
 def host_info():
@@ -295,6 +306,7 @@ def run_c4(args, rank, world):
     elapsed = e0.elapsed_time(e1)
     clk = clocks.stop()
     trans_ms = sum(a.elapsed_time(b) for a, b, _ in ev)
+    c4_kernel = "tile_reduce_kernel" if cube.tile_stats()[3] else "reduce_kernel"
     gpu_launches = cube.stats()[0] - k0 + olap.lib.olap_finalize_launches() - f0 + steps  # + one text_ranges_kernel
     reduce_ms, launches, alg_bytes = cube.profile_read()
     cube.profile(False)
@@ -321,8 +333,12 @@ def run_c4(args, rank, world):
         "translation": {"keys_per_s": nkeys / (trans_ms / 1e3), "share_of_step": trans_ms / elapsed,
                         "paper_share": 0.07},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                     "traffic": _traffic("C4"), "kernel": "reduce_kernel", "peak_source": peak_src,
-                     "note": "frac > 1 is L2/L1 reuse across overlapping queries (traffic = ncu DRAM bytes/launch)"},
+                     "traffic": _traffic("C4", c4_kernel), "kernel": c4_kernel, "peak_source": peak_src,
+                     "note": ("frac > 1: " + ("the tile-shared scan stages each cube tile in shared memory once per "
+                                              "batch and serves every query's reads from there"
+                                              if c4_kernel == "tile_reduce_kernel" else
+                                              "L2/L1 reuse across overlapping queries") +
+                              " (traffic = ncu DRAM bytes/launch)")},
         "gpu_launches": int(gpu_launches), "clocks": clk,
         "e2e": {"value": nq * e2e_steps / e2e_s, "unit": "queries/s",
                 "h2d_bytes_per_step": int(sum(x.nbytes for x in batches_[warm]["host"])) + int(nq * 4 * 2 * 16 + nq * 4),
@@ -615,6 +631,7 @@ def main():
     torch.cuda.synchronize()
     elapsed_ms = e0.elapsed_time(e1)
     clk = clocks.stop()
+    tiles_enabled, tile_cells, _nt, tiles_used = cube.tile_stats()
     gpu_launches = cube.stats()[0] - k0 + olap.lib.olap_finalize_launches() - f0
     reduce_ms, launches, alg_bytes = cube.profile_read()
     cube.profile(False)
@@ -675,7 +692,23 @@ def main():
                "h2d_bytes_per_step": int(nq * nd * 16 + nq * 4), "d2h_bytes_per_step": int(nq * 24),
                "api": "ShardedCube path: H2D, olap_query_partials_device, NCCL all-reduce, olap_finalize_device, D2H"}
 
-    traffic = _traffic(args.workload)
+    kernel = "tile_reduce_kernel" if tiles_used else "reduce_kernel"
+    traffic = _traffic(args.workload, kernel)
+    if tiles_used:
+        sm_mhz = (clk or {}).get("sm_mhz") or 1965.0
+        rnote = ("tile-shared scan: each 96-KiB cube tile is staged into shared memory once per batch (cp.async.bulk; "
+                 "traffic = its DRAM bytes per launch from ncu) and every query reads its cells from shared memory; "
+                 "achieved = algorithmic bytes (sum of V_q*4 over non-COUNT queries, Eq. 3) / tile_reduce_kernel "
+                 "time, so frac vs HBM > 1 by construction; smem.frac is the same bytes against the shared-memory "
+                 "bandwidth that bounds the kernel (128 B/clk/SM x 148 SMs at the measured SM clock)")
+        smem = {"peak": smem_peak_gbs(sm_mhz), "unit": "GB/s", "frac": achieved / smem_peak_gbs(sm_mhz),
+                "peak_source": f"derived: 128 B/clk/SM x 148 SMs x {sm_mhz:.0f} MHz (median SM clock in the timed region)"}
+    else:
+        rnote = ("achieved = algorithmic bytes (sum of V_q*4 over non-COUNT queries, Eq. 3) / "
+                 "reduce-kernel time; frac > 1 is L2 reuse: items are scheduled in cube-address "
+                 "order so queries overlapping in the cube read it from L2 (traffic = DRAM "
+                 "bytes per launch from ncu, profiles/traffic.json)")
+        smem = None
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -691,18 +724,18 @@ def main():
                        "queries": DESC[args.workload],
                        "l2": ("no flush: C1's 4 MiB cube is L2-resident by design (flagged)" if args.workload == "C1"
                               else "no flush: cube > L2 (126 MB) and every step reads >> L2"),
-                       "accumulation": "int32 cells, int64 SUM" if dtype == np.int32 else "f32 cells, f64 SUM",
+                       "accumulation": ("int32 cells, int64 SUM" if dtype == np.int32 else
+                                        ("f32 cells, SUM in fp32 trees of <= 8 cells then f64" if tiles_used
+                                         else "f32 cells, f64 SUM")),
+                       "path": "tile-shared scan" if tiles_used else "item path",
                        "parallelism": f"shard{world}" if world > 1 else "1gpu"},
             "gbs": gbs_total, "frac_of_nominal_8tbs": gbs_total / world / NOMINAL_HBM_GBS,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "kernel": "reduce_kernel",
+                         "frac": achieved / peak, "traffic": traffic, "kernel": kernel, "smem": smem,
                          "peak_source": peak_src,
                          "algorithmic_bytes_per_launch": alg_bytes / max(launches, 1),
                          "reduce_share_of_step": reduce_ms / elapsed_ms if elapsed_ms else None,
-                         "note": ("achieved = algorithmic bytes (sum of V_q*4 over non-COUNT queries, Eq. 3) / "
-                                  "reduce-kernel time; frac > 1 is L2 reuse: items are scheduled in cube-address "
-                                  "order so queries overlapping in the cube read it from L2 (traffic = DRAM "
-                                  "bytes per launch from ncu, profiles/traffic.json)")},
+                         "note": rnote},
             "gpu_launches": int(gpu_launches), "l2_order": l2_order,
             "clocks": clk,
             "e2e": e2e,

@@ -372,6 +372,9 @@ __device__ __forceinline__ void slot_masks(const QDesc& d, uint64_t& wf, uint64_
 #define OLAP_U8 3
 #endif
 constexpr int unroll_for(int V) { return V == 8 ? OLAP_U8 : 4; }
+#ifndef OLAP_SM_WIDE
+#define OLAP_SM_WIDE 1  // tile path: wide mode for runs of > 32 slots (stream_wide)
+#endif
 #ifndef OLAP_SM_COLS
 #define OLAP_SM_COLS 1  // tile path: column mode for runs of <= 32 slots (stream_cols)
 #endif
@@ -624,6 +627,73 @@ __device__ __forceinline__ void stream_cols(const uint32_t* __restrict__ sb, con
     }
 }
 
+// Tile path, runs of > 32 slots (NRD as in stream_cols): "wide mode".  One run per step; lane l
+// reads slots l, l+32, l+64, ... of it (32-slot chunks, 1 KiB apart: fixed offsets, no per-slot
+// index arithmetic).  Only the first chunk (slot 0 in lane 0) and the last chunk (slot
+// nslot-1, and lanes past the run end, which re-read the last slot with an all-zero mask)
+// are masked; every chunk in between folds without masks.
+template <class Acc, int OPC, int V, int NRD>
+__device__ __forceinline__ void stream_wide(const uint32_t* __restrict__ sb, const QDesc& d, Acc& acc, int lane) {
+    static_assert(V == 4 || V == 8, "wide mode reads 16-B slots");
+    const uint32_t nslot = (uint32_t)d.nslot;
+    const uint32_t K = (nslot + 31u) >> 5;  // chunks per run, >= 2
+    const uint32_t R = (uint32_t)d.R;
+    uint64_t wf, wl, wb;
+    slot_masks<V>(d, wf, wl, wb);
+    const uint32_t sl_last = (uint32_t)lane + 32u * (K - 1);
+    const uint64_t w0 = lane == 0 ? wf : ~0ull;
+    const uint64_t wL = sl_last == nslot - 1 ? wl : (sl_last < nslot ? ~0ull : 0ull);
+    const bool swp = V == 8 && sm_swapped();
+    const uint32_t a0 = smem_addr_u32(sb) + ((uint32_t)d.base_al + (uint32_t)lane * V) * 4u;
+    const uint32_t pa = a0 + (swp ? 16u : 0u), pb = a0 + (swp ? 0u : 16u);
+    constexpr uint32_t kChunk = 32u * V * 4u;  // bytes between a lane's consecutive slots
+    const uint32_t lastoff = (min(sl_last, nslot - 1) - (uint32_t)lane) * V * 4u;
+    uint32_t off = 0, x0 = 0, rad0 = 1, s1 = 0, rs0 = 0, rs1 = 0;
+    if constexpr (NRD >= 1) rs0 = (uint32_t)d.rs[0] * 4u;
+    if constexpr (NRD == 2) {
+        rad0 = d.frl[0].d;
+        rs1 = (uint32_t)d.rs[1] * 4u;
+        s1 = rs1 - (rad0 - 1) * rs0;  // carry: x0 wraps to 0, next outer digit
+    }
+    for (uint32_t r = 0; r < R; ++r) {
+        {
+            uint32_t v0[V];
+            lds_slot<V>(pa + off, pb + off, v0);
+            fold_slot<Acc, OPC, V, true>(acc, v0, w0);
+        }
+        uint32_t k = 1;
+        for (; k + 2 < K; k += 2) {
+            uint32_t v0[V], v1[V];
+            const uint32_t o0 = off + k * kChunk, o1 = o0 + kChunk;
+            lds_slot<V>(pa + o0, pb + o0, v0);
+            lds_slot<V>(pa + o1, pb + o1, v1);
+            fold_full<Acc, OPC, V, true>(acc, v0);
+            fold_full<Acc, OPC, V, true>(acc, v1);
+        }
+        if (k + 1 < K) {
+            uint32_t v0[V];
+            const uint32_t o0 = off + k * kChunk;
+            lds_slot<V>(pa + o0, pb + o0, v0);
+            fold_full<Acc, OPC, V, true>(acc, v0);
+        }
+        {
+            uint32_t v0[V];
+            lds_slot<V>(pa + off + lastoff, pb + off + lastoff, v0);
+            fold_slot<Acc, OPC, V, true>(acc, v0, wL);
+        }
+        if constexpr (NRD == 1) {
+            off += rs0;
+        } else if constexpr (NRD == 2) {
+            if (++x0 == rad0) {
+                x0 = 0;
+                off += s1;
+            } else {
+                off += rs0;
+            }
+        }
+    }
+}
+
 template <typename T, class Acc, int OPC, int V, bool SM = false>
 __device__ __forceinline__ void stream_tasks(const T* __restrict__ cube, const QDesc& d, int64_t t0, int64_t t1,
                                              Acc& acc, int lane, int w, int ws = kWarps) {
@@ -633,6 +703,12 @@ __device__ __forceinline__ void stream_tasks(const T* __restrict__ cube, const Q
             if (d.nrd == 2) stream_cols<Acc, OPC, V, 2>(c, d, acc, lane);
             else if (d.nrd == 1) stream_cols<Acc, OPC, V, 1>(c, d, acc, lane);
             else stream_cols<Acc, OPC, V, 0>(c, d, acc, lane);
+            return;
+        }
+        if (OLAP_SM_WIDE && d.nslot > 32 && d.nrd <= 2) {
+            if (d.nrd == 2) stream_wide<Acc, OPC, V, 2>(c, d, acc, lane);
+            else if (d.nrd == 1) stream_wide<Acc, OPC, V, 1>(c, d, acc, lane);
+            else stream_wide<Acc, OPC, V, 0>(c, d, acc, lane);
             return;
         }
     }

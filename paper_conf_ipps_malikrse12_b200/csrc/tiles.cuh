@@ -367,6 +367,7 @@ __device__ __forceinline__ void build_pair_desc(const TGeo& tg, const TDesc& d, 
     pd.tpi = 1;
     pd.shortp = nslot <= (uint32_t)kShortMaxSlots;
     if (OLAP_SM_COLS && pd.shortp && nslot <= 32 && nrd <= 2) return;  // column mode: nothing else needed
+    if (OLAP_SM_WIDE && nslot > 32 && nrd <= 2) return;                // wide mode: nothing else needed
     if (radix_na) pd.frl[nrd - 1] = dev_fastdiv(na);
     if (pd.shortp) {
         uint32_t rpt = (uint32_t)kTaskSlots / nslot;
