@@ -558,7 +558,10 @@ __device__ __forceinline__ void stream_cols(const uint32_t* __restrict__ sb, con
     const uint32_t grp = (uint32_t)lane / nslot;
     const uint32_t R = (uint32_t)d.R;
     const bool act = grp < g && grp < R;
-    const uint32_t sl = act ? (uint32_t)lane - grp * nslot : 0u;
+    // idle lanes read the last active lane's slot (same address or the other half of it), so in a
+    // partly idle quarter-warp they broadcast instead of bank-conflicting with the active lanes
+    const uint32_t glast = (g < R ? g : R) - 1u;
+    const uint32_t sl = act ? (uint32_t)lane - grp * nslot : nslot - 1u;
     uint64_t wf, wl, wb;
     slot_masks<V>(d, wf, wl, wb);
     uint64_t w = nslot == 1 ? wb : (sl == 0 ? wf : (sl == nslot - 1 ? wl : ~0ull));
@@ -571,7 +574,7 @@ __device__ __forceinline__ void stream_cols(const uint32_t* __restrict__ sb, con
     // lane byte addresses of its slot's two halves (half-swapped lanes read the upper half first)
     const uint32_t a0 = smem_addr_u32(sb) + ((uint32_t)d.base_al + sl * V) * 4u;
     const uint32_t pa = a0 + (swp ? 16u : 0u), pb = a0 + (swp ? 0u : 16u);
-    const uint32_t my = act ? grp : 0u;
+    const uint32_t my = act ? grp : glast;
     uint32_t off = 0, x0 = 0, rad0 = 1, s0 = 0, dstep = 0, dcarry = 0;
     if constexpr (NRD == 1) {
         const uint32_t rs0 = (uint32_t)d.rs[0] * 4u;
