@@ -1851,6 +1851,7 @@ int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_sh
         if (v > 0 && v < bps) bps = v;
     }
     c->blocks_per_sm = std::max(bps, 1);
+    if (const char* s = getenv("OLAP_L2_FETCH")) cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, atoi(s));
     // L2-aware item order for cubes larger than 64 MiB: buckets of >= 8 MiB, <= kMaxBuckets of them
     if (c->local_cells * 4 > (64ll << 20) && !getenv("OLAP_NO_ORDER")) {
         int sh = 21;  // 2^21 cells = 8 MiB
