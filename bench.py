@@ -545,6 +545,8 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--graph", action="store_true", help="replay each step as a captured CUDA graph (N=1)")
     ap.add_argument("--batch", type=int, default=0, help="queries per batch (default: the config's)")
+    ap.add_argument("--layout", default="auto", choices=["auto", "row", "brick"],
+                    help="cube layout in HBM (auto: bricked for C5's small boxes, row-major otherwise; DESIGN.md §5)")
     args = ap.parse_args()
 
     rank, world, local = env_int("RANK", 0), env_int("WORLD_SIZE", 1), env_int("LOCAL_RANK", 0)
@@ -577,7 +579,9 @@ def main():
     nq = args.batch or cfg["nq"]
     dtype = cfg["dtype"]
     nd = len(ext)
-    cube = olap.Cube(ext, dtype, shard=(world, rank, 1) if world > 1 else None, device=local)
+    layout = args.layout if args.layout != "auto" else ("brick" if args.workload == "C5" else "row")
+    cube = olap.Cube(ext, dtype, shard=(world, rank, 1) if world > 1 else None, device=local,
+                     layout=olap.LAYOUT_BRICK if layout == "brick" else olap.LAYOUT_ROWMAJOR)
     cube.fill(olap.GEN_UNIFORM, cfg["seed"])
     host_batches = batches(args.workload, ext, nq, args.warmup + args.steps, cfg["seed"])
     d_batches = [(torch.from_numpy(b).to(dev), torch.from_numpy(o).to(dev)) for b, o in host_batches]
@@ -728,6 +732,8 @@ def main():
                                         ("f32 cells, SUM in fp32 trees of <= 8 cells then f64" if tiles_used
                                          else "f32 cells, f64 SUM")),
                        "path": "tile-shared scan" if tiles_used else "item path",
+                       "layout": ("bricked: last two dims in 4x8-cell (128-B) bricks" if layout == "brick"
+                                  else "row-major"),
                        "parallelism": f"shard{world}" if world > 1 else "1gpu"},
             "gbs": gbs_total, "frac_of_nominal_8tbs": gbs_total / world / NOMINAL_HBM_GBS,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

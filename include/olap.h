@@ -95,6 +95,23 @@ typedef struct { int64_t nshards, shard, block; } olap_shard;
 int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_shard* shard,
                      int device, olap_cube** out);
 
+/* Cell layouts in HBM.  The API is layout-blind: ranges, load, fill
+ * and results always use the logical row-major index of Eq. 1's coordinates. */
+#define OLAP_LAYOUT_ROWMAJOR 0 /* row-major, dim 0 outermost (olap_cube_create) */
+#define OLAP_LAYOUT_BRICK 1    /* the last two dims stored in 4 x 8-cell bricks */
+
+/* olap_cube_create with a layout.  OLAP_LAYOUT_BRICK (the "array chunking" of related
+ * work [13], applied to the two innermost dimensions; reading R26): cells
+ * (x_{N-2}, x_{N-1}) are grouped into bricks of 4 x 8 cells = 128 B, one B200 DRAM fetch
+ * line, stored row-major inside the brick and in brick order (dims 0..N-3, brick row,
+ * brick column).  A small box then costs ~half the DRAM lines it costs row-major (C5).
+ * Needs ndims in [3,6] (dim 0 stays unbricked, so olap_shard is unchanged); extents
+ * need not be multiples of 4 / 8 (padding cells are zero and never read).  Roll-up,
+ * cube sets and olap_cube_add_facts_device return OLAP_E_UNSUPPORTED on such a cube;
+ * olap_cube_info reports the padded brick storage.  Other layouts: OLAP_E_INVALID. */
+int olap_cube_create_layout(int ndims, const int64_t* extents, int dtype, const olap_shard* shard,
+                            int device, int layout, olap_cube** out);
+
 /* Local geometry: owned dim-0 rows, owned cells, device pointer of the cells. */
 int olap_cube_info(const olap_cube* c, int64_t* local_rows, int64_t* local_cells, void** d_cells);
 

@@ -31,6 +31,7 @@ if os.environ.get("OLAP_LIB"):          # development only: A/B a differently-tu
 
 INT32, FLOAT32 = 1, 2
 SUM, COUNT, MIN, MAX, AVG = 0, 1, 2, 3, 4
+LAYOUT_ROWMAJOR, LAYOUT_BRICK = 0, 1  # olap.h OLAP_LAYOUT_*
 GEN_UNIFORM, GEN_AFFINE = 1, 2
 RESULT_EMPTY, RESULT_INVALID = 1, 2
 COND_ALL, COND_EQ, COND_RANGE, COND_IDS = 0, 1, 2, 3
@@ -57,6 +58,7 @@ _int = ctypes.c_int
 # every function declared in include/olap.h: name -> (restype, argtypes)
 EXPORTS = {
     "olap_cube_create": (_int, [_int, _i64p, _int, _p, _int, ctypes.POINTER(_p)]),
+    "olap_cube_create_layout": (_int, [_int, _i64p, _int, _p, _int, _int, ctypes.POINTER(_p)]),
     "olap_cube_info": (_int, [_p, _i64p, _i64p, ctypes.POINTER(_p)]),
     "olap_cube_load": (_int, [_p, _p, _i64]),
     "olap_cube_load_rows": (_int, [_p, _i64, _i64, _p]),
@@ -198,8 +200,9 @@ def _i64arr(a):
 class Cube:
     """A dense cube (or one block-cyclic dim-0 shard of it) resident in one GPU's HBM."""
 
-    def __init__(self, extents, dtype, shard=None, device: int = 0):
+    def __init__(self, extents, dtype, shard=None, device: int = 0, layout: int = LAYOUT_ROWMAJOR):
         self.extents = tuple(int(e) for e in extents)
+        self.layout = int(layout)
         self.ndims = len(self.extents)
         self.dtype_code = _dtype_code(dtype)
         self.np_dtype = np.int32 if self.dtype_code == INT32 else np.float32
@@ -208,8 +211,8 @@ class Cube:
         ext, extp = _i64arr(self.extents)
         h = ctypes.c_void_p()
         sh = _shard(shard)
-        _check(lib.olap_cube_create(self.ndims, extp, self.dtype_code, ctypes.byref(sh) if sh else None, device,
-                                    ctypes.byref(h)), "olap_cube_create")
+        _check(lib.olap_cube_create_layout(self.ndims, extp, self.dtype_code, ctypes.byref(sh) if sh else None,
+                                           device, self.layout, ctypes.byref(h)), "olap_cube_create_layout")
         self._h = h
 
     @property

@@ -856,16 +856,13 @@ __global__ void __launch_bounds__(kDescThreads) desc_kernel(Geo geo, int64_t nq,
     }
 }
 
-// One block: adaptive item size, tasks-per-item per query, exclusive scan of item counts.
-__global__ void __launch_bounds__(kPlanThreads) scan_kernel(int64_t nq, QDesc* desc, const int64_t* __restrict__ q_tasks,
-                                                            const int32_t* __restrict__ q_tv, int64_t* item_start,
-                                                            unsigned long long* counter, int64_t items_cap,
-                                                            const unsigned long long* totals,
-                                                            unsigned long long* bytes_acc, int grid,
-                                                            const int32_t* tmode) {
+// Grid-wide, one thread per query: adaptive item size and tasks-per-item, item count per
+// query (icnt[nq] = 0); a CUB exclusive scan then gives item_start[0..nq].
+__global__ void items_kernel(int64_t nq, QDesc* desc, const int64_t* __restrict__ q_tasks,
+                             const int32_t* __restrict__ q_tv, int64_t* __restrict__ icnt, int64_t items_cap,
+                             const unsigned long long* totals, int grid, const int32_t* tmode) {
     if (*tmode) return;
-    const int tid = threadIdx.x;
-    const int64_t total_cells = (int64_t)totals[0], total_slot_cells = (int64_t)totals[1];
+    const int64_t total_slot_cells = (int64_t)totals[1];
     // item size: 1 MiB, smaller for small batches so that there are >= 4 items per resident
     // block (latency), and large enough that sum_q items_q <= items_cap:
     // items_q <= tasks_q/tpi_q + 1 <= 2*G_q*V_q/teff + 2 (tpi_q*T_q*V_q >= teff/2)
@@ -877,44 +874,31 @@ __global__ void __launch_bounds__(kPlanThreads) scan_kernel(int64_t nq, QDesc* d
     const int64_t teff_cap = (4 * total_slot_cells + cap_left - 1) / cap_left;
     if (teff < teff_cap) teff = teff_cap;
     if (teff < 1) teff = 1;
-    const int64_t per = (nq + kPlanThreads - 1) / kPlanThreads;
-    const int64_t q0 = min(nq, (int64_t)tid * per), q1 = min(nq, q0 + per);
-    int64_t my_items = 0;
-    for (int64_t q = q0; q < q1; ++q) {
-        const int64_t tasks = q_tasks[q];
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q <= nq; q += (int64_t)gridDim.x * blockDim.x) {
         int64_t items = 0;
-        if (tasks) {
-            int64_t tpi = teff / q_tv[q];
-            if (tpi < 1) tpi = 1;
-            if (tpi > (1ll << 30)) tpi = (1ll << 30);
-            desc[q].tpi = (int32_t)tpi;
-            items = (tasks + tpi - 1) / tpi;
+        if (q < nq) {
+            const int64_t tasks = q_tasks[q];
+            if (tasks) {
+                int64_t tpi = teff / q_tv[q];
+                if (tpi < 1) tpi = 1;
+                if (tpi > (1ll << 30)) tpi = (1ll << 30);
+                desc[q].tpi = (int32_t)tpi;
+                items = (tasks + tpi - 1) / tpi;
+            }
         }
-        item_start[q] = items;
-        my_items += items;
+        icnt[q] = items;
     }
-    __shared__ int64_t scan[kPlanThreads];
-    scan[tid] = my_items;
-    __syncthreads();
-    for (int o = 1; o < kPlanThreads; o <<= 1) {
-        int64_t v = tid >= o ? scan[tid - o] : 0;
-        __syncthreads();
-        scan[tid] += v;
-        __syncthreads();
-    }
-    int64_t off = scan[tid] - my_items;
-    for (int64_t q = q0; q < q1; ++q) {
-        const int64_t items = item_start[q];
-        item_start[q] = off;
-        off += items;
-    }
-    if (tid == kPlanThreads - 1) {
-        // never write past the item-partial arrays: fail loudly instead (cannot happen by the bound above)
-        if (scan[tid] > items_cap) __trap();
-        item_start[nq] = scan[tid];
-        *counter = 0ull;
-        atomicAdd(bytes_acc, (unsigned long long)(total_cells * 4));
-    }
+}
+
+// After the scan: bound check, reset the item counter, count the batch's algorithmic bytes.
+__global__ void scan_fix_kernel(int64_t nq, const int64_t* __restrict__ item_start, unsigned long long* counter,
+                                int64_t items_cap, const unsigned long long* totals, unsigned long long* bytes_acc,
+                                const int32_t* tmode) {
+    if (*tmode) return;
+    // never write past the item-partial arrays: fail loudly instead (cannot happen by the bound above)
+    if (item_start[nq] > items_cap) __trap();
+    *counter = 0ull;
+    atomicAdd(bytes_acc, (unsigned long long)(totals[0] * 4));
 }
 
 // ------------------------------------------------------------------ L2-aware item order
@@ -1275,6 +1259,30 @@ struct FillParams {
     double c[kMaxDims + 1];
 };
 
+// Cell value of the global dim-0 row gr at logical offset off inside that row (the
+// generators of olap_cube_fill, a function of the logical index only: layout-blind).
+template <typename T>
+__device__ __forceinline__ void gen_cell(T* cells, int64_t li, const Geo& geo, int gen, uint64_t seed,
+                                         const FillParams& fp, int64_t gr, int64_t off) {
+    if (gen == OLAP_GEN_UNIFORM) {
+        const uint64_t z = splitmix64_at(seed, (uint64_t)(gr * geo.lrow + off));
+        if (sizeof(T) == 4 && geo.dtype == OLAP_INT32)
+            reinterpret_cast<int32_t*>(cells)[li] = (int32_t)(z >> 43) - (1 << 20);
+        else
+            reinterpret_cast<float*>(cells)[li] = (float)(z >> 40) * (1.0f / 16777216.0f);
+    } else {
+        double v = fp.c[0] + fp.c[1] * (double)gr;
+        int64_t rem = off;
+        for (int k = geo.nd - 1; k >= 1; --k) {
+            const int64_t x = rem % geo.n[k];
+            rem /= geo.n[k];
+            v += fp.c[1 + k] * (double)x;
+        }
+        if (geo.dtype == OLAP_INT32) reinterpret_cast<int32_t*>(cells)[li] = (int32_t)v;
+        else reinterpret_cast<float*>(cells)[li] = (float)v;
+    }
+}
+
 template <typename T>
 __global__ void fill_kernel(T* cells, Geo geo, int64_t row_cells, int gen, uint64_t seed, FillParams fp) {
     const int64_t n = geo.local_rows * row_cells;
@@ -1287,25 +1295,119 @@ __global__ void fill_kernel(T* cells, Geo geo, int64_t row_cells, int gen, uint6
             continue;
         }
         const int64_t off = rest * ninner + xin;  // logical offset inside the dim-0 row
-        const int64_t gr = shard_global_of(lr, geo.G, geo.g, geo.b);
-        const int64_t gi = gr * geo.lrow + off;
-        if (gen == OLAP_GEN_UNIFORM) {
-            const uint64_t z = splitmix64_at(seed, (uint64_t)gi);
-            if (sizeof(T) == 4 && geo.dtype == OLAP_INT32)
-                reinterpret_cast<int32_t*>(cells)[li] = (int32_t)(z >> 43) - (1 << 20);
-            else
-                reinterpret_cast<float*>(cells)[li] = (float)(z >> 40) * (1.0f / 16777216.0f);
-        } else {
-            double v = fp.c[0] + fp.c[1] * (double)gr;
-            int64_t rem = off;
-            for (int k = geo.nd - 1; k >= 1; --k) {
-                const int64_t x = rem % geo.n[k];
-                rem /= geo.n[k];
-                v += fp.c[1 + k] * (double)x;
-            }
-            if (geo.dtype == OLAP_INT32) reinterpret_cast<int32_t*>(cells)[li] = (int32_t)v;
-            else reinterpret_cast<float*>(cells)[li] = (float)v;
+        gen_cell<T>(cells, li, geo, gen, seed, fp, shard_global_of(lr, geo.G, geo.g, geo.b), off);
+    }
+}
+
+// ------------------------------------------------------------------ bricked layout (OLAP_LAYOUT_BRICK)
+// Cells (x_{N-2}, x_{N-1}) live in bricks of kBrickA x kBrickB = 4 x 8 cells (128 B: one DRAM
+// fetch line on B200, profiles/microbench_r01_sector.txt).  The storage is the row-major
+// (N+2)-D array (x_0 .. x_{N-3}, X, Z, y, z) with x_{N-2} = 4X + y, x_{N-1} = 8Z + z, so a
+// logical box is the union of <= 3 x 3 boxes of that array (head / middle / tail brick
+// sections per bricked dimension), each answered by the row-major path unchanged.
+constexpr int64_t kBrickA = 4, kBrickB = 8;
+constexpr int kBrickSecs = 9;
+static_assert(kBrickA == 4 && kBrickB == 8, "fill_brick_kernel and the host loader assume 4 x 8 bricks");
+
+struct BrickSec {
+    int64_t b0, b1, i0, i1;  // brick range, cell range inside the bricks
+};
+
+// Sections of [lo, hi] over bricks of B cells: a partial head brick, the whole bricks, a
+// partial tail brick (whole head / tail bricks merge into the middle section).
+__device__ __forceinline__ int brick_sections(int64_t lo, int64_t hi, int64_t B, BrickSec (&s)[3]) {
+    const int64_t b0 = lo / B, b1 = hi / B, h = lo - b0 * B, t = hi - b1 * B;
+    if (b0 == b1) {
+        s[0] = {b0, b0, h, t};
+        return 1;
+    }
+    int k = 0;
+    int64_t m0 = b0 + 1, m1 = b1 - 1;
+    if (h != 0) s[k++] = {b0, b0, h, B - 1};
+    else m0 = b0;
+    const bool tail_whole = t == B - 1;
+    if (tail_whole) m1 = b1;
+    if (m0 <= m1) s[k++] = {m0, m1, 0, B - 1};
+    if (!tail_whole) s[k++] = {b1, b1, 0, t};
+    return k;
+}
+
+// One thread per query: its kBrickSecs sub-queries on the brick array (query-major, section
+// order ia * 3 + ib).  Missing sections, empty boxes and invalid queries (flagged later by
+// finalize_kernel) become empty sub-boxes that read nothing.
+__global__ void brick_expand_kernel(int nd, Extents ln, int64_t nq, const olap_range* __restrict__ ranges,
+                                    const int32_t* __restrict__ ops, olap_range* __restrict__ xr,
+                                    int32_t* __restrict__ xops) {
+    const int K = nd + 2;
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nq; q += (int64_t)gridDim.x * blockDim.x) {
+        const olap_range* in = ranges + q * nd;
+        const int32_t op = ops[q];
+        bool ok = op >= OLAP_SUM && op <= OLAP_AVG;
+        for (int k = 0; k < nd; ++k) {
+            const olap_range r = in[k];
+            ok = ok && r.lo >= 0 && r.hi < ln.n[k] && r.lo <= r.hi;
         }
+        BrickSec sa[3], sb[3];
+        int na = 0, nb = 0;
+        if (ok) {
+            na = brick_sections(in[nd - 2].lo, in[nd - 2].hi, kBrickA, sa);
+            nb = brick_sections(in[nd - 1].lo, in[nd - 1].hi, kBrickB, sb);
+        }
+        for (int s = 0; s < kBrickSecs; ++s) {
+            const int ia = s / 3, ib = s - 3 * (s / 3);
+            olap_range* o = xr + (q * kBrickSecs + s) * K;
+            if (ia < na && ib < nb) {
+                for (int k = 0; k < nd - 2; ++k) o[k] = in[k];
+                o[nd - 2] = {sa[ia].b0, sa[ia].b1};
+                o[nd - 1] = {sb[ib].b0, sb[ib].b1};
+                o[nd] = {sa[ia].i0, sa[ia].i1};
+                o[nd + 1] = {sb[ib].i0, sb[ib].i1};
+                xops[q * kBrickSecs + s] = op;
+            } else {
+                for (int k = 0; k < K; ++k) o[k] = {1, 0};
+                xops[q * kBrickSecs + s] = OLAP_COUNT;
+            }
+        }
+    }
+}
+
+// Partials of a query's sections folded in section order (fixed: deterministic).
+__global__ void brick_fold_kernel(int dtype, int64_t nq, const int64_t* __restrict__ xs, const int32_t* __restrict__ xe,
+                                  int64_t* __restrict__ ps, int32_t* __restrict__ pe) {
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nq; q += (int64_t)gridDim.x * blockDim.x) {
+        long long s = 0;
+        int32_t mx = INT_MIN, mn = INT_MIN;
+        for (int k = 0; k < kBrickSecs; ++k) {
+            const int64_t j = q * kBrickSecs + k;
+            s = dtype == OLAP_INT32 ? SumOps<AccI>::add(s, xs[j]) : SumOps<AccF>::add(s, xs[j]);
+            mx = max(mx, xe[2 * j]);
+            mn = max(mn, xe[2 * j + 1]);
+        }
+        ps[q] = s;
+        pe[2 * q] = mx;
+        pe[2 * q + 1] = mn;
+    }
+}
+
+// olap_cube_fill on the brick array: storage index -> (local row, mid, X, Z, y, z) -> logical.
+template <typename T>
+__global__ void fill_brick_kernel(T* cells, Geo geo, int64_t row_cells, int64_t NX, int64_t NZ, int gen,
+                                  uint64_t seed, FillParams fp) {
+    const int64_t n = geo.local_rows * row_cells;
+    const int64_t na = geo.n[geo.nd - 2], nb = geo.n[geo.nd - 1];
+    for (int64_t li = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; li < n; li += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t lr = li / row_cells, rem = li - lr * row_cells;
+        const int64_t z = rem & (kBrickB - 1), y = (rem >> 3) & (kBrickA - 1);
+        int64_t t = rem >> 5;
+        const int64_t Z = t % NZ;
+        t /= NZ;
+        const int64_t X = t % NX, mid = t / NX;
+        const int64_t xa = kBrickA * X + y, xb = kBrickB * Z + z;
+        if (xa >= na || xb >= nb) {  // padding cell: never part of a box
+            cells[li] = (T)0;
+            continue;
+        }
+        gen_cell<T>(cells, li, geo, gen, seed, fp, shard_global_of(lr, geo.G, geo.g, geo.b), (mid * na + xa) * nb + xb);
     }
 }
 
@@ -1355,6 +1457,9 @@ struct olap_cube {
     int64_t* d_item_start = nullptr;
     int32_t* d_done = nullptr;
     int64_t* d_qtasks = nullptr;              // per query: tasks (planning scratch)
+    int64_t* d_icnt = nullptr;                // per query: items (planning scratch, nq + 1)
+    void* d_plantmp = nullptr;                // CUB scan scratch of the planners (item and pair offsets)
+    size_t plan_bytes = 0;
     int32_t* d_qtv = nullptr;                 // per query: cells per task (planning scratch)
     unsigned long long* d_counter = nullptr;  // [0] item counter, [1] algorithmic bytes, [2..3] batch totals
     long long* d_item_sum = nullptr;
@@ -1396,6 +1501,16 @@ struct olap_cube {
     int64_t launches = 0;
     int64_t kernel_launches = 0;  // every kernel this cube launched (all entry points)
     unsigned long long bytes_base = 0;
+
+    // OLAP_LAYOUT_BRICK: this handle keeps the logical geometry (nd, n, shards) and `inner` is
+    // the row-major cube of the brick array (.., ceil(n_{N-2}/4), ceil(n_{N-1}/8), 4, 8) that
+    // owns the cells; d_x* hold the kBrickSecs sub-queries per query and their partials.
+    olap_cube* inner = nullptr;
+    int64_t x_cap = 0;
+    olap_range* d_xranges = nullptr;
+    int32_t* d_xops = nullptr;
+    int64_t* d_xsum = nullptr;
+    int32_t* d_xext = nullptr;
 };
 
 namespace {
@@ -1438,8 +1553,13 @@ void free_ws(olap_cube* c) {
     cudaFree(c->d_done);
     cudaFree(c->d_qtasks);
     cudaFree(c->d_qtv);
+    cudaFree(c->d_icnt);
+    cudaFree(c->d_plantmp);
     c->d_qtasks = nullptr;
     c->d_qtv = nullptr;
+    c->d_icnt = nullptr;
+    c->d_plantmp = nullptr;
+    c->plan_bytes = 0;
     cudaFree(c->d_item_sum);
     cudaFree(c->d_item_ext);
     cudaFree(c->d_order);
@@ -1478,7 +1598,7 @@ void ensure_tile_ws(olap_cube* c, int64_t cap) {
     if (!c->tiles_on || cap <= c->tq_cap) return;
     const int64_t nt = c->tg.ntiles;
     bool ok = cudaMalloc(&c->d_tdesc, sizeof(TDesc) * cap) == cudaSuccess &&
-              cudaMalloc(&c->d_qpairs, sizeof(int64_t) * cap) == cudaSuccess &&
+              cudaMalloc(&c->d_qpairs, sizeof(int64_t) * (cap + 1)) == cudaSuccess &&
               cudaMalloc(&c->d_pstart, sizeof(int64_t) * (cap + 1)) == cudaSuccess;
     if (ok && !c->d_tcount) {
         ok = cudaMalloc(&c->d_tcount, sizeof(unsigned int) * (3 * nt + 1)) == cudaSuccess &&
@@ -1516,6 +1636,10 @@ int ensure_ws(olap_cube* c, int64_t nq) {
     OLAP_CUDA_TRY(cudaMalloc(&c->d_done, sizeof(int32_t) * cap));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_qtasks, sizeof(int64_t) * cap));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_qtv, sizeof(int32_t) * cap));
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_icnt, sizeof(int64_t) * (cap + 1)));
+    c->plan_bytes = 0;
+    OLAP_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, c->plan_bytes, c->d_icnt, c->d_item_start, (int)(cap + 1)));
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_plantmp, std::max<size_t>(c->plan_bytes, 16)));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_item_sum, sizeof(long long) * items));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_item_ext, sizeof(int32_t) * 2 * items));
     if (c->order_shift >= 0) {
@@ -1566,8 +1690,12 @@ bool capturing(cudaStream_t st) {
 // plan + reduce for nq queries already on the device; writes partials.  Capturable into a
 // CUDA graph once the workspace has grown to nq (a warm-up call outside capture): inside a
 // capture the cross-stream workspace event and the profiling events are left out.
+int run_partials_brick(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int32_t* d_ops, int64_t* d_psum,
+                       int32_t* d_pext, cudaStream_t st);
+
 int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int32_t* d_ops, int64_t* d_psum,
                  int32_t* d_pext, cudaStream_t st) {
+    if (c->inner) return run_partials_brick(c, nq, d_ranges, d_ops, d_psum, d_pext, st);
     const bool cap = capturing(st);
     if (cap && nq > c->nq_cap)
         return set_error(OLAP_E_STATE, "stream capture: run one batch of %lld queries outside capture first "
@@ -1595,8 +1723,10 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
         OLAP_CUDA_TRY(cudaMemsetAsync(c->d_ttot, 0, sizeof(unsigned long long), st));
         tile_desc_kernel<<<qb, kDescThreads, 0, st>>>(make_geo(c), tg, nq, d_ranges, d_ops, c->d_tdesc, c->d_qpairs,
                                                       d_psum, d_pext, c->d_ttot);
-        tile_scan_kernel<<<1, kPlanThreads, 0, st>>>(nq, c->d_qpairs, c->d_pstart, c->pairs_cap, tg, c->d_ttot,
-                                                     c->d_ctl, c->d_counter + 1);
+        OLAP_CUDA_TRY(cudaMemsetAsync(c->d_qpairs + nq, 0, sizeof(int64_t), st));
+        size_t pb = c->plan_bytes;
+        OLAP_CUDA_TRY(cub::DeviceScan::ExclusiveSum(c->d_plantmp, pb, c->d_qpairs, c->d_pstart, (int)(nq + 1), st));
+        tile_scan_kernel<<<1, 1, 0, st>>>(c->d_pstart, nq, c->pairs_cap, tg, c->d_ttot, c->d_ctl, c->d_counter + 1);
         OLAP_CUDA_TRY(cudaMemsetAsync(c->d_tcount, 0, sizeof(unsigned int) * (3 * tg.ntiles + 1), st));
         tile_count_kernel<<<eg, 256, 0, st>>>(tg, nq, c->d_pstart, c->d_tdesc, c->d_tcount, c->d_ctl);
         OLAP_CUDA_TRY(cudaGetLastError());
@@ -1631,19 +1761,26 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
             pair_fold_kernel<AccF><<<fg, 256, 0, st>>>(nq, c->d_pstart, c->d_tdesc, c->d_ctl, c->d_partial, d_psum,
                                                        d_pext);
         OLAP_CUDA_TRY(cudaGetLastError());
-        c->kernel_launches += 9;  // desc, scan, count, CUB scan (2), compact, scatter, reduce, fold
+        c->kernel_launches += 11;  // desc, CUB scan (2), choice, count, CUB scan (2), compact, scatter, reduce, fold
     }
     OLAP_CUDA_TRY(cudaMemsetAsync(c->d_counter + 2, 0, 2 * sizeof(unsigned long long), st));
     desc_kernel<<<(int)((nq + kDescThreads - 1) / kDescThreads), kDescThreads, 0, st>>>(
         make_geo(c), nq, d_ranges, d_ops, c->d_desc, c->d_qtasks, c->d_qtv, c->d_done, d_psum, d_pext, c->d_counter + 2,
         tmode);
     OLAP_CUDA_TRY(cudaGetLastError());
-    scan_kernel<<<1, kPlanThreads, 0, st>>>(nq, c->d_desc, c->d_qtasks, c->d_qtv, c->d_item_start, c->d_counter,
-                                            c->items_cap, c->d_counter + 2, c->d_counter + 1,
-                                            c->num_sms * c->blocks_per_sm, tmode);
+    items_kernel<<<(int)((nq + kDescThreads) / kDescThreads), kDescThreads, 0, st>>>(
+        nq, c->d_desc, c->d_qtasks, c->d_qtv, c->d_icnt, c->items_cap, c->d_counter + 2, c->num_sms * c->blocks_per_sm,
+        tmode);
+    OLAP_CUDA_TRY(cudaGetLastError());
+    {
+        size_t pb = c->plan_bytes;
+        OLAP_CUDA_TRY(cub::DeviceScan::ExclusiveSum(c->d_plantmp, pb, c->d_icnt, c->d_item_start, (int)(nq + 1), st));
+    }
+    scan_fix_kernel<<<1, 1, 0, st>>>(nq, c->d_item_start, c->d_counter, c->items_cap, c->d_counter + 2,
+                                     c->d_counter + 1, tmode);
     OLAP_CUDA_TRY(cudaGetLastError());
     const int32_t* order = nullptr;
-    c->kernel_launches += 3;  // desc, scan, reduce
+    c->kernel_launches += 6;  // desc, items, CUB scan (2), scan_fix, reduce
     if (c->order_shift >= 0) {
         c->kernel_launches += 3;
         OLAP_CUDA_TRY(cudaMemsetAsync(c->d_bcount, 0, sizeof(unsigned int) * kMaxBuckets, st));
@@ -1697,6 +1834,84 @@ int launch_finalize(int nd, const int64_t* ext, int dtype, int64_t nq, const ola
     g_finalize_launches.fetch_add(1);
     finalize_kernel<<<grid, 256, 0, st>>>(nd, e, dtype, nq, d_ranges, d_ops, d_psum, d_pext, d_results);
     OLAP_CUDA_TRY(cudaGetLastError());
+    return OLAP_OK;
+}
+
+void free_brick_x(olap_cube* c) {
+    cudaFree(c->d_xranges);
+    cudaFree(c->d_xops);
+    cudaFree(c->d_xsum);
+    cudaFree(c->d_xext);
+    c->d_xranges = nullptr;
+    c->d_xops = nullptr;
+    c->d_xsum = nullptr;
+    c->d_xext = nullptr;
+    c->x_cap = 0;
+}
+
+// Bricked cube: expand every query into its kBrickSecs sub-queries on the brick array, run
+// the row-major path on the inner cube, fold the section partials per query (fixed order).
+int run_partials_brick(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int32_t* d_ops, int64_t* d_psum,
+                       int32_t* d_pext, cudaStream_t st) {
+    const bool cap = capturing(st);
+    const int64_t nx = nq * kBrickSecs, K = c->nd + 2;
+    if (nx > c->x_cap) {
+        if (cap)
+            return set_error(OLAP_E_STATE, "stream capture: run one batch of %lld queries outside capture first "
+                             "(the workspace cannot grow inside a CUDA graph)", (long long)nq);
+        OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
+        free_brick_x(c);
+        const int64_t xc = std::max<int64_t>(nq, 1024) * kBrickSecs;
+        OLAP_CUDA_TRY(cudaMalloc(&c->d_xranges, sizeof(olap_range) * K * xc));
+        OLAP_CUDA_TRY(cudaMalloc(&c->d_xops, sizeof(int32_t) * xc));
+        OLAP_CUDA_TRY(cudaMalloc(&c->d_xsum, sizeof(int64_t) * xc));
+        OLAP_CUDA_TRY(cudaMalloc(&c->d_xext, sizeof(int32_t) * 2 * xc));
+        c->x_cap = xc;
+    }
+    if (!cap) OLAP_CUDA_TRY(cudaStreamWaitEvent(st, c->ws_done, 0));
+    Extents e;
+    std::memset(&e, 0, sizeof(e));
+    for (int k = 0; k < c->nd; ++k) e.n[k] = c->n[k];
+    const int grid = (int)std::min<int64_t>((nq + 255) / 256, (int64_t)c->num_sms * 8);
+    brick_expand_kernel<<<grid, 256, 0, st>>>(c->nd, e, nq, d_ranges, d_ops, c->d_xranges, c->d_xops);
+    OLAP_CUDA_TRY(cudaGetLastError());
+    int rc = run_partials(c->inner, nx, c->d_xranges, c->d_xops, c->d_xsum, c->d_xext, st);
+    if (rc) return rc;
+    brick_fold_kernel<<<grid, 256, 0, st>>>(c->dtype, nq, c->d_xsum, c->d_xext, d_psum, d_pext);
+    OLAP_CUDA_TRY(cudaGetLastError());
+    c->kernel_launches += 2;
+    if (!cap) OLAP_CUDA_TRY(cudaEventRecord(c->ws_done, st));
+    return OLAP_OK;
+}
+
+// Host rows [row_lo, row_hi) (logical row-major) -> brick order, one dim-0 row at a time.
+int load_rows_brick(olap_cube* c, int64_t row_lo, int64_t row_hi, const void* cells) {
+    olap_cube* ic = c->inner;
+    const int nd = c->nd;
+    const int64_t na = c->n[nd - 2], nb = c->n[nd - 1], P = c->lrow_cells / (na * nb);
+    const int64_t NX = ic->n[nd - 2], NZ = ic->n[nd - 1];
+    std::vector<uint32_t> buf;
+    try {
+        buf.assign((size_t)ic->row_cells, 0u);
+    } catch (...) {
+        return set_error(OLAP_E_NOMEM, "host staging of one brick row (%lld cells)", (long long)ic->row_cells);
+    }
+    const uint32_t* src = static_cast<const uint32_t*>(cells);
+    char* dst = static_cast<char*>(ic->d_cells);
+    const int64_t G = c->sh.nshards, g = c->sh.shard, b = c->sh.block;
+    for (int64_t r = row_lo; r < row_hi; ++r) {
+        if (G > 1 && (r / b) % G != g) continue;
+        const uint32_t* row = src + (r - row_lo) * c->lrow_cells;
+        for (int64_t mid = 0; mid < P; ++mid)
+            for (int64_t xa = 0; xa < na; ++xa) {
+                const uint32_t* in = row + (mid * na + xa) * nb;
+                uint32_t* out = buf.data() + ((mid * NX + xa / kBrickA) * NZ) * (kBrickA * kBrickB) +
+                                (xa % kBrickA) * kBrickB;
+                for (int64_t xb = 0; xb < nb; ++xb) out[(xb / kBrickB) * (kBrickA * kBrickB) + xb % kBrickB] = in[xb];
+            }
+        const int64_t lr = shard_local_of(r, G, b);
+        OLAP_CUDA_TRY(cudaMemcpy(dst + lr * ic->row_cells * 4, buf.data(), ic->row_cells * 4, cudaMemcpyHostToDevice));
+    }
     return OLAP_OK;
 }
 
@@ -1761,6 +1976,8 @@ int cube_geometry(const olap_cube* c, int* nd, int64_t* n, int* dtype, int64_t* 
     *nshards = c->sh.nshards;
     return OLAP_OK;
 }
+// OLAP_LAYOUT_ROWMAJOR or OLAP_LAYOUT_BRICK (roll-up reads raw cells and needs row-major)
+int cube_layout(const olap_cube* c) { return c->inner ? OLAP_LAYOUT_BRICK : OLAP_LAYOUT_ROWMAJOR; }
 }  // namespace olap
 
 extern "C" {
@@ -1865,6 +2082,57 @@ int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_sh
     return OLAP_OK;
 }
 
+int olap_cube_create_layout(int ndims, const int64_t* extents, int dtype, const olap_shard* shard, int device,
+                            int layout, olap_cube** out) {
+    clear_error();
+    if (layout == OLAP_LAYOUT_ROWMAJOR) return olap_cube_create(ndims, extents, dtype, shard, device, out);
+    if (layout != OLAP_LAYOUT_BRICK) return set_error(OLAP_E_INVALID, "unknown layout %d", layout);
+    if (!out || !extents) return set_error(OLAP_E_INVALID, "olap_cube_create_layout: NULL argument");
+    if (ndims < 3 || ndims > kMaxDims - 2)
+        return set_error(OLAP_E_INVALID, "bricked layout needs ndims in [3,%d], got %d", kMaxDims - 2, ndims);
+    for (int k = 0; k < ndims; ++k)
+        if (extents[k] < 1) return set_error(OLAP_E_INVALID, "extent[%d] = %lld < 1", k, (long long)extents[k]);
+    int64_t e[kMaxDims];
+    for (int k = 0; k < ndims - 2; ++k) e[k] = extents[k];
+    e[ndims - 2] = (extents[ndims - 2] + kBrickA - 1) / kBrickA;
+    e[ndims - 1] = (extents[ndims - 1] + kBrickB - 1) / kBrickB;
+    e[ndims] = kBrickA;
+    e[ndims + 1] = kBrickB;
+    olap_cube* ic = nullptr;
+    int rc = olap_cube_create(ndims + 2, e, dtype, shard, device, &ic);
+    if (rc) return rc;
+    DeviceGuard dg(device);
+    olap_cube* c = new (std::nothrow) olap_cube();
+    if (!c) {
+        olap_cube_destroy(ic);
+        return set_error(OLAP_E_NOMEM, "host allocation failed");
+    }
+    c->inner = ic;
+    c->nd = ndims;
+    c->dtype = dtype;
+    c->device = device;
+    c->sh = ic->sh;
+    for (int k = 0; k < ndims; ++k) c->n[k] = extents[k];
+    c->pitch = c->n[ndims - 1];
+    c->stride[ndims - 1] = 1;
+    for (int k = ndims - 2; k >= 0; --k) c->stride[k] = c->stride[k + 1] * c->n[k + 1];
+    c->lrow_cells = c->stride[0];
+    c->row_cells = ic->row_cells;  // storage
+    c->local_rows = ic->local_rows;
+    c->local_cells = ic->local_cells;
+    c->d_cells = ic->d_cells;
+    c->num_sms = ic->num_sms;
+    c->blocks_per_sm = ic->blocks_per_sm;
+    if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&c->ws_done, cudaEventDisableTiming) != cudaSuccess) {
+        rc = set_error(OLAP_E_CUDA, "stream/event setup failed");
+        olap_cube_destroy(c);
+        return rc;
+    }
+    *out = c;
+    return OLAP_OK;
+}
+
 int olap_cube_info(const olap_cube* c, int64_t* local_rows, int64_t* local_cells, void** d_cells) {
     clear_error();
     if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
@@ -1884,6 +2152,10 @@ int olap_cube_load_rows(olap_cube* c, int64_t row_lo, int64_t row_hi, const void
     std::lock_guard<std::mutex> lk(c->mu);
     DeviceGuard dg(c->device);
     OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
+    if (c->inner) {
+        OLAP_CUDA_TRY(cudaEventSynchronize(c->inner->ws_done));
+        return load_rows_brick(c, row_lo, row_hi, cells);
+    }
     const int64_t rb = c->row_cells * 4, lrb = c->lrow_cells * 4;  // device (padded) / host row bytes
     const int64_t nin = c->n[c->nd - 1];
     const bool padded = c->pitch != nin;
@@ -1935,6 +2207,20 @@ int olap_cube_fill(olap_cube* c, int generator, uint64_t seed, const double* par
         for (int k = 0; k <= c->nd; ++k) fp.c[k] = params[k];
     const int grid = c->num_sms * 8;
     ++c->kernel_launches;
+    if (c->inner) {
+        const olap_cube* ic = c->inner;
+        OLAP_CUDA_TRY(cudaEventSynchronize(ic->ws_done));
+        const int64_t NX = ic->n[c->nd - 2], NZ = ic->n[c->nd - 1];
+        if (c->dtype == OLAP_INT32)
+            fill_brick_kernel<int32_t><<<grid, 256, 0, c->stream>>>(static_cast<int32_t*>(c->d_cells), make_geo(c),
+                                                                    ic->row_cells, NX, NZ, generator, seed, fp);
+        else
+            fill_brick_kernel<float><<<grid, 256, 0, c->stream>>>(static_cast<float*>(c->d_cells), make_geo(c),
+                                                                  ic->row_cells, NX, NZ, generator, seed, fp);
+        OLAP_CUDA_TRY(cudaGetLastError());
+        OLAP_CUDA_TRY(cudaStreamSynchronize(c->stream));
+        return OLAP_OK;
+    }
     if (c->dtype == OLAP_INT32)
         fill_kernel<int32_t><<<grid, 256, 0, c->stream>>>(static_cast<int32_t*>(c->d_cells), make_geo(c), c->row_cells,
                                                           generator, seed, fp);
@@ -1953,6 +2239,7 @@ int olap_cube_add_facts_device(olap_cube* c, int64_t nrows, const int32_t* d_ids
     if (nrows < 0) return set_error(OLAP_E_INVALID, "nrows < 0");
     if (nrows == 0) return OLAP_OK;
     if (!d_ids) return set_error(OLAP_E_INVALID, "d_ids is NULL");
+    if (c->inner) return set_error(OLAP_E_UNSUPPORTED, "olap_cube_add_facts_device needs a row-major cube");
     std::lock_guard<std::mutex> lk(c->mu);
     DeviceGuard dg(c->device);
     cudaStream_t st = static_cast<cudaStream_t>(stream);
@@ -1976,6 +2263,12 @@ int olap_cube_destroy(olap_cube* c) {
     DeviceGuard dg(c->device);
     if (c->ws_done) cudaEventSynchronize(c->ws_done);
     if (c->stream) cudaStreamSynchronize(c->stream);
+    if (c->inner) {
+        free_brick_x(c);
+        olap_cube_destroy(c->inner);
+        c->inner = nullptr;
+        c->d_cells = nullptr;  // owned by the inner cube
+    }
     free_ws(c);
     cudaFree(c->d_ranges);
     cudaFree(c->d_ops);
@@ -2126,8 +2419,9 @@ int olap_shard_local_rows(int64_t n0, const olap_shard* s, int64_t lo, int64_t h
 int olap_cube_stats(const olap_cube* c, int64_t* kernel_launches, int* l2_order) {
     clear_error();
     if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
-    if (kernel_launches) *kernel_launches = c->kernel_launches;
-    if (l2_order) *l2_order = c->order_shift >= 0 ? 1 : 0;
+    const olap_cube* ic = c->inner ? c->inner : c;
+    if (kernel_launches) *kernel_launches = c->kernel_launches + (c->inner ? c->inner->kernel_launches : 0);
+    if (l2_order) *l2_order = ic->order_shift >= 0 ? 1 : 0;
     return OLAP_OK;
 }
 
@@ -2136,6 +2430,10 @@ int64_t olap_finalize_launches(void) { return g_finalize_launches.load(); }
 int olap_cube_tile_stats(olap_cube* c, int* enabled, int64_t* tile_cells, int64_t* ntiles, int* last_used) {
     clear_error();
     if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    if (c->inner) {
+        std::lock_guard<std::mutex> lk(c->mu);
+        return olap_cube_tile_stats(c->inner, enabled, tile_cells, ntiles, last_used);
+    }
     std::lock_guard<std::mutex> lk(c->mu);
     DeviceGuard dg(c->device);
     OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
@@ -2151,6 +2449,10 @@ int olap_cube_tile_stats(olap_cube* c, int* enabled, int64_t* tile_cells, int64_
 int olap_cube_profile(olap_cube* c, int enable) {
     clear_error();
     if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    if (c->inner) {
+        std::lock_guard<std::mutex> lk(c->mu);
+        return olap_cube_profile(c->inner, enable);
+    }
     std::lock_guard<std::mutex> lk(c->mu);
     DeviceGuard dg(c->device);
     OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
@@ -2164,6 +2466,11 @@ int olap_cube_profile(olap_cube* c, int enable) {
 int olap_cube_profile_read(olap_cube* c, double* reduce_ms, int64_t* launches, int64_t* bytes) {
     clear_error();
     if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    if (c->inner) {
+        std::lock_guard<std::mutex> lk(c->mu);
+        OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
+        return olap_cube_profile_read(c->inner, reduce_ms, launches, bytes);
+    }
     std::lock_guard<std::mutex> lk(c->mu);
     DeviceGuard dg(c->device);
     OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));

@@ -46,6 +46,7 @@ extern "C" int olap_query_batch(olap_cube* c, int64_t nq, const olap_range* rang
 namespace olap {
 
 int cube_geometry(const olap_cube* c, int* nd, int64_t* n, int* dtype, int64_t* pitch, int64_t* nshards);
+int cube_layout(const olap_cube* c);
 
 constexpr int kMaxHierDims = 8;
 
@@ -233,6 +234,8 @@ int olap_cube_rollup(const olap_hier* h, const olap_cube* fine, int fine_level, 
     cube_geometry(coarse, &ndc, nc, &dtc, &pc, &sc);
     if (ndf != h->nd || ndc != h->nd || dtf != dtc) return set_error(OLAP_E_INVALID, "cube dims / dtype mismatch");
     if (sf != 1 || sc != 1) return set_error(OLAP_E_UNSUPPORTED, "roll-up needs unsharded cubes");
+    if (cube_layout(fine) != OLAP_LAYOUT_ROWMAJOR || cube_layout(coarse) != OLAP_LAYOUT_ROWMAJOR)
+        return set_error(OLAP_E_UNSUPPORTED, "roll-up needs row-major cubes");
     for (int d = 0; d < h->nd; ++d)
         if (nf[d] != h->extent(d, fine_level) || nc[d] != h->extent(d, coarse_level))
             return set_error(OLAP_E_INVALID, "dimension %d: cube extents do not match the hierarchy levels", d);

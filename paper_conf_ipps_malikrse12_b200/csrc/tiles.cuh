@@ -208,44 +208,21 @@ __global__ void __launch_bounds__(kDescThreads) tile_desc_kernel(Geo geo, TGeo t
     if (threadIdx.x == 0 && cells) atomicAdd(totals, (unsigned long long)cells);
 }
 
-// One block: exclusive scan of pair counts -> pair_start[0..nq]; choose the path.
+// Path choice (after the exclusive scan of pair counts -> pair_start[0..nq]).
 // ctl: [0] mode (1 = tiles), [1] non-empty tiles, [2] tile pop counter.
 // Tiles pay when every staged byte is reused: cells >= 4 x staged cells (staged <= min(pairs,
 // ntiles) tiles) and pairs are big enough to amortise their set-up (>= 256 cells each).
-__global__ void __launch_bounds__(kPlanThreads) tile_scan_kernel(int64_t nq, const int64_t* __restrict__ q_pairs,
-                                                                 int64_t* pair_start, int64_t pairs_cap, TGeo tg,
-                                                                 const unsigned long long* totals, int32_t* ctl,
-                                                                 unsigned long long* bytes_acc) {
-    const int tid = threadIdx.x;
-    const int64_t per = (nq + kPlanThreads - 1) / kPlanThreads;
-    const int64_t q0 = min(nq, (int64_t)tid * per), q1 = min(nq, q0 + per);
-    int64_t mine = 0;
-    for (int64_t q = q0; q < q1; ++q) mine += q_pairs[q];
-    __shared__ int64_t scan[kPlanThreads];
-    scan[tid] = mine;
-    __syncthreads();
-    for (int o = 1; o < kPlanThreads; o <<= 1) {
-        int64_t v = tid >= o ? scan[tid - o] : 0;
-        __syncthreads();
-        scan[tid] += v;
-        __syncthreads();
-    }
-    int64_t off = scan[tid] - mine;
-    for (int64_t q = q0; q < q1; ++q) {
-        pair_start[q] = off;
-        off += q_pairs[q];
-    }
-    if (tid == kPlanThreads - 1) {
-        const int64_t pairs = scan[tid];
-        const int64_t cells = (int64_t)totals[0];
-        pair_start[nq] = pairs;
-        const int64_t staged = min(pairs, tg.ntiles) * tg.tcells;
-        const int use = tg.ok && pairs > 0 && pairs <= pairs_cap && cells >= 4 * staged && cells >= 256 * pairs;
-        ctl[0] = use;
-        ctl[1] = 0;
-        ctl[2] = 0;
-        if (use) atomicAdd(bytes_acc, (unsigned long long)(cells * 4));
-    }
+// One thread, after the CUB scan (pair_start[nq] = total pairs).
+__global__ void tile_scan_kernel(const int64_t* __restrict__ pair_start, int64_t nq, int64_t pairs_cap, TGeo tg,
+                                 const unsigned long long* totals, int32_t* ctl, unsigned long long* bytes_acc) {
+    const int64_t pairs = pair_start[nq];
+    const int64_t cells = (int64_t)totals[0];
+    const int64_t staged = min(pairs, tg.ntiles) * tg.tcells;
+    const int use = tg.ok && pairs > 0 && pairs <= pairs_cap && cells >= 4 * staged && cells >= 256 * pairs;
+    ctl[0] = use;
+    ctl[1] = 0;
+    ctl[2] = 0;
+    if (use) atomicAdd(bytes_acc, (unsigned long long)(cells * 4));
 }
 
 // tile id of query d's j-th pair (row-major over its tile box)

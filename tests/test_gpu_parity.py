@@ -423,10 +423,10 @@ def test_c4_tpcds_pipeline():
     assert np.array_equal(cnts["i"], ref_c)
 
 
-def _sampled_full_size(name, n_small, n_random, max_cells, affine_params):
+def _sampled_full_size(name, n_small, n_random, max_cells, affine_params, layout=olap.LAYOUT_ROWMAJOR):
     cfg = synth.CONFIGS[name]
     ext = cfg["extents"]
-    c = olap.Cube(ext, cfg["dtype"])
+    c = olap.Cube(ext, cfg["dtype"], layout=layout)
     try:
         c.fill(olap.GEN_UNIFORM, cfg["seed"])
         boxes, ops = synth.config_queries(name)
@@ -457,6 +457,11 @@ def test_c3_full_size_sampled():
 def test_c5_slice_full_size_sampled():
     """C5 per-GPU slice: 128 GiB float32 cube (1024,4096,8192), 65,536 small boxes; sampled parity."""
     _sampled_full_size("C5", 50, 400, 2_000_000, np.array([2, 1, 1, 1], float))
+
+
+def test_c5_slice_bricked_full_size_sampled():
+    """C5 as bench.py runs it: the 128 GiB slice in the bricked layout (R26)."""
+    _sampled_full_size("C5", 50, 400, 2_000_000, np.array([2, 1, 1, 1], float), layout=olap.LAYOUT_BRICK)
 
 
 # ------------------------------------------------------------------ fact tables (NEXT #1)
