@@ -40,9 +40,14 @@ constexpr int kUnroll = OLAP_UNROLL;        // independent loads in flight per l
 #endif
 constexpr int kMinBlocks = OLAP_MIN_BLOCKS;
 #ifndef OLAP_WARP_ITEMS
-#define OLAP_WARP_ITEMS 0
+#define OLAP_WARP_ITEMS -1
 #endif
-constexpr bool kWarpItems = OLAP_WARP_ITEMS != 0;  // warp-granular items (reduce_kernel_w) vs block items  // resident reduce blocks per SM the register budget targets
+// Item granularity: block items (reduce_kernel: 8 warps share an item) or warp items
+// (reduce_kernel_w: no block barriers).  -1 = per batch: warp items when the batch has more
+// than kWarpItemQueries queries per resident block (many small boxes: C5, bricked
+// sub-boxes; measured +13% there and -7% on C1's 1,000 queries); 0 / 1 force one.
+constexpr int kWarpItemsMode = OLAP_WARP_ITEMS;
+constexpr int64_t kWarpItemQueries = 8;
 constexpr int64_t kItemCells = 262144;      // minimum item: 1 MiB of 4-byte cells
 constexpr int64_t kMaxExtent = (1ll << 30); // per-dimension limit (32-bit digit arithmetic)
 constexpr int64_t kMaxCells = (1ll << 42);
@@ -860,15 +865,15 @@ __global__ void __launch_bounds__(kDescThreads) desc_kernel(Geo geo, int64_t nq,
 // query (icnt[nq] = 0); a CUB exclusive scan then gives item_start[0..nq].
 __global__ void items_kernel(int64_t nq, QDesc* desc, const int64_t* __restrict__ q_tasks,
                              const int32_t* __restrict__ q_tv, int64_t* __restrict__ icnt, int64_t items_cap,
-                             const unsigned long long* totals, int grid, const int32_t* tmode) {
+                             const unsigned long long* totals, int grid, int witems, const int32_t* tmode) {
     if (*tmode) return;
     const int64_t total_slot_cells = (int64_t)totals[1];
     // item size: 1 MiB, smaller for small batches so that there are >= 4 items per resident
     // block (latency), and large enough that sum_q items_q <= items_cap:
     // items_q <= tasks_q/tpi_q + 1 <= 2*G_q*V_q/teff + 2 (tpi_q*T_q*V_q >= teff/2)
     const int64_t cap_left = items_cap - 2 * nq;
-    const int64_t workers = kWarpItems ? 8ll * grid : (int64_t)grid;
-    const int64_t target = kWarpItems ? kItemCells / 4 : kItemCells;
+    const int64_t workers = witems ? 8ll * grid : (int64_t)grid;
+    const int64_t target = witems ? kItemCells / 4 : kItemCells;
     int64_t teff = total_slot_cells / (4ll * workers);
     if (teff > target) teff = target;
     const int64_t teff_cap = (4 * total_slot_cells + cap_left - 1) / cap_left;
@@ -1630,7 +1635,7 @@ int ensure_ws(olap_cube* c, int64_t nq) {
     // few MiB (the L2-aware order needs the ~600 in-flight items to fit in L2): one per 4 KiB of
     // cube, <= 2^24 (a batch reads the cube ~10^2-10^3 times over at C3-like overlap)
     const int64_t by_size = std::min<int64_t>(1ll << 24, (c->local_cells * 4) >> 12);
-    int64_t items = std::max<int64_t>(std::max<int64_t>(kWarpItems ? (1ll << 22) : (1ll << 20), 4 * cap), by_size);
+    int64_t items = std::max<int64_t>(std::max<int64_t>(1ll << 20, 4 * cap), by_size);
     OLAP_CUDA_TRY(cudaMalloc(&c->d_desc, sizeof(QDesc) * cap));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_item_start, sizeof(int64_t) * (cap + 1)));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_done, sizeof(int32_t) * cap));
@@ -1768,9 +1773,10 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
         make_geo(c), nq, d_ranges, d_ops, c->d_desc, c->d_qtasks, c->d_qtv, c->d_done, d_psum, d_pext, c->d_counter + 2,
         tmode);
     OLAP_CUDA_TRY(cudaGetLastError());
+    const int grid = c->num_sms * c->blocks_per_sm;
+    const bool witems = kWarpItemsMode >= 0 ? kWarpItemsMode != 0 : nq > kWarpItemQueries * grid;
     items_kernel<<<(int)((nq + kDescThreads) / kDescThreads), kDescThreads, 0, st>>>(
-        nq, c->d_desc, c->d_qtasks, c->d_qtv, c->d_icnt, c->items_cap, c->d_counter + 2, c->num_sms * c->blocks_per_sm,
-        tmode);
+        nq, c->d_desc, c->d_qtasks, c->d_qtv, c->d_icnt, c->items_cap, c->d_counter + 2, grid, witems ? 1 : 0, tmode);
     OLAP_CUDA_TRY(cudaGetLastError());
     {
         size_t pb = c->plan_bytes;
@@ -1792,14 +1798,13 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
         OLAP_CUDA_TRY(cudaGetLastError());
         order = c->d_order;
     }
-    const int grid = c->num_sms * c->blocks_per_sm;
     cudaEvent_t e0 = nullptr, e1 = nullptr;
     if (prof) {
         int rc2 = bracket(&e0, &e1);
         if (rc2) return rc2;
         OLAP_CUDA_TRY(cudaEventRecord(e0, st));
     }
-    if (kWarpItems) {
+    if (witems) {
         if (c->dtype == OLAP_INT32)
             reduce_kernel_w<int32_t, AccI><<<grid, kThreads, 0, st>>>(
                 static_cast<const int32_t*>(c->d_cells), nq, c->d_desc, c->d_item_start, c->d_counter, c->d_done,
@@ -2054,15 +2059,19 @@ int olap_cube_create(int ndims, const int64_t* extents, int dtype, const olap_sh
                          cudaSharedmemCarveoutMaxL1);
     cudaFuncSetAttribute(reduce_kernel<float, AccF>, cudaFuncAttributePreferredSharedMemoryCarveout,
                          cudaSharedmemCarveoutMaxL1);
-    if (kWarpItems) {
-        if (dtype == OLAP_INT32)
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, reduce_kernel_w<int32_t, AccI>, kThreads, 0);
-        else
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, reduce_kernel_w<float, AccF>, kThreads, 0);
-    } else if (dtype == OLAP_INT32)
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, reduce_kernel<int32_t, AccI>, kThreads, 0);
-    else
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, reduce_kernel<float, AccF>, kThreads, 0);
+    // (no max-L1 carveout for reduce_kernel_w: its 2 KiB of per-warp descriptors would then
+    // fit only 2 blocks per SM -- measured: C5 -40%)
+    {
+        int bw = 0;  // one grid serves both item kernels: the smaller residency of the two
+        if (dtype == OLAP_INT32) {
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, reduce_kernel<int32_t, AccI>, kThreads, 0);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bw, reduce_kernel_w<int32_t, AccI>, kThreads, 0);
+        } else {
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, reduce_kernel<float, AccF>, kThreads, 0);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bw, reduce_kernel_w<float, AccF>, kThreads, 0);
+        }
+        bps = std::min(bps, bw);
+    }
     if (const char* s = getenv("OLAP_BLOCKS_PER_SM")) {
         int v = atoi(s);
         if (v > 0 && v < bps) bps = v;

@@ -826,3 +826,24 @@ def test_table_partition_boxes():
     torch.cuda.synchronize()
     got = res.cpu().numpy().view(olap.RESULT_DTYPE)
     _check_table(got, oracle.tablescan(cols, qs, nthreads=oracle.max_threads()), cols, qs)
+
+
+@pytest.mark.parametrize("dtype", [np.int32, np.float32])
+@pytest.mark.parametrize("ext", [(64, 129, 7), (8, 8, 16, 16, 16, 16), (3, 1000), (2, 9, 16384), (40, 1024, 1024)])
+def test_warp_items_large_batches(ext, dtype):
+    """Batches of more than 8 queries per resident block take warp-granular items
+    (reduce_kernel_w): same bars as the block-item path, deterministic."""
+    n = int(np.prod(ext))
+    seed = 0x5EED5000 + n
+    rng = np.random.default_rng(seed)
+    boxes = np.concatenate([synth.random_boxes(ext, 2000, rng), synth.fraction_boxes(ext, 2000, rng, 1e-4),
+                            synth.small_boxes(ext, 4000, rng, bytes_lo=4, bytes_hi=1 << 16)])
+    ops = synth.ops_uniform(len(boxes), rng)
+    c = olap.Cube(ext, dtype)
+    c.fill(olap.GEN_UNIFORM, seed)
+    got = c.query(boxes, ops)
+    idx = np.arange(len(boxes)) if n <= (1 << 22) else rng.choice(len(boxes), 600, replace=False)
+    ref = oracle.query(ext, boxes[idx], ops[idx], dtype=dtype, gen=oracle.GEN_UNIFORM, seed=seed,
+                       nthreads=oracle.max_threads())
+    compare(got[idx], ref, ops[idx], dtype)
+    assert np.array_equal(c.query(boxes, ops), got)
