@@ -696,7 +696,7 @@ def main():
                "h2d_bytes_per_step": int(nq * nd * 16 + nq * 4), "d2h_bytes_per_step": int(nq * 24),
                "api": "ShardedCube path: H2D, olap_query_partials_device, NCCL all-reduce, olap_finalize_device, D2H"}
 
-    kernel = "tile_reduce_kernel" if tiles_used else "reduce_kernel"
+    kernel = "tile_reduce_kernel" if tiles_used else ("brick_reduce_kernel" if layout == "brick" else "reduce_kernel")
     traffic = _traffic(args.workload, kernel)
     if tiles_used:
         sm_mhz = (clk or {}).get("sm_mhz") or 1965.0
@@ -707,6 +707,12 @@ def main():
                  "bandwidth that bounds the kernel (128 B/clk/SM x 148 SMs at the measured SM clock)")
         smem = {"peak": smem_peak_gbs(sm_mhz), "unit": "GB/s", "frac": achieved / smem_peak_gbs(sm_mhz),
                 "peak_source": f"derived: 128 B/clk/SM x 148 SMs x {sm_mhz:.0f} MHz (median SM clock in the timed region)"}
+    elif layout == "brick":
+        rnote = ("bricked layout: achieved = algorithmic bytes (sum of V_q*4 over non-COUNT queries, Eq. 3) / "
+                 "brick_reduce_kernel time; the kernel reads whole 128-B bricks (one DRAM fetch line each), so "
+                 "traffic (ncu DRAM bytes per launch, profiles/traffic.json) exceeds the algorithmic bytes by the "
+                 "edge bricks' unselected cells")
+        smem = None
     else:
         rnote = ("achieved = algorithmic bytes (sum of V_q*4 over non-COUNT queries, Eq. 3) / "
                  "reduce-kernel time; frac > 1 is L2 reuse: items are scheduled in cube-address "

@@ -899,7 +899,7 @@ __global__ void items_kernel(int64_t nq, QDesc* desc, const int64_t* __restrict_
 __global__ void scan_fix_kernel(int64_t nq, const int64_t* __restrict__ item_start, unsigned long long* counter,
                                 int64_t items_cap, const unsigned long long* totals, unsigned long long* bytes_acc,
                                 const int32_t* tmode) {
-    if (*tmode) return;
+    if (tmode && *tmode) return;
     // never write past the item-partial arrays: fail loudly instead (cannot happen by the bound above)
     if (item_start[nq] > items_cap) __trap();
     *counter = 0ull;
@@ -1192,6 +1192,286 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) reduce_kernel(const T* _
     }
 }
 
+// ------------------------------------------------------------------ bricked cubes: brick_reduce_kernel
+// A query on a bricked cube (OLAP_LAYOUT_BRICK; the brick layout itself is defined below,
+// before the host runtime) is its box of bricks: the leading dims' ranges x the bricks
+// [X0, X1] x [Z0, Z1] its x_{N-2} / x_{N-1} ranges meet.  A lane takes one 128-B brick per
+// step (four LDG.256, all in flight), masks the rows and columns outside the box (only in
+// the box's edge bricks) and folds the 32 cells: one DRAM fetch line per brick, half the
+// lines of the row-major layout on C5's small boxes (reading R26).
+constexpr int kBrickDims = kMaxDims - 2;
+struct BDesc {
+    int32_t opc, nld;          // op class; leading digits (dims 0..N-3 with extent > 1)
+    int32_t ya, yb, za, zb;    // first brick row's first y, last brick row's last y; same for z
+    int64_t nb;                // bricks in the box (0: reads nothing)
+    int64_t base;              // cell offset of the box's first brick
+    int64_t nX, nZ, sX;        // brick extents of the box; cells between brick rows
+    FastDiv fZ, fX;            // / nZ, / nX
+    FastDiv fl[kBrickDims];    // / leading extents, innermost first (the outermost is not divided)
+    int64_t sl[kBrickDims];    // leading strides (cells), innermost first
+};
+static_assert(sizeof(BDesc) <= sizeof(QDesc), "brick descriptors live in the QDesc workspace");
+
+// Geometry of the brick array of a bricked cube (shard-local).
+struct BGeo {
+    int nd;                    // logical dims N
+    int64_t G, g, b;           // dim-0 shards
+    int64_t n[kMaxDims];       // logical global extents
+    int64_t stride[kMaxDims];  // brick-array strides (cells) of dims 0..N-3, then X (N-2); Z stride is 32
+    int64_t local_rows;
+};
+
+// One thread per query: the box of bricks on this shard, identity partials when it reads
+// nothing, per-query brick counts for the item planner, batch totals (cells, bricks).
+__global__ void __launch_bounds__(256) brick_desc_kernel(BGeo g, int64_t nq, const olap_range* __restrict__ ranges,
+                                                         const int32_t* __restrict__ ops, BDesc* __restrict__ desc,
+                                                         int64_t* __restrict__ q_bricks, int32_t* __restrict__ done,
+                                                         int64_t* __restrict__ psum, int32_t* __restrict__ pext,
+                                                         unsigned long long* totals) {
+    __shared__ int64_t sh[32];
+    const int64_t q = blockIdx.x * 256ll + threadIdx.x;
+    int64_t cells = 0, bricks = 0;
+    if (q < nq) {
+        const olap_range* r = ranges + q * g.nd;
+        const int32_t op = ops[q];
+        BDesc d;
+        d.nb = 0;
+        d.opc = (op == OLAP_MIN) ? OPC_MIN : (op == OLAP_MAX) ? OPC_MAX : OPC_SUM;
+        bool ok = op == OLAP_SUM || op == OLAP_MIN || op == OLAP_MAX || op == OLAP_AVG;
+        for (int k = 0; k < g.nd; ++k) ok = ok && r[k].lo >= 0 && r[k].hi < g.n[k] && r[k].lo <= r[k].hi;
+        int64_t l0 = 0, h0 = -1;
+        if (ok) ok = shard_local_range(g.n[0], g.G, g.g, g.b, r[0].lo, r[0].hi, &l0, &h0);
+        if (ok) {
+            const int a = g.nd - 2, bz = g.nd - 1;
+            const int64_t X0 = r[a].lo >> 2, X1 = r[a].hi >> 2, Z0 = r[bz].lo >> 3, Z1 = r[bz].hi >> 3;
+            d.ya = (int32_t)(r[a].lo & 3);
+            d.yb = (int32_t)(r[a].hi & 3);
+            d.za = (int32_t)(r[bz].lo & 7);
+            d.zb = (int32_t)(r[bz].hi & 7);
+            d.nX = X1 - X0 + 1;
+            d.nZ = Z1 - Z0 + 1;
+            d.sX = g.stride[a];
+            d.fX = dev_fastdiv((uint32_t)d.nX);
+            d.fZ = dev_fastdiv((uint32_t)d.nZ);
+            int64_t base = X0 * g.stride[a] + Z0 * 32, nb = d.nX * d.nZ, v = (r[a].hi - r[a].lo + 1) *
+                                                                            (r[bz].hi - r[bz].lo + 1);
+            int nld = 0;
+            for (int k = a - 1; k >= 0; --k) {
+                const int64_t lo = k == 0 ? l0 : r[k].lo, hi = k == 0 ? h0 : r[k].hi, ell = hi - lo + 1;
+                base += lo * g.stride[k];
+                nb *= ell;
+                v *= ell;
+                if (ell > 1) {
+                    d.fl[nld] = dev_fastdiv((uint32_t)ell);
+                    d.sl[nld] = g.stride[k];
+                    ++nld;
+                }
+            }
+            d.nld = nld;
+            d.base = base;
+            d.nb = nb;
+            cells = v;
+            bricks = nb;
+        }
+        desc[q] = d;
+        done[q] = 0;
+        q_bricks[q] = d.nb;
+        if (d.nb == 0 || op == OLAP_COUNT) {
+            if (op == OLAP_COUNT) q_bricks[q] = 0, cells = 0, bricks = 0;
+            psum[q] = 0;
+            pext[2 * q] = INT_MIN;
+            pext[2 * q + 1] = INT_MIN;
+        }
+    }
+    cells = block_sum<int64_t>(cells, sh);
+    bricks = block_sum<int64_t>(bricks, sh);
+    if (threadIdx.x == 0) {
+        if (cells) atomicAdd(totals + 0, (unsigned long long)cells);
+        if (bricks) atomicAdd(totals + 1, (unsigned long long)bricks);
+    }
+}
+
+// Bricks per item: <= 1,024 (32 warp steps of 32 bricks), fewer for small batches (>= 4 items per warp
+// slot), more if the item-partial arrays would overflow (items_q <= bricks_q / bpi + 1).
+__global__ void brick_items_kernel(int64_t nq, BDesc* desc, const int64_t* __restrict__ q_bricks,
+                                   int64_t* __restrict__ icnt, int64_t items_cap, const unsigned long long* totals,
+                                   int warps) {
+    const int64_t total = (int64_t)totals[1];
+    int64_t bpi = total / (4ll * warps);
+    if (bpi > 1024) bpi = 1024;
+    const int64_t cap_left = items_cap - nq;
+    const int64_t bpi_cap = (total + cap_left - 1) / cap_left;
+    if (bpi < bpi_cap) bpi = bpi_cap;
+    if (bpi < 32) bpi = 32;
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q <= nq; q += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t nb = q < nq ? q_bricks[q] : 0;
+        icnt[q] = (nb + bpi - 1) / bpi;
+        if (q == 0) icnt[nq + 1] = bpi;  // read by brick_reduce_kernel (icnt has nq + 2 entries)
+    }
+}
+
+__device__ __forceinline__ uint64_t byte_range_word(int lo, int hi) {  // bytes lo..hi of 8 = 0xFF
+    return (~0ull << (8 * lo)) & (~0ull >> (8 * (7 - hi)));
+}
+
+// Cell offset of brick j (< 2^32) of the box: Z fastest, then X, then the leading digits.
+__device__ __forceinline__ int64_t brick_addr(const BDesc& d, uint32_t j, uint32_t& X, uint32_t& Z) {
+    uint32_t t = fdiv(j, d.fZ);
+    Z = j - t * d.fZ.d;
+    const uint32_t t2 = fdiv(t, d.fX);
+    X = t - t2 * d.fX.d;
+    int64_t a = d.base + (int64_t)Z * 32 + (int64_t)X * d.sX;
+    t = t2;
+    for (int e = 0; e < d.nld; ++e) {
+        if (e == d.nld - 1) {  // outermost digit: no division
+            a += (int64_t)t * d.sl[e];
+            break;
+        }
+        const uint32_t qq = fdiv(t, d.fl[e]);
+        a += (int64_t)(t - qq * d.fl[e].d) * d.sl[e];
+        t = qq;
+    }
+    return a;
+}
+
+__device__ __noinline__ int64_t brick_addr_wide(const BDesc& d, int64_t j, uint32_t& X, uint32_t& Z) {  // nb >= 2^32
+    int64_t t = j / d.nZ;
+    Z = (uint32_t)(j - t * d.nZ);
+    const int64_t t2 = t / d.nX;
+    X = (uint32_t)(t - t2 * d.nX);
+    int64_t a = d.base + (int64_t)Z * 32 + (int64_t)X * d.sX;
+    t = t2;
+    for (int e = 0; e < d.nld; ++e) {
+        const int64_t l = d.fl[e].d, qq = e == d.nld - 1 ? 0 : t / l;
+        a += (e == d.nld - 1 ? t : t - qq * l) * d.sl[e];
+        t = qq;
+    }
+    return a;
+}
+
+template <class Acc, int OPC>
+__device__ __forceinline__ void fold_row(Acc& acc, const uint32_t (&v)[8], uint64_t w) {
+    if constexpr (OPC == OPC_SUM && std::is_same<Acc, AccF>::value) {  // fp32 tree of 8 cells (R8'), then fp64
+        uint32_t x[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) x[k] = v[k] & cell_mask<8>(w, k);
+        acc.s += (double)slot_tree<8>(x);
+    } else {
+#pragma unroll
+        for (int k = 0; k < 8; ++k) acc.template add<OPC>(v[k], cell_mask<8>(w, k));
+    }
+}
+
+// Four lanes per brick (lane quad = one 128-B line, one coalesced request; lane & 3 = the
+// brick row y), 8 bricks per warp step, kBrickU steps of loads in flight per lane.
+#ifndef OLAP_BRICK_U
+#define OLAP_BRICK_U 3
+#endif
+constexpr int kBrickU = OLAP_BRICK_U;
+template <class Acc, int OPC, bool WIDE>
+__device__ __forceinline__ void stream_bricks(const uint32_t* __restrict__ cube, const BDesc& d, int64_t b0,
+                                              int64_t b1, Acc& acc, int lane) {
+    const int sub = lane >> 2, y = lane & 3;
+    for (int64_t j0 = b0; j0 < b1; j0 += 8 * kBrickU) {
+        uint32_t v[kBrickU][8];
+        uint64_t w[kBrickU];
+#pragma unroll
+        for (int u = 0; u < kBrickU; ++u) {
+            const int64_t j = j0 + 8 * u + sub;
+            const bool ok = j < b1;
+            const int64_t jj = ok ? j : b1 - 1;
+            uint32_t X, Z;
+            const int64_t a = WIDE ? brick_addr_wide(d, jj, X, Z) : brick_addr(d, (uint32_t)jj, X, Z);
+            ld_stream8(cube + a + 8 * y, v[u]);
+            const int ylo = X == 0 ? d.ya : 0, yhi = X == d.fX.d - 1 ? d.yb : 3;
+            const int zlo = Z == 0 ? d.za : 0, zhi = Z == d.fZ.d - 1 ? d.zb : 7;
+            w[u] = ok && y >= ylo && y <= yhi ? byte_range_word(zlo, zhi) : 0ull;
+        }
+#pragma unroll
+        for (int u = 0; u < kBrickU; ++u) fold_row<Acc, OPC>(acc, v[u], w[u]);
+    }
+}
+
+// Persistent warp-item kernel over (query, brick range) items; partials folded per query in
+// fixed item order by the query's last warp (as reduce_kernel_w: deterministic).
+#ifndef OLAP_BRICK_BLOCKS
+#define OLAP_BRICK_BLOCKS 3
+#endif
+constexpr int kBrickBlocks = OLAP_BRICK_BLOCKS;  // resident blocks per SM the register budget targets
+template <typename T, class Acc>
+__global__ void __launch_bounds__(kThreads, kBrickBlocks) brick_reduce_kernel(
+    const T* __restrict__ cube, int64_t nq, const BDesc* __restrict__ desc, const int64_t* __restrict__ item_start,
+    const int64_t* __restrict__ icnt, unsigned long long* counter, int32_t* done, long long* item_sum,
+    int32_t* item_ext, int64_t* psum, int32_t* pext) {
+    __shared__ BDesc sdw[kWarps];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    BDesc& sd = sdw[w];
+    const int64_t total = __ldg(item_start + nq), bpi = __ldg(icnt + nq + 1);
+    const uint32_t* c = reinterpret_cast<const uint32_t*>(cube);
+    for (;;) {
+        long long item = 0;
+        if (lane == 0) item = (long long)atomicAdd(counter, 1ull);
+        item = __shfl_sync(0xffffffffu, item, 0);
+        if (item >= total) break;
+        const int64_t q = find_query(item_start, nq, item, lane);
+        {
+            const int* src = reinterpret_cast<const int*>(desc + q);
+            int* dst = reinterpret_cast<int*>(&sd);
+            for (int i = lane; i < (int)(sizeof(BDesc) / 4); i += 32) dst[i] = __ldg(src + i);
+        }
+        __syncwarp();
+        const int64_t first_item = __ldg(item_start + q);
+        const int64_t b0 = (item - first_item) * bpi, b1 = min(sd.nb, b0 + bpi);
+        Acc acc;
+        acc.init();
+        const int opc = sd.opc;
+        if (sd.nb >= (1ll << 32)) {  // > 2^32 bricks in one box (> 512 GiB): 64-bit digit arithmetic
+            if (opc == OPC_SUM) stream_bricks<Acc, OPC_SUM, true>(c, sd, b0, b1, acc, lane);
+            else if (opc == OPC_MIN) stream_bricks<Acc, OPC_MIN, true>(c, sd, b0, b1, acc, lane);
+            else stream_bricks<Acc, OPC_MAX, true>(c, sd, b0, b1, acc, lane);
+        } else if (opc == OPC_SUM) stream_bricks<Acc, OPC_SUM, false>(c, sd, b0, b1, acc, lane);
+        else if (opc == OPC_MIN) stream_bricks<Acc, OPC_MIN, false>(c, sd, b0, b1, acc, lane);
+        else stream_bricks<Acc, OPC_MAX, false>(c, sd, b0, b1, acc, lane);
+        long long s = acc.sum_bits();
+        int32_t cmx = opc == OPC_MAX ? acc.code_max() : INT_MIN, cmn = opc == OPC_MIN ? ~acc.code_min() : INT_MIN;
+#pragma unroll
+        for (int o = 16; o; o >>= 1) s = SumOps<Acc>::add(s, __shfl_xor_sync(0xffffffffu, s, o));
+        cmx = __reduce_max_sync(0xffffffffu, cmx);
+        cmn = __reduce_max_sync(0xffffffffu, cmn);
+        const int64_t nitems = (sd.nb + bpi - 1) / bpi;
+        int last = 0;
+        if (lane == 0) {
+            item_sum[item] = s;
+            item_ext[2 * item] = cmx;
+            item_ext[2 * item + 1] = cmn;
+            __threadfence();
+            last = atomicAdd(done + q, 1) == (int)nitems - 1;
+        }
+        last = __shfl_sync(0xffffffffu, last, 0);
+        if (last) {
+            __threadfence();
+            long long ts = 0;
+            int32_t tmx = INT_MIN, tmn = INT_MIN;
+            for (int64_t i = lane; i < nitems; i += 32) {
+                const int64_t it = first_item + i;
+                ts = SumOps<Acc>::add(ts, __ldcg(item_sum + it));
+                tmx = max(tmx, __ldcg(item_ext + 2 * it));
+                tmn = max(tmn, __ldcg(item_ext + 2 * it + 1));
+            }
+#pragma unroll
+            for (int o = 16; o; o >>= 1) ts = SumOps<Acc>::add(ts, __shfl_xor_sync(0xffffffffu, ts, o));
+            tmx = __reduce_max_sync(0xffffffffu, tmx);
+            tmn = __reduce_max_sync(0xffffffffu, tmn);
+            if (lane == 0) {
+                psum[q] = ts;
+                pext[2 * q] = tmx;
+                pext[2 * q + 1] = tmn;
+            }
+        }
+        __syncwarp();
+    }
+}
+
 // ------------------------------------------------------------------ tile-shared scan
 
 #include "tiles.cuh"
@@ -1307,92 +1587,10 @@ __global__ void fill_kernel(T* cells, Geo geo, int64_t row_cells, int gen, uint6
 // ------------------------------------------------------------------ bricked layout (OLAP_LAYOUT_BRICK)
 // Cells (x_{N-2}, x_{N-1}) live in bricks of kBrickA x kBrickB = 4 x 8 cells (128 B: one DRAM
 // fetch line on B200, profiles/microbench_r01_sector.txt).  The storage is the row-major
-// (N+2)-D array (x_0 .. x_{N-3}, X, Z, y, z) with x_{N-2} = 4X + y, x_{N-1} = 8Z + z, so a
-// logical box is the union of <= 3 x 3 boxes of that array (head / middle / tail brick
-// sections per bricked dimension), each answered by the row-major path unchanged.
+// (N+2)-D array (x_0 .. x_{N-3}, X, Z, y, z) with x_{N-2} = 4X + y, x_{N-1} = 8Z + z, held by
+// an inner row-major cube; queries run brick_reduce_kernel on it (a lane quad per brick).
 constexpr int64_t kBrickA = 4, kBrickB = 8;
-constexpr int kBrickSecs = 9;
 static_assert(kBrickA == 4 && kBrickB == 8, "fill_brick_kernel and the host loader assume 4 x 8 bricks");
-
-struct BrickSec {
-    int64_t b0, b1, i0, i1;  // brick range, cell range inside the bricks
-};
-
-// Sections of [lo, hi] over bricks of B cells: a partial head brick, the whole bricks, a
-// partial tail brick (whole head / tail bricks merge into the middle section).
-__device__ __forceinline__ int brick_sections(int64_t lo, int64_t hi, int64_t B, BrickSec (&s)[3]) {
-    const int64_t b0 = lo / B, b1 = hi / B, h = lo - b0 * B, t = hi - b1 * B;
-    if (b0 == b1) {
-        s[0] = {b0, b0, h, t};
-        return 1;
-    }
-    int k = 0;
-    int64_t m0 = b0 + 1, m1 = b1 - 1;
-    if (h != 0) s[k++] = {b0, b0, h, B - 1};
-    else m0 = b0;
-    const bool tail_whole = t == B - 1;
-    if (tail_whole) m1 = b1;
-    if (m0 <= m1) s[k++] = {m0, m1, 0, B - 1};
-    if (!tail_whole) s[k++] = {b1, b1, 0, t};
-    return k;
-}
-
-// One thread per query: its kBrickSecs sub-queries on the brick array (query-major, section
-// order ia * 3 + ib).  Missing sections, empty boxes and invalid queries (flagged later by
-// finalize_kernel) become empty sub-boxes that read nothing.
-__global__ void brick_expand_kernel(int nd, Extents ln, int64_t nq, const olap_range* __restrict__ ranges,
-                                    const int32_t* __restrict__ ops, olap_range* __restrict__ xr,
-                                    int32_t* __restrict__ xops) {
-    const int K = nd + 2;
-    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nq; q += (int64_t)gridDim.x * blockDim.x) {
-        const olap_range* in = ranges + q * nd;
-        const int32_t op = ops[q];
-        bool ok = op >= OLAP_SUM && op <= OLAP_AVG;
-        for (int k = 0; k < nd; ++k) {
-            const olap_range r = in[k];
-            ok = ok && r.lo >= 0 && r.hi < ln.n[k] && r.lo <= r.hi;
-        }
-        BrickSec sa[3], sb[3];
-        int na = 0, nb = 0;
-        if (ok) {
-            na = brick_sections(in[nd - 2].lo, in[nd - 2].hi, kBrickA, sa);
-            nb = brick_sections(in[nd - 1].lo, in[nd - 1].hi, kBrickB, sb);
-        }
-        for (int s = 0; s < kBrickSecs; ++s) {
-            const int ia = s / 3, ib = s - 3 * (s / 3);
-            olap_range* o = xr + (q * kBrickSecs + s) * K;
-            if (ia < na && ib < nb) {
-                for (int k = 0; k < nd - 2; ++k) o[k] = in[k];
-                o[nd - 2] = {sa[ia].b0, sa[ia].b1};
-                o[nd - 1] = {sb[ib].b0, sb[ib].b1};
-                o[nd] = {sa[ia].i0, sa[ia].i1};
-                o[nd + 1] = {sb[ib].i0, sb[ib].i1};
-                xops[q * kBrickSecs + s] = op;
-            } else {
-                for (int k = 0; k < K; ++k) o[k] = {1, 0};
-                xops[q * kBrickSecs + s] = OLAP_COUNT;
-            }
-        }
-    }
-}
-
-// Partials of a query's sections folded in section order (fixed: deterministic).
-__global__ void brick_fold_kernel(int dtype, int64_t nq, const int64_t* __restrict__ xs, const int32_t* __restrict__ xe,
-                                  int64_t* __restrict__ ps, int32_t* __restrict__ pe) {
-    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nq; q += (int64_t)gridDim.x * blockDim.x) {
-        long long s = 0;
-        int32_t mx = INT_MIN, mn = INT_MIN;
-        for (int k = 0; k < kBrickSecs; ++k) {
-            const int64_t j = q * kBrickSecs + k;
-            s = dtype == OLAP_INT32 ? SumOps<AccI>::add(s, xs[j]) : SumOps<AccF>::add(s, xs[j]);
-            mx = max(mx, xe[2 * j]);
-            mn = max(mn, xe[2 * j + 1]);
-        }
-        ps[q] = s;
-        pe[2 * q] = mx;
-        pe[2 * q + 1] = mn;
-    }
-}
 
 // olap_cube_fill on the brick array: storage index -> (local row, mid, X, Z, y, z) -> logical.
 template <typename T>
@@ -1509,13 +1707,9 @@ struct olap_cube {
 
     // OLAP_LAYOUT_BRICK: this handle keeps the logical geometry (nd, n, shards) and `inner` is
     // the row-major cube of the brick array (.., ceil(n_{N-2}/4), ceil(n_{N-1}/8), 4, 8) that
-    // owns the cells; d_x* hold the kBrickSecs sub-queries per query and their partials.
+    // owns the cells (queries use its workspace: run_partials_brick).
     olap_cube* inner = nullptr;
-    int64_t x_cap = 0;
-    olap_range* d_xranges = nullptr;
-    int32_t* d_xops = nullptr;
-    int64_t* d_xsum = nullptr;
-    int32_t* d_xext = nullptr;
+    int brick_bps = 0;  // resident brick_reduce_kernel blocks per SM
 };
 
 namespace {
@@ -1641,7 +1835,7 @@ int ensure_ws(olap_cube* c, int64_t nq) {
     OLAP_CUDA_TRY(cudaMalloc(&c->d_done, sizeof(int32_t) * cap));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_qtasks, sizeof(int64_t) * cap));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_qtv, sizeof(int32_t) * cap));
-    OLAP_CUDA_TRY(cudaMalloc(&c->d_icnt, sizeof(int64_t) * (cap + 1)));
+    OLAP_CUDA_TRY(cudaMalloc(&c->d_icnt, sizeof(int64_t) * (cap + 2)));
     c->plan_bytes = 0;
     OLAP_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, c->plan_bytes, c->d_icnt, c->d_item_start, (int)(cap + 1)));
     OLAP_CUDA_TRY(cudaMalloc(&c->d_plantmp, std::max<size_t>(c->plan_bytes, 16)));
@@ -1842,50 +2036,78 @@ int launch_finalize(int nd, const int64_t* ext, int dtype, int64_t nq, const ola
     return OLAP_OK;
 }
 
-void free_brick_x(olap_cube* c) {
-    cudaFree(c->d_xranges);
-    cudaFree(c->d_xops);
-    cudaFree(c->d_xsum);
-    cudaFree(c->d_xext);
-    c->d_xranges = nullptr;
-    c->d_xops = nullptr;
-    c->d_xsum = nullptr;
-    c->d_xext = nullptr;
-    c->x_cap = 0;
-}
-
-// Bricked cube: expand every query into its kBrickSecs sub-queries on the brick array, run
-// the row-major path on the inner cube, fold the section partials per query (fixed order).
+// Bricked cube: plan (brick_desc_kernel, brick_items_kernel, CUB scan) and reduce
+// (brick_reduce_kernel) on the inner cube's workspace.
 int run_partials_brick(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int32_t* d_ops, int64_t* d_psum,
                        int32_t* d_pext, cudaStream_t st) {
+    olap_cube* ic = c->inner;
     const bool cap = capturing(st);
-    const int64_t nx = nq * kBrickSecs, K = c->nd + 2;
-    if (nx > c->x_cap) {
-        if (cap)
-            return set_error(OLAP_E_STATE, "stream capture: run one batch of %lld queries outside capture first "
-                             "(the workspace cannot grow inside a CUDA graph)", (long long)nq);
-        OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
-        free_brick_x(c);
-        const int64_t xc = std::max<int64_t>(nq, 1024) * kBrickSecs;
-        OLAP_CUDA_TRY(cudaMalloc(&c->d_xranges, sizeof(olap_range) * K * xc));
-        OLAP_CUDA_TRY(cudaMalloc(&c->d_xops, sizeof(int32_t) * xc));
-        OLAP_CUDA_TRY(cudaMalloc(&c->d_xsum, sizeof(int64_t) * xc));
-        OLAP_CUDA_TRY(cudaMalloc(&c->d_xext, sizeof(int32_t) * 2 * xc));
-        c->x_cap = xc;
-    }
-    if (!cap) OLAP_CUDA_TRY(cudaStreamWaitEvent(st, c->ws_done, 0));
-    Extents e;
-    std::memset(&e, 0, sizeof(e));
-    for (int k = 0; k < c->nd; ++k) e.n[k] = c->n[k];
-    const int grid = (int)std::min<int64_t>((nq + 255) / 256, (int64_t)c->num_sms * 8);
-    brick_expand_kernel<<<grid, 256, 0, st>>>(c->nd, e, nq, d_ranges, d_ops, c->d_xranges, c->d_xops);
-    OLAP_CUDA_TRY(cudaGetLastError());
-    int rc = run_partials(c->inner, nx, c->d_xranges, c->d_xops, c->d_xsum, c->d_xext, st);
+    if (cap && nq > ic->nq_cap)
+        return set_error(OLAP_E_STATE, "stream capture: run one batch of %lld queries outside capture first "
+                         "(the workspace cannot grow inside a CUDA graph)", (long long)nq);
+    int rc = ensure_ws(ic, nq);
     if (rc) return rc;
-    brick_fold_kernel<<<grid, 256, 0, st>>>(c->dtype, nq, c->d_xsum, c->d_xext, d_psum, d_pext);
+    if (!cap) OLAP_CUDA_TRY(cudaStreamWaitEvent(st, ic->ws_done, 0));
+    BGeo g;
+    std::memset(&g, 0, sizeof(g));
+    g.nd = c->nd;
+    g.G = c->sh.nshards;
+    g.g = c->sh.shard;
+    g.b = c->sh.block;
+    for (int k = 0; k < c->nd; ++k) g.n[k] = c->n[k];
+    for (int k = 0; k <= c->nd - 2; ++k) g.stride[k] = ic->stride[k];
+    g.local_rows = c->local_rows;
+    BDesc* bd = reinterpret_cast<BDesc*>(ic->d_desc);
+    if (!c->brick_bps) {
+        int bps = 0;
+        if (c->dtype == OLAP_INT32)
+            OLAP_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, brick_reduce_kernel<int32_t, AccI>,
+                                                                        kThreads, 0));
+        else
+            OLAP_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, brick_reduce_kernel<float, AccF>,
+                                                                        kThreads, 0));
+        c->brick_bps = std::max(bps, 1);
+    }
+    const int grid = ic->num_sms * c->brick_bps;
+    OLAP_CUDA_TRY(cudaMemsetAsync(ic->d_counter + 2, 0, 2 * sizeof(unsigned long long), st));
+    brick_desc_kernel<<<(int)((nq + 255) / 256), 256, 0, st>>>(g, nq, d_ranges, d_ops, bd, ic->d_qtasks, ic->d_done,
+                                                               d_psum, d_pext, ic->d_counter + 2);
+    brick_items_kernel<<<(int)((nq + 256) / 256), 256, 0, st>>>(nq, bd, ic->d_qtasks, ic->d_icnt, ic->items_cap,
+                                                                ic->d_counter + 2, grid * kWarps);
     OLAP_CUDA_TRY(cudaGetLastError());
-    c->kernel_launches += 2;
-    if (!cap) OLAP_CUDA_TRY(cudaEventRecord(c->ws_done, st));
+    size_t pb = ic->plan_bytes;
+    OLAP_CUDA_TRY(cub::DeviceScan::ExclusiveSum(ic->d_plantmp, pb, ic->d_icnt, ic->d_item_start, (int)(nq + 1), st));
+    scan_fix_kernel<<<1, 1, 0, st>>>(nq, ic->d_item_start, ic->d_counter, ic->items_cap, ic->d_counter + 2,
+                                     ic->d_counter + 1, nullptr);
+    OLAP_CUDA_TRY(cudaGetLastError());
+    const bool prof = ic->prof && !cap;
+    if (prof) {
+        while (ic->ev.size() < ic->ev_used + 2) {
+            cudaEvent_t e;
+            OLAP_CUDA_TRY(cudaEventCreate(&e));
+            ic->ev.push_back(e);
+        }
+        OLAP_CUDA_TRY(cudaEventRecord(ic->ev[ic->ev_used], st));
+    }
+    if (c->dtype == OLAP_INT32)
+        brick_reduce_kernel<int32_t, AccI><<<grid, kThreads, 0, st>>>(
+            static_cast<const int32_t*>(ic->d_cells), nq, bd, ic->d_item_start, ic->d_icnt, ic->d_counter, ic->d_done,
+            ic->d_item_sum, ic->d_item_ext, d_psum, d_pext);
+    else
+        brick_reduce_kernel<float, AccF><<<grid, kThreads, 0, st>>>(
+            static_cast<const float*>(ic->d_cells), nq, bd, ic->d_item_start, ic->d_icnt, ic->d_counter, ic->d_done,
+            ic->d_item_sum, ic->d_item_ext, d_psum, d_pext);
+    OLAP_CUDA_TRY(cudaGetLastError());
+    if (prof) {
+        OLAP_CUDA_TRY(cudaEventRecord(ic->ev[ic->ev_used + 1], st));
+        ic->ev_used += 2;
+        ++ic->launches;
+    }
+    c->kernel_launches += 6;  // desc, items, CUB scan (2), fix, reduce
+    if (!cap) {
+        OLAP_CUDA_TRY(cudaEventRecord(ic->ws_done, st));
+        OLAP_CUDA_TRY(cudaEventRecord(c->ws_done, st));
+    }
     return OLAP_OK;
 }
 
@@ -2116,6 +2338,7 @@ int olap_cube_create_layout(int ndims, const int64_t* extents, int dtype, const 
         olap_cube_destroy(ic);
         return set_error(OLAP_E_NOMEM, "host allocation failed");
     }
+    ic->tiles_on = false;  // bricked queries run brick_reduce_kernel on the inner cube, never its tile path
     c->inner = ic;
     c->nd = ndims;
     c->dtype = dtype;
@@ -2273,7 +2496,6 @@ int olap_cube_destroy(olap_cube* c) {
     if (c->ws_done) cudaEventSynchronize(c->ws_done);
     if (c->stream) cudaStreamSynchronize(c->stream);
     if (c->inner) {
-        free_brick_x(c);
         olap_cube_destroy(c->inner);
         c->inner = nullptr;
         c->d_cells = nullptr;  // owned by the inner cube

@@ -20,7 +20,7 @@ def parse(path):
         if len(r) != len(h):
             continue
         name = r[h.index("Kernel Name")]
-        k = re.search(r"(tile_reduce_kernel|reduce_kernel|table_scan_kernel)", name)
+        k = re.search(r"(tile_reduce_kernel|brick_reduce_kernel|reduce_kernel|table_scan_kernel)", name)
         if not k:
             continue
         lid = r[h.index("ID")]
