@@ -518,9 +518,29 @@ __device__ __forceinline__ void stream_long(const uint32_t* __restrict__ cube, c
 // g = 32 / nslot whole runs per step, each as one contiguous span of shared memory (no
 // per-slot division, no shuffle, no separate edge pass).  Idle lanes read lane 0's slot
 // with an all-zero mask.  Offsets inside a staged tile fit in 32 bits.
+// float MIN / MAX in column mode mask by addition on the FMA pipe instead of a LOP3 on the
+// (binding) ALU pipe: m[k] holds a bias, +0.0 for a cell in the box and the op's identity
+// (+inf for MIN, -inf for MAX) outside it, so v + bias is v or the identity (a NaN from
+// -inf + inf is ignored by fminf / fmaxf; -0.0 + 0.0 reads as +0.0, reading R9).
+template <class Acc, int OPC>
+constexpr bool bias_fold() {
+    return std::is_same<Acc, AccF>::value && (OPC == OPC_MIN || OPC == OPC_MAX);
+}
+template <int OPC>
+constexpr uint32_t bias_identity() {
+    return OPC == OPC_MIN ? 0x7f800000u : 0xff800000u;
+}
+
 template <class Acc, int OPC, int V>
 __device__ __forceinline__ void fold_masked(Acc& acc, const uint32_t (&v)[V], const uint32_t (&m)[V]) {
-    if constexpr (tree_sum<Acc, OPC, V, true>()) {
+    if constexpr (bias_fold<Acc, OPC>()) {
+#pragma unroll
+        for (int k = 0; k < V; ++k) {
+            const float x = __uint_as_float(v[k]) + __uint_as_float(m[k]);
+            if constexpr (OPC == OPC_MIN) acc.mn = fminf(acc.mn, x);
+            else acc.mx = fmaxf(acc.mx, x);
+        }
+    } else if constexpr (tree_sum<Acc, OPC, V, true>()) {
         uint32_t x[V];
 #pragma unroll
         for (int k = 0; k < V; ++k) x[k] = v[k] & m[k];
@@ -575,7 +595,10 @@ __device__ __forceinline__ void stream_cols(const uint32_t* __restrict__ sb, con
     if (swp) w = (w >> 32) | (w << 32);
     uint32_t m[V];
 #pragma unroll
-    for (int k = 0; k < V; ++k) m[k] = cell_mask<V>(w, k);
+    for (int k = 0; k < V; ++k) {
+        m[k] = cell_mask<V>(w, k);
+        if constexpr (bias_fold<Acc, OPC>()) m[k] = ~m[k] & bias_identity<OPC>();
+    }
     // lane byte addresses of its slot's two halves (half-swapped lanes read the upper half first)
     const uint32_t a0 = smem_addr_u32(sb) + ((uint32_t)d.base_al + sl * V) * 4u;
     const uint32_t pa = a0 + (swp ? 16u : 0u), pb = a0 + (swp ? 0u : 16u);
@@ -630,7 +653,10 @@ __device__ __forceinline__ void stream_cols(const uint32_t* __restrict__ sb, con
         uint32_t v0[V], mm[V];
         lds_slot<V>(pa + o, pb + o, v0);
 #pragma unroll
-        for (int k = 0; k < V; ++k) mm[k] = m[k] & okm;
+        for (int k = 0; k < V; ++k) {
+            if constexpr (bias_fold<Acc, OPC>()) mm[k] = m[k] | (~okm & bias_identity<OPC>());
+            else mm[k] = m[k] & okm;
+        }
         fold_masked<Acc, OPC, V>(acc, v0, mm);
     }
 }
