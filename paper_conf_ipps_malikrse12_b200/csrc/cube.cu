@@ -887,16 +887,13 @@ __global__ void __launch_bounds__(kDescThreads) desc_kernel(Geo geo, int64_t nq,
     }
 }
 
-// Grid-wide, one thread per query: adaptive item size and tasks-per-item, item count per
-// query (icnt[nq] = 0); a CUB exclusive scan then gives item_start[0..nq].
-__global__ void items_kernel(int64_t nq, QDesc* desc, const int64_t* __restrict__ q_tasks,
-                             const int32_t* __restrict__ q_tv, int64_t* __restrict__ icnt, int64_t items_cap,
-                             const unsigned long long* totals, int grid, int witems, const int32_t* tmode) {
-    if (*tmode) return;
+// Item size (cells per item, "teff"): 1 MiB for block items, 256 KiB for warp items, smaller
+// for small batches so that there are >= 4 items per worker (latency), and large enough that
+// sum_q items_q <= items_cap: items_q <= tasks_q/tpi_q + 1 <= 2*G_q*V_q/teff + 2
+// (tpi_q*T_q*V_q >= teff/2).
+__device__ __forceinline__ int64_t item_cells(int64_t nq, int64_t items_cap, const unsigned long long* totals,
+                                              int grid, int witems) {
     const int64_t total_slot_cells = (int64_t)totals[1];
-    // item size: 1 MiB, smaller for small batches so that there are >= 4 items per resident
-    // block (latency), and large enough that sum_q items_q <= items_cap:
-    // items_q <= tasks_q/tpi_q + 1 <= 2*G_q*V_q/teff + 2 (tpi_q*T_q*V_q >= teff/2)
     const int64_t cap_left = items_cap - 2 * nq;
     const int64_t workers = witems ? 8ll * grid : (int64_t)grid;
     const int64_t target = witems ? kItemCells / 4 : kItemCells;
@@ -904,20 +901,74 @@ __global__ void items_kernel(int64_t nq, QDesc* desc, const int64_t* __restrict_
     if (teff > target) teff = target;
     const int64_t teff_cap = (4 * total_slot_cells + cap_left - 1) / cap_left;
     if (teff < teff_cap) teff = teff_cap;
-    if (teff < 1) teff = 1;
-    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q <= nq; q += (int64_t)gridDim.x * blockDim.x) {
-        int64_t items = 0;
-        if (q < nq) {
-            const int64_t tasks = q_tasks[q];
-            if (tasks) {
-                int64_t tpi = teff / q_tv[q];
-                if (tpi < 1) tpi = 1;
-                if (tpi > (1ll << 30)) tpi = (1ll << 30);
-                desc[q].tpi = (int32_t)tpi;
-                items = (tasks + tpi - 1) / tpi;
-            }
-        }
-        icnt[q] = items;
+    return teff < 1 ? 1 : teff;
+}
+
+// Items of query q (tasks-per-item written into its descriptor).
+__device__ __forceinline__ int64_t query_items(QDesc* desc, const int64_t* __restrict__ q_tasks,
+                                               const int32_t* __restrict__ q_tv, int64_t q, int64_t teff) {
+    const int64_t tasks = q_tasks[q];
+    if (!tasks) return 0;
+    int64_t tpi = teff / q_tv[q];
+    if (tpi < 1) tpi = 1;
+    if (tpi > (1ll << 30)) tpi = (1ll << 30);
+    desc[q].tpi = (int32_t)tpi;
+    return (tasks + tpi - 1) / tpi;
+}
+
+// Grid-wide, one thread per query: item count per query (icnt[nq] = 0); a CUB exclusive
+// scan then gives item_start[0..nq].  Large batches (> kPlanSmall queries).
+__global__ void items_kernel(int64_t nq, QDesc* desc, const int64_t* __restrict__ q_tasks,
+                             const int32_t* __restrict__ q_tv, int64_t* __restrict__ icnt, int64_t items_cap,
+                             const unsigned long long* totals, int grid, int witems, const int32_t* tmode) {
+    if (*tmode) return;
+    const int64_t teff = item_cells(nq, items_cap, totals, grid, witems);
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q <= nq; q += (int64_t)gridDim.x * blockDim.x)
+        icnt[q] = q < nq ? query_items(desc, q_tasks, q_tv, q, teff) : 0;
+}
+
+// Small batches (<= kPlanSmall queries): items, exclusive scan and the scan_fix_kernel work
+// in one block (one launch instead of four; C1's 1,000-query batches are launch-bound).
+constexpr int64_t kPlanSmall = 16384;
+__global__ void __launch_bounds__(kPlanThreads) plan_small_kernel(int64_t nq, QDesc* desc,
+                                                                  const int64_t* __restrict__ q_tasks,
+                                                                  const int32_t* __restrict__ q_tv,
+                                                                  int64_t* __restrict__ item_start,
+                                                                  unsigned long long* counter, int64_t items_cap,
+                                                                  const unsigned long long* totals,
+                                                                  unsigned long long* bytes_acc, int grid, int witems,
+                                                                  const int32_t* tmode) {
+    if (*tmode) return;
+    const int tid = threadIdx.x;
+    const int64_t teff = item_cells(nq, items_cap, totals, grid, witems);
+    const int64_t per = (nq + kPlanThreads - 1) / kPlanThreads;
+    const int64_t q0 = min(nq, (int64_t)tid * per), q1 = min(nq, q0 + per);
+    int64_t mine = 0;
+    for (int64_t q = q0; q < q1; ++q) {
+        const int64_t it = query_items(desc, q_tasks, q_tv, q, teff);
+        item_start[q] = it;
+        mine += it;
+    }
+    __shared__ int64_t scan[kPlanThreads];
+    scan[tid] = mine;
+    __syncthreads();
+    for (int o = 1; o < kPlanThreads; o <<= 1) {
+        const int64_t v = tid >= o ? scan[tid - o] : 0;
+        __syncthreads();
+        scan[tid] += v;
+        __syncthreads();
+    }
+    int64_t off = scan[tid] - mine;
+    for (int64_t q = q0; q < q1; ++q) {
+        const int64_t it = item_start[q];
+        item_start[q] = off;
+        off += it;
+    }
+    if (tid == kPlanThreads - 1) {
+        if (scan[tid] > items_cap) __trap();  // impossible by item_cells' bound
+        item_start[nq] = scan[tid];
+        *counter = 0ull;
+        atomicAdd(bytes_acc, (unsigned long long)(totals[0] * 4));
     }
 }
 
@@ -1995,16 +2046,23 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
     OLAP_CUDA_TRY(cudaGetLastError());
     const int grid = c->num_sms * c->blocks_per_sm;
     const bool witems = kWarpItemsMode >= 0 ? kWarpItemsMode != 0 : nq > kWarpItemQueries * grid;
-    items_kernel<<<(int)((nq + kDescThreads) / kDescThreads), kDescThreads, 0, st>>>(
-        nq, c->d_desc, c->d_qtasks, c->d_qtv, c->d_icnt, c->items_cap, c->d_counter + 2, grid, witems ? 1 : 0, tmode);
-    OLAP_CUDA_TRY(cudaGetLastError());
-    {
+    if (nq <= kPlanSmall) {
+        plan_small_kernel<<<1, kPlanThreads, 0, st>>>(nq, c->d_desc, c->d_qtasks, c->d_qtv, c->d_item_start,
+                                                      c->d_counter, c->items_cap, c->d_counter + 2, c->d_counter + 1,
+                                                      grid, witems ? 1 : 0, tmode);
+        OLAP_CUDA_TRY(cudaGetLastError());
+        c->kernel_launches -= 3;
+    } else {
+        items_kernel<<<(int)((nq + kDescThreads) / kDescThreads), kDescThreads, 0, st>>>(
+            nq, c->d_desc, c->d_qtasks, c->d_qtv, c->d_icnt, c->items_cap, c->d_counter + 2, grid, witems ? 1 : 0,
+            tmode);
+        OLAP_CUDA_TRY(cudaGetLastError());
         size_t pb = c->plan_bytes;
         OLAP_CUDA_TRY(cub::DeviceScan::ExclusiveSum(c->d_plantmp, pb, c->d_icnt, c->d_item_start, (int)(nq + 1), st));
+        scan_fix_kernel<<<1, 1, 0, st>>>(nq, c->d_item_start, c->d_counter, c->items_cap, c->d_counter + 2,
+                                         c->d_counter + 1, tmode);
+        OLAP_CUDA_TRY(cudaGetLastError());
     }
-    scan_fix_kernel<<<1, 1, 0, st>>>(nq, c->d_item_start, c->d_counter, c->items_cap, c->d_counter + 2,
-                                     c->d_counter + 1, tmode);
-    OLAP_CUDA_TRY(cudaGetLastError());
     const int32_t* order = nullptr;
     c->kernel_launches += 6;  // desc, items, CUB scan (2), scan_fix, reduce
     if (c->order_shift >= 0) {
