@@ -637,8 +637,19 @@ __device__ __forceinline__ void stream_cols(const uint32_t* __restrict__ sb, con
         step();
         lds_slot<V>(pa + off, pb + off, v1);
         step();
-        fold_masked<Acc, OPC, V>(acc, v0, m);
-        fold_masked<Acc, OPC, V>(acc, v1, m);
+        if constexpr (tree_sum<Acc, OPC, V, true>() && V == 8) {
+            // float SUM: one fp32 tree over both slots (16 cells, depth 4; reading R8'), one fp64 add
+            uint32_t x0[V], x1[V];
+#pragma unroll
+            for (int k = 0; k < V; ++k) {
+                x0[k] = v0[k] & m[k];
+                x1[k] = v1[k] & m[k];
+            }
+            acc.s += (double)(slot_tree<V>(x0) + slot_tree<V>(x1));
+        } else {
+            fold_masked<Acc, OPC, V>(acc, v0, m);
+            fold_masked<Acc, OPC, V>(acc, v1, m);
+        }
     }
     if (r0 < full) {
         uint32_t v0[V];
