@@ -152,48 +152,53 @@ __global__ void table_prep_boxes_kernel(int64_t nq, int ncols, TableCols tc, Box
     note_columns(t, colmask);
 }
 
-// One query on one staged tile.  Lane l owns rows l, l+32, ..., l+992: every condition
-// is loaded once per tile (uniform) and evaluated into a 32-bit pass mask (bit i = row
-// l + 32 i); COUNT is a popcount, and only matching rows touch the data column.
-template <bool FLOAT_DATA>
+// One query on one staged tile.  Lane l owns the row quads 4l..4l+3 + 128 i (i < 8): every
+// condition column is read with one LDS.128 per quad (lane-consecutive 16-B chunks, no bank
+// conflicts) and evaluated into a 32-bit pass mask (bit 4i + j = row 128 i + 4 l + j);
+// COUNT is a popcount, and only matching rows touch the data column, folding only the
+// accumulator the op needs (OPK: 0 SUM / AVG, 1 MIN, 2 MAX, 3 COUNT).
+__device__ __forceinline__ uint32_t quad_pass(uint4 x, uint32_t lo, uint32_t span) {
+    return (uint32_t)(x.x - lo <= span) | (uint32_t)(x.y - lo <= span) << 1 | (uint32_t)(x.z - lo <= span) << 2 |
+           (uint32_t)(x.w - lo <= span) << 3;
+}
+template <bool FLOAT_DATA, int OPK>
 __device__ __forceinline__ void scan_query_tile(const uint32_t* __restrict__ smem, int rows, const TQuery& tq, int lane,
                                                 long long& s, int64_t& cnt, int32_t& cmx, int32_t& cmn) {
     static_assert(kTileRows == 1024, "one 32-bit pass mask per lane");
     uint32_t pass = rows >= kTileRows ? 0xFFFFFFFFu : 0u;
     if (rows < kTileRows)
-        for (int i = 0; i < 32; ++i)
-            if (lane + 32 * i < rows) pass |= 1u << i;
+        for (int b = 0; b < 32; ++b)
+            if (128 * (b >> 2) + 4 * lane + (b & 3) < rows) pass |= 1u << b;
     const int nc = tq.ncond;
     for (int k = 0; k < nc && pass; ++k) {
         const TCond c = tq.c[k];
-        const uint32_t* col = smem + c.col * kTileRows + lane;
+        const uint4* col = reinterpret_cast<const uint4*>(smem + c.col * kTileRows) + lane;
         uint32_t m = 0;
 #pragma unroll
-        for (int i = 0; i < 32; ++i) m |= (uint32_t)((col[32 * i] - c.lo) <= c.span) << i;
+        for (int i = 0; i < 8; ++i) m |= quad_pass(col[32 * i], c.lo, c.span) << (4 * i);
         pass &= m;
     }
     int32_t n = __popc(pass);
-    const bool need_data = tq.op != OLAP_COUNT;
-    const uint32_t* data = smem + tq.data_col * kTileRows + lane;
+    const uint32_t* data = smem + tq.data_col * kTileRows + 4 * lane;
     unsigned long long si = 0ull;
     double sf = 0.0;
     float fmn = __int_as_float(0x7f800000), fmx = __int_as_float(0xff800000);
     int32_t imn = INT_MAX, imx = INT_MIN;
-    uint32_t bits_left = need_data ? pass : 0u;
+    uint32_t bits_left = OPK == 3 ? 0u : pass;
     while (bits_left) {
-        const int i = __ffs(bits_left) - 1;
+        const int b = __ffs(bits_left) - 1;
         bits_left &= bits_left - 1;
-        const uint32_t bits = data[32 * i];
+        const uint32_t bits = data[128 * (b >> 2) + (b & 3)];
         if (FLOAT_DATA) {
             const float v = __uint_as_float(bits);
-            sf += (double)v;
-            fmn = fminf(fmn, v);
-            fmx = fmaxf(fmx, v);
+            if (OPK == 0) sf += (double)v;
+            if (OPK == 1) fmn = fminf(fmn, v);
+            if (OPK == 2) fmx = fmaxf(fmx, v);
         } else {
             const int32_t v = (int32_t)bits;
-            si += (unsigned long long)(long long)v;
-            imn = min(imn, v);
-            imx = max(imx, v);
+            if (OPK == 0) si += (unsigned long long)(long long)v;
+            if (OPK == 1) imn = min(imn, v);
+            if (OPK == 2) imx = max(imx, v);
         }
     }
     // warp reduction in fixed order
@@ -258,8 +263,18 @@ __global__ void __launch_bounds__(kScanThreads) table_scan_kernel(TableCols tc, 
             long long s = p.sum;
             int64_t cnt = p.count;
             int32_t cmx = p.code_max, cmn = p.code_min;
-            if (tc.dtype[tq.data_col] == OLAP_FLOAT32) scan_query_tile<true>(smem, rows, tq, lane, s, cnt, cmx, cmn);
-            else scan_query_tile<false>(smem, rows, tq, lane, s, cnt, cmx, cmn);
+            const int opk = tq.op == OLAP_MIN ? 1 : tq.op == OLAP_MAX ? 2 : tq.op == OLAP_COUNT ? 3 : 0;
+            if (tc.dtype[tq.data_col] == OLAP_FLOAT32) {
+                if (opk == 0) scan_query_tile<true, 0>(smem, rows, tq, lane, s, cnt, cmx, cmn);
+                else if (opk == 1) scan_query_tile<true, 1>(smem, rows, tq, lane, s, cnt, cmx, cmn);
+                else if (opk == 2) scan_query_tile<true, 2>(smem, rows, tq, lane, s, cnt, cmx, cmn);
+                else scan_query_tile<true, 3>(smem, rows, tq, lane, s, cnt, cmx, cmn);
+            } else {
+                if (opk == 0) scan_query_tile<false, 0>(smem, rows, tq, lane, s, cnt, cmx, cmn);
+                else if (opk == 1) scan_query_tile<false, 1>(smem, rows, tq, lane, s, cnt, cmx, cmn);
+                else if (opk == 2) scan_query_tile<false, 2>(smem, rows, tq, lane, s, cnt, cmx, cmn);
+                else scan_query_tile<false, 3>(smem, rows, tq, lane, s, cnt, cmx, cmn);
+            }
             if (lane == 0) {
                 p.sum = s;
                 p.count = cnt;
