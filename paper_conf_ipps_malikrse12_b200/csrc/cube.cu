@@ -1422,21 +1422,6 @@ __device__ __forceinline__ int64_t brick_addr(const BDesc& d, uint32_t j, uint32
     return a;
 }
 
-__device__ __noinline__ int64_t brick_addr_wide(const BDesc& d, int64_t j, uint32_t& X, uint32_t& Z) {  // nb >= 2^32
-    int64_t t = j / d.nZ;
-    Z = (uint32_t)(j - t * d.nZ);
-    const int64_t t2 = t / d.nX;
-    X = (uint32_t)(t - t2 * d.nX);
-    int64_t a = d.base + (int64_t)Z * 32 + (int64_t)X * d.sX;
-    t = t2;
-    for (int e = 0; e < d.nld; ++e) {
-        const int64_t l = d.fl[e].d, qq = e == d.nld - 1 ? 0 : t / l;
-        a += (e == d.nld - 1 ? t : t - qq * l) * d.sl[e];
-        t = qq;
-    }
-    return a;
-}
-
 template <class Acc, int OPC>
 __device__ __forceinline__ void fold_row(Acc& acc, const uint32_t (&v)[8], uint64_t w) {
     if constexpr (OPC == OPC_SUM && std::is_same<Acc, AccF>::value) {  // fp32 tree of 8 cells (R8'), then fp64
@@ -1456,7 +1441,7 @@ __device__ __forceinline__ void fold_row(Acc& acc, const uint32_t (&v)[8], uint6
 #define OLAP_BRICK_U 3
 #endif
 constexpr int kBrickU = OLAP_BRICK_U;
-template <class Acc, int OPC, bool WIDE>
+template <class Acc, int OPC>
 __device__ __forceinline__ void stream_bricks(const uint32_t* __restrict__ cube, const BDesc& d, int64_t b0,
                                               int64_t b1, Acc& acc, int lane) {
     const int sub = lane >> 2, y = lane & 3;
@@ -1467,9 +1452,9 @@ __device__ __forceinline__ void stream_bricks(const uint32_t* __restrict__ cube,
         for (int u = 0; u < kBrickU; ++u) {
             const int64_t j = j0 + 8 * u + sub;
             const bool ok = j < b1;
-            const int64_t jj = ok ? j : b1 - 1;
+            const int64_t jj = ok ? j : b1 - 1;  // < 2^32: a shard holds < 2^32 bricks (checked at creation)
             uint32_t X, Z;
-            const int64_t a = WIDE ? brick_addr_wide(d, jj, X, Z) : brick_addr(d, (uint32_t)jj, X, Z);
+            const int64_t a = brick_addr(d, (uint32_t)jj, X, Z);
             ld_stream8(cube + a + 8 * y, v[u]);
             const int ylo = X == 0 ? d.ya : 0, yhi = X == d.fX.d - 1 ? d.yb : 3;
             const int zlo = Z == 0 ? d.za : 0, zhi = Z == d.fZ.d - 1 ? d.zb : 7;
@@ -1513,13 +1498,9 @@ __global__ void __launch_bounds__(kThreads, kBrickBlocks) brick_reduce_kernel(
         Acc acc;
         acc.init();
         const int opc = sd.opc;
-        if (sd.nb >= (1ll << 32)) {  // > 2^32 bricks in one box (> 512 GiB): 64-bit digit arithmetic
-            if (opc == OPC_SUM) stream_bricks<Acc, OPC_SUM, true>(c, sd, b0, b1, acc, lane);
-            else if (opc == OPC_MIN) stream_bricks<Acc, OPC_MIN, true>(c, sd, b0, b1, acc, lane);
-            else stream_bricks<Acc, OPC_MAX, true>(c, sd, b0, b1, acc, lane);
-        } else if (opc == OPC_SUM) stream_bricks<Acc, OPC_SUM, false>(c, sd, b0, b1, acc, lane);
-        else if (opc == OPC_MIN) stream_bricks<Acc, OPC_MIN, false>(c, sd, b0, b1, acc, lane);
-        else stream_bricks<Acc, OPC_MAX, false>(c, sd, b0, b1, acc, lane);
+        if (opc == OPC_SUM) stream_bricks<Acc, OPC_SUM>(c, sd, b0, b1, acc, lane);
+        else if (opc == OPC_MIN) stream_bricks<Acc, OPC_MIN>(c, sd, b0, b1, acc, lane);
+        else stream_bricks<Acc, OPC_MAX>(c, sd, b0, b1, acc, lane);
         long long s = acc.sum_bits();
         int32_t cmx = opc == OPC_MAX ? acc.code_max() : INT_MIN, cmn = opc == OPC_MIN ? ~acc.code_min() : INT_MIN;
 #pragma unroll
@@ -2427,6 +2408,10 @@ int olap_cube_create_layout(int ndims, const int64_t* extents, int dtype, const 
     olap_cube* ic = nullptr;
     int rc = olap_cube_create(ndims + 2, e, dtype, shard, device, &ic);
     if (rc) return rc;
+    if ((ic->local_cells >> 5) >= (1ll << 32)) {  // brick indices are 32-bit (2^32 bricks = 512 GiB per shard)
+        olap_cube_destroy(ic);
+        return set_error(OLAP_E_UNSUPPORTED, "a bricked shard must hold < 2^32 bricks");
+    }
     DeviceGuard dg(device);
     olap_cube* c = new (std::nothrow) olap_cube();
     if (!c) {
