@@ -608,12 +608,15 @@ def main():
     if args.graph and world == 1:
         # one CUDA graph per batch (plan, order, reduce, finalize), captured after the warm-up sized the workspace
         graphs = []
+        gk0, gf0 = cube.stats()[0], olap.lib.olap_finalize_launches()
         for k in range(args.warmup + args.steps):
             g = torch.cuda.CUDAGraph()
             with torch.cuda.graph(g, stream=stream):
                 cube.query_device(d_batches[k][0], d_batches[k][1], res, nq=nq, stream=torch.cuda.current_stream())
             graphs.append(g)
         torch.cuda.synchronize()
+        # kernels recorded into each graph (counted by the library at capture) -> launched per replay
+        graph_kernels = (cube.stats()[0] - gk0 + olap.lib.olap_finalize_launches() - gf0) / len(graphs)
 
         def step(k):  # noqa: F811
             graphs[k].replay()
@@ -637,6 +640,8 @@ def main():
     clk = clocks.stop()
     tiles_enabled, tile_cells, _nt, tiles_used = cube.tile_stats()
     gpu_launches = cube.stats()[0] - k0 + olap.lib.olap_finalize_launches() - f0
+    if graphs is not None:
+        gpu_launches = graph_kernels * args.steps
     reduce_ms, launches, alg_bytes = cube.profile_read()
     cube.profile(False)
     t = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev)
