@@ -686,18 +686,21 @@ def test_cuda_graph_capture_replay():
 
 @pytest.mark.parametrize("ext", [(9, 40, 33), (5, 7, 1000), (3, 3, 3, 64)])
 def test_full_range_int32_cells(ext):
-    """int32 cells over the whole int32 range: SUM through mad.wide (sign extension, int64),
-    MIN/MAX at the extremes, AVG = SUM/V — bit-exact vs the oracle."""
+    """int32 cells over the whole int32 range: SUM of biased cells (v ^ 2^31) minus nb * 2^31
+    (int64 mod 2^64, R7), MIN/MAX at the extremes, AVG = SUM/V — bit-exact vs the oracle, on
+    the row-major item / tile paths and the bricked layout."""
     rng = np.random.default_rng(int(np.prod(ext)))
     n = int(np.prod(ext))
     cells = rng.integers(-(2 ** 31), 2 ** 31, size=n, dtype=np.int64).astype(np.int32)
     cells[:3] = [-(2 ** 31), 2 ** 31 - 1, 0]
-    c = olap.Cube(ext, np.int32)
-    c.load(cells)
     boxes = np.concatenate([synth.random_boxes(ext, 300, rng), np.array([[[0, e - 1] for e in ext]])])
-    for op in range(5):
-        ops = np.full(len(boxes), op, np.int32)
-        compare(c.query(boxes, ops), oracle.query(ext, boxes, ops, cells), ops, np.int32)
+    for layout in (olap.LAYOUT_ROWMAJOR, olap.LAYOUT_BRICK):
+        c = olap.Cube(ext, np.int32, layout=layout)
+        c.load(cells)
+        for op in range(5):
+            ops = np.full(len(boxes), op, np.int32)
+            compare(c.query(boxes, ops), oracle.query(ext, boxes, ops, cells), ops, np.int32)
+        c.close()
 
 
 def test_text_ranges_device_matches_host():

@@ -140,3 +140,22 @@ def test_tile_path_on_shards(G, b):
     ref = oracle.query(ext, boxes, ops, dtype=np.int32, gen=oracle.GEN_UNIFORM, seed=23,
                        nthreads=oracle.max_threads())
     compare(got, ref, ops, np.int32)
+
+
+def test_tile_path_full_range_int32_bit_exact():
+    """Full-range int32 cells on the tile path (column and wide modes): the biased-cell SUM
+    (v ^ 2^31, minus nb * 2^31; reading R7) and MIN/MAX extremes, bit-exact vs the oracle."""
+    ext = (40, 16, 16, 16, 160)
+    n = int(np.prod(ext))
+    rng = np.random.default_rng(31)
+    cells = rng.integers(-(2 ** 31), 2 ** 31, size=n, dtype=np.int64).astype(np.int32)
+    cells[:2] = [-(2 ** 31), 2 ** 31 - 1]
+    c = olap.Cube(ext, np.int32)
+    c.load(cells)
+    boxes, _ = synth.config_queries("C2a", nq=512, extents=ext, seed=7)
+    boxes[0] = [[0, e - 1] for e in ext]
+    ops = synth.ops_uniform(len(boxes), rng)
+    got = c.query(boxes, ops)
+    assert c.tile_stats()[3], "batch expected to take the tile path"
+    ref = oracle.query(ext, boxes, ops, cells, nthreads=oracle.max_threads())
+    compare(got, ref, ops, np.int32)
