@@ -25,6 +25,10 @@ namespace olap {
 constexpr int kMaxTableCols = 16;
 constexpr int kMaxConds = 16;
 constexpr int kTileRows = 1024;
+#ifndef OLAP_SPARSE_ROWS
+#define OLAP_SPARSE_ROWS 6
+#endif
+constexpr int kSparseRows = OLAP_SPARSE_ROWS;  // a lane with <= this many surviving rows checks them one by one
 constexpr int kScanWarps = 8;
 constexpr int kScanThreads = kScanWarps * 32;
 
@@ -72,6 +76,20 @@ __device__ __forceinline__ void note_columns(const TQuery& t, uint32_t* colmask)
     if (m) atomicOr(colmask, m);
 }
 
+// Conditions in ascending span order (equality predicates first): after the most selective
+// one, few rows of a lane survive and scan_query_tile checks the rest row by row.
+__device__ __forceinline__ void order_conds(TQuery& t) {
+    for (int i = 1; i < t.ncond; ++i) {
+        const TCond x = t.c[i];
+        int j = i - 1;
+        while (j >= 0 && t.c[j].span > x.span) {
+            t.c[j + 1] = t.c[j];
+            --j;
+        }
+        t.c[j + 1] = x;
+    }
+}
+
 // conditions -> TQuery (one thread per query)
 __global__ void table_prep_kernel(int64_t nq, int ncols, TableCols tc, const int64_t* __restrict__ off,
                                   const olap_cond* __restrict__ conds, const int32_t* __restrict__ data_cols,
@@ -108,6 +126,7 @@ __global__ void table_prep_kernel(int64_t nq, int ncols, TableCols tc, const int
         }
     }
     if (impossible && !t.flags) t.ncond = -1;  // no row can match
+    if (!t.flags) order_conds(t);
     qs[q] = t;
     note_columns(t, colmask);
 }
@@ -148,6 +167,7 @@ __global__ void table_prep_boxes_kernel(int64_t nq, int ncols, TableCols tc, Box
         c.span = (uint32_t)(hi - lo);
     }
     if (impossible && !t.flags) t.ncond = -1;
+    if (!t.flags) order_conds(t);
     qs[q] = t;
     note_columns(t, colmask);
 }
@@ -172,6 +192,16 @@ __device__ __forceinline__ void scan_query_tile(const uint32_t* __restrict__ sme
     const int nc = tq.ncond;
     for (int k = 0; k < nc && pass; ++k) {
         const TCond c = tq.c[k];
+        if (__popc(pass) <= kSparseRows) {  // few survivors: check them one by one
+            const uint32_t* col = smem + c.col * kTileRows + 4 * lane;
+            uint32_t left = pass;
+            while (left) {
+                const int b = __ffs(left) - 1;
+                left &= left - 1;
+                if (col[128 * (b >> 2) + (b & 3)] - c.lo > c.span) pass &= ~(1u << b);
+            }
+            continue;
+        }
         const uint4* col = reinterpret_cast<const uint4*>(smem + c.col * kTileRows) + lane;
         uint32_t m = 0;
 #pragma unroll
