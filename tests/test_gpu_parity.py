@@ -61,6 +61,24 @@ def test_c1_full_bit_exact():
         compare(c.query(boxes, o), oracle.query(cfg["extents"], boxes, o, cells), o, np.int32)
 
 
+
+@pytest.mark.parametrize("nq", [1, 4095, 4096, 4097, 16384, 16385])
+def test_planner_batch_size_boundaries(nq):
+    """Batch sizes around the planner switch: <= 16,384 queries plan in one
+    block (plan_small_kernel), larger ones through items_kernel + CUB scan + scan_fix_kernel;
+    int32 bit-exact, including empty boxes (lo > hi)."""
+    ext = (12, 16, 33)
+    cells = synth.uniform_cells(int(np.prod(ext)), np.int32, 1234 + nq)
+    rng = np.random.default_rng(nq)
+    boxes = synth.random_boxes(ext, nq, rng)
+    ops = synth.ops_uniform(nq, rng)
+    if nq > 2:
+        boxes[nq // 2, 1] = [9, 3]    # lo > hi: empty, reported in flags
+        boxes[nq - 1, 2] = [20, 19]
+    c = olap.Cube(ext, np.int32)
+    c.load(cells)
+    compare(c.query(boxes, ops), oracle.query(ext, boxes, ops, cells), ops, np.int32)
+
 SHAPES = [
     ((8, 8, 8, 8, 8, 64), "C2a-like, runs >= 128 cells merge"),
     ((8, 8, 16, 16, 16, 16), "C2b-like, short runs"),
