@@ -208,6 +208,9 @@ __device__ __forceinline__ void scan_query_tile(const uint32_t* __restrict__ sme
         for (int i = 0; i < 8; ++i) m |= quad_pass(col[32 * i], c.lo, c.span) << (4 * i);
         pass &= m;
     }
+    // no row of the tile matches (most tiles of a query with equality predicates): the
+    // fold below would add +0 / INT_MIN codes, which leaves s, cnt, cmx, cmn bit-identical
+    if (!__any_sync(0xffffffffu, pass)) return;
     int32_t n = __popc(pass);
     const uint32_t* data = smem + tq.data_col * kTileRows + 4 * lane;
     unsigned long long si = 0ull;

@@ -1,0 +1,14 @@
+# Session-4: warp-level early exit of scan_query_tile on tiles with no matching row.
+# Table parity, then an A/B of T against abvar/head.so (the previous table.cu), alternating.
+set -u
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build_s4d.log 2>&1
+timeout 900 python -m pytest tests -m gpu -q -k "table or tpcds or smoke" > gpurun_out/pytest_gpu_r01s4d.log 2>&1; echo "pytest exit $?" >> gpurun_out/pytest_gpu_r01s4d.log
+for rep in 1 2; do
+  for v in head new; do
+    if [ $v = head ]; then env="OLAP_LIB=abvar/head.so"; else env=""; fi
+    env $env timeout 600 python bench.py --workload T > gpurun_out/bench_r01s4d_T_${v}_$rep.log 2>&1
+    tail -1 gpurun_out/bench_r01s4d_T_${v}_$rep.log > gpurun_out/bench_r01s4d_T_${v}_$rep.jsonl
+  done
+done
+echo s4ddone
