@@ -435,7 +435,7 @@ def run_table(args, rank, world):
                      "frac": achieved / peak_evals, "traffic": None, "kernel": "table_scan_kernel",
                      "peak_source": "derived: issue rate (148 SMs x 4 x 32 lanes x 1.965 GHz) / 3 instr per "
                                     "(query,row,column) evaluation (LDS + IADD + ISETP)"},
-        "gpu_launches": int(steps * 3), "clocks": clk,
+        "gpu_launches": int(steps * 4), "clocks": clk,  # prep, order, scan, final per step
         "e2e": {"value": nq * e2e_steps / e2e_s, "unit": "queries/s", "api": "olap_table_query_batch (host buffers)"},
         "cpu_baseline": None,
     }

@@ -254,12 +254,46 @@ __device__ __forceinline__ void scan_query_tile(const uint32_t* __restrict__ sme
     cmn = max(cmn, mn);
 }
 
+// Scan instantiation of a query: (float data, op) -> 0..7; 8 = skipped (invalid / empty).
+__device__ __forceinline__ int scan_class(const TableCols& tc, const TQuery& tq) {
+    if (tq.flags || tq.ncond < 0) return 8;
+    const int opk = tq.op == OLAP_MIN ? 1 : tq.op == OLAP_MAX ? 2 : tq.op == OLAP_COUNT ? 3 : 0;
+    return (tc.dtype[tq.data_col] == OLAP_FLOAT32 ? 4 : 0) + opk;
+}
+
+// Batch order for the scan, grouped by scan_class: the warps of a block (and the blocks
+// of the grid) then run the same scan_query_tile instantiation at the same time instead of
+// cycling through eight code paths per tile (instruction-cache misses were the top stall,
+// "no_instruction", in profiles/ncu_table_scan_r01s4.txt).  The order inside a class is
+// whatever the shared atomics give: each query's partials are still folded in tile and
+// block order, so results do not depend on it.
+__global__ void __launch_bounds__(1024) table_order_kernel(TableCols tc, int64_t nq, const TQuery* __restrict__ qs,
+                                                           int32_t* __restrict__ perm) {
+    __shared__ unsigned long long cnt[9];
+    if (threadIdx.x < 9) cnt[threadIdx.x] = 0;
+    __syncthreads();
+    for (int64_t q = threadIdx.x; q < nq; q += blockDim.x) atomicAdd(&cnt[scan_class(tc, qs[q])], 1ull);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long b = 0;
+        for (int k = 0; k < 9; ++k) {
+            const unsigned long long n = cnt[k];
+            cnt[k] = b;
+            b += n;
+        }
+    }
+    __syncthreads();
+    for (int64_t q = threadIdx.x; q < nq; q += blockDim.x)
+        perm[atomicAdd(&cnt[scan_class(tc, qs[q])], 1ull)] = (int32_t)q;
+}
+
 // The shared scan.  Block b stages tiles b, b+G, ... (all columns) into shared memory;
 // warp w evaluates queries w, w+8, ... on every staged tile.
 __global__ void __launch_bounds__(kScanThreads) table_scan_kernel(TableCols tc, int ncols, int64_t nrows, int64_t nq,
                                                                   const TQuery* __restrict__ qs,
                                                                   TPartial* __restrict__ part,
-                                                                  const uint32_t* __restrict__ colmask) {
+                                                                  const uint32_t* __restrict__ colmask,
+                                                                  const int32_t* __restrict__ perm) {
     extern __shared__ uint32_t smem[];  // ncols x kTileRows (only the batch's columns are staged)
     const uint32_t used = *colmask;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -289,7 +323,8 @@ __global__ void __launch_bounds__(kScanThreads) table_scan_kernel(TableCols tc, 
             }
         }
         __syncthreads();
-        for (int64_t q = w; q < nq; q += kScanWarps) {
+        for (int64_t i = w; i < nq; i += kScanWarps) {
+            const int64_t q = perm[i];
             const TQuery& tq = qs[q];
             if (tq.flags || tq.ncond < 0) continue;
             TPartial p = mine[q];  // warp w owns these partials: no race
@@ -381,6 +416,7 @@ struct TWork {
     TQuery* d_qs = nullptr;
     TPartial* d_part = nullptr;
     uint32_t* d_colmask = nullptr;
+    int32_t* d_perm = nullptr;  // batch order grouped by scan instantiation (table_order_kernel)
     std::mutex mu;
 };
 
@@ -436,6 +472,8 @@ void free_work(TWork& w) {
     cudaFree(w.d_qs);
     cudaFree(w.d_part);
     cudaFree(w.d_colmask);
+    cudaFree(w.d_perm);
+    w.d_perm = nullptr;
     w.d_qs = nullptr;
     w.d_part = nullptr;
     w.d_colmask = nullptr;
@@ -454,12 +492,15 @@ int ensure_work(TWork& w, int64_t nq, cudaStream_t st) {
         OLAP_CUDA_TRY(cudaStreamSynchronize(st));
         cudaFree(w.d_qs);
         cudaFree(w.d_part);
+        cudaFree(w.d_perm);
         w.d_qs = nullptr;
         w.d_part = nullptr;
+        w.d_perm = nullptr;
         w.nq_cap = 0;
         const int64_t cap = std::max<int64_t>(nq, 256);
         OLAP_CUDA_TRY(cudaMalloc(&w.d_qs, sizeof(TQuery) * cap));
         OLAP_CUDA_TRY(cudaMalloc(&w.d_part, sizeof(TPartial) * cap * w.blocks));
+        OLAP_CUDA_TRY(cudaMalloc(&w.d_perm, sizeof(int32_t) * cap));
         w.nq_cap = cap;
     }
     return OLAP_OK;
@@ -500,10 +541,13 @@ int ensure_staging(olap_table* t, int64_t nq, int64_t nconds) {
 int launch_scan_fold(olap_table* t, TWork& w, int64_t nq, olap_result* d_res, cudaStream_t st) {
     const TableCols tc = cols_of(t);
     const size_t smem = sizeof(uint32_t) * kTileRows * t->ncols;
-    table_scan_kernel<<<w.blocks, kScanThreads, smem, st>>>(tc, t->ncols, t->nrows, nq, w.d_qs, w.d_part, w.d_colmask);
+    if (nq > INT32_MAX) return set_error(OLAP_E_INVALID, "table batch of %lld queries: at most 2^31-1", (long long)nq);
+    table_order_kernel<<<1, 1024, 0, st>>>(tc, nq, w.d_qs, w.d_perm);
+    table_scan_kernel<<<w.blocks, kScanThreads, smem, st>>>(tc, t->ncols, t->nrows, nq, w.d_qs, w.d_part, w.d_colmask,
+                                                            w.d_perm);
     table_final_kernel<<<(int)((nq + 255) / 256), 256, 0, st>>>(tc, nq, w.blocks, w.d_qs, w.d_part, d_res);
     OLAP_CUDA_TRY(cudaGetLastError());
-    __atomic_fetch_add(&t->launches, 3, __ATOMIC_RELAXED);
+    __atomic_fetch_add(&t->launches, 4, __ATOMIC_RELAXED);
     return OLAP_OK;
 }
 
