@@ -289,7 +289,10 @@ __global__ void __launch_bounds__(1024) table_order_kernel(TableCols tc, int64_t
 
 // The shared scan.  Block b stages tiles b, b+G, ... (all columns) into shared memory;
 // warp w evaluates queries w, w+8, ... on every staged tile.
-__global__ void __launch_bounds__(kScanThreads) table_scan_kernel(TableCols tc, int ncols, int64_t nrows, int64_t nq,
+#ifndef OLAP_SCAN_MINBLOCKS
+#define OLAP_SCAN_MINBLOCKS 1  // tuning knob (resident blocks per SM the register budget must allow)
+#endif
+__global__ void __launch_bounds__(kScanThreads, OLAP_SCAN_MINBLOCKS) table_scan_kernel(TableCols tc, int ncols, int64_t nrows, int64_t nq,
                                                                   const TQuery* __restrict__ qs,
                                                                   TPartial* __restrict__ part,
                                                                   const uint32_t* __restrict__ colmask,
