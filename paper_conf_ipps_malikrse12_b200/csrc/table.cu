@@ -289,10 +289,15 @@ __global__ void __launch_bounds__(1024) table_order_kernel(TableCols tc, int64_t
 
 // The shared scan.  Block b stages tiles b, b+G, ... (all columns) into shared memory;
 // warp w evaluates queries w, w+8, ... on every staged tile.
-#ifndef OLAP_SCAN_MINBLOCKS
-#define OLAP_SCAN_MINBLOCKS 1  // tuning knob (resident blocks per SM the register budget must allow)
+// OLAP_SCAN_MINBLOCKS: tuning knob (resident blocks per SM the register budget must allow).
+// Not the default: an explicit minimum of 1 let ptxas take 96 registers (2 blocks/SM,
+// T 38.3k -> 25.2k q/s), while the bare bound gives 48 (5 blocks/SM).
+#ifdef OLAP_SCAN_MINBLOCKS
+#define OLAP_SCAN_BOUNDS __launch_bounds__(kScanThreads, OLAP_SCAN_MINBLOCKS)
+#else
+#define OLAP_SCAN_BOUNDS __launch_bounds__(kScanThreads)
 #endif
-__global__ void __launch_bounds__(kScanThreads, OLAP_SCAN_MINBLOCKS) table_scan_kernel(TableCols tc, int ncols, int64_t nrows, int64_t nq,
+__global__ void OLAP_SCAN_BOUNDS table_scan_kernel(TableCols tc, int ncols, int64_t nrows, int64_t nq,
                                                                   const TQuery* __restrict__ qs,
                                                                   TPartial* __restrict__ part,
                                                                   const uint32_t* __restrict__ colmask,
