@@ -7,10 +7,14 @@ device-filled with the counter-hash generator; every step answers one batch of
 4,096 synthetic queries (target fraction log-uniform in [1e-4,1], ops SUM 40% /
 MIN 20% / MAX 20% / AVG 10% / COUNT 10%) with inputs resident in HBM: plan ->
 persistent range-reduce -> finalize.  Each step draws a different batch.
-N>1 (torchrun, one rank per GPU): weak scaling — the global cube grows to
-(16N,16,16,16,16,256), block-cyclic dim-0 shards of 1 GiB per GPU, the same
-4,096-query batch recipe over the global cube; partials cross GPUs through one
-pair of NCCL all-reduces per batch.
+N>1 (one rank per GPU; `--gpus N` re-launches itself under torch.distributed.run when
+WORLD_SIZE is unset): every rank holds a block-cyclic dim-0 shard and the library's own
+NCCL communicator (olap_comm_init_rank + olap_cube_attach_comm) exchanges the 16-B/query
+partials inside olap_query_batch(_device).  Scaling (--scaling): weak (default; the global
+cube (16N,16,16,16,16,256) and the global batch 4,096 N grow with N, 1 GiB and 4,096
+queries' worth of cells per GPU), strong (default for C3: the 32 GiB cube and the 4,096-query
+batch fixed, 32/N GiB per GPU), replica (a full cube per GPU, independent batches, no
+collective: SURVEY §8(e)'s comparison point).
 
 Prints ONE JSON line (rank 0).  `--impl reference` times the CPU oracle (the
 paper's OpenMP partition analogue) on the host cores instead.
@@ -66,9 +70,7 @@ DESC = {
 
 def workload(name: str, world: int):
     cfg = synth.CONFIGS[name]
-    ext = list(cfg["extents"])
-    ext[0] *= world
-    return tuple(ext), cfg
+    return tuple(cfg["extents"]), cfg
 
 
 def batches(name, ext, nq, count, seed0):
@@ -178,13 +180,6 @@ def _traffic(workload, kernel="reduce_kernel"):
             return v.get(kernel)
         return v if kernel == "reduce_kernel" else None
     return None
-
-
-# shared-memory bandwidth of one B200: 32 banks x 4 B per clock per SM (B300_MICROARCH.md / Blackwell guide;
-# same SM design), x 148 SMs x the measured max SM clock.  The tile path serves every per-query read from
-# shared memory, so this — not HBM — is the ceiling its kernel is measured against.
-def smem_peak_gbs(sm_mhz):
-    return 128 * 148 * sm_mhz * 1e6 / 1e9
 
 
 def host_info():
@@ -534,39 +529,60 @@ def run_resolution(args, rank, world):
     return 0
 
 
-def main():
-    ap = argparse.ArgumentParser()
-    ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
-    ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="C2a", choices=["C2a", "C2b", "C3", "C1", "C4", "C5", "T", "R"])
-    ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--e2e-steps", type=int, default=3)
-    ap.add_argument("--graph", action="store_true", help="replay each step as a captured CUDA graph (N=1)")
-    ap.add_argument("--batch", type=int, default=0, help="queries per batch (default: the config's)")
-    ap.add_argument("--layout", default="auto", choices=["auto", "row", "brick"],
-                    help="cube layout in HBM (auto: bricked for C5's small boxes, row-major otherwise; DESIGN.md §5)")
-    args = ap.parse_args()
 
-    rank, world, local = env_int("RANK", 0), env_int("WORLD_SIZE", 1), env_int("LOCAL_RANK", 0)
-    if args.impl == "reference":
-        return run_reference(args, rank, world)
-    if args.workload == "C4":
-        return run_c4(args, rank, world)
-    if args.workload == "T":
-        return run_table(args, rank, world)
-    if args.workload == "R":
-        return run_resolution(args, rank, world)
 
+def smem_peak_gbs(sm_mhz):
+    """Shared-memory read bandwidth of one B200 at `sm_mhz`: the bytes per SM clock MEASURED by
+    tools/smem_peak.cu (profiles/smem_peak.json) x 148 SMs; 128 B/clk/SM if that file is missing."""
+    p = os.path.join(ROOT, "profiles", "smem_peak.json")
+    bpc, src = 128.0, "derived: 32 banks x 4 B per clock per SM (no measurement found)"
+    if os.path.exists(p):
+        with open(p) as f:
+            j = json.load(f)
+        bpc = float(j["bytes_per_clk_per_sm"])
+        src = f"measured: {bpc:.1f} B/clk/SM ({j['how']}) x 148 SMs x {sm_mhz:.0f} MHz (median SM clock, timed region)"
+    return bpc * 148 * sm_mhz * 1e6 / 1e9, src
+
+
+def default_scaling(name):
+    # C3 (32 GiB) fits one B200: the fixed global cube is split N ways (strong); the other cube
+    # workloads grow the global cube and the global batch with N (weak: fixed work per GPU)
+    return "strong" if name == "C3" else "weak"
+
+
+def scaled_workload(name, world, scaling):
+    """(global extents, global batch) of `name` at `world` GPUs under `scaling`."""
+    cfg = synth.CONFIGS[name]
+    ext, nq = list(cfg["extents"]), cfg["nq"]
+    if scaling == "weak" and world > 1:
+        ext[0] *= world
+        nq *= world
+    return tuple(ext), nq
+
+
+def launch_ranks(n):
+    """`python bench.py --gpus N` outside torchrun: re-run this command as N ranks (one per GPU)."""
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
+def run_cube(args, rank, world, local):
+    """C1 / C2a / C2b / C3 / C5: batches of sub-cube queries (the north_star hot path)."""
     import torch
     import torch.distributed as dist
 
     import paper_conf_ipps_malikrse12_b200 as olap
-    from paper_conf_ipps_malikrse12_b200.dist import exchange_partials
 
-    # one rank per GPU; OLAP_DIST_BACKEND=gloo lets ranks share a device to dry-run the N>1 path
-    backend = os.environ.get("OLAP_DIST_BACKEND", "nccl")
+    scaling = args.scaling or default_scaling(args.workload)
+    if world == 1:
+        scaling = "weak"  # one GPU: the config as BASELINE names it
+    backend = os.environ.get("OLAP_DIST_BACKEND", "nccl")  # gloo: dry-run N ranks on one GPU
     local = local % max(torch.cuda.device_count(), 1) if backend != "nccl" else local
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
@@ -575,34 +591,38 @@ def main():
             dist.init_process_group("nccl", device_id=dev)
         else:
             dist.init_process_group(backend)
-    ext, cfg = workload(args.workload, world)
-    nq = args.batch or cfg["nq"]
+    cfg = synth.CONFIGS[args.workload]
+    sharded = world > 1 and scaling != "replica"
+    ext, nq = scaled_workload(args.workload, world, scaling if sharded else "strong")
+    if args.batch:
+        nq = args.batch * (world if (sharded and scaling == "weak") else 1)
     dtype = cfg["dtype"]
     nd = len(ext)
     layout = args.layout if args.layout != "auto" else ("brick" if args.workload == "C5" else "row")
-    cube = olap.Cube(ext, dtype, shard=(world, rank, 1) if world > 1 else None, device=local,
-                     layout=olap.LAYOUT_BRICK if layout == "brick" else olap.LAYOUT_ROWMAJOR)
+    lay = olap.LAYOUT_BRICK if layout == "brick" else olap.LAYOUT_ROWMAJOR
+    comm = None
+    if sharded:
+        # this rank's block-cyclic dim-0 shard; the library's NCCL communicator does the exchange
+        from paper_conf_ipps_malikrse12_b200.dist import init_comm
+        cube = olap.Cube(ext, dtype, shard=(world, rank, 1), device=local, layout=lay)
+        comm = init_comm(rank, world, local)
+        cube.attach_comm(comm)
+    else:
+        cube = olap.Cube(ext, dtype, device=local, layout=lay)
     cube.fill(olap.GEN_UNIFORM, cfg["seed"])
-    host_batches = batches(args.workload, ext, nq, args.warmup + args.steps, cfg["seed"])
+    # replicas answer different batches; shards answer the same global batch
+    seed0 = cfg["seed"] + (7919 * rank if (world > 1 and not sharded) else 0)
+    host_batches = batches(args.workload, ext, nq, args.warmup + args.steps, seed0)
     d_batches = [(torch.from_numpy(b).to(dev), torch.from_numpy(o).to(dev)) for b, o in host_batches]
     res = torch.empty(nq * olap.RESULT_DTYPE.itemsize, dtype=torch.uint8, device=dev)
-    psum = torch.empty(nq, dtype=torch.int64, device=dev)
-    pext = torch.empty(2 * nq, dtype=torch.int32, device=dev)
     stream = torch.cuda.Stream(device=dev)
 
     def step(k):
         dr, do = d_batches[k]
-        if world == 1:
-            cube.query_device(dr, do, res, nq=nq, stream=stream)
-        else:
-            cube.partials_device(dr, do, psum, pext, nq=nq, stream=stream)
-            with torch.cuda.stream(stream):
-                exchange_partials(psum, pext, cube.dtype_code)
-            olap.finalize_device(ext, cube.dtype_code, nq, dr, do, psum, pext, res, stream=stream)
+        cube.query_device(dr, do, res, nq=nq, stream=stream)
 
-    with torch.cuda.stream(stream):
-        for k in range(args.warmup):
-            step(k)
+    for k in range(args.warmup):
+        step(k)
     stream.synchronize()
     graphs = None
     if args.graph and world == 1:
@@ -615,11 +635,11 @@ def main():
                 cube.query_device(d_batches[k][0], d_batches[k][1], res, nq=nq, stream=torch.cuda.current_stream())
             graphs.append(g)
         torch.cuda.synchronize()
-        # kernels recorded into each graph (counted by the library at capture) -> launched per replay
         graph_kernels = (cube.stats()[0] - gk0 + olap.lib.olap_finalize_launches() - gf0) / len(graphs)
 
         def step(k):  # noqa: F811
-            graphs[k].replay()
+            with torch.cuda.stream(stream):
+                graphs[k].replay()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -630,9 +650,8 @@ def main():
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
     e0.record(stream)
-    with torch.cuda.stream(stream):
-        for k in range(args.warmup, args.warmup + args.steps):
-            step(k)
+    for k in range(args.warmup, args.warmup + args.steps):
+        step(k)
     e1.record(stream)
     e1.synchronize()
     torch.cuda.synchronize()
@@ -651,88 +670,98 @@ def main():
         dist.all_reduce(tb, op=dist.ReduceOp.SUM)
     elapsed_ms = float(t.item())
     total_bytes = float(tb.item())
-    total_q = nq * args.steps
+    total_q = nq * args.steps * (world if not sharded else 1)
     qps = total_q / (elapsed_ms / 1e3)
     gbs_total = total_bytes / (elapsed_ms / 1e3) / 1e9
-    peak, peak_src = measured_peaks()
-    achieved = (alg_bytes / max(launches, 1)) / (reduce_ms / max(launches, 1) / 1e3) / 1e9 if reduce_ms else 0.0
+    hbm_peak, hbm_src = measured_peaks()
+    kern_s = reduce_ms / max(launches, 1) / 1e3
+    achieved = (alg_bytes / max(launches, 1)) / kern_s / 1e9 if reduce_ms else 0.0
 
-    # end to end through the public host-buffer C-ABI (H2D of ranges/ops, D2H of results inside)
+    # end to end through the public host-buffer C-ABI (H2D of ranges/ops, D2H of results inside):
+    # olap_query_batch on every rank (on a shard with a communicator it is the library's collective)
     e2e = None
-    if world == 1 and args.e2e_steps > 0:
+    if args.e2e_steps > 0:
         outs = np.zeros(nq, dtype=olap.RESULT_DTYPE)
         b0, o0 = host_batches[0]
         cube.query(b0, o0, out=outs)
+        if world > 1:
+            dist.barrier()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         for k in range(args.e2e_steps):
             b, o = host_batches[args.warmup + (k % args.steps)]
             cube.query(b, o, out=outs)
-        e2e_s = time.perf_counter() - t0
-        e2e = {"value": nq * args.e2e_steps / e2e_s, "unit": "queries/s",
-               "h2d_bytes_per_step": int(nq * nd * 16 + nq * 4), "d2h_bytes_per_step": int(nq * 24),
-               "api": "olap_query_batch (host buffers; pinned staging inside the library)"}
-    elif world > 1 and args.e2e_steps > 0:
-        # host arrays in, host results out, through the sharded path on every rank:
-        # pinned H2D -> shard partials -> NCCL exchange -> finalize -> D2H (timed max over ranks)
-        pin_r = torch.empty((nq, nd, 2), dtype=torch.int64).pin_memory()
-        pin_o = torch.empty(nq, dtype=torch.int32).pin_memory()
-        pin_res = torch.empty(nq * olap.RESULT_DTYPE.itemsize, dtype=torch.uint8).pin_memory()
-        d_r = torch.empty((nq, nd, 2), dtype=torch.int64, device=dev)
-        d_o = torch.empty(nq, dtype=torch.int32, device=dev)
-        dist.barrier()
-        torch.cuda.synchronize()
-        t0 = time.perf_counter()
-        for k in range(args.e2e_steps):
-            b, o = host_batches[args.warmup + (k % args.steps)]
-            pin_r.numpy()[...] = b
-            pin_o.numpy()[...] = o
-            with torch.cuda.stream(stream):
-                d_r.copy_(pin_r, non_blocking=True)
-                d_o.copy_(pin_o, non_blocking=True)
-                cube.partials_device(d_r, d_o, psum, pext, nq=nq, stream=stream)
-                exchange_partials(psum, pext, cube.dtype_code)
-                olap.finalize_device(ext, cube.dtype_code, nq, d_r, d_o, psum, pext, res, stream=stream)
-                pin_res.copy_(res, non_blocking=True)
-            stream.synchronize()
         e2e_t = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
-        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
-        e2e = {"value": nq * args.e2e_steps / float(e2e_t.item()), "unit": "queries/s",
+        if world > 1:
+            dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+        e2e_q = nq * args.e2e_steps * (world if not sharded else 1)
+        e2e = {"value": e2e_q / float(e2e_t.item()), "unit": "queries/s",
                "h2d_bytes_per_step": int(nq * nd * 16 + nq * 4), "d2h_bytes_per_step": int(nq * 24),
-               "api": "ShardedCube path: H2D, olap_query_partials_device, NCCL all-reduce, olap_finalize_device, D2H"}
+               "api": ("olap_query_batch on this rank's shard with the library's NCCL communicator attached "
+                       "(pinned H2D, shard partials, ncclAllReduce of 16 B/query, finalize, D2H; max over ranks)"
+                       if sharded else "olap_query_batch (host buffers; pinned staging inside the library)")}
+        if args.stream_batch:
+            # the same queries as one stream through olap_query_stream (pipelined batches)
+            allb = np.concatenate([host_batches[args.warmup + (k % args.steps)][0] for k in range(args.e2e_steps)])
+            allo = np.concatenate([host_batches[args.warmup + (k % args.steps)][1] for k in range(args.e2e_steps)])
+            cube.query_stream(allb[:nq], allo[:nq], batch=args.stream_batch)
+            if world > 1:
+                dist.barrier()
+            t0 = time.perf_counter()
+            cube.query_stream(allb, allo, batch=args.stream_batch)
+            st_t = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
+            if world > 1:
+                dist.all_reduce(st_t, op=dist.ReduceOp.MAX)
+            e2e["stream"] = {"value": len(allo) * (world if not sharded else 1) / float(st_t.item()),
+                             "unit": "queries/s", "batch": args.stream_batch,
+                             "api": "olap_query_stream (batch k+1 reduces while batch k exchanges / finalizes)"}
 
     kernel = "tile_reduce_kernel" if tiles_used else ("brick_reduce_kernel" if layout == "brick" else "reduce_kernel")
-    traffic = _traffic(args.workload, kernel)
+    traffic = _traffic(args.workload, kernel) if world == 1 else None
+    dram = {"gbs": traffic / kern_s / 1e9, "frac_of_hbm": traffic / kern_s / 1e9 / hbm_peak,
+            "source": "ncu dram__bytes_read.sum + dram__bytes_write.sum per launch (profiles/traffic.json) / "
+                      "the kernel's CUDA-event time here"} if (traffic and reduce_ms) else None
+    sm_mhz = (clk or {}).get("sm_mhz") or 1965.0
     if tiles_used:
-        sm_mhz = (clk or {}).get("sm_mhz") or 1965.0
-        rnote = ("tile-shared scan: each 96-KiB cube tile is staged into shared memory once per batch (cp.async.bulk; "
-                 "traffic = its DRAM bytes per launch from ncu) and every query reads its cells from shared memory; "
-                 "achieved = algorithmic bytes (sum of V_q*4 over non-COUNT queries, Eq. 3) / tile_reduce_kernel "
-                 "time, so frac vs HBM > 1 by construction; smem.frac is the same bytes against the shared-memory "
-                 "bandwidth that bounds the kernel (128 B/clk/SM x 148 SMs at the measured SM clock)")
-        smem = {"peak": smem_peak_gbs(sm_mhz), "unit": "GB/s", "frac": achieved / smem_peak_gbs(sm_mhz),
-                "peak_source": f"derived: 128 B/clk/SM x 148 SMs x {sm_mhz:.0f} MHz (median SM clock in the timed region)"}
+        speak, ssrc = smem_peak_gbs(sm_mhz)
+        roofline = {"bound": "smem", "achieved": achieved, "peak": speak, "unit": "GB/s", "frac": achieved / speak,
+                    "traffic": traffic, "kernel": kernel, "peak_source": ssrc,
+                    "note": "tile-shared scan: each 96-KiB cube tile is staged into shared memory once per batch "
+                            "(cp.async.bulk) and every query reduces its cells of the tile from shared memory, so "
+                            "the shared-memory read bandwidth bounds the kernel; achieved = algorithmic bytes "
+                            "(sum of V_q*4 over non-COUNT queries, Eq. 3) / tile_reduce_kernel time (CUDA events); "
+                            "traffic = ncu DRAM bytes per launch",
+                    "hbm_equiv": {"achieved": achieved, "peak": hbm_peak, "frac": achieved / hbm_peak,
+                                  "note": "the same algorithmic bytes against the HBM copy peak: > 1 because the "
+                                          "cube is read from HBM once per batch, not once per query"}}
     elif layout == "brick":
-        rnote = ("bricked layout: achieved = algorithmic bytes (sum of V_q*4 over non-COUNT queries, Eq. 3) / "
-                 "brick_reduce_kernel time; the kernel reads whole 128-B bricks (one DRAM fetch line each), so "
-                 "traffic (ncu DRAM bytes per launch, profiles/traffic.json) exceeds the algorithmic bytes by the "
-                 "edge bricks' unselected cells")
-        smem = None
+        roofline = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
+                    "frac": achieved / hbm_peak, "traffic": traffic, "kernel": kernel, "peak_source": hbm_src,
+                    "note": "bricked layout: achieved = algorithmic bytes (V_q*4, Eq. 3) / brick_reduce_kernel "
+                            "time; the kernel reads whole 128-B bricks (one DRAM fetch line each), so traffic "
+                            "exceeds the algorithmic bytes by the edge bricks' unselected cells (dram.gbs is the "
+                            "rate the HBM actually moved)"}
     else:
-        rnote = ("achieved = algorithmic bytes (sum of V_q*4 over non-COUNT queries, Eq. 3) / "
-                 "reduce-kernel time; frac > 1 is L2 reuse: items are scheduled in cube-address "
-                 "order so queries overlapping in the cube read it from L2 (traffic = DRAM "
-                 "bytes per launch from ncu, profiles/traffic.json)")
-        smem = None
+        roofline = {"bound": "hbm" if args.workload != "C1" else "l2", "achieved": achieved, "peak": hbm_peak,
+                    "unit": "GB/s", "frac": achieved / hbm_peak, "traffic": traffic, "kernel": kernel,
+                    "peak_source": hbm_src,
+                    "note": "item path: achieved = algorithmic bytes (V_q*4, Eq. 3) / reduce-kernel time; frac > 1 "
+                            "is L2 reuse (items run in cube-address order)" +
+                            ("; C1's 4 MiB cube is L2-resident by design: the HBM peak is only a reference"
+                             if args.workload == "C1" else "")}
+    roofline.update({"dram": dram, "algorithmic_bytes_per_launch": alg_bytes / max(launches, 1),
+                     "reduce_share_of_step": reduce_ms / elapsed_ms if elapsed_ms else None})
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(args.workload, ext, cfg, seed=cfg["seed"] + 1000 + args.warmup)
     if rank == 0:
+        par = "1gpu" if world == 1 else (f"shard{world}" if sharded else f"replica{world}")
         line = {
             "metric": METRIC, "value": qps, "unit": "queries/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "i32" if dtype == np.int32 else "f32",
+            "scaling": "strong" if (sharded and scaling == "strong") else "weak",
+            "vs_baseline": None, "dtype": "i32" if dtype == np.int32 else "f32",
             "data": "synthetic",
             "config": {"workload": args.workload, "extents": list(ext), "cube_gib_per_gpu":
                        cube.info()[1] * 4 / 2**30, "batch": nq,
@@ -740,19 +769,18 @@ def main():
                        "l2": ("no flush: C1's 4 MiB cube is L2-resident by design (flagged)" if args.workload == "C1"
                               else "no flush: cube > L2 (126 MB) and every step reads >> L2"),
                        "accumulation": ("int32 cells, int64 SUM" if dtype == np.int32 else
-                                        ("f32 cells, SUM in fp32 trees of <= 8 cells then f64" if tiles_used
-                                         else "f32 cells, f64 SUM")),
-                       "path": "tile-shared scan" if tiles_used else "item path",
+                                        ("f32 cells, SUM in fp32 trees of <= 16 cells then f64 (reading R8')"
+                                         if tiles_used else
+                                         ("f32 cells, SUM in fp32 trees of one 8-cell brick row then f64"
+                                          if layout == "brick" else "f32 cells, f64 SUM"))),
+                       "path": "tile-shared scan" if tiles_used else ("brick" if layout == "brick" else "item path"),
                        "layout": ("bricked: last two dims in 4x8-cell (128-B) bricks" if layout == "brick"
                                   else "row-major"),
-                       "parallelism": f"shard{world}" if world > 1 else "1gpu"},
+                       "parallelism": par,
+                       "exchange": ("library NCCL: ncclAllReduce of the 16-B/query partials per batch "
+                                    "(olap_cube_attach_comm)" if sharded else None)},
             "gbs": gbs_total, "frac_of_nominal_8tbs": gbs_total / world / NOMINAL_HBM_GBS,
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "kernel": kernel, "smem": smem,
-                         "peak_source": peak_src,
-                         "algorithmic_bytes_per_launch": alg_bytes / max(launches, 1),
-                         "reduce_share_of_step": reduce_ms / elapsed_ms if elapsed_ms else None,
-                         "note": rnote},
+            "roofline": roofline,
             "gpu_launches": int(gpu_launches), "l2_order": l2_order,
             "clocks": clk,
             "e2e": e2e,
@@ -761,8 +789,51 @@ def main():
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.barrier()
+        cube.close()
+        if comm is not None:
+            comm.close()
         dist.destroy_process_group()
     return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=None,
+                    help="GPUs (one rank each); without torchrun, N > 1 re-launches itself under torch.distributed.run")
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="C2a", choices=["C2a", "C2b", "C3", "C1", "C4", "C5", "T", "R"])
+    ap.add_argument("--scaling", default=None, choices=["weak", "strong", "replica"],
+                    help="N > 1: weak (global cube and batch grow with N; default), strong (fixed global cube "
+                         "and batch; default for C3), replica (a full cube per GPU, independent batches)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--stream-batch", type=int, default=0,
+                    help="also time the e2e queries as one olap_query_stream in batches of this size")
+    ap.add_argument("--graph", action="store_true", help="replay each step as a captured CUDA graph (N=1)")
+    ap.add_argument("--batch", type=int, default=0, help="queries per batch per GPU (default: the config's)")
+    ap.add_argument("--layout", default="auto", choices=["auto", "row", "brick"],
+                    help="cube layout in HBM (auto: bricked for C5's small boxes, row-major otherwise; DESIGN.md §5)")
+    args = ap.parse_args()
+
+    rank, world, local = env_int("RANK", 0), env_int("WORLD_SIZE", 1), env_int("LOCAL_RANK", 0)
+    launched = "WORLD_SIZE" in os.environ
+    if args.gpus is None:
+        args.gpus = world
+    if not launched and args.gpus > 1:
+        return launch_ranks(args.gpus)
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}: launch one rank per GPU")
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+    if args.workload == "C4":
+        return run_c4(args, rank, world)
+    if args.workload == "T":
+        return run_table(args, rank, world)
+    if args.workload == "R":
+        return run_resolution(args, rank, world)
+    return run_cube(args, rank, world, local)
 
 
 if __name__ == "__main__":

@@ -41,7 +41,7 @@
 extern "C" {
 #endif
 
-typedef struct olap_cube olap_cube; /* opaque: one (shard of a) dense cube on one GPU */
+typedef struct olap_cube olap_cube; /* opaque: a dense cube, one shard of it, or a group of shards */
 typedef struct olap_dict olap_dict; /* opaque: one text column's dictionary, immutable */
 
 typedef enum {
@@ -50,6 +50,7 @@ typedef enum {
     OLAP_E_RANGE = -2,       /* a query range lies outside the cube */
     OLAP_E_NOMEM = -3,       /* device or host allocation failed */
     OLAP_E_CUDA = -4,        /* CUDA runtime error / no device */
+    OLAP_E_NCCL = -5,        /* NCCL missing, a NCCL call failed, or a communicator failed (asynchronously) */
     OLAP_E_STATE = -6,       /* handle in the wrong state */
     OLAP_E_UNSUPPORTED = -7
 } olap_status;
@@ -146,13 +147,18 @@ int olap_cube_add_facts_device(olap_cube* c, int64_t nrows, const int32_t* d_ids
 
 /* Whole path on HOST buffers: validate, copy ranges (nq*ndims, query-major) and
  * ops in, plan + range-reduce + finalize on the GPU, copy results out, sync.
- * Only valid on an unsharded cube (nshards == 1).  nq == 0 is a no-op. */
+ * Valid on an unsharded cube, on a group handle (olap_cube_create_multi: every shard
+ * reduces, the partials are exchanged over NCCL, devices[0] finalizes) and on a shard with
+ * an attached communicator (olap_cube_attach_comm: a collective, every rank passes the same
+ * batch and receives every answer).  A plain shard returns OLAP_E_STATE.  nq == 0 is a no-op. */
 int olap_query_batch(olap_cube* c, int64_t nq, const olap_range* ranges, const int32_t* ops,
                      olap_result* results);
 
 /* Same path on DEVICE buffers, asynchronous on `stream` (cudaStream_t, NULL =
  * legacy default stream).  Invalid queries are flagged OLAP_RESULT_INVALID in
- * their result instead of failing the batch.  Unsharded cubes only.  The call can be
+ * their result instead of failing the batch.  On a group handle the buffers and `stream`
+ * live on devices[0] (the inputs are copied to the other devices over NVLink); on a shard
+ * with a communicator, on its device (a collective, as above).  An unsharded cube's call can be
  * captured into a CUDA graph (and olap_query_partials_device likewise) after one
  * uncaptured call with at least nq queries has sized the cube's workspace; a replayed
  * graph must not overlap another batch on the same cube. */
@@ -161,7 +167,8 @@ int olap_query_batch_device(olap_cube* c, int64_t nq, const olap_range* d_ranges
 
 /* Shard-local half of the path: plan + range-reduce of this shard's part of
  * every query into partials (d_sum[nq], d_ext[2*nq], see above).  COUNT queries
- * and boxes that miss the shard produce the identity.  Asynchronous. */
+ * and boxes that miss the shard produce the identity.  Asynchronous.  Not on a group
+ * handle (OLAP_E_UNSUPPORTED: call it on the shards). */
 int olap_query_partials_device(olap_cube* c, int64_t nq, const olap_range* d_ranges,
                                const int32_t* d_ops, int64_t* d_sum, int32_t* d_ext, void* stream);
 
@@ -205,6 +212,71 @@ int64_t olap_finalize_launches(void);
  * tile_cells = cells of a full tile; ntiles = tiles of the (local) cube; last_used = the
  * last batch took it (waits for that batch).  Any out-pointer may be NULL. */
 int olap_cube_tile_stats(olap_cube* c, int* enabled, int64_t* tile_cells, int64_t* ntiles, int* last_used);
+
+/* ---------------------------------------------------------------- multi-GPU */
+
+/* The cube sharded on dimension 0 over several GPUs (BASELINE.json north_star part (4); the
+ * paper used one GPU).  Every shard reduces its part of each query into the
+ * partials above; ONE exchange combines them (16 B per query: sum with +, the two codes with
+ * max, in one ncclGroup); the finalize turns them into answers.  Two ways to run it:
+ *   - one process, several GPUs: olap_cube_create_multi -> a group handle.  The shards'
+ *     partials are reduced over NCCL (ncclCommInitAll, ncclReduce) to devices[0];
+ *   - one process per GPU: olap_comm_init_rank on every rank (the id from olap_comm_unique_id
+ *     on rank 0, passed out of band), olap_cube_create with olap_shard {nranks, rank, b},
+ *     then olap_cube_attach_comm.  ncclAllReduce: every rank gets every answer.
+ * NCCL is loaded at run time (libnccl.so.2, or the file named by $OLAP_NCCL_LIB); without it
+ * these calls return OLAP_E_NCCL.  After each exchange the communicators' asynchronous error
+ * state is polled; a failed communicator is aborted and every later batch returns OLAP_E_NCCL.
+ * Float sums are combined in NCCL's fixed order for a given configuration (deterministic);
+ * int32 results are bit-exact for any number of shards (wraparound sums, R7). */
+
+typedef struct {
+    int32_t ndevices;          /* >= 1 distinct CUDA ordinals in `devices`; devices[0] is the root */
+    int32_t shards_per_device; /* >= 1: G = ndevices * shards_per_device shards, shard g on devices[g / spd];
+                                  shards of one device are folded in shard order before the exchange */
+    const int32_t* devices;
+    int64_t shard_block;       /* block-cyclic dim-0 block b >= 1 (olap_shard) */
+    int32_t layout;            /* OLAP_LAYOUT_* of every shard */
+    int32_t _pad;
+} olap_cube_opts;
+
+/* A group handle: G shard cubes (olap_shard {G, g, shard_block}) over opts->devices.  load,
+ * load_rows, fill, destroy, info (summed rows / cells, d_cells = NULL), profile, stats and the
+ * query calls act on every shard.  OLAP_E_NCCL if NCCL cannot be loaded or initialised. */
+int olap_cube_create_multi(int ndims, const int64_t* extents, int dtype, const olap_cube_opts* opts,
+                           olap_cube** out);
+
+typedef struct olap_comm olap_comm;               /* opaque: one rank of a NCCL communicator */
+typedef struct { char internal[128]; } olap_comm_id;  /* = ncclUniqueId */
+
+/* Rank 0 creates the id and broadcasts its 128 bytes to every rank (any channel). */
+int olap_comm_unique_id(olap_comm_id* id);
+/* Collective over nranks processes: this rank's communicator on CUDA `device`. */
+int olap_comm_init_rank(const olap_comm_id* id, int nranks, int rank, int device, olap_comm** out);
+int olap_comm_info(const olap_comm* comm, int* nranks, int* rank, int* device);
+/* Poll the asynchronous error state (OLAP_E_NCCL, and the communicator is aborted, on failure). */
+int olap_comm_check(olap_comm* comm);
+/* Destroys (or aborts, after a failure) the communicator; detach it from cubes first. */
+int olap_comm_destroy(olap_comm* comm);
+
+/* Attach (comm != NULL) or detach a communicator to a shard whose olap_shard is {nranks, rank,
+ * b} on the communicator's device: olap_query_batch(_device) and olap_query_stream then run the
+ * whole sharded path as a collective.  The cube borrows the communicator. */
+int olap_cube_attach_comm(olap_cube* c, olap_comm* comm);
+
+/* The exchange alone (all-reduce in place of d_sum[nq], d_ext[2*nq] over the communicator),
+ * asynchronous on `stream`, for callers that run olap_query_partials_device themselves. */
+int olap_exchange_partials_device(olap_comm* comm, int dtype, int64_t nq, int64_t* d_sum, int32_t* d_ext,
+                                  void* stream);
+int olap_nccl_version(int* version);
+
+/* A stream of nq queries (HOST buffers) answered in batches of `batch` (<= 0: one batch),
+ * pipelined: batch k+1's copy-in and range-reduce run while batch k's exchange, finalize and
+ * copy-out complete ("overlap batch k's exchange with batch k+1's reduction").
+ * Any cube kind (plain, group, shard with a communicator).  Results are those of
+ * olap_query_batch on each batch; the whole stream fails with OLAP_E_RANGE on a bad query. */
+int olap_query_stream(olap_cube* c, int64_t nq, const olap_range* ranges, const int32_t* ops,
+                      olap_result* results, int64_t batch);
 
 /* ---------------------------------------------------------------- dictionaries */
 
@@ -293,7 +365,9 @@ int olap_table_load_column(olap_table* t, int col, const void* values);
 /* Device pointer of column `col` (nrows 4-byte values), e.g. to fill it on the device. */
 int olap_table_column_device(olap_table* t, int col, void** d_ptr);
 
-/* Answer nq queries Q_D on HOST buffers.  Query q has conditions
+/* A table's calls (and a partition's) may come from different streams: each workspace orders
+ * a batch after the previous batch on that workspace (an event), whatever its stream.
+ * Answer nq queries Q_D on HOST buffers.  Query q has conditions
  * conds[cond_offsets[q] .. cond_offsets[q+1]) (at most 16; cond_offsets[0] = 0), data
  * column data_cols[q] and op ops[q].  A row matches when it satisfies every condition
  * (PAPER.md:208); the result aggregates the data column over matching rows: COUNT =
@@ -330,7 +404,8 @@ int olap_table_part_query_device(olap_table_part* p, int64_t nq, const int64_t* 
 /* Queries given as boxes over dimension columns, e.g. olap_text_ranges output: query q's
  * condition on dimension d is column dim_cols[d] in d_boxes[q*ndims + d] (inclusive); a
  * range covering all of [0, extents[d]) is no condition and reads no column (Eq. 12); an
- * empty range matches nothing.  dim_cols and extents are HOST arrays of ndims <= 16. */
+ * empty range (lo > hi) matches nothing; lo < 0 or hi >= extents[d] flags the query
+ * OLAP_RESULT_INVALID (the cube path's rule, reading R10).  dim_cols and extents are HOST arrays of ndims <= 16. */
 int olap_table_part_query_boxes_device(olap_table_part* p, int64_t nq, int ndims, const int32_t* dim_cols,
                                        const int64_t* extents, const olap_range* d_boxes,
                                        const int32_t* d_data_cols, const int32_t* d_ops, olap_result* d_results,

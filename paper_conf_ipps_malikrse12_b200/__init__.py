@@ -23,7 +23,8 @@ __all__ = ["Cube", "Dict", "OlapError", "translate", "shard_local_rows", "combin
            "RESULT_EMPTY", "RESULT_INVALID", "EXPORTS", "text_ranges", "text_ranges_device", "pack_text_conditions", "text_ranges_packed",
            "COND_ALL", "COND_EQ", "COND_RANGE", "COND_IDS", "Table", "COND_DTYPE", "Hierarchy", "CubeSet",
            "TablePart", "Scheduler", "PART_CUBE", "PART_TABLE", "SCHED_PART_DTYPE", "SCHED_QUERY_DTYPE",
-           "SCHED_DECISION_DTYPE", "perf_fn"]
+           "SCHED_DECISION_DTYPE", "perf_fn", "Comm", "comm_unique_id", "nccl_version", "exchange_partials_device",
+           "E_NCCL"]
 
 LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libolap_b200.so")
 if os.environ.get("OLAP_LIB"):          # development only: A/B a differently-tuned build of the same sources
@@ -36,7 +37,7 @@ GEN_UNIFORM, GEN_AFFINE = 1, 2
 RESULT_EMPTY, RESULT_INVALID = 1, 2
 COND_ALL, COND_EQ, COND_RANGE, COND_IDS = 0, 1, 2, 3
 
-OK, E_INVALID, E_RANGE, E_NOMEM, E_CUDA, E_STATE, E_UNSUPPORTED = 0, -1, -2, -3, -4, -6, -7
+OK, E_INVALID, E_RANGE, E_NOMEM, E_CUDA, E_NCCL, E_STATE, E_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6, -7
 
 PART_CUBE, PART_TABLE = 0, 1
 
@@ -111,6 +112,16 @@ EXPORTS = {
     "olap_finalize_launches": (_i64, []),
     "olap_cube_tile_stats": (_int, [_p, ctypes.POINTER(_int), ctypes.POINTER(_i64), ctypes.POINTER(_i64),
                                     ctypes.POINTER(_int)]),
+    "olap_cube_create_multi": (_int, [_int, _i64p, _int, _p, ctypes.POINTER(_p)]),
+    "olap_comm_unique_id": (_int, [_p]),
+    "olap_comm_init_rank": (_int, [_p, _int, _int, _int, ctypes.POINTER(_p)]),
+    "olap_comm_info": (_int, [_p, ctypes.POINTER(_int), ctypes.POINTER(_int), ctypes.POINTER(_int)]),
+    "olap_comm_check": (_int, [_p]),
+    "olap_comm_destroy": (_int, [_p]),
+    "olap_cube_attach_comm": (_int, [_p, _p]),
+    "olap_exchange_partials_device": (_int, [_p, _int, _i64, _p, _p, _p]),
+    "olap_nccl_version": (_int, [ctypes.POINTER(_int)]),
+    "olap_query_stream": (_int, [_p, _i64, _p, _p, _p, _i64]),
     "olap_last_error": (ctypes.c_char_p, []),
     "olap_version": (ctypes.c_char_p, []),
 }
@@ -197,22 +208,44 @@ def _i64arr(a):
     return a, a.ctypes.data_as(_i64p)
 
 
-class Cube:
-    """A dense cube (or one block-cyclic dim-0 shard of it) resident in one GPU's HBM."""
+class _CubeOpts(ctypes.Structure):
+    _fields_ = [("ndevices", ctypes.c_int32), ("shards_per_device", ctypes.c_int32),
+                ("devices", ctypes.POINTER(ctypes.c_int32)), ("shard_block", ctypes.c_int64),
+                ("layout", ctypes.c_int32), ("pad", ctypes.c_int32)]
 
-    def __init__(self, extents, dtype, shard=None, device: int = 0, layout: int = LAYOUT_ROWMAJOR):
+
+class Cube:
+    """A dense cube (or one block-cyclic dim-0 shard of it) resident in one GPU's HBM.
+
+    devices=[d0, d1, ...] (and/or shards_per_device > 1) makes a group handle
+    (olap_cube_create_multi): the cube sharded over those GPUs of this process, answered
+    through the library's NCCL exchange."""
+
+    def __init__(self, extents, dtype, shard=None, device: int = 0, layout: int = LAYOUT_ROWMAJOR,
+                 devices=None, shards_per_device: int = 1, shard_block: int = 1):
         self.extents = tuple(int(e) for e in extents)
         self.layout = int(layout)
         self.ndims = len(self.extents)
         self.dtype_code = _dtype_code(dtype)
         self.np_dtype = np.int32 if self.dtype_code == INT32 else np.float32
         self.shard = tuple(shard) if shard is not None else (1, 0, 1)
-        self.device = device
+        self.device = device if devices is None else int(devices[0])
+        self._comm = None
         ext, extp = _i64arr(self.extents)
         h = ctypes.c_void_p()
-        sh = _shard(shard)
-        _check(lib.olap_cube_create_layout(self.ndims, extp, self.dtype_code, ctypes.byref(sh) if sh else None,
-                                           device, self.layout, ctypes.byref(h)), "olap_cube_create_layout")
+        if devices is not None or shards_per_device > 1:
+            devs = np.ascontiguousarray(devices if devices is not None else [device], dtype=np.int32)
+            o = _CubeOpts(len(devs), int(shards_per_device), devs.ctypes.data_as(ctypes.POINTER(ctypes.c_int32)),
+                          int(shard_block), self.layout, 0)
+            _check(lib.olap_cube_create_multi(self.ndims, extp, self.dtype_code, ctypes.byref(o), ctypes.byref(h)),
+                   "olap_cube_create_multi")
+            self.shard = (len(devs) * int(shards_per_device), 0, int(shard_block))
+            self.devices = tuple(int(d) for d in devs)
+        else:
+            sh = _shard(shard)
+            _check(lib.olap_cube_create_layout(self.ndims, extp, self.dtype_code, ctypes.byref(sh) if sh else None,
+                                               device, self.layout, ctypes.byref(h)), "olap_cube_create_layout")
+            self.devices = (int(device),)
         self._h = h
 
     @property
@@ -249,6 +282,21 @@ class Cube:
         _check(lib.olap_query_batch(self._h, nq, rng.ctypes.data, opa.ctypes.data, res.ctypes.data),
                "olap_query_batch")
         return res
+
+    def query_stream(self, ranges, ops, batch: int = 0, out: np.ndarray | None = None) -> np.ndarray:
+        """olap_query_stream: a stream of queries answered in pipelined batches of `batch`."""
+        rng = np.ascontiguousarray(ranges, dtype=np.int64).reshape(-1, self.ndims, 2)
+        nq = rng.shape[0]
+        opa = np.ascontiguousarray(ops, dtype=np.int32).reshape(nq)
+        res = out if out is not None else np.zeros(nq, dtype=RESULT_DTYPE)
+        _check(lib.olap_query_stream(self._h, nq, rng.ctypes.data, opa.ctypes.data, res.ctypes.data, int(batch)),
+               "olap_query_stream")
+        return res
+
+    def attach_comm(self, comm: "Comm | None"):
+        """olap_cube_attach_comm: this shard's batches become collectives over `comm` (None detaches)."""
+        _check(lib.olap_cube_attach_comm(self._h, comm.handle if comm is not None else None), "olap_cube_attach_comm")
+        self._comm = comm  # the cube borrows it
 
     def query_device(self, d_ranges, d_ops, d_results, nq: int | None = None, stream=None):
         nq = d_ops.numel() if nq is None else nq
@@ -292,12 +340,64 @@ class Cube:
         if getattr(self, "_h", None):
             lib.olap_cube_destroy(self._h)
             self._h = None
+        self._comm = None
 
     def __del__(self):
         try:
             self.close()
         except Exception:
             pass
+
+
+class Comm:
+    """One rank of a NCCL communicator owned by the library (olap_comm_init_rank)."""
+
+    def __init__(self, unique_id: bytes, nranks: int, rank: int, device: int = 0):
+        if len(unique_id) != 128:
+            raise ValueError("a communicator id is 128 bytes (olap_comm_unique_id)")
+        buf = ctypes.create_string_buffer(bytes(unique_id), 128)
+        h = ctypes.c_void_p()
+        _check(lib.olap_comm_init_rank(buf, int(nranks), int(rank), int(device), ctypes.byref(h)),
+               "olap_comm_init_rank")
+        self._h = h
+        self.nranks, self.rank, self.device = int(nranks), int(rank), int(device)
+
+    @property
+    def handle(self):
+        return self._h
+
+    def check(self):
+        _check(lib.olap_comm_check(self._h), "olap_comm_check")
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib.olap_comm_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def comm_unique_id() -> bytes:
+    """olap_comm_unique_id: 128 bytes that rank 0 passes to every rank."""
+    buf = ctypes.create_string_buffer(128)
+    _check(lib.olap_comm_unique_id(buf), "olap_comm_unique_id")
+    return buf.raw
+
+
+def nccl_version() -> int:
+    v = _int()
+    _check(lib.olap_nccl_version(ctypes.byref(v)), "olap_nccl_version")
+    return v.value
+
+
+def exchange_partials_device(comm: Comm, dtype, nq: int, d_sum, d_ext, stream=None):
+    """olap_exchange_partials_device: all-reduce partials in place over the library's communicator."""
+    _check(lib.olap_exchange_partials_device(comm.handle, _dtype_code(dtype), nq, _ptr(d_sum), _ptr(d_ext),
+                                             _stream(stream)), "olap_exchange_partials_device")
 
 
 def combine_partials_device(dtype, nq: int, sum_in, ext_in, sum_acc, ext_acc, stream=None):

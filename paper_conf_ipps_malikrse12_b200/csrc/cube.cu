@@ -22,6 +22,7 @@
 #include <cub/device/device_scan.cuh>
 
 #include "common.cuh"
+#include "mgpu.h"
 
 namespace olap {
 
@@ -1770,6 +1771,7 @@ struct olap_cube {
     void* d_cubtmp = nullptr;
     size_t cub_bytes = 0;
     int32_t* d_ctl = nullptr;                  // [0] mode (1 = tiles), [1] non-empty tiles, [2] pop counter
+    bool ctl_dirty = false;                    // a tile planner ran: d_ctl[0] may hold 1 (cleared when tiles go off)
     unsigned long long* d_ttot = nullptr;      // tile path batch totals (cells)
 
     bool prof = false;
@@ -1784,6 +1786,15 @@ struct olap_cube {
     // owns the cells (queries use its workspace: run_partials_brick).
     olap_cube* inner = nullptr;
     int brick_bps = 0;  // resident brick_reduce_kernel blocks per SM
+
+    // multi-GPU (mgpu.cu): a group handle (olap_cube_create_multi) owns `shards` (G shard cubes
+    // over its devices) and answers through `exec`; a shard with an attached communicator
+    // (olap_cube_attach_comm) answers through `exec` too; a plain cube builds `exec` lazily for
+    // olap_query_stream.
+    std::vector<olap_cube*> shards;
+    olap::Exec* exec = nullptr;
+    olap_comm* comm = nullptr;
+    bool multi() const { return !shards.empty(); }
 };
 
 namespace {
@@ -1870,7 +1881,9 @@ void free_ws(olap_cube* c) {
 void ensure_tile_ws(olap_cube* c, int64_t cap) {
     if (!c->tiles_on || cap <= c->tq_cap) return;
     const int64_t nt = c->tg.ntiles;
-    bool ok = cudaMalloc(&c->d_tdesc, sizeof(TDesc) * cap) == cudaSuccess &&
+    // test hook: simulate an allocation failure above a query capacity (tests/test_gpu_tiles.py)
+    const char* lim = getenv("OLAP_TEST_TILE_WS_LIMIT");
+    bool ok = !(lim && cap > atoll(lim)) && cudaMalloc(&c->d_tdesc, sizeof(TDesc) * cap) == cudaSuccess &&
               cudaMalloc(&c->d_qpairs, sizeof(int64_t) * (cap + 1)) == cudaSuccess &&
               cudaMalloc(&c->d_pstart, sizeof(int64_t) * (cap + 1)) == cudaSuccess;
     if (ok && !c->d_tcount) {
@@ -1989,7 +2002,14 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
         return OLAP_OK;
     };
     const int32_t* tmode = c->d_ctl;  // stays 0 when the cube has no tile path
+    if (!c->tiles_on && c->ctl_dirty) {
+        // the tile path was switched off (workspace growth failed) after a batch that took it:
+        // clear the stale mode word, or every item-path kernel below would return at once
+        OLAP_CUDA_TRY(cudaMemsetAsync(c->d_ctl, 0, sizeof(int32_t), st));
+        c->ctl_dirty = false;
+    }
     if (c->tiles_on) {
+        c->ctl_dirty = true;
         // tile-shared scan (tiles.cuh); tile_scan_kernel picks it or the item path on the device
         const TGeo& tg = c->tg;
         const int qb = (int)((nq + kDescThreads - 1) / kDescThreads), eg = c->num_sms * 8;
@@ -2268,6 +2288,7 @@ void make_tiles(olap_cube* c) {
 
 int check_cube(const olap_cube* c) {
     if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    if (c->multi()) return OLAP_OK;
     if (!c->d_cells) return set_error(OLAP_E_STATE, "cube has no device storage");
     return OLAP_OK;
 }
@@ -2453,6 +2474,17 @@ int olap_cube_create_layout(int ndims, const int64_t* extents, int dtype, const 
 int olap_cube_info(const olap_cube* c, int64_t* local_rows, int64_t* local_cells, void** d_cells) {
     clear_error();
     if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    if (c->multi()) {  // a group: every shard's rows and cells; no single device pointer
+        int64_t r = 0, n = 0;
+        for (const olap_cube* s : c->shards) {
+            r += s->local_rows;
+            n += s->local_cells;
+        }
+        if (local_rows) *local_rows = r;
+        if (local_cells) *local_cells = n;
+        if (d_cells) *d_cells = nullptr;
+        return OLAP_OK;
+    }
     if (local_rows) *local_rows = c->local_rows;
     if (local_cells) *local_cells = c->local_cells;
     if (d_cells) *d_cells = c->d_cells;
@@ -2466,6 +2498,13 @@ int olap_cube_load_rows(olap_cube* c, int64_t row_lo, int64_t row_hi, const void
     if (!cells || row_lo < 0 || row_hi > c->n[0] || row_lo > row_hi)
         return set_error(OLAP_E_INVALID, "olap_cube_load_rows: bad rows [%lld,%lld)", (long long)row_lo,
                          (long long)row_hi);
+    if (c->multi()) {  // every shard copies the rows it owns
+        for (olap_cube* sc : c->shards) {
+            rc = olap_cube_load_rows(sc, row_lo, row_hi, cells);
+            if (rc) return rc;
+        }
+        return OLAP_OK;
+    }
     std::lock_guard<std::mutex> lk(c->mu);
     DeviceGuard dg(c->device);
     OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
@@ -2516,6 +2555,13 @@ int olap_cube_fill(olap_cube* c, int generator, uint64_t seed, const double* par
     if (generator != OLAP_GEN_UNIFORM && generator != OLAP_GEN_AFFINE)
         return set_error(OLAP_E_INVALID, "unknown generator %d", generator);
     if (generator == OLAP_GEN_AFFINE && !params) return set_error(OLAP_E_INVALID, "affine generator needs params");
+    if (c->multi()) {  // the generators are functions of the global index: every shard fills its own rows
+        for (olap_cube* sc : c->shards) {
+            rc = olap_cube_fill(sc, generator, seed, params);
+            if (rc) return rc;
+        }
+        return OLAP_OK;
+    }
     std::lock_guard<std::mutex> lk(c->mu);
     DeviceGuard dg(c->device);
     FillParams fp;
@@ -2557,6 +2603,7 @@ int olap_cube_add_facts_device(olap_cube* c, int64_t nrows, const int32_t* d_ids
     if (nrows == 0) return OLAP_OK;
     if (!d_ids) return set_error(OLAP_E_INVALID, "d_ids is NULL");
     if (c->inner) return set_error(OLAP_E_UNSUPPORTED, "olap_cube_add_facts_device needs a row-major cube");
+    if (c->multi()) return set_error(OLAP_E_UNSUPPORTED, "olap_cube_add_facts_device: add facts to each shard");
     std::lock_guard<std::mutex> lk(c->mu);
     DeviceGuard dg(c->device);
     cudaStream_t st = static_cast<cudaStream_t>(stream);
@@ -2577,6 +2624,13 @@ int olap_cube_add_facts_device(olap_cube* c, int64_t nrows, const int32_t* d_ids
 int olap_cube_destroy(olap_cube* c) {
     clear_error();
     if (!c) return OLAP_OK;
+    olap::exec_destroy(c->exec);  // drains its streams first
+    c->exec = nullptr;
+    if (c->multi()) {
+        for (olap_cube* sc : c->shards) olap_cube_destroy(sc);
+        delete c;
+        return OLAP_OK;
+    }
     DeviceGuard dg(c->device);
     if (c->ws_done) cudaEventSynchronize(c->ws_done);
     if (c->stream) cudaStreamSynchronize(c->stream);
@@ -2609,18 +2663,12 @@ int olap_query_batch(olap_cube* c, int64_t nq, const olap_range* ranges, const i
     if (nq < 0) return set_error(OLAP_E_INVALID, "nq < 0");
     if (nq == 0) return OLAP_OK;
     if (!ranges || !ops || !results) return set_error(OLAP_E_INVALID, "olap_query_batch: NULL buffer");
+    rc = olap::validate_queries(c->nd, c->n, nq, ranges, ops);
+    if (rc) return rc;
+    if (c->multi() || c->comm) return olap::exec_query_batch(c->exec, nq, ranges, ops, results);
     if (c->sh.nshards != 1)
-        return set_error(OLAP_E_STATE, "olap_query_batch needs an unsharded cube; use olap_query_partials_device");
-    for (int64_t q = 0; q < nq; ++q) {
-        if (ops[q] < OLAP_SUM || ops[q] > OLAP_AVG)
-            return set_error(OLAP_E_INVALID, "query %lld: unknown op %d", (long long)q, ops[q]);
-        for (int k = 0; k < c->nd; ++k) {
-            const olap_range r = ranges[q * c->nd + k];
-            if (r.lo < 0 || r.hi >= c->n[k])
-                return set_error(OLAP_E_RANGE, "query %lld dimension %d: range [%lld,%lld] outside [0,%lld)",
-                                 (long long)q, k, (long long)r.lo, (long long)r.hi, (long long)c->n[k]);
-        }
-    }
+        return set_error(OLAP_E_STATE, "olap_query_batch on a shard needs an attached communicator "
+                         "(olap_cube_attach_comm) or olap_query_partials_device");
     std::lock_guard<std::mutex> lk(c->mu);
     DeviceGuard dg(c->device);
     rc = ensure_stage(c, nq);
@@ -2654,6 +2702,9 @@ int olap_query_partials_device(olap_cube* c, int64_t nq, const olap_range* d_ran
     if (nq < 0) return set_error(OLAP_E_INVALID, "nq < 0");
     if (nq == 0) return OLAP_OK;
     if (!d_ranges || !d_ops || !d_sum || !d_ext) return set_error(OLAP_E_INVALID, "NULL device buffer");
+    if (c->multi())
+        return set_error(OLAP_E_UNSUPPORTED, "olap_query_partials_device on a group handle: query its shards, or use "
+                         "olap_query_batch(_device)");
     std::lock_guard<std::mutex> lk(c->mu);
     DeviceGuard dg(c->device);
     return run_partials(c, nq, d_ranges, d_ops, d_sum, d_ext, static_cast<cudaStream_t>(stream));
@@ -2667,7 +2718,13 @@ int olap_query_batch_device(olap_cube* c, int64_t nq, const olap_range* d_ranges
     if (nq < 0) return set_error(OLAP_E_INVALID, "nq < 0");
     if (nq == 0) return OLAP_OK;
     if (!d_ranges || !d_ops || !d_results) return set_error(OLAP_E_INVALID, "NULL device buffer");
-    if (c->sh.nshards != 1) return set_error(OLAP_E_STATE, "olap_query_batch_device needs an unsharded cube");
+    if (c->multi() || c->comm) {
+        if (capturing(static_cast<cudaStream_t>(stream)))
+            return set_error(OLAP_E_UNSUPPORTED, "stream capture of a multi-GPU batch");
+        return olap::exec_query_batch_device(c->exec, nq, d_ranges, d_ops, d_results, static_cast<cudaStream_t>(stream));
+    }
+    if (c->sh.nshards != 1)
+        return set_error(OLAP_E_STATE, "olap_query_batch_device on a shard needs an attached communicator");
     std::lock_guard<std::mutex> lk(c->mu);
     DeviceGuard dg(c->device);
     cudaStream_t st = static_cast<cudaStream_t>(stream);
@@ -2735,8 +2792,23 @@ int olap_shard_local_rows(int64_t n0, const olap_shard* s, int64_t lo, int64_t h
 int olap_cube_stats(const olap_cube* c, int64_t* kernel_launches, int* l2_order) {
     clear_error();
     if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    if (c->multi()) {
+        int64_t k = olap::exec_launches(c->exec);
+        int o = 1;
+        for (const olap_cube* sc : c->shards) {
+            int64_t ks = 0;
+            int os = 0;
+            olap_cube_stats(sc, &ks, &os);
+            k += ks;
+            o &= os;
+        }
+        if (kernel_launches) *kernel_launches = k;
+        if (l2_order) *l2_order = o;
+        return OLAP_OK;
+    }
     const olap_cube* ic = c->inner ? c->inner : c;
-    if (kernel_launches) *kernel_launches = c->kernel_launches + (c->inner ? c->inner->kernel_launches : 0);
+    if (kernel_launches)
+        *kernel_launches = c->kernel_launches + (c->inner ? c->inner->kernel_launches : 0) + olap::exec_launches(c->exec);
     if (l2_order) *l2_order = ic->order_shift >= 0 ? 1 : 0;
     return OLAP_OK;
 }
@@ -2746,6 +2818,7 @@ int64_t olap_finalize_launches(void) { return g_finalize_launches.load(); }
 int olap_cube_tile_stats(olap_cube* c, int* enabled, int64_t* tile_cells, int64_t* ntiles, int* last_used) {
     clear_error();
     if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    if (c->multi()) return olap_cube_tile_stats(c->shards[0], enabled, tile_cells, ntiles, last_used);
     if (c->inner) {
         std::lock_guard<std::mutex> lk(c->mu);
         return olap_cube_tile_stats(c->inner, enabled, tile_cells, ntiles, last_used);
@@ -2765,6 +2838,13 @@ int olap_cube_tile_stats(olap_cube* c, int* enabled, int64_t* tile_cells, int64_
 int olap_cube_profile(olap_cube* c, int enable) {
     clear_error();
     if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    if (c->multi()) {
+        for (olap_cube* sc : c->shards) {
+            int rc = olap_cube_profile(sc, enable);
+            if (rc) return rc;
+        }
+        return OLAP_OK;
+    }
     if (c->inner) {
         std::lock_guard<std::mutex> lk(c->mu);
         return olap_cube_profile(c->inner, enable);
@@ -2782,6 +2862,23 @@ int olap_cube_profile(olap_cube* c, int enable) {
 int olap_cube_profile_read(olap_cube* c, double* reduce_ms, int64_t* launches, int64_t* bytes) {
     clear_error();
     if (!c) return set_error(OLAP_E_INVALID, "cube handle is NULL");
+    if (c->multi()) {  // sums over the shards (reduce time: summed over shards, whatever device)
+        double ms = 0.0;
+        int64_t n = 0, b = 0;
+        for (olap_cube* sc : c->shards) {
+            double m = 0.0;
+            int64_t nn = 0, bb = 0;
+            int rc = olap_cube_profile_read(sc, &m, &nn, &bb);
+            if (rc) return rc;
+            ms += m;
+            n += nn;
+            b += bb;
+        }
+        if (reduce_ms) *reduce_ms = ms;
+        if (launches) *launches = n;
+        if (bytes) *bytes = b;
+        return OLAP_OK;
+    }
     if (c->inner) {
         std::lock_guard<std::mutex> lk(c->mu);
         OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
@@ -2803,6 +2900,116 @@ int olap_cube_profile_read(olap_cube* c, double* reduce_ms, int64_t* launches, i
     if (launches) *launches = c->launches;
     if (bytes) *bytes = (int64_t)(b - c->bytes_base);
     return OLAP_OK;
+}
+
+int olap_cube_create_multi(int ndims, const int64_t* extents, int dtype, const olap_cube_opts* opts, olap_cube** out) {
+    clear_error();
+    if (!out || !extents || !opts || !opts->devices)
+        return set_error(OLAP_E_INVALID, "olap_cube_create_multi: NULL argument");
+    if (opts->ndevices < 1 || opts->ndevices > 64)
+        return set_error(OLAP_E_INVALID, "ndevices %d not in [1,64]", opts->ndevices);
+    if (opts->shards_per_device < 1 || opts->shard_block < 1)
+        return set_error(OLAP_E_INVALID, "shards_per_device and shard_block must be >= 1");
+    if (ndims < 1 || ndims > kMaxDims) return set_error(OLAP_E_INVALID, "ndims %d not in [1,8]", ndims);
+    for (int i = 0; i < opts->ndevices; ++i)
+        for (int j = 0; j < i; ++j)
+            if (opts->devices[i] == opts->devices[j])
+                return set_error(OLAP_E_INVALID, "device %d listed twice (use shards_per_device)", opts->devices[i]);
+    const int spd = opts->shards_per_device;
+    const int64_t G = (int64_t)opts->ndevices * spd;
+    olap_cube* c = new (std::nothrow) olap_cube();
+    if (!c) return set_error(OLAP_E_NOMEM, "host allocation failed");
+    c->nd = ndims;
+    c->dtype = dtype;
+    c->device = opts->devices[0];
+    c->sh = olap_shard{G, 0, opts->shard_block};
+    for (int k = 0; k < ndims; ++k) c->n[k] = extents[k];
+    c->lrow_cells = 1;
+    for (int k = 1; k < ndims; ++k) c->lrow_cells *= extents[k];
+    olap::ExecSpec spec;
+    spec.nd = ndims;
+    spec.dtype = dtype;
+    for (int k = 0; k < ndims; ++k) spec.n[k] = extents[k];
+    spec.spd = spd;
+    spec.own_comms = true;
+    for (int i = 0; i < opts->ndevices; ++i) spec.devices.push_back(opts->devices[i]);
+    for (int64_t g = 0; g < G; ++g) {
+        const olap_shard sh{G, g, opts->shard_block};
+        olap_cube* sc = nullptr;
+        int rc = olap_cube_create_layout(ndims, extents, dtype, &sh, opts->devices[g / spd], opts->layout, &sc);
+        if (rc) {
+            std::string msg = olap_last_error();
+            olap_cube_destroy(c);
+            return set_error(rc, "shard %lld of %lld on device %d: %s", (long long)g, (long long)G,
+                             opts->devices[g / spd], msg.c_str());
+        }
+        c->shards.push_back(sc);
+    }
+    spec.shards = c->shards;
+    int rc = olap::exec_create(spec, &c->exec);
+    if (rc) {
+        std::string msg = olap_last_error();
+        olap_cube_destroy(c);
+        return set_error(rc, "%s", msg.c_str());
+    }
+    *out = c;
+    return OLAP_OK;
+}
+
+int olap_cube_attach_comm(olap_cube* c, olap_comm* comm) {
+    clear_error();
+    int rc = check_cube(c);
+    if (rc) return rc;
+    if (c->multi()) return set_error(OLAP_E_INVALID, "a group handle has its own communicators");
+    int nranks = 0, rank = 0, device = 0;
+    if (comm) {
+        rc = olap_comm_info(comm, &nranks, &rank, &device);
+        if (rc) return rc;
+        if (c->sh.nshards != nranks || c->sh.shard != rank || c->device != device)
+            return set_error(OLAP_E_INVALID, "cube shard %lld of %lld on device %d does not match communicator rank %d "
+                             "of %d on device %d", (long long)c->sh.shard, (long long)c->sh.nshards, c->device, rank,
+                             nranks, device);
+    }
+    olap::exec_destroy(c->exec);
+    c->exec = nullptr;
+    c->comm = nullptr;
+    if (!comm) return OLAP_OK;
+    olap::ExecSpec spec;
+    spec.nd = c->nd;
+    spec.dtype = c->dtype;
+    for (int k = 0; k < c->nd; ++k) spec.n[k] = c->n[k];
+    spec.devices.push_back(c->device);
+    spec.shards.push_back(c);
+    spec.comm = comm;
+    rc = olap::exec_create(spec, &c->exec);
+    if (rc) return rc;
+    c->comm = comm;
+    return OLAP_OK;
+}
+
+int olap_query_stream(olap_cube* c, int64_t nq, const olap_range* ranges, const int32_t* ops, olap_result* results,
+                      int64_t batch) {
+    clear_error();
+    int rc = check_cube(c);
+    if (rc) return rc;
+    if (nq < 0) return set_error(OLAP_E_INVALID, "nq < 0");
+    if (nq == 0) return OLAP_OK;
+    if (!ranges || !ops || !results) return set_error(OLAP_E_INVALID, "olap_query_stream: NULL buffer");
+    rc = olap::validate_queries(c->nd, c->n, nq, ranges, ops);
+    if (rc) return rc;
+    if (!c->exec) {
+        if (c->sh.nshards != 1)
+            return set_error(OLAP_E_STATE, "olap_query_stream on a shard needs an attached communicator");
+        olap::ExecSpec spec;  // a plain cube: the pipeline without an exchange
+        spec.nd = c->nd;
+        spec.dtype = c->dtype;
+        for (int k = 0; k < c->nd; ++k) spec.n[k] = c->n[k];
+        spec.devices.push_back(c->device);
+        spec.shards.push_back(c);
+        rc = olap::exec_create(spec, &c->exec);
+        if (rc) return rc;
+    }
+    return olap::exec_query_stream(c->exec, nq, ranges, ops, results, batch);
 }
 
 }  // extern "C"

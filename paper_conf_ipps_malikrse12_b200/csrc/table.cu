@@ -154,13 +154,22 @@ __global__ void table_prep_boxes_kernel(int64_t nq, int ncols, TableCols tc, Box
     bool impossible = false;
     for (int d = 0; d < bm.ndims && !t.flags; ++d) {
         const olap_range r = boxes[q * bm.ndims + d];
+        if (r.lo < 0 || r.hi >= bm.extent[d]) {  // outside [0, extent): INVALID, the cube path's rule (R10)
+            t.flags = OLAP_RESULT_INVALID;
+            break;
+        }
         if (r.lo > r.hi) {
             impossible = true;
             continue;
         }
         if (r.lo <= 0 && r.hi >= bm.extent[d] - 1) continue;  // the whole dimension: no condition
-        const int64_t lo = r.lo < INT_MIN ? (int64_t)INT_MIN : r.lo;
-        const int64_t hi = r.hi > INT_MAX ? (int64_t)INT_MAX : r.hi;
+        // ids are in [0, extent) (< 2^31 by the 32-bit id columns): clamp, then the span cannot wrap
+        const int64_t lo = r.lo < INT_MIN ? (int64_t)INT_MIN : (r.lo > INT_MAX ? (int64_t)INT_MAX : r.lo);
+        const int64_t hi = r.hi > INT_MAX ? (int64_t)INT_MAX : (r.hi < INT_MIN ? (int64_t)INT_MIN : r.hi);
+        if (lo > hi) {
+            impossible = true;
+            continue;
+        }
         TCond& c = t.c[t.ncond++];
         c.col = bm.col[d];
         c.lo = (uint32_t)(int32_t)lo;
@@ -425,6 +434,8 @@ struct TWork {
     TPartial* d_part = nullptr;
     uint32_t* d_colmask = nullptr;
     int32_t* d_perm = nullptr;  // batch order grouped by scan instantiation (table_order_kernel)
+    cudaEvent_t done = nullptr; // recorded after the last kernel of every batch on this workspace: a
+                                // batch on another stream waits for it before touching d_qs / d_part
     std::mutex mu;
 };
 
@@ -486,6 +497,8 @@ void free_work(TWork& w) {
     w.d_part = nullptr;
     w.d_colmask = nullptr;
     w.nq_cap = 0;
+    if (w.done) cudaEventDestroy(w.done);
+    w.done = nullptr;
 }
 
 void init_work(const olap_table* t, TWork& w, int sm_count) {
@@ -493,11 +506,21 @@ void init_work(const olap_table* t, TWork& w, int sm_count) {
     w.blocks = w.sm_count * std::max(t->blocks_per_sm, 1);
 }
 
-// (re)size a workspace; `st` is the stream its previous launches were queued on
+bool stream_capturing(cudaStream_t st) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    return cudaStreamIsCapturing(st, &cs) == cudaSuccess && cs == cudaStreamCaptureStatusActive;
+}
+
+// (re)size a workspace and order `st` after the workspace's previous batch, whatever stream
+// that batch ran on (w.done); the caller records w.done on `st` after its last kernel
 int ensure_work(TWork& w, int64_t nq, cudaStream_t st) {
     if (!w.d_colmask) OLAP_CUDA_TRY(cudaMalloc(&w.d_colmask, sizeof(uint32_t)));
+    if (!w.done) OLAP_CUDA_TRY(cudaEventCreateWithFlags(&w.done, cudaEventDisableTiming));
     if (nq > w.nq_cap) {
-        OLAP_CUDA_TRY(cudaStreamSynchronize(st));
+        if (stream_capturing(st))
+            return set_error(OLAP_E_STATE, "stream capture: run one batch of %lld queries outside capture first",
+                             (long long)nq);
+        OLAP_CUDA_TRY(cudaEventSynchronize(w.done));
         cudaFree(w.d_qs);
         cudaFree(w.d_part);
         cudaFree(w.d_perm);
@@ -511,6 +534,7 @@ int ensure_work(TWork& w, int64_t nq, cudaStream_t st) {
         OLAP_CUDA_TRY(cudaMalloc(&w.d_perm, sizeof(int32_t) * cap));
         w.nq_cap = cap;
     }
+    if (!stream_capturing(st)) OLAP_CUDA_TRY(cudaStreamWaitEvent(st, w.done, 0));
     return OLAP_OK;
 }
 
@@ -555,6 +579,7 @@ int launch_scan_fold(olap_table* t, TWork& w, int64_t nq, olap_result* d_res, cu
                                                             w.d_perm);
     table_final_kernel<<<(int)((nq + 255) / 256), 256, 0, st>>>(tc, nq, w.blocks, w.d_qs, w.d_part, d_res);
     OLAP_CUDA_TRY(cudaGetLastError());
+    if (!stream_capturing(st)) OLAP_CUDA_TRY(cudaEventRecord(w.done, st));
     __atomic_fetch_add(&t->launches, 4, __ATOMIC_RELAXED);
     return OLAP_OK;
 }

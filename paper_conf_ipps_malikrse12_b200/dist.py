@@ -1,65 +1,66 @@
-"""Multi-GPU plumbing for the sharded cube.
+"""One process per GPU: the sharded cube on a torch.distributed job.
 
-One process per GPU.  Rank g holds shard g of a block-cyclic dim-0 split of the
-global cube.  A batch runs the shard-local plan + range-reduce in the library's
-kernels (``olap_query_partials_device``), exchanges the per-query partials with
-ONE pair of element-wise all-reduces over NCCL (torch.distributed: SUM on the
-int64 / float64 sums, MAX on the order-preserving MIN/MAX codes), then finalizes
-in the library's kernel.  The exchange is 16 B per query, latency-bound.
+Rank g holds shard g of a block-cyclic dim-0 split of the global cube.  The whole query path
+(shard-local plan + range-reduce, the NCCL exchange of the per-query partials, the finalize) runs
+inside the library: this module only bootstraps the library's NCCL communicator — rank 0 asks the
+library for a communicator id (olap_comm_unique_id) and torch.distributed broadcasts its 128
+bytes — and attaches it to the rank's shard (olap_cube_attach_comm).  torch.distributed is the
+out-of-band channel, nothing more; no partial crosses it.
 """
 from __future__ import annotations
 
 import numpy as np
 
-from . import FLOAT32, INT32, RESULT_DTYPE, Cube, finalize_device
+from . import RESULT_DTYPE, Comm, Cube, comm_unique_id
 
 
-def exchange_partials(psum, pext, dtype_code: int, group=None):
-    """All-reduce partials in place: sums with +, ext codes with max (olap.h partial format).
-
-    Works on CUDA tensors with the nccl backend and on CPU tensors with gloo."""
-    import torch
+def broadcast_comm_id(rank: int, group=None) -> bytes:
+    """Rank 0's olap_comm_unique_id, broadcast to every rank of `group` (any backend)."""
     import torch.distributed as dist
 
-    if dtype_code == FLOAT32:
-        dist.all_reduce(psum.view(torch.float64), op=dist.ReduceOp.SUM, group=group)
-    else:
-        dist.all_reduce(psum, op=dist.ReduceOp.SUM, group=group)   # two's complement wraparound
-    dist.all_reduce(pext, op=dist.ReduceOp.MAX, group=group)
+    box = [comm_unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(box, src=0, group=group)
+    uid = box[0]
+    if not isinstance(uid, (bytes, bytearray)) or len(uid) != 128:
+        raise RuntimeError("communicator id broadcast failed")
+    return bytes(uid)
+
+
+def init_comm(rank: int, world: int, device: int, group=None) -> Comm:
+    """The library's NCCL communicator for this rank (collective over the process group)."""
+    return Comm(broadcast_comm_id(rank, group), world, rank, device)
 
 
 class ShardedCube:
-    """This rank's shard of a cube sharded over the default process group."""
+    """This rank's shard of a cube sharded over the default process group, answering batches
+    as collectives through the library (olap_query_batch / _device / olap_query_stream)."""
 
-    def __init__(self, extents, dtype, rank: int, world: int, block: int = 1, device: int = 0, group=None):
+    def __init__(self, extents, dtype, rank: int, world: int, block: int = 1, device: int = 0, group=None,
+                 layout: int = 0, comm: Comm | None = None):
         self.extents = tuple(int(e) for e in extents)
-        self.cube = Cube(self.extents, dtype, shard=(world, rank, block), device=device)
+        self.cube = Cube(self.extents, dtype, shard=(world, rank, block), device=device, layout=layout)
         self.dtype_code = self.cube.dtype_code
-        self.rank, self.world, self.group = rank, world, group
-        self._ws = None
+        self.rank, self.world = rank, world
+        self.comm = comm if comm is not None else init_comm(rank, world, device, group)
+        self.cube.attach_comm(self.comm)
 
-    def _workspace(self, nq: int):
-        import torch
-        if self._ws is None or self._ws[0].numel() < nq:
-            dev = torch.device("cuda", self.cube.device)
-            self._ws = (torch.empty(nq, dtype=torch.int64, device=dev),
-                        torch.empty(2 * nq, dtype=torch.int32, device=dev))
-        return self._ws[0][:nq], self._ws[1][:2 * nq]
+    def fill(self, *a, **k):
+        self.cube.fill(*a, **k)
 
-    def query_device(self, d_ranges, d_ops, d_results, stream=None):
-        nq = d_ops.numel()
-        psum, pext = self._workspace(nq)
-        self.cube.partials_device(d_ranges, d_ops, psum, pext, nq=nq, stream=stream)
-        if self.world > 1:
-            exchange_partials(psum, pext, self.dtype_code, self.group)
-        finalize_device(self.extents, self.dtype_code, nq, d_ranges, d_ops, psum, pext, d_results, stream=stream)
+    def query_device(self, d_ranges, d_ops, d_results, nq: int | None = None, stream=None):
+        self.cube.query_device(d_ranges, d_ops, d_results, nq=nq, stream=stream)
 
-    def query(self, ranges, ops) -> np.ndarray:
+    def query(self, ranges, ops, out: np.ndarray | None = None) -> np.ndarray:
         """Host arrays in, host results out (every rank gets every answer)."""
-        import torch
-        dev = torch.device("cuda", self.cube.device)
-        rng = torch.from_numpy(np.ascontiguousarray(ranges, dtype=np.int64)).to(dev)
-        opt = torch.from_numpy(np.ascontiguousarray(ops, dtype=np.int32)).to(dev)
-        res = torch.empty(opt.numel() * RESULT_DTYPE.itemsize, dtype=torch.uint8, device=dev)
-        self.query_device(rng, opt, res)
-        return res.cpu().numpy().view(RESULT_DTYPE)
+        return self.cube.query(ranges, ops, out=out)
+
+    def query_stream(self, ranges, ops, batch: int = 0) -> np.ndarray:
+        return self.cube.query_stream(ranges, ops, batch=batch)
+
+    def close(self):
+        self.cube.attach_comm(None)
+        self.cube.close()
+        self.comm.close()
+
+
+__all__ = ["broadcast_comm_id", "init_comm", "ShardedCube", "RESULT_DTYPE"]

@@ -1,11 +1,14 @@
-"""N>1 host path on CPU: world_size-2 gloo process group.
+"""N>1 host path on CPU: world_size-2 gloo process groups.
 
-Each rank owns a block-cyclic dim-0 shard of the cube (olap_shard_local_rows from the
-product's C-ABI gives its local row range), computes its partials over its local box
-(here with the oracle on the shard's rows, since kernels need a GPU), encodes them in
-the olap.h partial format, and the product's exchange (dist.exchange_partials: SUM on
-sums, MAX on MIN/MAX codes) combines them.  The decoded result must equal the oracle
-on the global cube.
+1. The exchange algebra.  Each rank owns a block-cyclic dim-0 shard of the cube
+   (olap_shard_local_rows from the product's C-ABI gives its local row range), computes its
+   partials over its local box (here with the oracle on the shard's rows, since kernels need a
+   GPU), encodes them in the olap.h partial format, and the two element-wise reductions the
+   library's NCCL exchange performs (mgpu.cu: ncclSum on the sums as uint64 / float64, ncclMax
+   on the int32 codes) are applied across the ranks with gloo all-reduces of the same types.
+   The decoded result must equal the oracle on the global cube.
+2. The communicator bootstrap of dist.py: rank 0's olap_comm_unique_id reaches every rank
+   through the process group, and olap_comm_init_rank without a GPU fails loudly (E_CUDA).
 """
 import os
 import socket
@@ -50,7 +53,6 @@ def _worker(rank, world, port, dtype_name, block, q):
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         import paper_conf_ipps_malikrse12_b200 as olap
-        from paper_conf_ipps_malikrse12_b200.dist import exchange_partials
 
         dtype = np.dtype(dtype_name)
         ext = (23, 6, 9)
@@ -82,7 +84,13 @@ def _worker(rank, world, port, dtype_name, block, q):
                 pext[2 * i] = int(_code(mx["d"][0], dtype))
                 pext[2 * i + 1] = int(~_code(mn["d"][0], dtype))
         code = olap.INT32 if dtype == np.int32 else olap.FLOAT32
-        exchange_partials(psum, pext, code)
+        # the library's exchange (mgpu.cu): ncclSum on uint64 (int32 cube, wraparound) or
+        # float64 sums, ncclMax on the int32 codes -- the same reductions over gloo
+        if code == olap.FLOAT32:
+            dist.all_reduce(psum.view(torch.float64), op=dist.ReduceOp.SUM)
+        else:
+            dist.all_reduce(psum, op=dist.ReduceOp.SUM)
+        dist.all_reduce(pext, op=dist.ReduceOp.MAX)
         ref = oracle.query(ext, boxes, ops, cells.ravel())
         bad = 0
         for i in range(nq):
@@ -123,3 +131,45 @@ def test_two_rank_exchange_equals_oracle(dtype_name, block):
         p.join(timeout=60)
     for rank, bad in out:
         assert bad == 0, f"rank {rank}: {bad}"
+
+
+def _boot_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import paper_conf_ipps_malikrse12_b200 as olap
+        from paper_conf_ipps_malikrse12_b200.dist import broadcast_comm_id
+
+        uid = broadcast_comm_id(rank)
+        got = [None] * world
+        dist.all_gather_object(got, uid)
+        status = None
+        if not torch.cuda.is_available():
+            try:
+                olap.Comm(uid, world, rank, 0)
+            except olap.OlapError as e:
+                status = e.status
+        q.put((rank, len(uid), all(g == got[0] for g in got), status))
+    except Exception as e:  # pragma: no cover - reported to the parent
+        q.put((rank, repr(e), False, None))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_two_rank_comm_id_bootstrap():
+    """dist.broadcast_comm_id: every rank receives rank 0's 128-byte communicator id."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_boot_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    out = [q.get(timeout=180) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+    import paper_conf_ipps_malikrse12_b200 as olap
+    for rank, n, same, status in out:
+        assert n == 128 and same, (rank, n, same)
+        if not torch.cuda.is_available():
+            assert status == olap.E_CUDA, status

@@ -159,3 +159,29 @@ def test_tile_path_full_range_int32_bit_exact():
     assert c.tile_stats()[3], "batch expected to take the tile path"
     ref = oracle.query(ext, boxes, ops, cells, nthreads=oracle.max_threads())
     compare(got, ref, ops, np.int32)
+
+
+def test_tile_workspace_failure_falls_back_to_items(monkeypatch):
+    """when the tile workspace cannot grow after a batch took the tile path, the cube
+    switches the tile path off and must clear the device's mode word, or every later batch would
+    skip the item path and finalize stale partials.  OLAP_TEST_TILE_WS_LIMIT makes the library's
+    allocation 'fail' above a query capacity."""
+    ext = (32, 16, 16, 16, 192)  # 96 MiB
+    seed = 0x5EED2200
+    c = olap.Cube(ext, np.float32)
+    c.fill(olap.GEN_UNIFORM, seed)
+    rng = np.random.default_rng(seed)
+    b1 = synth.fraction_boxes(ext, 512, rng, 1e-2, 0.5)
+    o1 = synth.ops_mix(512, rng)
+    c.query(b1, o1)
+    assert c.tile_stats()[3], "first batch should take the tile path"
+    monkeypatch.setenv("OLAP_TEST_TILE_WS_LIMIT", "1500")
+    b2 = synth.fraction_boxes(ext, 2000, rng, 1e-2, 0.5)
+    o2 = synth.ops_mix(2000, rng)
+    got = c.query(b2, o2)
+    en, _, _, used = c.tile_stats()
+    assert not en and not used
+    idx = rng.choice(2000, 120, replace=False)
+    ref = oracle.query(ext, b2[idx], o2[idx], dtype=np.float32, gen=oracle.GEN_UNIFORM, seed=seed,
+                       nthreads=oracle.max_threads())
+    compare(got[idx], ref, o2[idx], np.float32)
