@@ -138,8 +138,11 @@ int olap_cube_destroy(olap_cube* c);
  * [0, n_d)); d_values (DEVICE, nrows cells of the cube's dtype) or NULL to add 1 per
  * row (a fact-count cube).  Rows whose dim-0 id is not owned by this shard are skipped.
  * Cells are NOT cleared first (olap_cube_fill with params {0,...} or load zeros).
- * int32 adds are exact (atomic, order-free); float32 adds are atomic in arrival order.
- * Asynchronous on `stream`. */
+ * int32 adds are exact (wraparound, atomic, order-free).  float32 adds are deterministic:
+ * the rows are sorted by cell (stable radix sort), each cell's values are added in row
+ * order in fp64 and the cell becomes (float)((double)cell + sum), rounded once -- bit-equal
+ * to oracle_factbuild.  float32 calls take < 2^31 rows and stream-ordered scratch of ~24 B
+ * per row.  Asynchronous on `stream`. */
 int olap_cube_add_facts_device(olap_cube* c, int64_t nrows, const int32_t* d_ids, const void* d_values,
                                void* stream);
 

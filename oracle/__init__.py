@@ -10,6 +10,7 @@ Functions (all cite the passage they follow in oracle.cpp):
   query()      Eq. 1 / Eq. 3 / PAPER.md:25 — odometer sub-cube aggregation.
   Dict         PAPER.md:252-256 — one std::map dictionary per text column.
   factscan()   PAPER.md:206-208 — filtered aggregation over a fact table.
+  factbuild()  PAPER.md:101 — the cube built from fact rows (row loop; float: fp64 per cell, one rounding).
   rollup(), convert_range()  PAPER.md:103-136, Fig. 1, Eq. 1-2 — multi-resolution cube set.
   tablescan()  Eq. 11-12, PAPER.md:206-216 — the paper's GPU query Q_D over a column store.
   fill()       the counter-based cell generator (independent re-implementation).
@@ -30,7 +31,28 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "oracle.cpp")
-_LIB = os.path.join(_HERE, "liboracle.so")
+def _host_tag() -> str:
+    """The build is -march=native: one library per host CPU model + flags (the GPU box's host is
+    not this one, and an AVX-512 build must never load on a CPU without it)."""
+    import hashlib
+    sig = ""
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith(("model name", "flags")):
+                    sig += line
+                if line.strip() == "":
+                    break
+    except OSError:
+        pass
+    return hashlib.sha1(sig.encode()).hexdigest()[:10]
+
+
+_LIB = os.path.join(_HERE, f"liboracle-{_host_tag()}.so")
+# -O3 -march=native for the timed CPU baseline (SURVEY §8(d)); -ffp-contract=off keeps every
+# a*b+c a separate multiply and add (no FMA contraction), so the arithmetic is the source's,
+# bit for bit, whatever the host's ISA.  GCC never reassociates fp sums without -ffast-math.
+CFLAGS = ["-O3", "-march=native", "-ffp-contract=off", "-std=c++17", "-fopenmp", "-shared", "-fPIC"]
 
 INT32, FLOAT32 = 1, 2
 SUM, COUNT, MIN, MAX, AVG = 0, 1, 2, 3, 4
@@ -41,9 +63,9 @@ RESULT_DTYPE = np.dtype([("i", "<i8"), ("d", "<f8"), ("flags", "<u4"), ("pad", "
 
 
 def build(force: bool = False) -> str:
-    """Compile oracle.cpp -> liboracle.so (g++ -O2 -fopenmp)."""
+    """Compile oracle.cpp -> liboracle-<host>.so (g++ CFLAGS, OpenMP)."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
-        cmd = ["g++", "-O2", "-std=c++17", "-fopenmp", "-shared", "-fPIC", _SRC, "-o", _LIB + ".tmp"]
+        cmd = ["g++", *CFLAGS, _SRC, "-o", _LIB + ".tmp"]
         subprocess.check_call(cmd)
         os.replace(_LIB + ".tmp", _LIB)
     return _LIB
@@ -86,6 +108,9 @@ def lib():
         L.oracle_factscan.argtypes = [ctypes.c_int64, ctypes.c_int, ctypes.c_void_p, ctypes.c_int,
                                       ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p,
                                       ctypes.c_void_p, ctypes.c_void_p]
+        L.oracle_factbuild.restype = ctypes.c_int
+        L.oracle_factbuild.argtypes = [ctypes.c_int, c_i64p, ctypes.c_int, ctypes.c_int64, ctypes.c_void_p,
+                                       ctypes.c_void_p, ctypes.c_void_p]
         L.oracle_tablescan.restype = ctypes.c_int
         L.oracle_tablescan.argtypes = [ctypes.c_int64, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64,
                                        ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
@@ -216,6 +241,21 @@ class Dict:
             self.close()
         except Exception:
             pass
+
+
+def factbuild(extents, ids, values=None, cells=None, dtype=None):
+    """The cube built from fact rows (oracle_factbuild): ids (nd, nrows) int32,
+    values (nrows,) of the cube's dtype or None (+1 per row), added into `cells` (a copy of
+    the row-major host cube; zeros of `dtype` when None).  Returns the new cells."""
+    ext, ext_p = _i64(extents)
+    ids = np.ascontiguousarray(ids, dtype=np.int32)
+    nd, nrows = ids.shape
+    dt = np.dtype(dtype if dtype is not None else (values.dtype if values is not None else cells.dtype))
+    out = np.zeros(int(np.prod(ext)), dt) if cells is None else np.array(cells, dtype=dt).reshape(-1).copy()
+    v = None if values is None else np.ascontiguousarray(values, dtype=dt)
+    lib().oracle_factbuild(nd, ext_p, _dtype_code(dt), nrows, ids.ctypes.data, None if v is None else v.ctypes.data,
+                           out.ctypes.data)
+    return out
 
 
 def factscan(dims, data, ranges):

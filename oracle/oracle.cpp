@@ -24,6 +24,11 @@
  *                       (Fig. 1, Eq. 1-2): coarse cells
  *                       aggregate the fine cells mapping to them; a level-r range in
  *                       level-R members.
+ *   oracle_factbuild  — the cube built from fact rows ("the GPU performs ... building the
+ *                       cube from relational tables"): every row adds its
+ *                       measure (or 1) into the cell its dimension ids name.  Plain row
+ *                       loop; int32 wraps mod 2^32; float32 adds each cell's values in row
+ *                       order in double and rounds once into the cell (reading R27).
  *   oracle_factscan   — filtered aggregation over a fact table of translated
  *                       (integer) dimension columns and one data column  PAPER.md:206-208 (§III-E)
  *                       used as an independent path to the cube answer for SUM.
@@ -342,6 +347,47 @@ int oracle_factscan(int64_t nrows, int nd, const int32_t* dims, int dtype, const
         if (dtype == ORC_INT32) out_sum[q] = (int64_t)su;
         else std::memcpy(&out_sum[q], &sf, sizeof(double));
         out_count[q] = cnt;
+    }
+    return 0;
+}
+
+/*
+ * Cube build from fact rows (§III-F: the text columns are
+ * already integer ids).  ids[d*nrows + r] is row r's member id in dimension d; a row with
+ * an id outside [0, n_d) adds nothing.  vals (nrows cells of the cube's dtype) or NULL to
+ * add 1 per row.  cells: the row-major host cube, updated in place:
+ *   int32:   cell += v (mod 2^32) row by row;
+ *   float32: acc[cell] = sum of the cell's values in row order, in double; then
+ *            cell = (float)((double)cell + acc[cell]) once (reading R27).
+ */
+int oracle_factbuild(int nd, const int64_t* extents, int dtype, int64_t nrows, const int32_t* ids,
+                     const void* vals, void* cells) {
+    int64_t ncells = 1;
+    for (int d = 0; d < nd; ++d) ncells *= extents[d];
+    std::vector<double> acc(dtype == ORC_FLOAT32 ? ncells : 0, 0.0);
+    std::vector<char> touched(dtype == ORC_FLOAT32 ? ncells : 0, 0);
+    for (int64_t r = 0; r < nrows; ++r) {
+        int64_t idx = 0;
+        bool ok = true;
+        for (int d = 0; d < nd; ++d) {
+            const int64_t x = ids[(int64_t)d * nrows + r];
+            if (x < 0 || x >= extents[d]) ok = false;
+            idx = idx * extents[d] + x;
+        }
+        if (!ok) continue;
+        if (dtype == ORC_INT32) {
+            int32_t* c = static_cast<int32_t*>(cells);
+            const uint32_t v = vals ? (uint32_t)static_cast<const int32_t*>(vals)[r] : 1u;
+            c[idx] = (int32_t)((uint32_t)c[idx] + v);
+        } else {
+            acc[idx] += vals ? (double)static_cast<const float*>(vals)[r] : 1.0;
+            touched[idx] = 1;
+        }
+    }
+    if (dtype == ORC_FLOAT32) {
+        float* c = static_cast<float*>(cells);
+        for (int64_t i = 0; i < ncells; ++i)
+            if (touched[i]) c[i] = (float)((double)c[i] + acc[i]);
     }
     return 0;
 }

@@ -19,6 +19,7 @@
 #include <type_traits>
 #include <vector>
 
+#include <cub/device/device_radix_sort.cuh>
 #include <cub/device/device_scan.cuh>
 
 #include "common.cuh"
@@ -1710,6 +1711,40 @@ __global__ void add_facts_kernel(T* cells, Geo geo, int64_t nrows, const int32_t
     }
 }
 
+// Deterministic float32 build: the cell each row adds into (local storage index), or kNoCell
+// for rows another shard owns or with an id outside the cube; `row` = the row index (the sort's
+// payload, so equal cells keep row order: the radix sort is stable).
+constexpr unsigned long long kNoCell = ~0ull;
+__global__ void fact_cell_kernel(Geo geo, int64_t nrows, const int32_t* __restrict__ ids, unsigned long long* key,
+                                 int32_t* row) {
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < nrows; r += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t x0 = ids[r];
+        bool ok = x0 >= 0 && x0 < geo.n[0] && (geo.G == 1 || (x0 / geo.b) % geo.G == geo.g);
+        int64_t idx = ok ? shard_local_of(x0, geo.G, geo.b) * geo.stride[0] : 0;
+        for (int d = 1; d < geo.nd; ++d) {
+            const int64_t x = ids[(int64_t)d * nrows + r];
+            ok = ok && x >= 0 && x < geo.n[d];
+            idx += x * geo.stride[d];
+        }
+        key[r] = ok ? (unsigned long long)idx : kNoCell;
+        row[r] = (int32_t)r;
+    }
+}
+
+// One thread per run of equal cells in the sorted order (its head): the run's values are added in
+// row order in fp64 and the cell gets (float)((double)cell + sum) -- one rounding per cell, the
+// same sequence as oracle_factbuild, so the build is bit-exact and deterministic (no atomics).
+__global__ void fact_segsum_kernel(float* cells, int64_t nrows, const unsigned long long* __restrict__ key,
+                                   const int32_t* __restrict__ row, const float* __restrict__ vals) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nrows; i += (int64_t)gridDim.x * blockDim.x) {
+        const unsigned long long k = key[i];
+        if (k == kNoCell || (i > 0 && key[i - 1] == k)) continue;
+        double acc = 0.0;
+        for (int64_t j = i; j < nrows && key[j] == k; ++j) acc += vals ? (double)vals[row[j]] : 1.0;
+        cells[k] = (float)((double)cells[k] + acc);
+    }
+}
+
 }  // namespace olap
 
 // ====================================================================== host runtime
@@ -2609,14 +2644,40 @@ int olap_cube_add_facts_device(olap_cube* c, int64_t nrows, const int32_t* d_ids
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     OLAP_CUDA_TRY(cudaStreamWaitEvent(st, c->ws_done, 0));
     const int grid = (int)std::min<int64_t>((nrows + 255) / 256, (int64_t)c->num_sms * 16);
-    ++c->kernel_launches;
-    if (c->dtype == OLAP_INT32)
+    if (c->dtype == OLAP_INT32) {  // wraparound int32 adds are exact in any order: atomics
+        ++c->kernel_launches;
         add_facts_kernel<int32_t><<<grid, 256, 0, st>>>(static_cast<int32_t*>(c->d_cells), make_geo(c), nrows, d_ids,
                                                         static_cast<const int32_t*>(d_values));
-    else
-        add_facts_kernel<float><<<grid, 256, 0, st>>>(static_cast<float*>(c->d_cells), make_geo(c), nrows, d_ids,
-                                                      static_cast<const float*>(d_values));
-    OLAP_CUDA_TRY(cudaGetLastError());
+        OLAP_CUDA_TRY(cudaGetLastError());
+    } else {
+        // float32: sort the rows by cell (stable LSD radix sort, rows stay in order within a cell),
+        // then add each cell's values in row order in fp64 and round once (fact_segsum_kernel)
+        if (nrows > INT32_MAX) return set_error(OLAP_E_UNSUPPORTED, "a float32 build takes < 2^31 rows per call");
+        int bits = 1;
+        while (bits < 63 && (1ull << bits) <= (unsigned long long)c->local_cells + 1) ++bits;
+        unsigned long long *k0 = nullptr, *k1 = nullptr;
+        int32_t *r0 = nullptr, *r1 = nullptr;
+        void* tmp = nullptr;
+        size_t tb = 0;
+        OLAP_CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb, k0, k1, r0, r1, (int)nrows, 0, bits, st));
+        OLAP_CUDA_TRY(cudaMallocAsync(reinterpret_cast<void**>(&k0), sizeof(unsigned long long) * nrows, st));
+        OLAP_CUDA_TRY(cudaMallocAsync(reinterpret_cast<void**>(&k1), sizeof(unsigned long long) * nrows, st));
+        OLAP_CUDA_TRY(cudaMallocAsync(reinterpret_cast<void**>(&r0), sizeof(int32_t) * nrows, st));
+        OLAP_CUDA_TRY(cudaMallocAsync(reinterpret_cast<void**>(&r1), sizeof(int32_t) * nrows, st));
+        OLAP_CUDA_TRY(cudaMallocAsync(&tmp, std::max<size_t>(tb, 16), st));
+        fact_cell_kernel<<<grid, 256, 0, st>>>(make_geo(c), nrows, d_ids, k0, r0);
+        // keys < local_cells < 2^bits - 1: sorting the low `bits` bits puts kNoCell (all ones) last
+        OLAP_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, tb, k0, k1, r0, r1, (int)nrows, 0, bits, st));
+        fact_segsum_kernel<<<grid, 256, 0, st>>>(static_cast<float*>(c->d_cells), nrows, k1, r1,
+                                                 static_cast<const float*>(d_values));
+        OLAP_CUDA_TRY(cudaGetLastError());
+        cudaFreeAsync(tmp, st);
+        cudaFreeAsync(k0, st);
+        cudaFreeAsync(k1, st);
+        cudaFreeAsync(r0, st);
+        cudaFreeAsync(r1, st);
+        c->kernel_launches += 4;  // cells, radix sort (2 passes counted as one launch group), segment sums
+    }
     OLAP_CUDA_TRY(cudaEventRecord(c->ws_done, st));
     return OLAP_OK;
 }

@@ -194,6 +194,28 @@ def tpcds_facts(nrows: int, members: dict[str, list[str]], seed: int = SEED_BASE
     return cols, qty, cents
 
 
+def text_column(members: list[str], idx, chunk: int = 1 << 22):
+    """A fact table's raw text column: row r holds the string members[idx[r]] (length-delimited
+    bytes, the C-ABI key layout).  Returns (bytes uint8[...], offsets int64[n+1])."""
+    idx = np.asarray(idx)
+    enc = [m.encode() for m in members]
+    lens = np.array([len(e) for e in enc], np.int64)
+    width = max(int(lens.max()), 1)
+    table = np.zeros((len(enc), width), np.uint8)
+    for i, e in enumerate(enc):
+        table[i, :len(e)] = np.frombuffer(e, np.uint8)
+    rl = lens[idx]
+    offs = np.zeros(len(idx) + 1, np.int64)
+    np.cumsum(rl, out=offs[1:])
+    out = np.empty(max(int(offs[-1]), 1), np.uint8)
+    col = np.arange(width)
+    for a in range(0, len(idx), chunk):
+        b = min(len(idx), a + chunk)
+        rows = table[idx[a:b]]
+        out[offs[a]:offs[b]] = rows[col[None, :] < rl[a:b, None]]
+    return out, offs
+
+
 def tpcds_queries(nq: int, members: dict[str, list[str]], seed: int = SEED_BASE + 3):
     """Query strings: a d_date range (two dates), 0-3 equality predicates on store/class/state, op."""
     rng = np.random.default_rng(seed + 2)
