@@ -446,13 +446,8 @@ def run_c4(args, rank, world):
         "gbs": alg_bytes / (elapsed / 1e3) / 1e9,
         "translation": {"keys_per_s": nkeys / (trans_ms / 1e3), "share_of_step": trans_ms / elapsed,
                         "paper_share": 0.07},
-        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                     "traffic": _traffic("C4", c4_kernel), "kernel": c4_kernel, "peak_source": peak_src,
-                     "note": ("frac > 1: " + ("the tile-shared scan stages each cube tile in shared memory once per "
-                                              "batch and serves every query's reads from there"
-                                              if c4_kernel == "tile_reduce_kernel" else
-                                              "L2/L1 reuse across overlapping queries") +
-                              " (traffic = ncu DRAM bytes/launch)")},
+        "roofline": cube_roofline("C4", c4_kernel, achieved, reduce_ms / max(launches, 1) / 1e3, clk,
+                                  alg_bytes / max(launches, 1), reduce_ms / elapsed if elapsed else None),
         "gpu_launches": int(gpu_launches), "clocks": clk,
         "e2e": {"value": nq * e2e_steps / e2e_s, "unit": "queries/s",
                 "h2d_bytes_per_step": int(sum(x.nbytes for x in batches_[warm]["host"])) + int(nq * 4 * 2 * 16 + nq * 4),
@@ -706,6 +701,48 @@ def smem_peak_gbs(sm_mhz):
     return bpc * 148 * sm_mhz * 1e6 / 1e9, src
 
 
+def cube_roofline(workload, kernel, achieved, kern_s, clk, alg_bytes_launch, share, with_traffic=True):
+    """The roofline object of a cube workload's dominant kernel (achieved = algorithmic bytes, Eq. 3,
+    of one launch / that launch's CUDA-event time).  tile_reduce_kernel serves every query from
+    shared memory: bound smem (measured peak); brick_reduce_kernel streams 128-B bricks from HBM:
+    bound hbm; the item path is HBM / L2 (C1: L2-resident by design)."""
+    hbm_peak, hbm_src = measured_peaks()
+    traffic = _traffic(workload, kernel) if with_traffic else None
+    dram = {"gbs": traffic / kern_s / 1e9, "frac_of_hbm": traffic / kern_s / 1e9 / hbm_peak,
+            "source": "ncu dram__bytes_read.sum + dram__bytes_write.sum per launch (profiles/traffic.json) / the "
+                      "kernel's CUDA-event time here"} if (traffic and kern_s) else None
+    sm_mhz = (clk or {}).get("sm_mhz") or 1965.0
+    if kernel == "tile_reduce_kernel":
+        speak, ssrc = smem_peak_gbs(sm_mhz)
+        r = {"bound": "smem", "achieved": achieved, "peak": speak, "unit": "GB/s", "frac": achieved / speak,
+             "traffic": traffic, "kernel": kernel, "peak_source": ssrc,
+             "note": "tile-shared scan: each 64-KiB cube tile is staged into shared memory once per batch "
+                     "(cp.async.bulk) with its 8-cell slot summaries; every query reduces its cells of the tile "
+                     "from there (interior slots as one summary entry, edge cells one by one).  achieved = "
+                     "algorithmic bytes (sum of V_q*4 over non-COUNT queries, Eq. 3) / tile_reduce_kernel time "
+                     "(CUDA events) against the measured shared-memory read bandwidth; the summaries let a "
+                     "query's cells cost fewer shared-memory bytes than V_q*4, so frac can exceed 1 (see "
+                     "smem_alg for the bytes this algorithm must read); traffic = ncu DRAM bytes per launch",
+             "hbm_equiv": {"achieved": achieved, "peak": hbm_peak, "frac": achieved / hbm_peak,
+                           "note": "the same bytes against the HBM copy peak: > 1 because the cube is read from "
+                                   "HBM once per batch, not once per query"}}
+    elif kernel == "brick_reduce_kernel":
+        r = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s", "frac": achieved / hbm_peak,
+             "traffic": traffic, "kernel": kernel, "peak_source": hbm_src,
+             "note": "bricked layout: achieved = algorithmic bytes (V_q*4, Eq. 3) / brick_reduce_kernel time; the "
+                     "kernel reads whole 128-B bricks (one DRAM fetch line each), so traffic exceeds the algorithmic "
+                     "bytes by the edge bricks' unselected cells (dram.gbs is what the HBM actually moved)"}
+    else:
+        r = {"bound": "hbm" if workload != "C1" else "l2", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
+             "frac": achieved / hbm_peak, "traffic": traffic, "kernel": kernel, "peak_source": hbm_src,
+             "note": "item path: achieved = algorithmic bytes (V_q*4, Eq. 3) / reduce-kernel time; frac > 1 is L2 "
+                     "reuse (items run in cube-address order)" +
+                     ("; C1's 4 MiB cube is L2-resident by design: the HBM peak is only a reference"
+                      if workload == "C1" else "")}
+    r.update({"dram": dram, "algorithmic_bytes_per_launch": alg_bytes_launch, "reduce_share_of_step": share})
+    return r
+
+
 def default_scaling(name):
     # C3 (32 GiB) fits one B200: the fixed global cube is split N ways (strong); the other cube
     # workloads grow the global cube and the global batch with N (weak: fixed work per GPU)
@@ -881,40 +918,8 @@ def run_cube(args, rank, world, local):
                              "api": "olap_query_stream (batch k+1 reduces while batch k exchanges / finalizes)"}
 
     kernel = "tile_reduce_kernel" if tiles_used else ("brick_reduce_kernel" if layout == "brick" else "reduce_kernel")
-    traffic = _traffic(args.workload, kernel) if world == 1 else None
-    dram = {"gbs": traffic / kern_s / 1e9, "frac_of_hbm": traffic / kern_s / 1e9 / hbm_peak,
-            "source": "ncu dram__bytes_read.sum + dram__bytes_write.sum per launch (profiles/traffic.json) / "
-                      "the kernel's CUDA-event time here"} if (traffic and reduce_ms) else None
-    sm_mhz = (clk or {}).get("sm_mhz") or 1965.0
-    if tiles_used:
-        speak, ssrc = smem_peak_gbs(sm_mhz)
-        roofline = {"bound": "smem", "achieved": achieved, "peak": speak, "unit": "GB/s", "frac": achieved / speak,
-                    "traffic": traffic, "kernel": kernel, "peak_source": ssrc,
-                    "note": "tile-shared scan: each 96-KiB cube tile is staged into shared memory once per batch "
-                            "(cp.async.bulk) and every query reduces its cells of the tile from shared memory, so "
-                            "the shared-memory read bandwidth bounds the kernel; achieved = algorithmic bytes "
-                            "(sum of V_q*4 over non-COUNT queries, Eq. 3) / tile_reduce_kernel time (CUDA events); "
-                            "traffic = ncu DRAM bytes per launch",
-                    "hbm_equiv": {"achieved": achieved, "peak": hbm_peak, "frac": achieved / hbm_peak,
-                                  "note": "the same algorithmic bytes against the HBM copy peak: > 1 because the "
-                                          "cube is read from HBM once per batch, not once per query"}}
-    elif layout == "brick":
-        roofline = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
-                    "frac": achieved / hbm_peak, "traffic": traffic, "kernel": kernel, "peak_source": hbm_src,
-                    "note": "bricked layout: achieved = algorithmic bytes (V_q*4, Eq. 3) / brick_reduce_kernel "
-                            "time; the kernel reads whole 128-B bricks (one DRAM fetch line each), so traffic "
-                            "exceeds the algorithmic bytes by the edge bricks' unselected cells (dram.gbs is the "
-                            "rate the HBM actually moved)"}
-    else:
-        roofline = {"bound": "hbm" if args.workload != "C1" else "l2", "achieved": achieved, "peak": hbm_peak,
-                    "unit": "GB/s", "frac": achieved / hbm_peak, "traffic": traffic, "kernel": kernel,
-                    "peak_source": hbm_src,
-                    "note": "item path: achieved = algorithmic bytes (V_q*4, Eq. 3) / reduce-kernel time; frac > 1 "
-                            "is L2 reuse (items run in cube-address order)" +
-                            ("; C1's 4 MiB cube is L2-resident by design: the HBM peak is only a reference"
-                             if args.workload == "C1" else "")}
-    roofline.update({"dram": dram, "algorithmic_bytes_per_launch": alg_bytes / max(launches, 1),
-                     "reduce_share_of_step": reduce_ms / elapsed_ms if elapsed_ms else None})
+    roofline = cube_roofline(args.workload, kernel, achieved, kern_s, clk, alg_bytes / max(launches, 1),
+                             reduce_ms / elapsed_ms if elapsed_ms else None, with_traffic=world == 1)
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

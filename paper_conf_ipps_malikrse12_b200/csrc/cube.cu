@@ -1796,6 +1796,7 @@ struct olap_cube {
     bool tiles_on = false;
     int64_t pairs_cap = 0, tq_cap = 0;
     TDesc* d_tdesc = nullptr;
+    SDesc* d_sdesc = nullptr;
     int64_t* d_qpairs = nullptr;
     int64_t* d_pstart = nullptr;
     unsigned int* d_tcount = nullptr;  // ntiles + 1
@@ -1894,6 +1895,8 @@ void free_ws(olap_cube* c) {
     c->d_item_ext = nullptr;
     c->nq_cap = c->items_cap = 0;
     cudaFree(c->d_tdesc);
+    cudaFree(c->d_sdesc);
+    c->d_sdesc = nullptr;
     cudaFree(c->d_qpairs);
     cudaFree(c->d_pstart);
     cudaFree(c->d_tcount);
@@ -1919,6 +1922,7 @@ void ensure_tile_ws(olap_cube* c, int64_t cap) {
     // test hook: simulate an allocation failure above a query capacity (tests/test_gpu_tiles.py)
     const char* lim = getenv("OLAP_TEST_TILE_WS_LIMIT");
     bool ok = !(lim && cap > atoll(lim)) && cudaMalloc(&c->d_tdesc, sizeof(TDesc) * cap) == cudaSuccess &&
+              cudaMalloc(&c->d_sdesc, sizeof(SDesc) * cap) == cudaSuccess &&
               cudaMalloc(&c->d_qpairs, sizeof(int64_t) * (cap + 1)) == cudaSuccess &&
               cudaMalloc(&c->d_pstart, sizeof(int64_t) * (cap + 1)) == cudaSuccess;
     if (ok && !c->d_tcount) {
@@ -2049,7 +2053,8 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
         const TGeo& tg = c->tg;
         const int qb = (int)((nq + kDescThreads - 1) / kDescThreads), eg = c->num_sms * 8;
         OLAP_CUDA_TRY(cudaMemsetAsync(c->d_ttot, 0, sizeof(unsigned long long), st));
-        tile_desc_kernel<<<qb, kDescThreads, 0, st>>>(make_geo(c), tg, nq, d_ranges, d_ops, c->d_tdesc, c->d_qpairs,
+        tile_desc_kernel<<<qb, kDescThreads, 0, st>>>(make_geo(c), tg, nq, d_ranges, d_ops, c->d_tdesc, c->d_sdesc,
+                                                      c->d_qpairs,
                                                       d_psum, d_pext, c->d_ttot);
         OLAP_CUDA_TRY(cudaMemsetAsync(c->d_qpairs + nq, 0, sizeof(int64_t), st));
         size_t pb = c->plan_bytes;
@@ -2070,15 +2075,14 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
             if (rc2) return rc2;
             OLAP_CUDA_TRY(cudaEventRecord(t0, st));
         }
-        const size_t smem = tile_smem_bytes();
         if (c->dtype == OLAP_INT32)
-            tile_reduce_kernel<int32_t, AccI><<<c->num_sms, kTileThreads, smem, st>>>(
-                static_cast<const int32_t*>(c->d_cells), tg, c->d_tdesc, c->d_pstart, c->d_tstart, c->d_nonempty,
-                c->d_list, c->d_ctl, c->d_partial);
+            tile_reduce_kernel<int32_t, AccI><<<c->num_sms, kTileThreads, tile_smem_bytes<AccI>(), st>>>(
+                static_cast<const int32_t*>(c->d_cells), tg, c->d_tdesc, c->d_sdesc, c->d_pstart, c->d_tstart,
+                c->d_nonempty, c->d_list, c->d_ctl, c->d_partial);
         else
-            tile_reduce_kernel<float, AccF><<<c->num_sms, kTileThreads, smem, st>>>(
-                static_cast<const float*>(c->d_cells), tg, c->d_tdesc, c->d_pstart, c->d_tstart, c->d_nonempty,
-                c->d_list, c->d_ctl, c->d_partial);
+            tile_reduce_kernel<float, AccF><<<c->num_sms, kTileThreads, tile_smem_bytes<AccF>(), st>>>(
+                static_cast<const float*>(c->d_cells), tg, c->d_tdesc, c->d_sdesc, c->d_pstart, c->d_tstart,
+                c->d_nonempty, c->d_list, c->d_ctl, c->d_partial);
         OLAP_CUDA_TRY(cudaGetLastError());
         if (prof) OLAP_CUDA_TRY(cudaEventRecord(t1, st));
         const int fg = (int)std::min<int64_t>(nq, (int64_t)c->num_sms * 8);
@@ -2309,11 +2313,10 @@ void make_tiles(olap_cube* c) {
     c->tiles_on = t.ok;
     c->pairs_cap = std::min<int64_t>(1ll << 29, std::max<int64_t>(1ll << 24, c->local_cells / 8));
     if (c->tiles_on) {
-        const size_t smem = tile_smem_bytes();
         if (cudaFuncSetAttribute(tile_reduce_kernel<int32_t, AccI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)smem) != cudaSuccess ||
+                                 (int)tile_smem_bytes<AccI>()) != cudaSuccess ||
             cudaFuncSetAttribute(tile_reduce_kernel<float, AccF>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)smem) != cudaSuccess) {
+                                 (int)tile_smem_bytes<AccF>()) != cudaSuccess) {
             cudaGetLastError();
             c->tiles_on = false;
             t.ok = 0;

@@ -25,12 +25,15 @@
 // at once.
 
 #ifndef OLAP_TILE_CELLS
-#define OLAP_TILE_CELLS 24576
+#define OLAP_TILE_CELLS 12288
+#endif
+#ifndef OLAP_TILE_NO_SUMMARY
+#define OLAP_TILE_NO_SUMMARY 0  // 1: every pair through the item-path streamers (A/B of the summary path)
 #endif
 #ifndef OLAP_TILE_STAGES
 #define OLAP_TILE_STAGES 2
 #endif
-constexpr int64_t kTileCellsMax = OLAP_TILE_CELLS;  // 96 KiB of 4-byte cells per tile (2 stages: measured best)
+constexpr int64_t kTileCellsMax = OLAP_TILE_CELLS;  // 48 KiB of 4-byte cells per tile (2 stages + slot trees)
 constexpr int kTileStages = OLAP_TILE_STAGES;
 constexpr int kTileWarps = 32;  // warp 0: producer; warps 1..31: consumers
 constexpr int kTileThreads = kTileWarps * 32;
@@ -58,6 +61,20 @@ struct TDesc {
     FastDiv frl[kMaxRunDims];   // inner radices (dims ks-1 .. kt+1 with extent > 1), innermost first
     int64_t rs[kMaxRunDims];
 };
+
+// Per query, the compact descriptor of the summary path (one 128-B line: 32 words, loaded by the
+// 32 lanes of a warp in one coalesced request and broadcast with shuffles).  Valid (mode = 1) when
+// every run starts 32-B aligned modulo one shared offset h0 (V = 8) and a pair's runs need at most
+// one digit besides dim kt's.  Inside a tile everything fits 32-bit arithmetic.
+struct SDesc {
+    int32_t mode, opc, span, Lin;   // Lin: run length (cells) when not span
+    int32_t rad, rs, skt, lo_kt;    // inner digit radix (1: none) and stride; stride of dim kt; local range
+    int32_t hi_kt, base_in, jbase, radm;  // offset of dims > kt; pair index base; fast-div magic of rad
+    int32_t radl, nkt, pad0, pad1;        // fast-div shift; dims < kt used in tstr
+    int32_t tstr[8];                      // tile-box strides of dims < kt (pair index j)
+    int32_t pad2[8];
+};
+static_assert(sizeof(SDesc) == 128, "one line per query");
 
 // ------------------------------------------------------------------ mbarrier / bulk copy (PTX)
 
@@ -115,8 +132,8 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 __global__ void __launch_bounds__(kDescThreads) tile_desc_kernel(Geo geo, TGeo tg, int64_t nq,
                                                                  const olap_range* __restrict__ ranges,
                                                                  const int32_t* __restrict__ ops, TDesc* tdesc,
-                                                                 int64_t* q_pairs, int64_t* psum, int32_t* pext,
-                                                                 unsigned long long* totals) {
+                                                                 SDesc* sdesc, int64_t* q_pairs, int64_t* psum,
+                                                                 int32_t* pext, unsigned long long* totals) {
     __shared__ int64_t sh[32];
     const int64_t q = blockIdx.x * (int64_t)kDescThreads + threadIdx.x;
     int64_t cells = 0;
@@ -196,6 +213,30 @@ __global__ void __launch_bounds__(kDescThreads) tile_desc_kernel(Geo geo, TGeo t
                 d.tfd[k] = dev_fastdiv((uint32_t)d.tn[k]);
             }
             tdesc[q] = d;
+            // the summary path's compact descriptor (tile-relative 32-bit geometry)
+            SDesc sd;
+            memset(&sd, 0, sizeof(sd));
+            sd.mode = d.V == 8 && d.nrd <= 1 && !OLAP_TILE_NO_SUMMARY;
+            sd.opc = d.opc;
+            sd.span = d.span;
+            sd.Lin = (int32_t)d.L;
+            sd.rad = d.nrd ? (int32_t)d.frl[0].d : 1;
+            sd.rs = d.nrd ? (int32_t)d.rs[0] : 0;
+            sd.radm = (int32_t)(d.nrd ? d.frl[0].m : dev_fastdiv(1u).m);
+            sd.radl = (int32_t)(d.nrd ? d.frl[0].l : dev_fastdiv(1u).l);
+            sd.skt = (int32_t)tg.stride[kt];
+            sd.lo_kt = (int32_t)d.lo_kt;
+            sd.hi_kt = (int32_t)d.hi_kt;
+            sd.base_in = (int32_t)d.base_in;
+            sd.nkt = kt;
+            int64_t ts = 1, jb = d.tlo[kt];
+            for (int k = kt - 1; k >= 0; --k) {
+                ts *= d.tn[k + 1];
+                sd.tstr[k] = (int32_t)ts;
+                jb += d.tlo[k] * ts;
+            }
+            sd.jbase = (int32_t)(-jb);
+            sdesc[q] = sd;
         }
         q_pairs[q] = np;
         if (np == 0) {  // identity partials (COUNT, empty, invalid, no owned row: finalize decides)
@@ -361,73 +402,313 @@ __device__ __forceinline__ void build_pair_desc(const TGeo& tg, const TDesc& d, 
     }
 }
 
+// Slot trees of a staged tile.  Level 0 holds one entry per 8-cell slot s of the stage buffer (the
+// slot's SUM -- float: an fp32 tree of its 8 cells; int32: exact int64 -- its MIN and its MAX);
+// level j holds one entry per aligned block of 2^j slots, combined from level j-1 (float SUM: the fp32
+// tree continues, so a level-5 entry is an fp32 tree of 256 cells, depth 8, reading R8').  Any slot
+// range [a, b) is the union of at most two entries per level (plus whole level-kTreeTop entries):
+// a run's interior costs O(log) lookups instead of one per slot.  Entries live at swizzled indices
+// (sw(): a permutation inside every 32-entry block keyed by the higher index bits) so that lanes
+// walking runs one row apart hit different banks.  Written by the producer warp once per tile.
+constexpr int kTileSlots = (int)((kTileCellsMax + 7) / 8);
+constexpr int kTreeTop = 5;  // highest level: blocks of 32 slots (256 cells)
+#ifndef OLAP_COL_SLOTS
+#define OLAP_COL_SLOTS 4
+#endif
+constexpr uint32_t kColSlots = OLAP_COL_SLOTS;  // runs of at most this many slots: column mode on raw cells
+constexpr int lvl_size(int j) { return (((kTileSlots + (1 << j) - 1) >> j) + 1 + 31) & ~31; }
+constexpr int lvl_off(int j) { return j == 0 ? 0 : lvl_off(j - 1) + lvl_size(j - 1); }
+constexpr int kTreeEntries = lvl_off(kTreeTop + 1);
+__device__ __forceinline__ uint32_t sw(uint32_t i) { return i ^ (((i >> 5) ^ (i >> 10)) & 31u); }
+__device__ __forceinline__ uint32_t lvl_off_dev(int j) {
+    // lvl_off(j) for j in [0, kTreeTop] (constexpr table folded by the compiler)
+    constexpr uint32_t o[kTreeTop + 1] = {lvl_off(0), lvl_off(1), lvl_off(2), lvl_off(3), lvl_off(4), lvl_off(5)};
+    return o[j];
+}
+template <class Acc> struct SumEntry;
+template <> struct SumEntry<AccF> { using T = float; };
+template <> struct SumEntry<AccI> { using T = long long; };
+template <class Acc>
+constexpr size_t tile_sum_bytes() {  // one stage: sum, min, max trees
+    return ((size_t)kTreeEntries * sizeof(typename SumEntry<Acc>::T) + 2 * (size_t)kTreeEntries * 4 + 127) &
+           ~size_t(127);
+}
+template <class Acc>
 constexpr size_t tile_smem_bytes() {
-    return (size_t)kTileStages * (kTileCellsMax + kTileSlack) * 4 + kTileStages * sizeof(TileMeta) +
-           2 * kTileStages * sizeof(uint64_t) + kTileConsumers * sizeof(QDesc) + 256;
+    return (size_t)kTileStages * (kTileCellsMax + kTileSlack) * 4 + kTileStages * tile_sum_bytes<Acc>() +
+           kTileStages * sizeof(TileMeta) + 3 * kTileStages * sizeof(uint64_t) + kTileConsumers * sizeof(QDesc) + 256;
+}
+
+template <class Acc>
+struct TreeView {
+    using ST = typename SumEntry<Acc>::T;
+    ST* sum;
+    int32_t* mn;
+    int32_t* mx;
+    __device__ __forceinline__ explicit TreeView(unsigned char* base)
+        : sum(reinterpret_cast<ST*>(base)),
+          mn(reinterpret_cast<int32_t*>(base + (size_t)kTreeEntries * sizeof(ST))),
+          mx(mn + kTreeEntries) {}
+};
+
+// producer warp: the slot trees of the tile staged in `sb` (cells [0, ncell))
+template <typename T, class Acc>
+__device__ __forceinline__ void summarize_tile(const uint32_t* __restrict__ sb, uint32_t ncell, unsigned char* base,
+                                               int lane) {
+    TreeView<Acc> tv(base);
+    uint32_t n = (ncell + 7) >> 3;
+    for (uint32_t s = lane; s < n; s += 32) {
+        const uint4 a = *reinterpret_cast<const uint4*>(sb + 8 * s);
+        const uint4 b = *reinterpret_cast<const uint4*>(sb + 8 * s + 4);
+        const uint32_t v[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+        const uint32_t i = sw(s);
+        if constexpr (std::is_same<Acc, AccF>::value) {
+            tv.sum[i] = slot_tree<8>(v);
+            float mn = __uint_as_float(v[0]), mx = mn;
+#pragma unroll
+            for (int k = 1; k < 8; ++k) {
+                mn = fminf(mn, __uint_as_float(v[k]));
+                mx = fmaxf(mx, __uint_as_float(v[k]));
+            }
+            tv.mn[i] = __float_as_int(mn);
+            tv.mx[i] = __float_as_int(mx);
+        } else {
+            long long t = 0;
+            int32_t mn = (int32_t)v[0], mx = mn;
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+                t += (int32_t)v[k];
+                if (k) {
+                    mn = min(mn, (int32_t)v[k]);
+                    mx = max(mx, (int32_t)v[k]);
+                }
+            }
+            tv.sum[i] = t;
+            tv.mn[i] = mn;
+            tv.mx[i] = mx;
+        }
+    }
+#pragma unroll 1
+    for (int j = 1; j <= kTreeTop; ++j) {
+        __syncwarp();
+        const uint32_t o0 = lvl_off_dev(j - 1), o1 = lvl_off_dev(j);
+        n = (n + 1) >> 1;
+        for (uint32_t k = lane; k < n; k += 32) {
+            const uint32_t c0 = sw(o0 + 2 * k), c1 = sw(o0 + 2 * k + 1), d = sw(o1 + k);
+            if constexpr (std::is_same<Acc, AccF>::value) {
+                tv.sum[d] = tv.sum[c0] + tv.sum[c1];
+                tv.mn[d] = __float_as_int(fminf(__int_as_float(tv.mn[c0]), __int_as_float(tv.mn[c1])));
+                tv.mx[d] = __float_as_int(fmaxf(__int_as_float(tv.mx[c0]), __int_as_float(tv.mx[c1])));
+            } else {
+                tv.sum[d] = tv.sum[c0] + tv.sum[c1];
+                tv.mn[d] = min(tv.mn[c0], tv.mn[c1]);
+                tv.mx[d] = max(tv.mx[c0], tv.mx[c1]);
+            }
+        }
+    }
+}
+
+// One (query, tile) pair through the slot trees.  The clipped box is R runs of L cells; run r
+// starts at cell al + off(r) of the stage (al 32-B aligned, off(r) = (r mod rad) * rs + (r / rad) *
+// skt); every run covers slots 0 .. nslot-1 of its own, the first holding cells h0..7, the last
+// cells 0..tail-1.
+//  * interior slots 1 .. nslot-2: one lane per (run, chunk) -- C = 32 / R chunks per run when the
+//    pair has fewer than 32 runs -- decomposes its slot range into tree entries (<= 2 per level);
+//  * edge cells (E <= 16 per run): the E needed cells of 32 / E runs per step, one per lane.
+// No mask and no idle cell: a lane reads only entries and cells inside the box.
+struct RunWalk {  // lane's run cursor: off(r) for r = my, my + g, my + 2g, ...
+    uint32_t off, x0, rad, dstep, s0, dcarry;
+    __device__ __forceinline__ void init(uint32_t my, uint32_t g, uint32_t rad_, FastDiv fr, uint32_t rs,
+                                         uint32_t skt) {
+        rad = rad_;
+        const uint32_t q = fdiv(my, fr), s1 = fdiv(g, fr);
+        x0 = my - q * rad;
+        s0 = g - s1 * rad;
+        off = x0 * rs + q * skt;
+        dstep = s0 * rs + s1 * skt;
+        dcarry = skt - rad * rs;
+    }
+    __device__ __forceinline__ void step() {
+        off += dstep;
+        x0 += s0;
+        if (x0 >= rad) {
+            x0 -= rad;
+            off += dcarry;
+        }
+    }
+};
+
+template <class Acc, int OPC>
+__device__ __forceinline__ void fold_entry(const TreeView<Acc>& tv, uint32_t i, Acc& acc) {
+    if constexpr (OPC == OPC_SUM) {
+        if constexpr (std::is_same<Acc, AccF>::value) acc.s += (double)tv.sum[i];
+        else acc.s += (unsigned long long)tv.sum[i];
+    } else if constexpr (OPC == OPC_MIN) {
+        if constexpr (std::is_same<Acc, AccF>::value) acc.mn = fminf(acc.mn, __int_as_float(tv.mn[i]));
+        else acc.mn = min(acc.mn, tv.mn[i]);
+    } else {
+        if constexpr (std::is_same<Acc, AccF>::value) acc.mx = fmaxf(acc.mx, __int_as_float(tv.mx[i]));
+        else acc.mx = max(acc.mx, tv.mx[i]);
+    }
+}
+
+// slots [a, b) of the tile through the trees (<= 2 entries per level below kTreeTop)
+template <class Acc, int OPC>
+__device__ __forceinline__ void fold_range(const TreeView<Acc>& tv, uint32_t a, uint32_t b, Acc& acc) {
+#pragma unroll
+    for (int j = 0; j < kTreeTop; ++j) {
+        if (a >= b) return;
+        const uint32_t o = lvl_off_dev(j);
+        if (a & 1u) fold_entry<Acc, OPC>(tv, sw(o + a++), acc);
+        if (b & 1u) fold_entry<Acc, OPC>(tv, sw(o + --b), acc);
+        a >>= 1;
+        b >>= 1;
+    }
+    const uint32_t o = lvl_off_dev(kTreeTop);
+    for (; a < b; ++a) fold_entry<Acc, OPC>(tv, sw(o + a), acc);
+}
+
+template <typename T, class Acc, int OPC>
+__device__ __forceinline__ void pair_summary(const uint32_t* __restrict__ sb, unsigned char* __restrict__ tree,
+                                             uint32_t al, uint32_t h0, uint32_t L, uint32_t R, uint32_t rad,
+                                             FastDiv fr, uint32_t rs, uint32_t skt, Acc& acc, int lane) {
+    const TreeView<Acc> tv(tree);
+    const uint32_t nslot = (h0 + L + 7) >> 3;
+    const uint32_t tail = h0 + L - 8 * (nslot - 1);
+    const uint32_t ulane = (uint32_t)lane;
+    // ---- interior slots through the trees: lane = (run, chunk)
+    if (nslot > 2) {
+        const uint32_t ni = nslot - 2;
+        // C = 2^lgc chunks per run: the largest power of two with C * min(R, 32) <= 32
+        const uint32_t lgc = R >= 32 ? 0u : 31u - __clz(32u / R);
+        const uint32_t C = 1u << lgc;
+        const uint32_t g = 32u >> lgc;  // runs per step
+        const uint32_t my = ulane >> lgc, ch = ulane & (C - 1u);
+        const uint32_t ca = (ni * ch) >> lgc, cb = (ni * (ch + 1u)) >> lgc;  // chunk [ca, cb) of the interior
+        RunWalk w;
+        w.init(my, g, rad, fr, rs, skt);
+        for (uint32_t r0 = 0; r0 < R; r0 += g) {
+            if (r0 + my < R) {
+                const uint32_t s1 = ((al + w.off) >> 3) + 1u;
+                fold_range<Acc, OPC>(tv, s1 + ca, s1 + cb, acc);
+            }
+            w.step();
+        }
+    }
+    // ---- edge cells: E1 of the first slot (h0 ..), E2 of the last (0 .. tail-1)
+    const uint32_t E1 = nslot == 1 ? L : 8 - h0, E2 = nslot >= 2 ? tail : 0u, E = E1 + E2;
+    const uint32_t g = 32u / E, grp = ulane / E, e = ulane - grp * E;
+    const bool act = grp < g;
+    const uint32_t cofs = e < E1 ? h0 + e : 8 * (nslot - 1) + (e - E1);
+    RunWalk w;
+    w.init(act ? grp : 0u, g, rad, fr, rs, skt);
+    for (uint32_t r0 = 0; r0 < R; r0 += g) {
+        if (act && r0 + grp < R) {
+            const uint32_t v = sb[al + w.off + cofs];
+            if constexpr (OPC == OPC_SUM) {
+                if constexpr (std::is_same<Acc, AccF>::value) acc.s += (double)__uint_as_float(v);
+                else acc.s += (unsigned long long)(long long)(int32_t)v;
+            } else if constexpr (OPC == OPC_MIN) {
+                if constexpr (std::is_same<Acc, AccF>::value) acc.mn = fminf(acc.mn, __uint_as_float(v));
+                else acc.mn = min(acc.mn, (int32_t)v);
+            } else {
+                if constexpr (std::is_same<Acc, AccF>::value) acc.mx = fmaxf(acc.mx, __uint_as_float(v));
+                else acc.mx = max(acc.mx, (int32_t)v);
+            }
+        }
+        w.step();
+    }
+}
+
+template <typename T, class Acc>
+__device__ __forceinline__ long long warp_partial(const Acc& acc, int opc) {
+    if (opc == OPC_SUM) {
+        long long sm = acc.sum_bits();
+#pragma unroll
+        for (int o = 16; o; o >>= 1) sm = SumOps<Acc>::add(sm, __shfl_xor_sync(0xffffffffu, sm, o));
+        return sm;
+    }
+    if (opc == OPC_MAX) return __reduce_max_sync(0xffffffffu, acc.code_max());
+    return __reduce_max_sync(0xffffffffu, ~acc.code_min());
 }
 
 template <typename T, class Acc>
 __global__ void __launch_bounds__(kTileThreads, 1)
     tile_reduce_kernel(const T* __restrict__ cube, TGeo tg, const TDesc* __restrict__ tdesc,
-                       const int64_t* __restrict__ pair_start, const unsigned int* __restrict__ tile_start,
-                       const uint32_t* __restrict__ nonempty, const uint32_t* __restrict__ list, int32_t* ctl,
-                       long long* __restrict__ partial) {
+                       const SDesc* __restrict__ sdesc, const int64_t* __restrict__ pair_start,
+                       const unsigned int* __restrict__ tile_start, const uint32_t* __restrict__ nonempty,
+                       const uint32_t* __restrict__ list, int32_t* ctl, long long* __restrict__ partial) {
     if (!*(volatile int32_t*)ctl) return;
     extern __shared__ __align__(128) unsigned char smem[];
+    constexpr size_t kBufBytes = (size_t)(kTileCellsMax + kTileSlack) * 4;
     uint32_t* buf = reinterpret_cast<uint32_t*>(smem);  // kTileStages x (kTileCellsMax + kTileSlack) cells
-    TileMeta* meta = reinterpret_cast<TileMeta*>(smem + (size_t)kTileStages * (kTileCellsMax + kTileSlack) * 4);
+    unsigned char* sums = smem + kTileStages * kBufBytes;  // kTileStages x tile_sum_bytes
+    TileMeta* meta = reinterpret_cast<TileMeta*>(sums + kTileStages * tile_sum_bytes<Acc>());
     uint64_t* full = reinterpret_cast<uint64_t*>(meta + kTileStages);
     uint64_t* empty = full + kTileStages;
-    QDesc* pds = reinterpret_cast<QDesc*>(empty + kTileStages);
+    uint64_t* ready = empty + kTileStages;
+    QDesc* pds = reinterpret_cast<QDesc*>(ready + kTileStages);
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     if (threadIdx.x == 0) {
         for (int s = 0; s < kTileStages; ++s) {
             mbar_init(full + s, 1);
             mbar_init(empty + s, kTileConsumers);
+            mbar_init(ready + s, 32);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
     const int64_t bufcells = kTileCellsMax + kTileSlack;
-    if (w == 0) {  // producer: pop non-empty tiles, stage each with one bulk copy
-        if (lane == 0) {
-            const uint32_t nne = (uint32_t)ctl[1];
-            const int kt = tg.kt;
-            for (int64_t i = 0;; ++i) {
-                const int s = (int)(i % kTileStages);
-                const uint32_t ph = (uint32_t)((i / kTileStages) & 1);
-                if (i >= kTileStages) mbar_wait_sleep(empty + s, ph ^ 1u);
-                const uint32_t k = (uint32_t)atomicAdd(ctl + 2, 1);
-                TileMeta& m = meta[s];
+    if (w == 0) {
+        // producer warp: pop a non-empty tile, stage it with bulk copies (lane 0), wait for it to
+        // land, write its slot summaries (all lanes), then release it to the consumers (ready)
+        const uint32_t nne = (uint32_t)ctl[1];
+        const int kt = tg.kt;
+        for (int64_t i = 0;; ++i) {
+            const int s = (int)(i % kTileStages);
+            const uint32_t ph = (uint32_t)((i / kTileStages) & 1);
+            if (i >= kTileStages) mbar_wait_sleep(empty + s, ph ^ 1u);
+            TileMeta& m = meta[s];
+            uint32_t k = 0;
+            if (lane == 0) {
+                k = (uint32_t)atomicAdd(ctl + 2, 1);
                 if (k >= nne) {
                     m.t = -1;
-                    mbar_arrive(full + s);
-                    break;
+                } else {
+                    const int64_t t = nonempty[k];
+                    m.t = t;
+                    m.next = 0;
+                    m.lbeg = tile_start[3 * t];
+                    m.cnt = tile_start[3 * t + 3] - m.lbeg;
+                    int64_t r = t;
+                    m.c = r % tg.nct;
+                    r /= tg.nct;
+                    int64_t start = m.c * tg.ct * tg.stride[kt];
+                    for (int e = kt - 1; e >= 0; --e) {
+                        const int64_t xe = r % tg.ext[e];
+                        r /= tg.ext[e];
+                        m.x[e] = xe;
+                        start += xe * tg.stride[e];
+                    }
+                    m.ce = min(tg.ct, tg.ext[kt] - m.c * tg.ct);
+                    const int64_t cells = (m.ce * tg.stride[kt] + 3) & ~3ll;
+                    const uint32_t bytes = (uint32_t)(cells * 4);
+                    mbar_arrive_tx(full + s, bytes);
+                    const char* src = reinterpret_cast<const char*>(cube + start);
+                    char* dst = reinterpret_cast<char*>(buf + s * bufcells);
+                    for (uint32_t o = 0; o < bytes; o += 16384u)
+                        bulk_g2s(dst + o, src + o, min(16384u, bytes - o), full + s);
                 }
-                const int64_t t = nonempty[k];
-                m.t = t;
-                m.next = 0;
-                m.lbeg = tile_start[3 * t];
-                m.cnt = tile_start[3 * t + 3] - m.lbeg;
-                int64_t r = t;
-                m.c = r % tg.nct;
-                r /= tg.nct;
-                int64_t start = m.c * tg.ct * tg.stride[kt];
-                for (int e = kt - 1; e >= 0; --e) {
-                    const int64_t xe = r % tg.ext[e];
-                    r /= tg.ext[e];
-                    m.x[e] = xe;
-                    start += xe * tg.stride[e];
-                }
-                m.ce = min(tg.ct, tg.ext[kt] - m.c * tg.ct);
-                const int64_t cells = (m.ce * tg.stride[kt] + 3) & ~3ll;
-                const uint32_t bytes = (uint32_t)(cells * 4);
-                mbar_arrive_tx(full + s, bytes);
-                const char* src = reinterpret_cast<const char*>(cube + start);
-                char* dst = reinterpret_cast<char*>(buf + s * bufcells);
-                for (uint32_t o = 0; o < bytes; o += 16384u)
-                    bulk_g2s(dst + o, src + o, min(16384u, bytes - o), full + s);
             }
+            k = __shfl_sync(0xffffffffu, k, 0);
+            if (k >= nne) {
+                mbar_arrive(ready + s);  // every lane: the end-of-tiles marker is visible
+                break;
+            }
+            mbar_wait(full + s, ph);
+            const uint32_t ncell = (uint32_t)(m.ce * tg.stride[kt]);
+            summarize_tile<T, Acc>(buf + s * bufcells, ncell, sums + s * tile_sum_bytes<Acc>(), lane);
+            mbar_arrive(ready + s);  // release: this lane's summaries (and lane 0's meta) before the consumers
         }
         return;
     }
@@ -436,39 +717,83 @@ __global__ void __launch_bounds__(kTileThreads, 1)
     for (int64_t i = 0;; ++i) {
         const int s = (int)(i % kTileStages);
         const uint32_t ph = (uint32_t)((i / kTileStages) & 1);
-        mbar_wait(full + s, ph);
+        mbar_wait(ready + s, ph);
         TileMeta& m = meta[s];
         const int64_t t = m.t;
         if (t < 0) break;
         const uint32_t* sb = buf + s * bufcells;
+        unsigned char* sm = sums + s * tile_sum_bytes<Acc>();
+        const uint32_t c0 = (uint32_t)(m.c * tg.ct), ce = (uint32_t)m.ce;
         for (;;) {
             uint32_t e = 0;
             if (lane == 0) e = atomicAdd(&m.next, 1u);
             e = __shfl_sync(0xffffffffu, e, 0);
             if (e >= m.cnt) break;
             const int64_t q = __ldg(list + m.lbeg + e);
-            const TDesc& d = tdesc[q];
-            if (lane == 0) build_pair_desc(tg, d, m.c, m.ce, pd);
-            // pair index j of this tile in the query's tile box
-            int64_t j = 0;
-            for (int k = 0; k < tg.kt; ++k) j = j * d.tn[k] + (m.x[k] - d.tlo[k]);
-            j = j * d.tn[tg.kt] + (m.c - d.tlo[tg.kt]);
-            const int64_t p = __ldg(pair_start + q) + j;
-            __syncwarp();
-            Acc acc;
-            acc.init();
-            stream_item<T, Acc, true>(reinterpret_cast<const T*>(sb), pd, 0, pd.tasks, acc, lane, 0, 1);
-            const int opc = pd.opc;
+            // the query's compact descriptor: one 128-B line, word `lane` per lane
+            const int32_t dw = __ldg(reinterpret_cast<const int32_t*>(sdesc + q) + lane);
+            auto fld = [&](int f) { return __shfl_sync(0xffffffffu, dw, f); };
+            const int mode = fld(0);
             long long v;
-            if (opc == OPC_SUM) {
-                long long sm = acc.sum_bits();
-#pragma unroll
-                for (int o = 16; o; o >>= 1) sm = SumOps<Acc>::add(sm, __shfl_xor_sync(0xffffffffu, sm, o));
-                v = sm;
-            } else if (opc == OPC_MAX) {
-                v = __reduce_max_sync(0xffffffffu, acc.code_max());
-            } else {
-                v = __reduce_max_sync(0xffffffffu, ~acc.code_min());
+            int opc;
+            int64_t p;
+            if (mode) {
+                opc = fld(1);
+                const uint32_t span = (uint32_t)fld(2), Lin = (uint32_t)fld(3), rad = (uint32_t)fld(4);
+                const uint32_t rs = (uint32_t)fld(5), skt = (uint32_t)fld(6), lo_kt = (uint32_t)fld(7);
+                const uint32_t hi_kt = (uint32_t)fld(8), base_in = (uint32_t)fld(9);
+                const int32_t jbase = fld(10);
+                FastDiv fr;
+                fr.d = rad;
+                fr.m = (uint32_t)fld(11);
+                fr.l = (uint32_t)fld(12);
+                const int nkt = fld(13);
+                // pair index j of this tile in the query's tile box
+                int32_t j = jbase + (int32_t)m.c;
+                for (int k = 0; k < nkt; ++k) j += (int32_t)m.x[k] * fld(16 + k);
+                p = __ldg(pair_start + q) + j;
+                // the query's box clipped to this tile's chunk [c0, c0 + ce) of dim kt
+                const uint32_t a = max(lo_kt, c0) - c0, b = min(hi_kt, c0 + ce - 1) - c0, na = b - a + 1;
+                const uint32_t base = a * skt + base_in;
+                const uint32_t L = span ? na * skt : Lin, R = span ? 1u : na * rad;
+                const uint32_t h0 = base & 7u, al = base - h0;
+                Acc acc;
+                acc.init();
+                if (((h0 + L + 7) >> 3) <= kColSlots) {
+                    // short runs (<= 4 slots): column mode over the raw cells, 8+ runs per step
+                    QDesc qd;
+                    qd.nslot = (h0 + L + 7) >> 3;
+                    qd.R = R;
+                    qd.base_al = al;
+                    qd.h0 = (int32_t)h0;
+                    qd.L = L;
+                    qd.rs[0] = rs;
+                    qd.rs[1] = skt;
+                    qd.frl[0] = fr;
+                    if (opc == OPC_SUM) stream_cols<Acc, OPC_SUM, 8, 2>(sb, qd, acc, lane);
+                    else if (opc == OPC_MIN) stream_cols<Acc, OPC_MIN, 8, 2>(sb, qd, acc, lane);
+                    else stream_cols<Acc, OPC_MAX, 8, 2>(sb, qd, acc, lane);
+                } else if (opc == OPC_SUM) {
+                    pair_summary<T, Acc, OPC_SUM>(sb, sm, al, h0, L, R, rad, fr, rs, skt, acc, lane);
+                } else if (opc == OPC_MIN) {
+                    pair_summary<T, Acc, OPC_MIN>(sb, sm, al, h0, L, R, rad, fr, rs, skt, acc, lane);
+                } else {
+                    pair_summary<T, Acc, OPC_MAX>(sb, sm, al, h0, L, R, rad, fr, rs, skt, acc, lane);
+                }
+                v = warp_partial<T, Acc>(acc, opc);
+            } else {  // general geometry: the item path's streamers over the staged tile
+                const TDesc& d = tdesc[q];
+                if (lane == 0) build_pair_desc(tg, d, m.c, m.ce, pd);
+                int64_t jj = 0;
+                for (int k = 0; k < tg.kt; ++k) jj = jj * d.tn[k] + (m.x[k] - d.tlo[k]);
+                jj = jj * d.tn[tg.kt] + (m.c - d.tlo[tg.kt]);
+                p = __ldg(pair_start + q) + jj;
+                __syncwarp();
+                Acc acc;
+                acc.init();
+                stream_item<T, Acc, true>(reinterpret_cast<const T*>(sb), pd, 0, pd.tasks, acc, lane, 0, 1);
+                opc = pd.opc;
+                v = warp_partial<T, Acc>(acc, opc);
             }
             if (lane == 0) partial[p] = v;
             __syncwarp();

@@ -200,3 +200,17 @@ def test_brick_c5_small_boxes_equal_rowmajor():
     idx = np.random.default_rng(0).choice(len(boxes), 300, replace=False)
     ref = oracle.query(ext, boxes[idx], ops[idx], dtype=np.int32, gen=oracle.GEN_UNIFORM, seed=21)
     compare(got[idx], ref, ops[idx], np.int32)
+
+
+def test_brick_signed_noninteger_float():
+    """VERDICT r1 weak #2 on the bricked kernel (fp32 tree of one 8-cell brick row, then fp64):
+    mixed-sign, non-integer cells within 1e-6 * sum|x|; MIN / MAX / COUNT exact."""
+    from test_gpu_parity import compare_signed, signed_cells
+    ext = (6, 61, 203)
+    cells = signed_cells(int(np.prod(ext)), 0x5EED2400)
+    c = olap.Cube(ext, np.float32, layout=BRICK)
+    c.load(cells)
+    rng = np.random.default_rng(24)
+    boxes = _boxes(ext, rng, 200)
+    ops = synth.ops_uniform(len(boxes), rng)
+    compare_signed(c.query(boxes, ops), cells, ext, boxes, ops)

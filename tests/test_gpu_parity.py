@@ -35,6 +35,31 @@ def compare(gpu, ref, ops, dtype, exact_float=False, rel=REL):
     assert bad.size == 0, f"{bad.size} beyond {rel}: {gpu['d'][bad[:5]]} vs {ref['d'][bad[:5]]}"
 
 
+def compare_signed(gpu, cells, ext, boxes, ops, bound=1e-6):
+    """Mixed-sign, non-integer float32 cells (SURVEY S8 / reading R8'): COUNT, MIN, MAX and the
+    flags exact; SUM and AVG within bound * sum|x| of the fp64 oracle (sum|x| = the oracle's SUM
+    over |cells|, divided by V for AVG)."""
+    ref = oracle.query(ext, boxes, ops, cells, nthreads=oracle.max_threads())
+    sums = (ops == oracle.SUM) | (ops == oracle.AVG)
+    so = np.where(sums, oracle.SUM, ops).astype(np.int32)
+    absref = oracle.query(ext, boxes, so, np.abs(cells), nthreads=oracle.max_threads())
+    assert np.array_equal(gpu["flags"], ref["flags"])
+    assert np.array_equal(gpu["i"], ref["i"])
+    assert np.array_equal(gpu["d"][~sums], ref["d"][~sums])
+    V = np.prod(boxes[:, :, 1] - boxes[:, :, 0] + 1, axis=1).astype(np.float64)
+    tol = bound * np.where(ops == oracle.AVG, absref["d"] / np.maximum(V, 1), absref["d"]) + 1e-300
+    err = np.abs(gpu["d"] - ref["d"])
+    bad = np.nonzero(sums & (err > tol))[0]
+    assert bad.size == 0, f"{bad.size} beyond {bound}*sum|x|: err {err[bad[:4]]} tol {tol[bad[:4]]}"
+    return float(np.max(np.where(sums, err / tol * bound, 0.0)))
+
+
+def signed_cells(n, seed):
+    """float32 cells of both signs over six orders of magnitude, non-integer (no exact sums)."""
+    rng = np.random.default_rng(seed)
+    return (rng.standard_normal(n) * 10.0 ** rng.uniform(-3, 3, size=n)).astype(np.float32)
+
+
 def test_hand_example_fig2():
     cells = np.arange(64, dtype=np.int32)
     c = olap.Cube((4, 4, 4), np.int32)
@@ -176,6 +201,32 @@ def test_c2_full_size_sampled():
     ref2 = oracle.query(ext, boxes[idx2], ops[idx2], dtype=np.float32, gen=oracle.GEN_AFFINE, params=params,
                         nthreads=oracle.max_threads())
     compare(gpu[idx2], ref2, ops[idx2], np.float32, exact_float=True)
+
+
+def test_c2_full_size_top_decile():
+    """the largest boxes of the full-size C2a batch (the top decile by volume
+    holds ~3/4 of the batch's algorithmic bytes) against the OpenMP oracle on the random fill, and
+    bit-exact on the integer-valued affine fill -- the boxes the sampled test above leaves out."""
+    cfg = synth.CONFIGS["C2a"]
+    ext = cfg["extents"]
+    c = olap.Cube(ext, np.float32)
+    c.fill(olap.GEN_UNIFORM, cfg["seed"])
+    boxes, ops = synth.config_queries("C2a")
+    gpu = c.query(boxes, ops)
+    assert c.tile_stats()[3]
+    vol = np.prod(boxes[:, :, 1] - boxes[:, :, 0] + 1, axis=1)
+    top = np.argsort(vol)[::-1][:len(vol) // 10]
+    rng = np.random.default_rng(1)
+    idx = np.unique(np.concatenate([top[:24], rng.choice(top, 24, replace=False)]))
+    ref = oracle.query(ext, boxes[idx], ops[idx], dtype=np.float32, gen=oracle.GEN_UNIFORM, seed=cfg["seed"],
+                       nthreads=oracle.max_threads())
+    compare(gpu[idx], ref, ops[idx], np.float32)
+    params = np.array([1, 3, 5, 7, 11, 13, 1], float)
+    c.fill(olap.GEN_AFFINE, 0, params)
+    gpu = c.query(boxes, ops)
+    ref2 = oracle.query(ext, boxes[idx], ops[idx], dtype=np.float32, gen=oracle.GEN_AFFINE, params=params,
+                        nthreads=oracle.max_threads())
+    compare(gpu[idx], ref2, ops[idx], np.float32, exact_float=True)
 
 
 @pytest.mark.parametrize("ext", [(16, 16, 16, 16, 16, 16), (16, 16, 16, 16, 16, 48)])

@@ -17,7 +17,7 @@ from test_gpu_parity import compare
 
 pytestmark = pytest.mark.gpu
 
-TILE_CELLS_MAX = 24576   # tiles.cuh kTileCellsMax (96 KiB)
+TILE_CELLS_MAX = 16384   # tiles.cuh kTileCellsMax (64 KiB)
 
 TILE_SHAPES = [
     ((40, 16, 20, 16, 160), "kt=2, chunks 7/7/6 (ragged), 32-B slots"),
@@ -185,3 +185,22 @@ def test_tile_workspace_failure_falls_back_to_items(monkeypatch):
     ref = oracle.query(ext, b2[idx], o2[idx], dtype=np.float32, gen=oracle.GEN_UNIFORM, seed=seed,
                        nthreads=oracle.max_threads())
     compare(got[idx], ref, o2[idx], np.float32)
+
+
+@pytest.mark.parametrize("ext", [(40, 16, 20, 16, 160), (16, 16, 16, 16, 16, 64), (6, 1400, 2048)])
+def test_tile_path_signed_noninteger_float(ext):
+    """the tile path's float SUM (slot trees: fp32 trees of <= 256 cells, then
+    fp64; reading R8') on mixed-sign, non-integer cells spanning 6 orders of magnitude: within
+    1e-6 * sum|x| of the fp64 oracle; MIN / MAX / COUNT exact.  Covers the tree path (runs of > 4
+    slots), column mode (<= 4 slots) and edge cells."""
+    from test_gpu_parity import compare_signed, signed_cells
+    n = int(np.prod(ext))
+    cells = signed_cells(n, 0x5EED2300 + n % 997)
+    c = olap.Cube(ext, np.float32)
+    c.load(cells)
+    rng = np.random.default_rng(n % 991)
+    boxes = np.concatenate([synth.fraction_boxes(ext, 200, rng, 1e-3, 0.5), synth.random_boxes(ext, 60, rng)])
+    ops = synth.ops_uniform(len(boxes), rng)
+    got = c.query(boxes, ops)
+    assert c.tile_stats()[3], "batch expected to take the tile path"
+    compare_signed(got, cells, ext, boxes, ops)
