@@ -35,7 +35,10 @@
 #endif
 constexpr int64_t kTileCellsMax = OLAP_TILE_CELLS;  // 48 KiB of 4-byte cells per tile (2 stages + slot trees)
 constexpr int kTileStages = OLAP_TILE_STAGES;
-constexpr int kTileWarps = 32;  // warp 0: producer; warps 1..31: consumers
+#ifndef OLAP_TILE_WARPS
+#define OLAP_TILE_WARPS 32
+#endif
+constexpr int kTileWarps = OLAP_TILE_WARPS;  // warp 0: producer; warps 1..: consumers
 constexpr int kTileThreads = kTileWarps * 32;
 constexpr int kTileConsumers = kTileWarps - 1;
 constexpr int kTileSlack = 16;  // cells after each stage buffer: masked over-reads of a run's last slot
@@ -337,6 +340,7 @@ struct TileMeta {
     int64_t t;          // tile id, -1: no more tiles
     int64_t c, ce;      // chunk index along kt and its extent
     int64_t x[kMaxDims];  // tile coordinates of dims < kt
+    int32_t x32[kMaxDims];  // the same, 32-bit (summary path: pair index by one warp reduction)
     uint32_t lbeg, cnt;   // the tile's query list
     unsigned int next;    // next list entry to claim
 };
@@ -407,9 +411,9 @@ __device__ __forceinline__ void build_pair_desc(const TGeo& tg, const TDesc& d, 
 // level j holds one entry per aligned block of 2^j slots, combined from level j-1 (float SUM: the fp32
 // tree continues, so a level-5 entry is an fp32 tree of 256 cells, depth 8, reading R8').  Any slot
 // range [a, b) is the union of at most two entries per level (plus whole level-kTreeTop entries):
-// a run's interior costs O(log) lookups instead of one per slot.  Entries live at swizzled indices
-// (sw(): a permutation inside every 32-entry block keyed by the higher index bits) so that lanes
-// walking runs one row apart hit different banks.  Written by the producer warp once per tile.
+// a run's interior costs O(log) lookups instead of one per slot.  Entries live at padded indices
+// (sw(i) = i + i / 32: one spare entry per 32) so that lanes walking runs one 32-slot row apart hit
+// different banks at every level.  Written by the producer warp once per tile.
 constexpr int kTileSlots = (int)((kTileCellsMax + 7) / 8);
 constexpr int kTreeTop = 5;  // highest level: blocks of 32 slots (256 cells)
 #ifndef OLAP_COL_SLOTS
@@ -418,8 +422,8 @@ constexpr int kTreeTop = 5;  // highest level: blocks of 32 slots (256 cells)
 constexpr uint32_t kColSlots = OLAP_COL_SLOTS;  // runs of at most this many slots: column mode on raw cells
 constexpr int lvl_size(int j) { return (((kTileSlots + (1 << j) - 1) >> j) + 1 + 31) & ~31; }
 constexpr int lvl_off(int j) { return j == 0 ? 0 : lvl_off(j - 1) + lvl_size(j - 1); }
-constexpr int kTreeEntries = lvl_off(kTreeTop + 1);
-__device__ __forceinline__ uint32_t sw(uint32_t i) { return i ^ (((i >> 5) ^ (i >> 10)) & 31u); }
+constexpr int kTreeEntries = lvl_off(kTreeTop + 1) + lvl_off(kTreeTop + 1) / 32 + 1;  // padded
+__device__ __forceinline__ uint32_t sw(uint32_t i) { return i + (i >> 5); }
 __device__ __forceinline__ uint32_t lvl_off_dev(int j) {
     // lvl_off(j) for j in [0, kTreeTop] (constexpr table folded by the compiler)
     constexpr uint32_t o[kTreeTop + 1] = {lvl_off(0), lvl_off(1), lvl_off(2), lvl_off(3), lvl_off(4), lvl_off(5)};
@@ -516,6 +520,13 @@ __device__ __forceinline__ void summarize_tile(const uint32_t* __restrict__ sb, 
 //    pair has fewer than 32 runs -- decomposes its slot range into tree entries (<= 2 per level);
 //  * edge cells (E <= 16 per run): the E needed cells of 32 / E runs per step, one per lane.
 // No mask and no idle cell: a lane reads only entries and cells inside the box.
+// floor(n / d) for n < 32 (lanes) and 1 <= d <= 32 without a division: n * ceil(2^16 / d) >> 16
+// (exact: the rounding excess is below 31 / 2^16 < 1 / d)
+__constant__ uint32_t kSmallInv[33] = {0,    65536, 32768, 21846, 16384, 13108, 10923, 9363, 8192, 7282, 6554,
+                                        5958, 5462,  5042,  4682,  4370,  4096,  3856,  3641, 3450, 3277, 3121,
+                                        2979, 2850,  2731,  2622,  2521,  2428,  2341,  2260, 2185, 2115, 2048};
+__device__ __forceinline__ uint32_t small_div(uint32_t n, uint32_t d) { return (n * kSmallInv[d]) >> 16; }
+
 struct RunWalk {  // lane's run cursor: off(r) for r = my, my + g, my + 2g, ...
     uint32_t off, x0, rad, dstep, s0, dcarry;
     __device__ __forceinline__ void init(uint32_t my, uint32_t g, uint32_t rad_, FastDiv fr, uint32_t rs,
@@ -571,7 +582,7 @@ __device__ __forceinline__ void fold_range(const TreeView<Acc>& tv, uint32_t a, 
 template <typename T, class Acc, int OPC>
 __device__ __forceinline__ void pair_summary(const uint32_t* __restrict__ sb, unsigned char* __restrict__ tree,
                                              uint32_t al, uint32_t h0, uint32_t L, uint32_t R, uint32_t rad,
-                                             FastDiv fr, uint32_t rs, uint32_t skt, Acc& acc, int lane) {
+                                             uint32_t na, FastDiv fr, uint32_t rs, uint32_t skt, Acc& acc, int lane) {
     const TreeView<Acc> tv(tree);
     const uint32_t nslot = (h0 + L + 7) >> 3;
     const uint32_t tail = h0 + L - 8 * (nslot - 1);
@@ -580,7 +591,7 @@ __device__ __forceinline__ void pair_summary(const uint32_t* __restrict__ sb, un
     if (nslot > 2) {
         const uint32_t ni = nslot - 2;
         // C = 2^lgc chunks per run: the largest power of two with C * min(R, 32) <= 32
-        const uint32_t lgc = R >= 32 ? 0u : 31u - __clz(32u / R);
+        const uint32_t lgc = R >= 32 ? 0u : 31u - __clz(small_div(32u, R));
         const uint32_t C = 1u << lgc;
         const uint32_t g = 32u >> lgc;  // runs per step
         const uint32_t my = ulane >> lgc, ch = ulane & (C - 1u);
@@ -595,28 +606,35 @@ __device__ __forceinline__ void pair_summary(const uint32_t* __restrict__ sb, un
             w.step();
         }
     }
-    // ---- edge cells: E1 of the first slot (h0 ..), E2 of the last (0 .. tail-1)
+    // ---- edge cells: E1 of the first slot (h0 ..), E2 of the last (0 .. tail-1); lanes = (run, cell),
+    // g = 32 / E runs per step; kt rows outside, the inner digit inside (offsets advance by g * rs)
     const uint32_t E1 = nslot == 1 ? L : 8 - h0, E2 = nslot >= 2 ? tail : 0u, E = E1 + E2;
-    const uint32_t g = 32u / E, grp = ulane / E, e = ulane - grp * E;
-    const bool act = grp < g;
+    const uint32_t g = small_div(32u, E), grp = small_div(ulane, E), e = ulane - grp * E;
+    if (grp >= g) return;
     const uint32_t cofs = e < E1 ? h0 + e : 8 * (nslot - 1) + (e - E1);
-    RunWalk w;
-    w.init(act ? grp : 0u, g, rad, fr, rs, skt);
-    for (uint32_t r0 = 0; r0 < R; r0 += g) {
-        if (act && r0 + grp < R) {
-            const uint32_t v = sb[al + w.off + cofs];
-            if constexpr (OPC == OPC_SUM) {
-                if constexpr (std::is_same<Acc, AccF>::value) acc.s += (double)__uint_as_float(v);
-                else acc.s += (unsigned long long)(long long)(int32_t)v;
-            } else if constexpr (OPC == OPC_MIN) {
-                if constexpr (std::is_same<Acc, AccF>::value) acc.mn = fminf(acc.mn, __uint_as_float(v));
-                else acc.mn = min(acc.mn, (int32_t)v);
-            } else {
-                if constexpr (std::is_same<Acc, AccF>::value) acc.mx = fmaxf(acc.mx, __uint_as_float(v));
-                else acc.mx = max(acc.mx, (int32_t)v);
-            }
+    auto fold_cell = [&](uint32_t v) {
+        if constexpr (OPC == OPC_SUM) {
+            if constexpr (std::is_same<Acc, AccF>::value) acc.s += (double)__uint_as_float(v);
+            else acc.s += (unsigned long long)(long long)(int32_t)v;
+        } else if constexpr (OPC == OPC_MIN) {
+            if constexpr (std::is_same<Acc, AccF>::value) acc.mn = fminf(acc.mn, __uint_as_float(v));
+            else acc.mn = min(acc.mn, (int32_t)v);
+        } else {
+            if constexpr (std::is_same<Acc, AccF>::value) acc.mx = fmaxf(acc.mx, __uint_as_float(v));
+            else acc.mx = max(acc.mx, (int32_t)v);
         }
-        w.step();
+    };
+    const uint32_t step = g * rs;
+    const uint32_t* pk = sb + al + cofs + grp * rs;
+    for (uint32_t kr = 0; kr < na; ++kr, pk += skt) {
+        const uint32_t* pc = pk;
+        uint32_t ri = grp;
+        for (; ri + g < rad; ri += 2 * g, pc += 2 * step) {  // two runs per lane in flight
+            const uint32_t va = pc[0], vb = pc[step];
+            fold_cell(va);
+            fold_cell(vb);
+        }
+        if (ri < rad) fold_cell(pc[0]);
     }
 }
 
@@ -688,6 +706,7 @@ __global__ void __launch_bounds__(kTileThreads, 1)
                         const int64_t xe = r % tg.ext[e];
                         r /= tg.ext[e];
                         m.x[e] = xe;
+                        m.x32[e] = (int32_t)xe;
                         start += xe * tg.stride[e];
                     }
                     m.ce = min(tg.ct, tg.ext[kt] - m.c * tg.ct);
@@ -748,9 +767,9 @@ __global__ void __launch_bounds__(kTileThreads, 1)
                 fr.m = (uint32_t)fld(11);
                 fr.l = (uint32_t)fld(12);
                 const int nkt = fld(13);
-                // pair index j of this tile in the query's tile box
-                int32_t j = jbase + (int32_t)m.c;
-                for (int k = 0; k < nkt; ++k) j += (int32_t)m.x[k] * fld(16 + k);
+                // pair index j of this tile in the query's tile box: lane 16 + k holds tstr[k]
+                const int32_t tj = (lane >= 16 && lane < 16 + nkt) ? m.x32[lane - 16] * dw : 0;
+                const int32_t j = jbase + (int32_t)m.c + __reduce_add_sync(0xffffffffu, tj);
                 p = __ldg(pair_start + q) + j;
                 // the query's box clipped to this tile's chunk [c0, c0 + ce) of dim kt
                 const uint32_t a = max(lo_kt, c0) - c0, b = min(hi_kt, c0 + ce - 1) - c0, na = b - a + 1;
@@ -774,11 +793,11 @@ __global__ void __launch_bounds__(kTileThreads, 1)
                     else if (opc == OPC_MIN) stream_cols<Acc, OPC_MIN, 8, 2>(sb, qd, acc, lane);
                     else stream_cols<Acc, OPC_MAX, 8, 2>(sb, qd, acc, lane);
                 } else if (opc == OPC_SUM) {
-                    pair_summary<T, Acc, OPC_SUM>(sb, sm, al, h0, L, R, rad, fr, rs, skt, acc, lane);
+                    pair_summary<T, Acc, OPC_SUM>(sb, sm, al, h0, L, R, span ? 1u : rad, span ? 1u : na, fr, rs, skt, acc, lane);
                 } else if (opc == OPC_MIN) {
-                    pair_summary<T, Acc, OPC_MIN>(sb, sm, al, h0, L, R, rad, fr, rs, skt, acc, lane);
+                    pair_summary<T, Acc, OPC_MIN>(sb, sm, al, h0, L, R, span ? 1u : rad, span ? 1u : na, fr, rs, skt, acc, lane);
                 } else {
-                    pair_summary<T, Acc, OPC_MAX>(sb, sm, al, h0, L, R, rad, fr, rs, skt, acc, lane);
+                    pair_summary<T, Acc, OPC_MAX>(sb, sm, al, h0, L, R, span ? 1u : rad, span ? 1u : na, fr, rs, skt, acc, lane);
                 }
                 v = warp_partial<T, Acc>(acc, opc);
             } else {  // general geometry: the item path's streamers over the staged tile
