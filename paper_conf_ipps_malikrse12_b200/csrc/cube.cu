@@ -53,6 +53,7 @@ constexpr int64_t kWarpItemQueries = 8;
 constexpr int64_t kItemCells = 262144;      // minimum item: 1 MiB of 4-byte cells
 constexpr int64_t kMaxExtent = (1ll << 30); // per-dimension limit (32-bit digit arithmetic)
 constexpr int64_t kMaxCells = (1ll << 42);
+constexpr int64_t kGraphMaxQueries = 16384;  // olap_query_batch replays CUDA graphs up to this batch size
 
 // op class of a query: which accumulator the hot loop keeps (SUM and AVG share one)
 enum : int32_t { OPC_NONE = 0, OPC_SUM = 1, OPC_MIN = 2, OPC_MAX = 3 };
@@ -1831,6 +1832,18 @@ struct olap_cube {
     olap::Exec* exec = nullptr;
     olap_comm* comm = nullptr;
     bool multi() const { return !shards.empty(); }
+
+    // olap_query_batch on small batches replays a CUDA graph of its whole device sequence
+    // (copy-in, plan, reduce, finalize, copy-out), one per batch size, captured on first use;
+    // any workspace reallocation (ws_gen) invalidates them
+    struct BatchGraph {
+        int64_t nq = 0;
+        uint64_t gen = 0, last = 0;
+        int64_t kernels = 0, finals = 0;
+        cudaGraphExec_t exec = nullptr;
+    };
+    std::vector<BatchGraph> graphs;
+    uint64_t ws_gen = 0, graph_clock = 0;
 };
 
 namespace {
@@ -1949,6 +1962,7 @@ void ensure_tile_ws(olap_cube* c, int64_t cap) {
 int ensure_ws(olap_cube* c, int64_t nq) {
     if (nq <= c->nq_cap) return OLAP_OK;
     OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
+    ++c->ws_gen;
     free_ws(c);
     int64_t cap = std::max<int64_t>(nq, 1024);
     // item partial capacity: >= 2^20 and 4 per query, and for big cubes enough that items stay a
@@ -1981,6 +1995,7 @@ int ensure_ws(olap_cube* c, int64_t nq) {
 int ensure_stage(olap_cube* c, int64_t nq) {
     if (nq <= c->stage_cap) return OLAP_OK;
     OLAP_CUDA_TRY(cudaEventSynchronize(c->ws_done));
+    ++c->ws_gen;
     cudaFree(c->d_ranges);
     cudaFree(c->d_ops);
     cudaFree(c->d_results);
@@ -2703,6 +2718,8 @@ int olap_cube_destroy(olap_cube* c) {
         c->inner = nullptr;
         c->d_cells = nullptr;  // owned by the inner cube
     }
+    for (auto& g : c->graphs) cudaGraphExecDestroy(g.exec);
+    c->graphs.clear();
     free_ws(c);
     cudaFree(c->d_ranges);
     cudaFree(c->d_ops);
@@ -2744,14 +2761,69 @@ int olap_query_batch(olap_cube* c, int64_t nq, const olap_range* ranges, const i
     std::memcpy(hp, ranges, rbytes);
     std::memcpy(hp + rbytes, ops, obytes);
     cudaStream_t st = c->stream;
-    OLAP_CUDA_TRY(cudaMemcpyAsync(c->d_ranges, hp, rbytes, cudaMemcpyHostToDevice, st));
-    OLAP_CUDA_TRY(cudaMemcpyAsync(c->d_ops, hp + rbytes, obytes, cudaMemcpyHostToDevice, st));
-    rc = run_partials(c, nq, c->d_ranges, c->d_ops, c->d_psum, c->d_pext, st);
-    if (rc) return rc;
-    rc = launch_finalize(c->nd, c->n, c->dtype, nq, c->d_ranges, c->d_ops, c->d_psum, c->d_pext, c->d_results, st);
-    if (rc) return rc;
     char* hres = hp + rbytes + obytes;
-    OLAP_CUDA_TRY(cudaMemcpyAsync(hres, c->d_results, res_bytes, cudaMemcpyDeviceToHost, st));
+    auto enqueue = [&]() -> int {
+        OLAP_CUDA_TRY(cudaMemcpyAsync(c->d_ranges, hp, rbytes, cudaMemcpyHostToDevice, st));
+        OLAP_CUDA_TRY(cudaMemcpyAsync(c->d_ops, hp + rbytes, obytes, cudaMemcpyHostToDevice, st));
+        int r = run_partials(c, nq, c->d_ranges, c->d_ops, c->d_psum, c->d_pext, st);
+        if (r) return r;
+        r = launch_finalize(c->nd, c->n, c->dtype, nq, c->d_ranges, c->d_ops, c->d_psum, c->d_pext, c->d_results,
+                            st);
+        if (r) return r;
+        OLAP_CUDA_TRY(cudaMemcpyAsync(hres, c->d_results, res_bytes, cudaMemcpyDeviceToHost, st));
+        return OLAP_OK;
+    };
+    // small batches: replay the batch's CUDA graph (launch-bound otherwise); not while
+    // the reduce kernel is being timed (olap_cube_profile), whose events a graph does not record
+    const bool graph = nq <= kGraphMaxQueries && !c->prof && !(c->inner && c->inner->prof) && !getenv("OLAP_NO_GRAPHS");
+    if (graph) {
+        olap_cube* wc = c->inner ? c->inner : c;
+        rc = ensure_ws(wc, nq);  // the workspace cannot grow inside a capture
+        if (rc) return rc;
+        olap_cube::BatchGraph* g = nullptr;
+        for (auto& e : c->graphs)
+            if (e.nq == nq && e.gen == c->ws_gen + wc->ws_gen * 1000003ull) g = &e;
+        if (!g) {
+            if (c->graphs.size() >= 4) {  // evict the least recently used
+                auto lru = std::min_element(c->graphs.begin(), c->graphs.end(),
+                                            [](const auto& a, const auto& b) { return a.last < b.last; });
+                cudaGraphExecDestroy(lru->exec);
+                c->graphs.erase(lru);
+            }
+            const int64_t k0 = c->kernel_launches + (c->inner ? c->inner->kernel_launches : 0);
+            const int64_t f0 = g_finalize_launches.load();
+            OLAP_CUDA_TRY(cudaEventSynchronize(wc->ws_done));
+            OLAP_CUDA_TRY(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
+            rc = enqueue();
+            cudaGraph_t gr = nullptr;
+            const cudaError_t ce = cudaStreamEndCapture(st, &gr);
+            if (rc) {
+                if (gr) cudaGraphDestroy(gr);
+                return rc;
+            }
+            OLAP_CUDA_TRY(ce);
+            olap_cube::BatchGraph ng;
+            ng.nq = nq;
+            ng.gen = c->ws_gen + wc->ws_gen * 1000003ull;
+            ng.kernels = c->kernel_launches + (c->inner ? c->inner->kernel_launches : 0) - k0;
+            ng.finals = g_finalize_launches.load() - f0;
+            const cudaError_t ie = cudaGraphInstantiate(&ng.exec, gr, 0);
+            cudaGraphDestroy(gr);
+            OLAP_CUDA_TRY(ie);
+            c->graphs.push_back(ng);
+            g = &c->graphs.back();
+        } else {  // the kernels a replay launches count like launched ones (olap_cube_stats)
+            c->kernel_launches += g->kernels;
+            g_finalize_launches.fetch_add(g->finals);
+        }
+        g->last = ++c->graph_clock;
+        OLAP_CUDA_TRY(cudaStreamWaitEvent(st, wc->ws_done, 0));  // a device batch on another stream
+        OLAP_CUDA_TRY(cudaGraphLaunch(g->exec, st));
+        if (c->inner) OLAP_CUDA_TRY(cudaEventRecord(c->inner->ws_done, st));
+    } else {
+        rc = enqueue();
+        if (rc) return rc;
+    }
     OLAP_CUDA_TRY(cudaEventRecord(c->ws_done, st));
     OLAP_CUDA_TRY(cudaStreamSynchronize(st));
     std::memcpy(results, hres, res_bytes);

@@ -749,26 +749,29 @@ __global__ void __launch_bounds__(kTileThreads, 1)
             e = __shfl_sync(0xffffffffu, e, 0);
             if (e >= m.cnt) break;
             const int64_t q = __ldg(list + m.lbeg + e);
-            // the query's compact descriptor: one 128-B line, word `lane` per lane
-            const int32_t dw = __ldg(reinterpret_cast<const int32_t*>(sdesc + q) + lane);
-            auto fld = [&](int f) { return __shfl_sync(0xffffffffu, dw, f); };
-            const int mode = fld(0);
+            // the query's compact descriptor: words 0-15 by four uniform (broadcast) 16-B loads, the
+            // tile-box strides (words 16..) by lane k < nkt
+            const int4* sd4 = reinterpret_cast<const int4*>(sdesc + q);
+            const int4 w0 = __ldg(sd4);
+            const int mode = w0.x;
             long long v;
             int opc;
             int64_t p;
             if (mode) {
-                opc = fld(1);
-                const uint32_t span = (uint32_t)fld(2), Lin = (uint32_t)fld(3), rad = (uint32_t)fld(4);
-                const uint32_t rs = (uint32_t)fld(5), skt = (uint32_t)fld(6), lo_kt = (uint32_t)fld(7);
-                const uint32_t hi_kt = (uint32_t)fld(8), base_in = (uint32_t)fld(9);
-                const int32_t jbase = fld(10);
+                const int4 w1 = __ldg(sd4 + 1), w2 = __ldg(sd4 + 2), w3 = __ldg(sd4 + 3);
+                opc = w0.y;
+                const uint32_t span = (uint32_t)w0.z, Lin = (uint32_t)w0.w, rad = (uint32_t)w1.x;
+                const uint32_t rs = (uint32_t)w1.y, skt = (uint32_t)w1.z, lo_kt = (uint32_t)w1.w;
+                const uint32_t hi_kt = (uint32_t)w2.x, base_in = (uint32_t)w2.y;
+                const int32_t jbase = w2.z;
                 FastDiv fr;
                 fr.d = rad;
-                fr.m = (uint32_t)fld(11);
-                fr.l = (uint32_t)fld(12);
-                const int nkt = fld(13);
-                // pair index j of this tile in the query's tile box: lane 16 + k holds tstr[k]
-                const int32_t tj = (lane >= 16 && lane < 16 + nkt) ? m.x32[lane - 16] * dw : 0;
+                fr.m = (uint32_t)w2.w;
+                fr.l = (uint32_t)w3.x;
+                const int nkt = w3.y;
+                // pair index j of this tile in the query's tile box (one warp reduction)
+                const int32_t tj = lane < nkt ? m.x32[lane] * __ldg(reinterpret_cast<const int32_t*>(sdesc + q) + 16 + lane)
+                                              : 0;
                 const int32_t j = jbase + (int32_t)m.c + __reduce_add_sync(0xffffffffu, tj);
                 p = __ldg(pair_start + q) + j;
                 // the query's box clipped to this tile's chunk [c0, c0 + ce) of dim kt

@@ -919,3 +919,37 @@ def test_warp_items_large_batches(ext, dtype):
                        nthreads=oracle.max_threads())
     compare(got[idx], ref, ops[idx], dtype)
     assert np.array_equal(c.query(boxes, ops), got)
+
+
+def test_host_batches_replay_cuda_graphs(monkeypatch):
+    """olap_query_batch replays a per-batch-size CUDA graph for batches of
+    <= 16,384 queries.  Replays equal the direct path bit for bit, across sizes (LRU of four
+    graphs), after a workspace growth (graphs invalidated), on a bricked cube, and interleaved
+    with device batches on another stream."""
+    for ext, layout in (((32, 32, 32, 32), olap.LAYOUT_ROWMAJOR), ((16, 96, 136), olap.LAYOUT_BRICK),
+                        ((64, 16, 16, 16, 192), olap.LAYOUT_ROWMAJOR)):
+        c = olap.Cube(ext, np.float32, layout=layout)
+        c.fill(olap.GEN_UNIFORM, 9)
+        rng = np.random.default_rng(9)
+        sizes = [1000, 17, 1000, 3000, 5, 999, 1000, 20000, 1000]
+        batches = {n: (synth.fraction_boxes(ext, n, rng, 1e-4), synth.ops_uniform(n, rng)) for n in set(sizes)}
+        monkeypatch.setenv("OLAP_NO_GRAPHS", "1")
+        ref = {n: c.query(*batches[n]) for n in batches}
+        monkeypatch.delenv("OLAP_NO_GRAPHS")
+        k0 = c.stats()[0]
+        for i, n in enumerate(sizes):
+            got = c.query(*batches[n])
+            assert got.tobytes() == ref[n].tobytes(), (ext, n, i)
+            if i == 4:  # a device batch on another stream between host batches
+                b, o = batches[1000]
+                res = torch.empty(1000 * 24, dtype=torch.uint8, device="cuda")
+                s = torch.cuda.Stream()
+                c.query_device(torch.from_numpy(b).cuda(), torch.from_numpy(o).cuda(), res, stream=s)
+                s.synchronize()
+                assert res.cpu().numpy().tobytes() == ref[1000].tobytes()
+        assert c.stats()[0] > k0  # replayed kernels are counted
+        idx = np.arange(0, 1000, 37)
+        b, o = batches[1000]
+        want = oracle.query(ext, b[idx], o[idx], dtype=np.float32, gen=oracle.GEN_UNIFORM, seed=9,
+                            nthreads=oracle.max_threads())
+        compare(ref[1000][idx], want, o[idx], np.float32)
