@@ -92,33 +92,39 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* b) {
 __device__ __forceinline__ void mbar_arrive_tx(uint64_t* b, uint32_t bytes) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
 }
-// producer side: back off between probes (a single lane; keeps the spin off the issue slots)
-__device__ __forceinline__ void mbar_wait_sleep(uint64_t* b, uint32_t parity) {
+// A wait that never completes is a bug (a phase nobody will reach); rather than hang the GPU, a
+// waiter that has spun for ~8 s traps the kernel (cudaErrorLaunchFailure: an error, not a hang).
+constexpr long long kWaitTrapCycles = 16ll * 1000 * 1000 * 1000;
+__device__ __forceinline__ bool mbar_try(uint64_t* b, uint32_t parity) {
     uint32_t ok = 0;
-    for (;;) {
-        asm volatile(
-            "{\n"
-            ".reg .pred p;\n"
-            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
-            "selp.u32 %0, 1, 0, p;\n"
-            "}\n"
-            : "=r"(ok)
-            : "r"(smem_u32(b)), "r"(parity)
-            : "memory");
-        if (ok) return;
-        __nanosleep(256);
-    }
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
     asm volatile(
         "{\n"
         ".reg .pred p;\n"
-        "OLAP_WAIT_%=:\n"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-        "@!p bra OLAP_WAIT_%=;\n"
-        "}\n" ::"r"(smem_u32(b)),
-        "r"(parity)
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+        "selp.u32 %0, 1, 0, p;\n"
+        "}\n"
+        : "=r"(ok)
+        : "r"(smem_u32(b)), "r"(parity)
         : "memory");
+    return ok != 0;
+}
+// producer side: back off between probes (keeps the spin off the issue slots)
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* b, uint32_t parity) {
+    if (mbar_try(b, parity)) return;
+    const long long t0 = clock64();
+    for (;;) {
+        if (mbar_try(b, parity)) return;
+        __nanosleep(256);
+        if (clock64() - t0 > kWaitTrapCycles) __trap();
+    }
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+    if (mbar_try(b, parity)) return;  // the common case: one probe
+    const long long t0 = clock64();
+    for (uint32_t i = 1;; ++i) {
+        if (mbar_try(b, parity)) return;
+        if ((i & 1023u) == 0 && clock64() - t0 > kWaitTrapCycles) __trap();
+    }
 }
 // global -> shared bulk copy completing on mbarrier b (bytes: multiple of 16, both ends 16-B aligned)
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* b) {
@@ -739,7 +745,12 @@ __global__ void __launch_bounds__(kTileThreads, 1)
         mbar_wait(ready + s, ph);
         TileMeta& m = meta[s];
         const int64_t t = m.t;
-        if (t < 0) break;
+        if (t < 0) break;  // the end-of-tiles marker has no copy behind it: never wait on full[s] for it
+        // also observe the bulk copy's own completion (already complete: the producer waited for it
+        // before summarising) -- a direct acquire of the async-proxy writes, not only through ready[s]
+#ifndef OLAP_NO_FULL_WAIT
+        mbar_wait(full + s, ph);
+#endif
         const uint32_t* sb = buf + s * bufcells;
         unsigned char* sm = sums + s * tile_sum_bytes<Acc>();
         const uint32_t c0 = (uint32_t)(m.c * tg.ct), ce = (uint32_t)m.ce;

@@ -8,9 +8,9 @@ for rep in 1 2; do
     name=${v%%=*}; path=${v#*=}
     for w in ${WORKLOADS:-C2a}; do
       if [ "$path" = "default" ]; then
-        timeout 600 python bench.py --workload $w --no-cpu-baseline --e2e-steps 0 > gpurun_out/ab_${TAG}_${name}_${w}_$rep.log 2>&1
+        timeout ${BENCH_TIMEOUT:-240} python bench.py --workload $w --no-cpu-baseline --e2e-steps 0 > gpurun_out/ab_${TAG}_${name}_${w}_$rep.log 2>&1
       else
-        OLAP_LIB=$path timeout 600 python bench.py --workload $w --no-cpu-baseline --e2e-steps 0 > gpurun_out/ab_${TAG}_${name}_${w}_$rep.log 2>&1
+        OLAP_LIB=$path timeout ${BENCH_TIMEOUT:-240} python bench.py --workload $w --no-cpu-baseline --e2e-steps 0 > gpurun_out/ab_${TAG}_${name}_${w}_$rep.log 2>&1
       fi
       tail -1 gpurun_out/ab_${TAG}_${name}_${w}_$rep.log > gpurun_out/ab_${TAG}_${name}_${w}_$rep.jsonl
     done
