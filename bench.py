@@ -536,6 +536,7 @@ def run_table(args, rank, world):
     for k in range(warm):
         table.query_device(nq, *devb[k], res, stream=stream)
     stream.synchronize()
+    table.profile(True)
     clocks = Clocks(0)
     clocks.mark(True)
     e0 = torch.cuda.Event(enable_timing=True)
@@ -547,6 +548,8 @@ def run_table(args, rank, world):
     e1.synchronize()
     clocks.mark(False)
     elapsed = e0.elapsed_time(e1)
+    scan_ms, scan_n = table.profile_read()
+    table.profile(False)
     clk = clocks.stop()
     # Eq. 12 cost model of the paper's design: each query reads its C_QD columns whole
     paper_bytes = sum(evals[warm:]) * nrows * 4
@@ -574,14 +577,16 @@ def run_table(args, rank, world):
                    "batch": nq, "queries": "d_date range + 0-3 equality predicates, op on quantity or net_paid",
                    "l2": "columns (1.6 GB) > L2; staged once per batch"},
         "paper_eq12_gbs": paper_bytes / (elapsed / 1e3) / 1e9,
-        "roofline": {"bound": "hbm", "achieved": col_bytes / (elapsed / steps / 1e3) / 1e9, "peak": peak,
-                     "unit": "GB/s", "frac": col_bytes / (elapsed / steps / 1e3) / 1e9 / peak,
-                     "traffic": _traffic("T", "table_scan_kernel"), "kernel": "table_scan_kernel",
-                     "peak_source": peak_src,
-                     "note": "algorithmic bytes = the referenced columns read once per batch (the shared scan); "
-                             "the kernel is not HBM-bound but issue-bound: ncu issue-slot utilisation 71% "
-                             "(profiles/ncu_table_scan_r01s4e.txt), so frac is far below 1 by design; "
-                             "effective_evals restates the paper's dense Eq. 12 work per second"},
+        "roofline": dict(issue_roofline("T", "table_scan_kernel", scan_ms / max(scan_n, 1) / 1e3,
+                                        (clk or {}).get("sm_mhz") or 1965.0),
+                         traffic=_traffic("T", "table_scan_kernel"),
+                         scan_share_of_step=scan_ms / elapsed if elapsed else None,
+                         note="the shared scan reads every referenced column once per batch (hbm below) and then "
+                              "evaluates every (query, row) from shared memory: instruction issue binds it (ncu); "
+                              "kernel time from CUDA events around table_scan_kernel (olap_table_profile)",
+                         hbm={"achieved": col_bytes / (elapsed / steps / 1e3) / 1e9, "peak": peak, "unit": "GB/s",
+                              "frac": col_bytes / (elapsed / steps / 1e3) / 1e9 / peak, "peak_source": peak_src,
+                              "note": "algorithmic bytes = the referenced columns, read once per batch"}),
         "effective_evals": {"value": achieved, "unit": "(query,row,column) evaluations/s (Eq. 12, dense)",
                             "frac_of_issue_bound": achieved / peak_evals,
                             "issue_bound": "148 SMs x 4 x 32 lanes x 1.965 GHz / 3 instr per evaluation; the "
@@ -701,6 +706,21 @@ def smem_peak_gbs(sm_mhz):
     return bpc * 148 * sm_mhz * 1e6 / 1e9, src
 
 
+def issue_roofline(workload, kernel, kern_s, sm_mhz):
+    """Instruction-issue roofline of an issue-bound kernel: warp instructions per launch (ncu, the same
+    bench batch, profiles/traffic.json '<kernel>:inst') / the launch's CUDA-event time, against
+    148 SMs x 4 SM sub-partitions x 1 warp instruction per clock at the measured SM clock."""
+    inst = _traffic(workload, kernel + ":inst")
+    peak = 148 * 4 * sm_mhz * 1e6
+    ach = inst / kern_s if (inst and kern_s) else None
+    return {"bound": "issue", "achieved": ach, "peak": peak, "unit": "warp-instr/s",
+            "frac": (ach / peak) if ach else None, "kernel": kernel,
+            "inst_per_launch": inst,
+            "peak_source": f"derived: 148 SMs x 4 schedulers x 1 warp instruction/clk x {sm_mhz:.0f} MHz (median SM "
+                           "clock of the timed region; B200_PROFILING.md / Blackwell guide: one issue per SMSP per "
+                           "clock)"}
+
+
 def cube_roofline(workload, kernel, achieved, kern_s, clk, alg_bytes_launch, share, with_traffic=True):
     """The roofline object of a cube workload's dominant kernel (achieved = algorithmic bytes, Eq. 3,
     of one launch / that launch's CUDA-event time).  tile_reduce_kernel serves every query from
@@ -713,19 +733,19 @@ def cube_roofline(workload, kernel, achieved, kern_s, clk, alg_bytes_launch, sha
                       "kernel's CUDA-event time here"} if (traffic and kern_s) else None
     sm_mhz = (clk or {}).get("sm_mhz") or 1965.0
     if kernel == "tile_reduce_kernel":
+        r = issue_roofline(workload, kernel, kern_s, sm_mhz)
         speak, ssrc = smem_peak_gbs(sm_mhz)
-        r = {"bound": "smem", "achieved": achieved, "peak": speak, "unit": "GB/s", "frac": achieved / speak,
-             "traffic": traffic, "kernel": kernel, "peak_source": ssrc,
-             "note": "tile-shared scan: each 64-KiB cube tile is staged into shared memory once per batch "
-                     "(cp.async.bulk) with its 8-cell slot summaries; every query reduces its cells of the tile "
-                     "from there (interior slots as one summary entry, edge cells one by one).  achieved = "
-                     "algorithmic bytes (sum of V_q*4 over non-COUNT queries, Eq. 3) / tile_reduce_kernel time "
-                     "(CUDA events) against the measured shared-memory read bandwidth; the summaries let a "
-                     "query's cells cost fewer shared-memory bytes than V_q*4, so frac can exceed 1 (see "
-                     "smem_alg for the bytes this algorithm must read); traffic = ncu DRAM bytes per launch",
-             "hbm_equiv": {"achieved": achieved, "peak": hbm_peak, "frac": achieved / hbm_peak,
-                           "note": "the same bytes against the HBM copy peak: > 1 because the cube is read from "
-                                   "HBM once per batch, not once per query"}}
+        r["note"] = ("tile-shared scan: each 48-KiB cube tile is staged into shared memory once per batch "
+                     "(cp.async.bulk) with its slot trees; every query reduces its cells of the tile from there (run "
+                     "interiors as O(log) tree entries, edge cells one by one), so neither HBM nor shared-memory "
+                     "bandwidth binds it: ncu shows instruction issue as the limit (profiles/).  achieved = the "
+                     "launch's warp instructions (ncu smsp__inst_executed.sum of the same batch, profiles/"
+                     "traffic.json) / its CUDA-event time here; peak = 148 SMs x 4 schedulers x 1 warp-instr/clk")
+        r["eq3"] = {"achieved": achieved, "unit": "GB/s",
+                    "note": "the paper's cost model (Eq. 3: V_q*4 bytes per non-COUNT query) per second of the kernel",
+                    "smem": {"peak": speak, "frac": achieved / speak, "peak_source": ssrc},
+                    "hbm": {"peak": hbm_peak, "frac": achieved / hbm_peak, "peak_source": hbm_src}}
+        r["traffic"] = traffic
     elif kernel == "brick_reduce_kernel":
         r = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s", "frac": achieved / hbm_peak,
              "traffic": traffic, "kernel": kernel, "peak_source": hbm_src,

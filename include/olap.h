@@ -385,6 +385,12 @@ int olap_table_query_batch_device(olap_table* t, int64_t nq, const int64_t* d_co
                                   const olap_cond* d_conds, const int32_t* d_data_cols, const int32_t* d_ops,
                                   olap_result* d_results, void* stream);
 
+/* Accumulated device time (CUDA events on the launching stream) and launch count of the scan
+ * kernel of the table's own calls (not its partitions') since profiling was enabled; enabling
+ * resets the counters. */
+int olap_table_profile(olap_table* t, int enable);
+int olap_table_profile_read(olap_table* t, double* scan_ms, int64_t* launches);
+
 int olap_table_destroy(olap_table* t);
 
 /* A GPU partition for fact-table queries (Fig. 7: the paper

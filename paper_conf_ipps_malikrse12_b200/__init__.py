@@ -90,6 +90,8 @@ EXPORTS = {
     "olap_table_query_batch": (_int, [_p, _i64, _p, _p, _p, _p, _p]),
     "olap_table_query_batch_device": (_int, [_p, _i64, _p, _p, _p, _p, _p, _p]),
     "olap_table_destroy": (_int, [_p]),
+    "olap_table_profile": (_int, [_p, _int]),
+    "olap_table_profile_read": (_int, [_p, ctypes.POINTER(ctypes.c_double), _i64p]),
     "olap_table_part_create": (_int, [_p, _int, ctypes.POINTER(_p)]),
     "olap_table_part_sms": (_int, [_p, ctypes.POINTER(_int), ctypes.POINTER(_int)]),
     "olap_table_part_query_device": (_int, [_p, _i64, _p, _p, _p, _p, _p, _p]),
@@ -625,6 +627,14 @@ class Table:
     def query_device(self, nq: int, d_off, d_conds, d_dcol, d_ops, d_results, stream=None):
         _check(lib.olap_table_query_batch_device(self._h, nq, _ptr(d_off), _ptr(d_conds), _ptr(d_dcol), _ptr(d_ops),
                                                  _ptr(d_results), _stream(stream)), "olap_table_query_batch_device")
+
+    def profile(self, enable: bool = True):
+        _check(lib.olap_table_profile(self._h, 1 if enable else 0), "olap_table_profile")
+
+    def profile_read(self):
+        ms, n = ctypes.c_double(), ctypes.c_int64()
+        _check(lib.olap_table_profile_read(self._h, ctypes.byref(ms), ctypes.byref(n)), "olap_table_profile_read")
+        return ms.value, n.value
 
     def close(self):
         if getattr(self, "_h", None):

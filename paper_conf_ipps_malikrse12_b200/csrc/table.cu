@@ -458,6 +458,10 @@ struct olap_table {
     int32_t* d_dcol = nullptr;
     int32_t* d_ops = nullptr;
     int64_t launches = 0;
+    // olap_table_profile: CUDA events around every table_scan_kernel launch of the table's own calls
+    bool prof = false;
+    std::vector<cudaEvent_t> ev;
+    size_t ev_used = 0;
 };
 
 struct olap_table_part {
@@ -575,8 +579,21 @@ int launch_scan_fold(olap_table* t, TWork& w, int64_t nq, olap_result* d_res, cu
     const size_t smem = sizeof(uint32_t) * kTileRows * t->ncols;
     if (nq > INT32_MAX) return set_error(OLAP_E_INVALID, "table batch of %lld queries: at most 2^31-1", (long long)nq);
     table_order_kernel<<<1, 1024, 0, st>>>(tc, nq, w.d_qs, w.d_perm);
+    const bool prof = t->prof && &w == &t->work && !stream_capturing(st);
+    if (prof) {
+        while (t->ev.size() < t->ev_used + 2) {
+            cudaEvent_t e;
+            OLAP_CUDA_TRY(cudaEventCreate(&e));
+            t->ev.push_back(e);
+        }
+        OLAP_CUDA_TRY(cudaEventRecord(t->ev[t->ev_used], st));
+    }
     table_scan_kernel<<<w.blocks, kScanThreads, smem, st>>>(tc, t->ncols, t->nrows, nq, w.d_qs, w.d_part, w.d_colmask,
                                                             w.d_perm);
+    if (prof) {
+        OLAP_CUDA_TRY(cudaEventRecord(t->ev[t->ev_used + 1], st));
+        t->ev_used += 2;
+    }
     table_final_kernel<<<(int)((nq + 255) / 256), 256, 0, st>>>(tc, nq, w.blocks, w.d_qs, w.d_part, d_res);
     OLAP_CUDA_TRY(cudaGetLastError());
     if (!stream_capturing(st)) OLAP_CUDA_TRY(cudaEventRecord(w.done, st));
@@ -723,11 +740,40 @@ int olap_table_query_batch(olap_table* t, int64_t nq, const int64_t* cond_offset
     return OLAP_OK;
 }
 
+int olap_table_profile(olap_table* t, int enable) {
+    clear_error();
+    if (!t) return set_error(OLAP_E_INVALID, "table handle is NULL");
+    std::lock_guard<std::mutex> lk(t->work.mu);
+    TDevGuard g(t->device);
+    if (t->work.done) OLAP_CUDA_TRY(cudaEventSynchronize(t->work.done));
+    t->prof = enable != 0;
+    t->ev_used = 0;
+    return OLAP_OK;
+}
+
+int olap_table_profile_read(olap_table* t, double* scan_ms, int64_t* launches) {
+    clear_error();
+    if (!t) return set_error(OLAP_E_INVALID, "table handle is NULL");
+    std::lock_guard<std::mutex> lk(t->work.mu);
+    TDevGuard g(t->device);
+    double ms = 0.0;
+    for (size_t i = 0; i + 1 < t->ev_used; i += 2) {
+        float x = 0.f;
+        OLAP_CUDA_TRY(cudaEventSynchronize(t->ev[i + 1]));
+        OLAP_CUDA_TRY(cudaEventElapsedTime(&x, t->ev[i], t->ev[i + 1]));
+        ms += x;
+    }
+    if (scan_ms) *scan_ms = ms;
+    if (launches) *launches = (int64_t)(t->ev_used / 2);
+    return OLAP_OK;
+}
+
 int olap_table_destroy(olap_table* t) {
     clear_error();
     if (!t) return OLAP_OK;
     TDevGuard g(t->device);
     cudaDeviceSynchronize();  // the table's and its partitions' launches (any stream)
+    for (auto e : t->ev) cudaEventDestroy(e);
     free_work(t->work);
     cudaFree(t->d_off);
     cudaFree(t->d_dcol);

@@ -8,7 +8,9 @@ import re
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-UNIT = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
+UNIT = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12,
+        "nsecond": 1, "usecond": 1e3, "msecond": 1e6, "second": 1e9,
+        "inst": 1, "Kinst": 1e3, "Minst": 1e6, "Ginst": 1e9}
 
 
 def parse(path):
@@ -30,6 +32,10 @@ def parse(path):
     out = {}
     for (k, lid), ms in sorted(per.items(), key=lambda x: x[0][1]):
         out[k] = int(ms.get("dram__bytes_read.sum", 0) + ms.get("dram__bytes_write.sum", 0))
+        if "smsp__inst_executed.sum" in ms:
+            out[k + ":inst"] = int(ms["smsp__inst_executed.sum"])
+        if "gpu__time_duration.sum" in ms:
+            out[k + ":ncu_ms"] = ms["gpu__time_duration.sum"] / 1e6  # nsecond -> ms
     return out
 
 
@@ -42,9 +48,11 @@ def main():
             data[w] = parse(p)
         except StopIteration:
             print("no kernels in", p, file=sys.stderr)
-    data["_source"] = ("ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum --clock-control none on the reduce "
-                       "kernels of a 1-warm-up + 1-step bench.py run per workload (tools/traffic.sh); value = read + "
-                       "write bytes of the last launch of each kernel, i.e. per launch = per batch")
+    data["_source"] = ("ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,smsp__inst_executed.sum,"
+                       "gpu__time_duration.sum --clock-control none on the reduce kernels of a 1-warm-up + 1-step "
+                       "bench.py run per workload (tools/traffic.sh); <kernel> = DRAM read + write bytes of its last "
+                       "launch (per launch = per batch), <kernel>:inst = warp instructions executed by that launch, "
+                       "<kernel>:ncu_ms its (serialised, cold-cache) duration")
     json.dump(data, open(tp, "w"), indent=1, sort_keys=True)
     print(json.dumps(data, indent=1, sort_keys=True))
 
