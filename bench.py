@@ -811,7 +811,9 @@ def run_cube(args, rank, world, local):
         else:
             dist.init_process_group(backend)
     cfg = synth.CONFIGS[args.workload]
-    sharded = world > 1 and scaling != "replica"
+    # OLAP_BENCH_SHARDED=1 runs the N > 1 code path (a shard with the library's communicator
+    # attached) at N = 1 as well: a 1-rank NCCL communicator, for testing on one GPU
+    sharded = (world > 1 and scaling != "replica") or os.environ.get("OLAP_BENCH_SHARDED") == "1"
     ext, nq = scaled_workload(args.workload, world, scaling if sharded else "strong")
     if args.batch:
         nq = args.batch * (world if (sharded and scaling == "weak") else 1)
@@ -824,7 +826,7 @@ def run_cube(args, rank, world, local):
         # this rank's block-cyclic dim-0 shard; the library's NCCL communicator does the exchange
         from paper_conf_ipps_malikrse12_b200.dist import init_comm
         cube = olap.Cube(ext, dtype, shard=(world, rank, 1), device=local, layout=lay)
-        comm = init_comm(rank, world, local)
+        comm = init_comm(rank, world, local) if world > 1 else olap.Comm(olap.comm_unique_id(), 1, 0, local)
         cube.attach_comm(comm)
     else:
         cube = olap.Cube(ext, dtype, device=local, layout=lay)

@@ -763,13 +763,15 @@ __global__ void __launch_bounds__(kTileThreads, 1)
             // the query's compact descriptor: words 0-15 by four uniform (broadcast) 16-B loads, the
             // tile-box strides (words 16..) by lane k < nkt
             const int4* sd4 = reinterpret_cast<const int4*>(sdesc + q);
-            const int4 w0 = __ldg(sd4);
+            // every load of the pair's set-up issued at once (one global latency, not three in a row)
+            const int4 w0 = __ldg(sd4), w1 = __ldg(sd4 + 1), w2 = __ldg(sd4 + 2), w3 = __ldg(sd4 + 3);
+            const int32_t tw = __ldg(reinterpret_cast<const int32_t*>(sdesc + q) + 16 + (lane & 7));
+            const int64_t ps = __ldg(pair_start + q);
             const int mode = w0.x;
             long long v;
             int opc;
             int64_t p;
             if (mode) {
-                const int4 w1 = __ldg(sd4 + 1), w2 = __ldg(sd4 + 2), w3 = __ldg(sd4 + 3);
                 opc = w0.y;
                 const uint32_t span = (uint32_t)w0.z, Lin = (uint32_t)w0.w, rad = (uint32_t)w1.x;
                 const uint32_t rs = (uint32_t)w1.y, skt = (uint32_t)w1.z, lo_kt = (uint32_t)w1.w;
@@ -781,10 +783,9 @@ __global__ void __launch_bounds__(kTileThreads, 1)
                 fr.l = (uint32_t)w3.x;
                 const int nkt = w3.y;
                 // pair index j of this tile in the query's tile box (one warp reduction)
-                const int32_t tj = lane < nkt ? m.x32[lane] * __ldg(reinterpret_cast<const int32_t*>(sdesc + q) + 16 + lane)
-                                              : 0;
+                const int32_t tj = lane < nkt ? m.x32[lane] * tw : 0;
                 const int32_t j = jbase + (int32_t)m.c + __reduce_add_sync(0xffffffffu, tj);
-                p = __ldg(pair_start + q) + j;
+                p = ps + j;
                 // the query's box clipped to this tile's chunk [c0, c0 + ce) of dim kt
                 const uint32_t a = max(lo_kt, c0) - c0, b = min(hi_kt, c0 + ce - 1) - c0, na = b - a + 1;
                 const uint32_t base = a * skt + base_in;
@@ -820,7 +821,7 @@ __global__ void __launch_bounds__(kTileThreads, 1)
                 int64_t jj = 0;
                 for (int k = 0; k < tg.kt; ++k) jj = jj * d.tn[k] + (m.x[k] - d.tlo[k]);
                 jj = jj * d.tn[tg.kt] + (m.c - d.tlo[tg.kt]);
-                p = __ldg(pair_start + q) + jj;
+                p = ps + jj;
                 __syncwarp();
                 Acc acc;
                 acc.init();
