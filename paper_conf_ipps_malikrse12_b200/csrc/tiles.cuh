@@ -43,6 +43,7 @@ constexpr int kTileThreads = kTileWarps * 32;
 constexpr int kTileConsumers = kTileWarps - 1;
 constexpr int kTileSlack = 16;  // cells after each stage buffer: masked over-reads of a run's last slot
 constexpr int kTilePairsPerThread = 8;
+constexpr int kTreeTop = 5;  // slot trees (below): highest level, blocks of 32 slots (256 cells)
 
 // Tile geometry of a cube (shard-local), fixed at cube creation.
 struct TGeo {
@@ -73,9 +74,9 @@ struct SDesc {
     int32_t mode, opc, span, Lin;   // Lin: run length (cells) when not span
     int32_t rad, rs, skt, lo_kt;    // inner digit radix (1: none) and stride; stride of dim kt; local range
     int32_t hi_kt, base_in, jbase, radm;  // offset of dims > kt; pair index base; fast-div magic of rad
-    int32_t radl, nkt, pad0, pad1;        // fast-div shift; dims < kt used in tstr
+    int32_t radl, nkt, npat, pad1;        // fast-div shift; dims < kt used in tstr; pattern length (-1: none)
     int32_t tstr[8];                      // tile-box strides of dims < kt (pair index j)
-    int32_t pad2[8];
+    uint16_t pat[16];                     // the run interior's tree entries: level << 13 | node offset
 };
 static_assert(sizeof(SDesc) == 128, "one line per query");
 
@@ -118,12 +119,18 @@ __device__ __forceinline__ void mbar_wait_sleep(uint64_t* b, uint32_t parity) {
         if (clock64() - t0 > kWaitTrapCycles) __trap();
     }
 }
+#ifndef OLAP_WAIT_NS
+#define OLAP_WAIT_NS 128
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
     if (mbar_try(b, parity)) return;  // the common case: one probe
+    // a consumer waiting for the next stage sleeps between probes: a spinning warp would take
+    // issue slots from the warps still reducing (ncu: 7% of the kernel's instructions)
     const long long t0 = clock64();
-    for (uint32_t i = 1;; ++i) {
+    for (;;) {
+        if (OLAP_WAIT_NS) __nanosleep(OLAP_WAIT_NS);
         if (mbar_try(b, parity)) return;
-        if ((i & 1023u) == 0 && clock64() - t0 > kWaitTrapCycles) __trap();
+        if (clock64() - t0 > kWaitTrapCycles) __trap();
     }
 }
 // global -> shared bulk copy completing on mbarrier b (bytes: multiple of 16, both ends 16-B aligned)
@@ -245,6 +252,32 @@ __global__ void __launch_bounds__(kDescThreads) tile_desc_kernel(Geo geo, TGeo t
                 jb += d.tlo[k] * ts;
             }
             sd.jbase = (int32_t)(-jb);
+            // When every run of every pair starts at the same slot of a 32-slot row (run and kt
+            // strides multiples of 256 cells), the interior's tree decomposition is the same for all
+            // of them: node (rb >> j) + off at level j, rb the run's row start slot.  Precompute it.
+            sd.npat = -1;
+            if (sd.mode && !d.span && (d.nrd == 0 || (d.rs[0] & 255) == 0) && (tg.stride[kt] & 255) == 0) {
+                const uint32_t h0 = (uint32_t)(d.base_in & 7);
+                const uint32_t c0 = (uint32_t)(((d.base_in - h0) >> 3) & 31);
+                const uint32_t nslot = (uint32_t)((h0 + d.L + 7) >> 3);
+                int np2 = 0;
+                bool ok = true;
+                if (nslot > 2) {
+                    uint32_t a = c0 + 1, b = c0 + nslot - 1;
+                    auto emit = [&](uint32_t j, uint32_t n) {
+                        if (np2 >= 16 || n >= 8192u) ok = false;
+                        else sd.pat[np2++] = (uint16_t)(j << 13 | n);
+                    };
+                    for (uint32_t j = 0; j < (uint32_t)kTreeTop && a < b; ++j) {
+                        if (a & 1u) emit(j, a++);
+                        if (b & 1u) emit(j, --b);
+                        a >>= 1;
+                        b >>= 1;
+                    }
+                    for (; a < b; ++a) emit((uint32_t)kTreeTop, a);
+                }
+                if (ok) sd.npat = np2;
+            }
             sdesc[q] = sd;
         }
         q_pairs[q] = np;
@@ -421,11 +454,16 @@ __device__ __forceinline__ void build_pair_desc(const TGeo& tg, const TDesc& d, 
 // (sw(i) = i + i / 32: one spare entry per 32) so that lanes walking runs one 32-slot row apart hit
 // different banks at every level.  Written by the producer warp once per tile.
 constexpr int kTileSlots = (int)((kTileCellsMax + 7) / 8);
-constexpr int kTreeTop = 5;  // highest level: blocks of 32 slots (256 cells)
 #ifndef OLAP_COL_SLOTS
 #define OLAP_COL_SLOTS 4
 #endif
 constexpr uint32_t kColSlots = OLAP_COL_SLOTS;  // runs of at most this many slots: column mode on raw cells
+#ifndef OLAP_PAT_MAX_RUNS
+#define OLAP_PAT_MAX_RUNS 16
+#endif
+// pairs of at most this many runs take the per-query pattern (long runs, few of them: C3); more
+// runs are walked through the trees one run per lane (C2a measured equal either way)
+constexpr uint32_t kPatMaxRuns = OLAP_PAT_MAX_RUNS;
 constexpr int lvl_size(int j) { return (((kTileSlots + (1 << j) - 1) >> j) + 1 + 31) & ~31; }
 constexpr int lvl_off(int j) { return j == 0 ? 0 : lvl_off(j - 1) + lvl_size(j - 1); }
 constexpr int kTreeEntries = lvl_off(kTreeTop + 1) + lvl_off(kTreeTop + 1) / 32 + 1;  // padded
@@ -435,6 +473,7 @@ __device__ __forceinline__ uint32_t lvl_off_dev(int j) {
     constexpr uint32_t o[kTreeTop + 1] = {lvl_off(0), lvl_off(1), lvl_off(2), lvl_off(3), lvl_off(4), lvl_off(5)};
     return o[j];
 }
+__constant__ uint32_t kLvlOff[kTreeTop + 1] = {lvl_off(0), lvl_off(1), lvl_off(2), lvl_off(3), lvl_off(4), lvl_off(5)};
 template <class Acc> struct SumEntry;
 template <> struct SumEntry<AccF> { using T = float; };
 template <> struct SumEntry<AccI> { using T = long long; };
@@ -644,6 +683,84 @@ __device__ __forceinline__ void pair_summary(const uint32_t* __restrict__ sb, un
     }
 }
 
+// A pair whose runs all start at the same slot of a 32-slot row (SDesc.npat >= 0): the interior
+// of every run is the same K tree entries (level j, node (rb >> j) + off, rb = the run's row start
+// slot) and the same E edge cells.  One unit = one tree entry or one edge cell of one run; lanes =
+// (run group, unit) with U = K + E <= 32 units per run and 32 / U runs per step, every lane keeping
+// one unit for the whole pair: a step is one load and one fold per lane, no decomposition, no
+// divisions, addresses advanced by fixed increments (kt rows outside, the inner digit inside).
+template <typename T, class Acc, int OPC>
+__device__ __forceinline__ void pair_pattern(const uint32_t* __restrict__ sb, unsigned char* __restrict__ tree,
+                                             uint32_t al, uint32_t h0, uint32_t L, uint32_t rad, uint32_t na,
+                                             uint32_t rs, uint32_t skt, uint32_t K, uint32_t patw, Acc& acc,
+                                             int lane) {
+    using ST = typename SumEntry<Acc>::T;
+    const uint32_t nslot = (h0 + L + 7) >> 3;
+    const uint32_t tail = h0 + L - 8 * (nslot - 1);
+    const uint32_t E1 = nslot == 1 ? L : 8 - h0, E2 = nslot >= 2 ? tail : 0u;
+    const uint32_t U = K + E1 + E2;
+    const uint32_t ulane = (uint32_t)lane;
+    const uint32_t g = small_div(32u, U), grp = small_div(ulane, U), u = ulane - grp * U;
+    const uint32_t pw = __shfl_sync(0xffffffffu, patw, (int)(u >> 1) & 7);
+    if (grp >= g) return;
+    const bool is_tree = u < K;
+    constexpr bool wide_sum = std::is_same<Acc, AccI>::value && OPC == OPC_SUM;  // int64 tree entries
+    const uint32_t rs8 = rs >> 3, skt8 = skt >> 3;  // row-aligned: multiples of 32 slots
+    uint32_t pos, dinner, dkt, base, sh;
+    if (is_tree) {
+        const uint32_t pt = (u & 1u) ? pw >> 16 : pw & 0xffffu;
+        const uint32_t j = pt >> 13, off = pt & 0x1fffu;
+        const uint32_t rb0 = (al >> 3) & ~31u;
+        pos = kLvlOff[j] + (rb0 >> j) + off + ((grp * rs8) >> j);
+        dinner = (g * rs8) >> j;
+        dkt = skt8 >> j;
+        const TreeView<Acc> tv(tree);
+        base = smem_addr_u32(OPC == OPC_SUM ? (const void*)tv.sum : (OPC == OPC_MIN ? (const void*)tv.mn
+                                                                                     : (const void*)tv.mx));
+        sh = wide_sum ? 3u : 2u;
+    } else {
+        const uint32_t e = u - K;
+        pos = al + (e < E1 ? h0 + e : 8 * (nslot - 1) + (e - E1)) + grp * rs;
+        dinner = g * rs;
+        dkt = skt;
+        base = smem_addr_u32(sb);
+        sh = 2u;
+    }
+    auto fold_one = [&](uint32_t p) {
+        const uint32_t addr = base + ((is_tree ? sw(p) : p) << sh);
+        if constexpr (wide_sum) {
+            long long x;
+            if (is_tree) asm volatile("ld.shared.s64 %0, [%1];" : "=l"(x) : "r"(addr));
+            else {
+                int32_t y;
+                asm volatile("ld.shared.s32 %0, [%1];" : "=r"(y) : "r"(addr));
+                x = y;
+            }
+            acc.s += (unsigned long long)x;
+        } else {
+            uint32_t v;
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+            if constexpr (OPC == OPC_SUM) acc.s += (double)__uint_as_float(v);
+            else if constexpr (OPC == OPC_MIN) {
+                if constexpr (std::is_same<Acc, AccF>::value) acc.mn = fminf(acc.mn, __uint_as_float(v));
+                else acc.mn = min(acc.mn, (int32_t)v);
+            } else {
+                if constexpr (std::is_same<Acc, AccF>::value) acc.mx = fmaxf(acc.mx, __uint_as_float(v));
+                else acc.mx = max(acc.mx, (int32_t)v);
+            }
+        }
+    };
+    (void)sizeof(ST);
+    for (uint32_t kr = 0; kr < na; ++kr, pos += dkt) {
+        uint32_t p = pos, ri = grp;
+        for (; ri + g < rad; ri += 2 * g, p += 2 * dinner) {  // two runs per lane in flight
+            fold_one(p);
+            fold_one(p + dinner);
+        }
+        if (ri < rad) fold_one(p);
+    }
+}
+
 template <typename T, class Acc>
 __device__ __forceinline__ long long warp_partial(const Acc& acc, int opc) {
     if (opc == OPC_SUM) {
@@ -766,6 +883,7 @@ __global__ void __launch_bounds__(kTileThreads, 1)
             // every load of the pair's set-up issued at once (one global latency, not three in a row)
             const int4 w0 = __ldg(sd4), w1 = __ldg(sd4 + 1), w2 = __ldg(sd4 + 2), w3 = __ldg(sd4 + 3);
             const int32_t tw = __ldg(reinterpret_cast<const int32_t*>(sdesc + q) + 16 + (lane & 7));
+            const uint32_t patw = (uint32_t)__ldg(reinterpret_cast<const int32_t*>(sdesc + q) + 24 + (lane & 7));
             const int64_t ps = __ldg(pair_start + q);
             const int mode = w0.x;
             long long v;
@@ -807,6 +925,14 @@ __global__ void __launch_bounds__(kTileThreads, 1)
                     if (opc == OPC_SUM) stream_cols<Acc, OPC_SUM, 8, 2>(sb, qd, acc, lane);
                     else if (opc == OPC_MIN) stream_cols<Acc, OPC_MIN, 8, 2>(sb, qd, acc, lane);
                     else stream_cols<Acc, OPC_MAX, 8, 2>(sb, qd, acc, lane);
+                } else if (w3.z >= 0 && !span && R <= kPatMaxRuns && (uint32_t)w3.z + ((h0 + L + 7) >> 3 == 1 ? L : 8 - h0) +
+                                                        (((h0 + L + 7) >> 3) >= 2 ? h0 + L - 8 * (((h0 + L + 7) >> 3) - 1)
+                                                                                  : 0u) <= 32u) {
+                    // row-aligned runs: the precomputed per-query pattern, one unit per lane
+                    const uint32_t K = (uint32_t)w3.z;
+                    if (opc == OPC_SUM) pair_pattern<T, Acc, OPC_SUM>(sb, sm, al, h0, L, rad, na, rs, skt, K, patw, acc, lane);
+                    else if (opc == OPC_MIN) pair_pattern<T, Acc, OPC_MIN>(sb, sm, al, h0, L, rad, na, rs, skt, K, patw, acc, lane);
+                    else pair_pattern<T, Acc, OPC_MAX>(sb, sm, al, h0, L, rad, na, rs, skt, K, patw, acc, lane);
                 } else if (opc == OPC_SUM) {
                     pair_summary<T, Acc, OPC_SUM>(sb, sm, al, h0, L, R, span ? 1u : rad, span ? 1u : na, fr, rs, skt, acc, lane);
                 } else if (opc == OPC_MIN) {
