@@ -154,3 +154,46 @@ def test_multi_errors():
         sh.attach_comm(comm)  # shard 1 of 2 vs rank 0 of 1
     assert ei.value.status == olap.E_INVALID
     comm.close()
+
+
+def test_group_handle_invalid_growth_and_stream_errors():
+    """Device batches flag out-of-range queries INVALID (the host path fails the whole batch with
+    E_RANGE naming the query); the executor's buffers grow across calls; a stream with a bad query
+    fails as a whole and leaves the cube usable."""
+    ext = (24, 9, 70)
+    seed = 0x5EED7200
+    c = olap.Cube(ext, np.float32, devices=[0], shards_per_device=3, shard_block=2)
+    c.fill(olap.GEN_UNIFORM, seed)
+    for n in (10, 1500, 5000, 300):  # growth past the first capacity, then a smaller batch again
+        boxes, ops = _batch(ext, n, seed + n)
+        compare(c.query(boxes, ops), _ref(ext, boxes, ops, np.float32, seed), ops, np.float32)
+    boxes, ops = _batch(ext, 200, seed + 1)
+    bad = boxes.copy()
+    bad[7, 2] = [5, 70]  # hi == extent: out of range
+    res = torch.empty(200 * olap.RESULT_DTYPE.itemsize, dtype=torch.uint8, device="cuda")
+    c.query_device(torch.from_numpy(bad).cuda(), torch.from_numpy(ops).cuda(), res)
+    torch.cuda.synchronize()
+    got = res.cpu().numpy().view(olap.RESULT_DTYPE)
+    assert got["flags"][7] == olap.RESULT_INVALID
+    ok = np.arange(200) != 7
+    compare(got[ok], _ref(ext, boxes[ok], ops[ok], np.float32, seed), ops[ok], np.float32)
+    with pytest.raises(olap.OlapError) as ei:
+        c.query(bad, ops)
+    assert ei.value.status == olap.E_RANGE and "query 7" in str(ei.value)
+    with pytest.raises(olap.OlapError) as ei:
+        c.query_stream(bad, ops, batch=64)
+    assert ei.value.status == olap.E_RANGE
+    compare(c.query_stream(boxes, ops, batch=64), _ref(ext, boxes, ops, np.float32, seed), ops, np.float32)
+
+
+def test_plain_cube_stream_equals_batches():
+    """olap_query_stream on a plain cube (no exchange): pipelined copy-in / reduce / copy-out in
+    batches of any size equals olap_query_batch on the whole, bit for bit (int32)."""
+    ext = (40, 33, 17)
+    c = olap.Cube(ext, np.int32)
+    c.fill(olap.GEN_UNIFORM, 77)
+    boxes, ops = _batch(ext, 3000, 77)
+    want = c.query(boxes, ops)
+    for batch in (1, 999, 1024, 2999, 3000, 0):
+        assert c.query_stream(boxes, ops, batch=batch).tobytes() == want.tobytes(), batch
+    compare(want, _ref(ext, boxes, ops, np.int32, 77), ops, np.int32)
