@@ -819,8 +819,9 @@ def run_cube(args, rank, world, local):
         nq = args.batch * (world if (sharded and scaling == "weak") else 1)
     dtype = cfg["dtype"]
     nd = len(ext)
-    layout = args.layout if args.layout != "auto" else ("brick" if args.workload == "C5" else "row")
-    lay = olap.LAYOUT_BRICK if layout == "brick" else olap.LAYOUT_ROWMAJOR
+    layout = args.layout if args.layout != "auto" else ("brick3" if args.workload == "C5" else "row")
+    lay = {"brick": olap.LAYOUT_BRICK, "brick3": olap.LAYOUT_BRICK3}.get(layout, olap.LAYOUT_ROWMAJOR)
+    bricked = layout in ("brick", "brick3")
     comm = None
     if sharded:
         # this rank's block-cyclic dim-0 shard; the library's NCCL communicator does the exchange
@@ -939,7 +940,7 @@ def run_cube(args, rank, world, local):
                              "unit": "queries/s", "batch": args.stream_batch,
                              "api": "olap_query_stream (batch k+1 reduces while batch k exchanges / finalizes)"}
 
-    kernel = "tile_reduce_kernel" if tiles_used else ("brick_reduce_kernel" if layout == "brick" else "reduce_kernel")
+    kernel = "tile_reduce_kernel" if tiles_used else ("brick_reduce_kernel" if bricked else "reduce_kernel")
     roofline = cube_roofline(args.workload, kernel, achieved, kern_s, clk, alg_bytes / max(launches, 1),
                              reduce_ms / elapsed_ms if elapsed_ms else None, with_traffic=world == 1)
 
@@ -962,11 +963,12 @@ def run_cube(args, rank, world, local):
                        "accumulation": ("int32 cells, int64 SUM" if dtype == np.int32 else
                                         ("f32 cells, SUM in fp32 trees of <= 16 cells then f64 (reading R8')"
                                          if tiles_used else
-                                         ("f32 cells, SUM in fp32 trees of one 8-cell brick row then f64"
-                                          if layout == "brick" else "f32 cells, f64 SUM"))),
-                       "path": "tile-shared scan" if tiles_used else ("brick" if layout == "brick" else "item path"),
-                       "layout": ("bricked: last two dims in 4x8-cell (128-B) bricks" if layout == "brick"
-                                  else "row-major"),
+                                         ("f32 cells, SUM in fp32 trees of 8 cells of a brick then f64"
+                                          if bricked else "f32 cells, f64 SUM"))),
+                       "path": "tile-shared scan" if tiles_used else ("brick" if bricked else "item path"),
+                       "layout": {"brick": "bricked: last two dims in 4x8-cell (128-B) bricks",
+                                  "brick3": "bricked: last three dims in 2x4x4-cell (128-B) bricks (dim 0: local "
+                                            "row pairs)"}.get(layout, "row-major"),
                        "parallelism": par,
                        "exchange": ("library NCCL: ncclAllReduce of the 16-B/query partials per batch "
                                     "(olap_cube_attach_comm)" if sharded else None)},
@@ -1004,8 +1006,9 @@ def main():
                     help="also time the e2e queries as one olap_query_stream in batches of this size")
     ap.add_argument("--graph", action="store_true", help="replay each step as a captured CUDA graph (N=1)")
     ap.add_argument("--batch", type=int, default=0, help="queries per batch per GPU (default: the config's)")
-    ap.add_argument("--layout", default="auto", choices=["auto", "row", "brick"],
-                    help="cube layout in HBM (auto: bricked for C5's small boxes, row-major otherwise; DESIGN.md §5)")
+    ap.add_argument("--layout", default="auto", choices=["auto", "row", "brick", "brick3"],
+                    help="cube layout in HBM (auto: 2x4x4 bricks for C5's small boxes, row-major otherwise; "
+                         "DESIGN.md §5)")
     args = ap.parse_args()
 
     rank, world, local = env_int("RANK", 0), env_int("WORLD_SIZE", 1), env_int("LOCAL_RANK", 0)

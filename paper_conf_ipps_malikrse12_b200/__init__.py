@@ -32,7 +32,7 @@ if os.environ.get("OLAP_LIB"):          # development only: A/B a differently-tu
 
 INT32, FLOAT32 = 1, 2
 SUM, COUNT, MIN, MAX, AVG = 0, 1, 2, 3, 4
-LAYOUT_ROWMAJOR, LAYOUT_BRICK = 0, 1  # olap.h OLAP_LAYOUT_*
+LAYOUT_ROWMAJOR, LAYOUT_BRICK, LAYOUT_BRICK3 = 0, 1, 2  # olap.h OLAP_LAYOUT_*
 GEN_UNIFORM, GEN_AFFINE = 1, 2
 RESULT_EMPTY, RESULT_INVALID = 1, 2
 COND_ALL, COND_EQ, COND_RANGE, COND_IDS = 0, 1, 2, 3

@@ -1289,20 +1289,24 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) reduce_kernel(const T* _
 }
 
 // ------------------------------------------------------------------ bricked cubes: brick_reduce_kernel
-// A query on a bricked cube (OLAP_LAYOUT_BRICK; the brick layout itself is defined below,
-// before the host runtime) is its box of bricks: the leading dims' ranges x the bricks
-// [X0, X1] x [Z0, Z1] its x_{N-2} / x_{N-1} ranges meet.  A lane takes one 128-B brick per
-// step (four LDG.256, all in flight), masks the rows and columns outside the box (only in
-// the box's edge bricks) and folds the 32 cells: one DRAM fetch line per brick, half the
-// lines of the row-major layout on C5's small boxes (reading R26).
-constexpr int kBrickDims = kMaxDims - 2;
+// A query on a bricked cube (OLAP_LAYOUT_BRICK / OLAP_LAYOUT_BRICK3; the layouts themselves are
+// defined below, before the host runtime) is its box of bricks: the leading dims' ranges x the
+// bricks [W0, W1] x [X0, X1] x [Z0, Z1] its x_{N-3} / x_{N-2} / x_{N-1} ranges meet.  A lane quad
+// takes one 128-B brick per step (one LDG.256 per lane, all in flight), masks the cells outside
+// the box (only in the box's edge bricks) and folds its 8 cells: one DRAM fetch line per brick
+// (reading R26).  Brick shapes (cells along x_{N-3}, x_{N-2}, x_{N-1}):
+//   BS = 0: 1 x 4 x 8 (OLAP_LAYOUT_BRICK), BS = 1: 2 x 4 x 4 (OLAP_LAYOUT_BRICK3).
+template <int BS> struct BrickShape;
+template <> struct BrickShape<0> { static constexpr int A0 = 1, A = 4, B = 8; };
+template <> struct BrickShape<1> { static constexpr int A0 = 2, A = 4, B = 4; };
+constexpr int kBrickDims = kMaxDims - 3;  // leading dims 0..N-4 (N <= kMaxDims - 2)
 struct BDesc {
-    int32_t opc, nld;          // op class; leading digits (dims 0..N-3 with extent > 1)
-    int32_t ya, yb, za, zb;    // first brick row's first y, last brick row's last y; same for z
+    int32_t opc, nld;          // op class; leading digits (dims 0..N-4 with extent > 1)
+    int32_t wa, wb, ya, yb, za, zb;  // first brick's first / last brick's last cell along x_{N-3}, x_{N-2}, x_{N-1}
     int64_t nb;                // bricks in the box (0: reads nothing)
     int64_t base;              // cell offset of the box's first brick
-    int64_t nX, nZ, sX;        // brick extents of the box; cells between brick rows
-    FastDiv fZ, fX;            // / nZ, / nX
+    int64_t sW, sX;            // cells between bricks along x_{N-3}, x_{N-2} (Z stride is 32)
+    FastDiv fZ, fX, fW;        // / nZ, / nX, / nW (brick extents of the box)
     FastDiv fl[kBrickDims];    // / leading extents, innermost first (the outermost is not divided)
     int64_t sl[kBrickDims];    // leading strides (cells), innermost first
 };
@@ -1313,17 +1317,19 @@ struct BGeo {
     int nd;                    // logical dims N
     int64_t G, g, b;           // dim-0 shards
     int64_t n[kMaxDims];       // logical global extents
-    int64_t stride[kMaxDims];  // brick-array strides (cells) of dims 0..N-3, then X (N-2); Z stride is 32
+    int64_t stride[kMaxDims];  // brick-array strides (cells) of dims 0..N-4, then W (N-3), X (N-2); Z stride is 32
     int64_t local_rows;
 };
 
 // One thread per query: the box of bricks on this shard, identity partials when it reads
 // nothing, per-query brick counts for the item planner, batch totals (cells, bricks).
+template <int BS>
 __global__ void __launch_bounds__(256) brick_desc_kernel(BGeo g, int64_t nq, const olap_range* __restrict__ ranges,
                                                          const int32_t* __restrict__ ops, BDesc* __restrict__ desc,
                                                          int64_t* __restrict__ q_bricks, int32_t* __restrict__ done,
                                                          int64_t* __restrict__ psum, int32_t* __restrict__ pext,
                                                          unsigned long long* totals) {
+    using S = BrickShape<BS>;
     __shared__ int64_t sh[32];
     const int64_t q = blockIdx.x * 256ll + threadIdx.x;
     int64_t cells = 0, bricks = 0;
@@ -1338,21 +1344,27 @@ __global__ void __launch_bounds__(256) brick_desc_kernel(BGeo g, int64_t nq, con
         int64_t l0 = 0, h0 = -1;
         if (ok) ok = shard_local_range(g.n[0], g.G, g.g, g.b, r[0].lo, r[0].hi, &l0, &h0);
         if (ok) {
-            const int a = g.nd - 2, bz = g.nd - 1;
-            const int64_t X0 = r[a].lo >> 2, X1 = r[a].hi >> 2, Z0 = r[bz].lo >> 3, Z1 = r[bz].hi >> 3;
-            d.ya = (int32_t)(r[a].lo & 3);
-            d.yb = (int32_t)(r[a].hi & 3);
-            d.za = (int32_t)(r[bz].lo & 7);
-            d.zb = (int32_t)(r[bz].hi & 7);
-            d.nX = X1 - X0 + 1;
-            d.nZ = Z1 - Z0 + 1;
+            const int wd = g.nd - 3, a = g.nd - 2, bz = g.nd - 1;
+            // x_{N-3} in shard-local coordinates (dim 0 when N = 3: the owned rows are one local range)
+            const int64_t wlo = wd == 0 ? l0 : r[wd].lo, whi = wd == 0 ? h0 : r[wd].hi;
+            const int64_t W0 = wlo / S::A0, W1 = whi / S::A0;
+            const int64_t X0 = r[a].lo / S::A, X1 = r[a].hi / S::A, Z0 = r[bz].lo / S::B, Z1 = r[bz].hi / S::B;
+            d.wa = (int32_t)(wlo % S::A0);
+            d.wb = (int32_t)(whi % S::A0);
+            d.ya = (int32_t)(r[a].lo % S::A);
+            d.yb = (int32_t)(r[a].hi % S::A);
+            d.za = (int32_t)(r[bz].lo % S::B);
+            d.zb = (int32_t)(r[bz].hi % S::B);
+            const int64_t nW = W1 - W0 + 1, nX = X1 - X0 + 1, nZ = Z1 - Z0 + 1;
+            d.sW = g.stride[wd];
             d.sX = g.stride[a];
-            d.fX = dev_fastdiv((uint32_t)d.nX);
-            d.fZ = dev_fastdiv((uint32_t)d.nZ);
-            int64_t base = X0 * g.stride[a] + Z0 * 32, nb = d.nX * d.nZ, v = (r[a].hi - r[a].lo + 1) *
-                                                                            (r[bz].hi - r[bz].lo + 1);
+            d.fW = dev_fastdiv((uint32_t)nW);
+            d.fX = dev_fastdiv((uint32_t)nX);
+            d.fZ = dev_fastdiv((uint32_t)nZ);
+            int64_t base = W0 * d.sW + X0 * d.sX + Z0 * 32, nb = nW * nX * nZ;
+            int64_t v = (whi - wlo + 1) * (r[a].hi - r[a].lo + 1) * (r[bz].hi - r[bz].lo + 1);
             int nld = 0;
-            for (int k = a - 1; k >= 0; --k) {
+            for (int k = wd - 1; k >= 0; --k) {
                 const int64_t lo = k == 0 ? l0 : r[k].lo, hi = k == 0 ? h0 : r[k].hi, ell = hi - lo + 1;
                 base += lo * g.stride[k];
                 nb *= ell;
@@ -1410,14 +1422,21 @@ __device__ __forceinline__ uint64_t byte_range_word(int lo, int hi) {  // bytes 
     return (~0ull << (8 * lo)) & (~0ull >> (8 * (7 - hi)));
 }
 
-// Cell offset of brick j (< 2^32) of the box: Z fastest, then X, then the leading digits.
-__device__ __forceinline__ int64_t brick_addr(const BDesc& d, uint32_t j, uint32_t& X, uint32_t& Z) {
+// Cell offset of brick j (< 2^32) of the box: Z fastest, then X, then W, then the leading digits.
+__device__ __forceinline__ int64_t brick_addr(const BDesc& d, uint32_t j, uint32_t& W, uint32_t& X, uint32_t& Z) {
     uint32_t t = fdiv(j, d.fZ);
     Z = j - t * d.fZ.d;
     const uint32_t t2 = fdiv(t, d.fX);
     X = t - t2 * d.fX.d;
-    int64_t a = d.base + (int64_t)Z * 32 + (int64_t)X * d.sX;
     t = t2;
+    if (d.nld == 0) {  // W is the outermost digit: no division
+        W = t;
+        return d.base + (int64_t)Z * 32 + (int64_t)X * d.sX + (int64_t)W * d.sW;
+    }
+    const uint32_t t3 = fdiv(t, d.fW);
+    W = t - t3 * d.fW.d;
+    int64_t a = d.base + (int64_t)Z * 32 + (int64_t)X * d.sX + (int64_t)W * d.sW;
+    t = t3;
     for (int e = 0; e < d.nld; ++e) {
         if (e == d.nld - 1) {  // outermost digit: no division
             a += (int64_t)t * d.sl[e];
@@ -1443,16 +1462,34 @@ __device__ __forceinline__ void fold_row(Acc& acc, const uint32_t (&v)[8], uint6
     }
 }
 
-// Four lanes per brick (lane quad = one 128-B line, one coalesced request; lane & 3 = the
-// brick row y), 8 bricks per warp step, kBrickU steps of loads in flight per lane.
+// Byte mask of the 8 cells lane quad member `y4` holds in brick (W, X, Z) (cells 8 y4 .. 8 y4 + 7 of
+// the brick, stored (w, y, z) with z fastest).
+template <int BS>
+__device__ __forceinline__ uint64_t brick_quad_mask(const BDesc& d, int y4, uint32_t W, uint32_t X, uint32_t Z) {
+    using S = BrickShape<BS>;
+    const int ylo = X == 0 ? d.ya : 0, yhi = X == d.fX.d - 1 ? d.yb : S::A - 1;
+    const int zlo = Z == 0 ? d.za : 0, zhi = Z == d.fZ.d - 1 ? d.zb : S::B - 1;
+    if constexpr (BS == 0) {  // the quad member is brick row y = y4: 8 cells along z
+        return y4 >= ylo && y4 <= yhi ? byte_range_word(zlo, zhi) : 0ull;
+    } else {  // w = y4 / 2; rows y = 2 (y4 & 1) and +1, 4 cells along z each
+        const int w = y4 >> 1, wlo = W == 0 ? d.wa : 0, whi = W == d.fW.d - 1 ? d.wb : S::A0 - 1;
+        if (w < wlo || w > whi) return 0ull;
+        const uint32_t zm = (uint32_t)byte_range_word(zlo, zhi);  // bytes zlo..zhi of 4
+        const int y = 2 * (y4 & 1);
+        return (y >= ylo && y <= yhi ? (uint64_t)zm : 0ull) | (y + 1 >= ylo && y + 1 <= yhi ? (uint64_t)zm << 32 : 0ull);
+    }
+}
+
+// Four lanes per brick (lane quad = one 128-B line, one coalesced request), 8 bricks per warp
+// step, kBrickU steps of loads in flight per lane.
 #ifndef OLAP_BRICK_U
 #define OLAP_BRICK_U 3
 #endif
 constexpr int kBrickU = OLAP_BRICK_U;
-template <class Acc, int OPC>
+template <class Acc, int OPC, int BS>
 __device__ __forceinline__ void stream_bricks(const uint32_t* __restrict__ cube, const BDesc& d, int64_t b0,
                                               int64_t b1, Acc& acc, int lane) {
-    const int sub = lane >> 2, y = lane & 3;
+    const int sub = lane >> 2, y4 = lane & 3;
     for (int64_t j0 = b0; j0 < b1; j0 += 8 * kBrickU) {
         uint32_t v[kBrickU][8];
         uint64_t w[kBrickU];
@@ -1461,12 +1498,10 @@ __device__ __forceinline__ void stream_bricks(const uint32_t* __restrict__ cube,
             const int64_t j = j0 + 8 * u + sub;
             const bool ok = j < b1;
             const int64_t jj = ok ? j : b1 - 1;  // < 2^32: a shard holds < 2^32 bricks (checked at creation)
-            uint32_t X, Z;
-            const int64_t a = brick_addr(d, (uint32_t)jj, X, Z);
-            ld_stream8(cube + a + 8 * y, v[u]);
-            const int ylo = X == 0 ? d.ya : 0, yhi = X == d.fX.d - 1 ? d.yb : 3;
-            const int zlo = Z == 0 ? d.za : 0, zhi = Z == d.fZ.d - 1 ? d.zb : 7;
-            w[u] = ok && y >= ylo && y <= yhi ? byte_range_word(zlo, zhi) : 0ull;
+            uint32_t W, X, Z;
+            const int64_t a = brick_addr(d, (uint32_t)jj, W, X, Z);
+            ld_stream8(cube + a + 8 * y4, v[u]);
+            w[u] = ok ? brick_quad_mask<BS>(d, y4, W, X, Z) : 0ull;
         }
 #pragma unroll
         for (int u = 0; u < kBrickU; ++u) fold_row<Acc, OPC>(acc, v[u], w[u]);
@@ -1479,7 +1514,7 @@ __device__ __forceinline__ void stream_bricks(const uint32_t* __restrict__ cube,
 #define OLAP_BRICK_BLOCKS 3
 #endif
 constexpr int kBrickBlocks = OLAP_BRICK_BLOCKS;  // resident blocks per SM the register budget targets
-template <typename T, class Acc>
+template <typename T, class Acc, int BS>
 __global__ void __launch_bounds__(kThreads, kBrickBlocks) brick_reduce_kernel(
     const T* __restrict__ cube, int64_t nq, const BDesc* __restrict__ desc, const int64_t* __restrict__ item_start,
     const int64_t* __restrict__ icnt, unsigned long long* counter, int32_t* done, long long* item_sum,
@@ -1506,9 +1541,9 @@ __global__ void __launch_bounds__(kThreads, kBrickBlocks) brick_reduce_kernel(
         Acc acc;
         acc.init();
         const int opc = sd.opc;
-        if (opc == OPC_SUM) stream_bricks<Acc, OPC_SUM>(c, sd, b0, b1, acc, lane);
-        else if (opc == OPC_MIN) stream_bricks<Acc, OPC_MIN>(c, sd, b0, b1, acc, lane);
-        else stream_bricks<Acc, OPC_MAX>(c, sd, b0, b1, acc, lane);
+        if (opc == OPC_SUM) stream_bricks<Acc, OPC_SUM, BS>(c, sd, b0, b1, acc, lane);
+        else if (opc == OPC_MIN) stream_bricks<Acc, OPC_MIN, BS>(c, sd, b0, b1, acc, lane);
+        else stream_bricks<Acc, OPC_MAX, BS>(c, sd, b0, b1, acc, lane);
         long long s = acc.sum_bits();
         int32_t cmx = opc == OPC_MAX ? acc.code_max() : INT_MIN, cmn = opc == OPC_MIN ? ~acc.code_min() : INT_MIN;
 #pragma unroll
@@ -1661,33 +1696,47 @@ __global__ void fill_kernel(T* cells, Geo geo, int64_t row_cells, int gen, uint6
     }
 }
 
-// ------------------------------------------------------------------ bricked layout (OLAP_LAYOUT_BRICK)
-// Cells (x_{N-2}, x_{N-1}) live in bricks of kBrickA x kBrickB = 4 x 8 cells (128 B: one DRAM
-// fetch line on B200, profiles/microbench_r01_sector.txt).  The storage is the row-major
-// (N+2)-D array (x_0 .. x_{N-3}, X, Z, y, z) with x_{N-2} = 4X + y, x_{N-1} = 8Z + z, held by
-// an inner row-major cube; queries run brick_reduce_kernel on it (a lane quad per brick).
-constexpr int64_t kBrickA = 4, kBrickB = 8;
-static_assert(kBrickA == 4 && kBrickB == 8, "fill_brick_kernel and the host loader assume 4 x 8 bricks");
+// ------------------------------------------------------------------ bricked layouts (OLAP_LAYOUT_BRICK, _BRICK3)
+// Cells (x_{N-3}, x_{N-2}, x_{N-1}) live in bricks of A0 x A x B = 32 cells (128 B: one DRAM fetch
+// line on B200, profiles/r01/microbench_r01_sector.txt): 1 x 4 x 8 (OLAP_LAYOUT_BRICK) or 2 x 4 x 4
+// (OLAP_LAYOUT_BRICK3).  The storage is the row-major array (x_0 .. x_{N-4}, W, X, Z, w, y, z) with
+// x_{N-3} = A0 W + w, x_{N-2} = A X + y, x_{N-1} = B Z + z, held by an inner row-major cube of
+// extents (.., NW, NX, NZ, 32); queries run brick_reduce_kernel on it (a lane quad per brick).
+// When N = 3, x_{N-3} is dim 0 in SHARD-LOCAL rows (a query's owned rows are one local range), so
+// a 2 x 4 x 4 brick pairs local rows 2W, 2W + 1 and the inner cube is the shard's own, unsharded.
+struct BrickDims {
+    int a0, a, b;
+};
+inline BrickDims brick_dims(int layout) { return layout == OLAP_LAYOUT_BRICK3 ? BrickDims{2, 4, 4} : BrickDims{1, 4, 8}; }
 
-// olap_cube_fill on the brick array: storage index -> (local row, mid, X, Z, y, z) -> logical.
+// olap_cube_fill on the brick array: storage index -> (leading, W, X, Z, w, y, z) -> logical cell.
 template <typename T>
-__global__ void fill_brick_kernel(T* cells, Geo geo, int64_t row_cells, int64_t NX, int64_t NZ, int gen,
-                                  uint64_t seed, FillParams fp) {
-    const int64_t n = geo.local_rows * row_cells;
-    const int64_t na = geo.n[geo.nd - 2], nb = geo.n[geo.nd - 1];
-    for (int64_t li = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; li < n; li += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t lr = li / row_cells, rem = li - lr * row_cells;
-        const int64_t z = rem & (kBrickB - 1), y = (rem >> 3) & (kBrickA - 1);
-        int64_t t = rem >> 5;
+__global__ void fill_brick_kernel(T* cells, Geo geo, int64_t ncells, int64_t NW, int64_t NX, int64_t NZ, int a0, int a,
+                                  int b, int64_t P1, int gen, uint64_t seed, FillParams fp) {
+    const int nd = geo.nd;
+    const int64_t na = geo.n[nd - 2], nb = geo.n[nd - 1], nw = nd == 3 ? geo.local_rows : geo.n[nd - 3];
+    for (int64_t li = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; li < ncells; li += (int64_t)gridDim.x * blockDim.x) {
+        const int c32 = (int)(li & 31);
+        int64_t t = li >> 5;
         const int64_t Z = t % NZ;
         t /= NZ;
-        const int64_t X = t % NX, mid = t / NX;
-        const int64_t xa = kBrickA * X + y, xb = kBrickB * Z + z;
-        if (xa >= na || xb >= nb) {  // padding cell: never part of a box
+        const int64_t X = t % NX;
+        t /= NX;
+        const int64_t W = t % NW, mid = t / NW;
+        const int64_t xw = a0 * W + c32 / (a * b), xa = a * X + (c32 / b) % a, xb = b * Z + c32 % b;
+        if (xw >= nw || xa >= na || xb >= nb) {  // padding cell: never part of a box
             cells[li] = (T)0;
             continue;
         }
-        gen_cell<T>(cells, li, geo, gen, seed, fp, shard_global_of(lr, geo.G, geo.g, geo.b), (mid * na + xa) * nb + xb);
+        int64_t lr, off;
+        if (nd == 3) {
+            lr = xw;
+            off = xa * nb + xb;
+        } else {  // mid = local row x P1 + the digits of dims 1..N-4
+            lr = mid / P1;
+            off = (((mid - lr * P1) * nw + xw) * na + xa) * nb + xb;
+        }
+        gen_cell<T>(cells, li, geo, gen, seed, fp, shard_global_of(lr, geo.G, geo.g, geo.b), off);
     }
 }
 
@@ -1818,11 +1867,12 @@ struct olap_cube {
     int64_t kernel_launches = 0;  // every kernel this cube launched (all entry points)
     unsigned long long bytes_base = 0;
 
-    // OLAP_LAYOUT_BRICK: this handle keeps the logical geometry (nd, n, shards) and `inner` is
-    // the row-major cube of the brick array (.., ceil(n_{N-2}/4), ceil(n_{N-1}/8), 4, 8) that
-    // owns the cells (queries use its workspace: run_partials_brick).
+    // OLAP_LAYOUT_BRICK / _BRICK3: this handle keeps the logical geometry (nd, n, shards) and
+    // `inner` is the row-major cube of the brick array (.., NW, NX, NZ, 32) that owns the cells
+    // (queries use its workspace: run_partials_brick).
     olap_cube* inner = nullptr;
     int brick_bps = 0;  // resident brick_reduce_kernel blocks per SM
+    int layout = OLAP_LAYOUT_ROWMAJOR;  // OLAP_LAYOUT_BRICK / _BRICK3: `inner` holds the bricks
 
     // multi-GPU (mgpu.cu): a group handle (olap_cube_create_multi) owns `shards` (G shard cubes
     // over its devices) and answers through `exec`; a shard with an attached communicator
@@ -2213,20 +2263,21 @@ int run_partials_brick(olap_cube* c, int64_t nq, const olap_range* d_ranges, con
     for (int k = 0; k <= c->nd - 2; ++k) g.stride[k] = ic->stride[k];
     g.local_rows = c->local_rows;
     BDesc* bd = reinterpret_cast<BDesc*>(ic->d_desc);
+    const bool b3 = c->layout == OLAP_LAYOUT_BRICK3;
     if (!c->brick_bps) {
         int bps = 0;
         if (c->dtype == OLAP_INT32)
-            OLAP_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, brick_reduce_kernel<int32_t, AccI>,
-                                                                        kThreads, 0));
+            OLAP_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+                &bps, b3 ? brick_reduce_kernel<int32_t, AccI, 1> : brick_reduce_kernel<int32_t, AccI, 0>, kThreads, 0));
         else
-            OLAP_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, brick_reduce_kernel<float, AccF>,
-                                                                        kThreads, 0));
+            OLAP_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+                &bps, b3 ? brick_reduce_kernel<float, AccF, 1> : brick_reduce_kernel<float, AccF, 0>, kThreads, 0));
         c->brick_bps = std::max(bps, 1);
     }
     const int grid = ic->num_sms * c->brick_bps;
     OLAP_CUDA_TRY(cudaMemsetAsync(ic->d_counter + 2, 0, 2 * sizeof(unsigned long long), st));
-    brick_desc_kernel<<<(int)((nq + 255) / 256), 256, 0, st>>>(g, nq, d_ranges, d_ops, bd, ic->d_qtasks, ic->d_done,
-                                                               d_psum, d_pext, ic->d_counter + 2);
+    (b3 ? brick_desc_kernel<1> : brick_desc_kernel<0>)<<<(int)((nq + 255) / 256), 256, 0, st>>>(
+        g, nq, d_ranges, d_ops, bd, ic->d_qtasks, ic->d_done, d_psum, d_pext, ic->d_counter + 2);
     brick_items_kernel<<<(int)((nq + 256) / 256), 256, 0, st>>>(nq, bd, ic->d_qtasks, ic->d_icnt, ic->items_cap,
                                                                 ic->d_counter + 2, grid * kWarps);
     OLAP_CUDA_TRY(cudaGetLastError());
@@ -2245,11 +2296,11 @@ int run_partials_brick(olap_cube* c, int64_t nq, const olap_range* d_ranges, con
         OLAP_CUDA_TRY(cudaEventRecord(ic->ev[ic->ev_used], st));
     }
     if (c->dtype == OLAP_INT32)
-        brick_reduce_kernel<int32_t, AccI><<<grid, kThreads, 0, st>>>(
+        (b3 ? brick_reduce_kernel<int32_t, AccI, 1> : brick_reduce_kernel<int32_t, AccI, 0>)<<<grid, kThreads, 0, st>>>(
             static_cast<const int32_t*>(ic->d_cells), nq, bd, ic->d_item_start, ic->d_icnt, ic->d_counter, ic->d_done,
             ic->d_item_sum, ic->d_item_ext, d_psum, d_pext);
     else
-        brick_reduce_kernel<float, AccF><<<grid, kThreads, 0, st>>>(
+        (b3 ? brick_reduce_kernel<float, AccF, 1> : brick_reduce_kernel<float, AccF, 0>)<<<grid, kThreads, 0, st>>>(
             static_cast<const float*>(ic->d_cells), nq, bd, ic->d_item_start, ic->d_icnt, ic->d_counter, ic->d_done,
             ic->d_item_sum, ic->d_item_ext, d_psum, d_pext);
     OLAP_CUDA_TRY(cudaGetLastError());
@@ -2266,17 +2317,25 @@ int run_partials_brick(olap_cube* c, int64_t nq, const olap_range* d_ranges, con
     return OLAP_OK;
 }
 
-// Host rows [row_lo, row_hi) (logical row-major) -> brick order, one dim-0 row at a time.
+// Host rows [row_lo, row_hi) (logical row-major) -> brick order, one dim-0 row at a time.  A row is
+// one inner row, except for 2 x 4 x 4 bricks of a 3-D cube: there local rows 2W and 2W + 1 share
+// inner row W, each holding the first or second 16-cell half of every brick (one strided copy).
 int load_rows_brick(olap_cube* c, int64_t row_lo, int64_t row_hi, const void* cells) {
     olap_cube* ic = c->inner;
     const int nd = c->nd;
-    const int64_t na = c->n[nd - 2], nb = c->n[nd - 1], P = c->lrow_cells / (na * nb);
-    const int64_t NX = ic->n[nd - 2], NZ = ic->n[nd - 1];
+    const BrickDims bd = brick_dims(c->layout);
+    const int64_t na = c->n[nd - 2], nb = c->n[nd - 1];
+    const int64_t NW = ic->n[nd - 3], NX = ic->n[nd - 2], NZ = ic->n[nd - 1];
+    const bool pair_rows = nd == 3 && bd.a0 == 2;
+    const int64_t nw = nd == 3 ? 1 : c->n[nd - 3];         // x_{N-3} values inside one dim-0 row
+    const int64_t P1 = nd == 3 ? 1 : c->lrow_cells / (nw * na * nb);  // digits of dims 1..N-4
+    const int64_t half = 32 / bd.a0;                        // cells of one x_{N-3} layer of a brick
+    const int64_t bufcells = pair_rows ? NX * NZ * half : ic->row_cells;
     std::vector<uint32_t> buf;
     try {
-        buf.assign((size_t)ic->row_cells, 0u);
+        buf.assign((size_t)bufcells, 0u);
     } catch (...) {
-        return set_error(OLAP_E_NOMEM, "host staging of one brick row (%lld cells)", (long long)ic->row_cells);
+        return set_error(OLAP_E_NOMEM, "host staging of one brick row (%lld cells)", (long long)bufcells);
     }
     const uint32_t* src = static_cast<const uint32_t*>(cells);
     char* dst = static_cast<char*>(ic->d_cells);
@@ -2284,15 +2343,23 @@ int load_rows_brick(olap_cube* c, int64_t row_lo, int64_t row_hi, const void* ce
     for (int64_t r = row_lo; r < row_hi; ++r) {
         if (G > 1 && (r / b) % G != g) continue;
         const uint32_t* row = src + (r - row_lo) * c->lrow_cells;
-        for (int64_t mid = 0; mid < P; ++mid)
-            for (int64_t xa = 0; xa < na; ++xa) {
-                const uint32_t* in = row + (mid * na + xa) * nb;
-                uint32_t* out = buf.data() + ((mid * NX + xa / kBrickA) * NZ) * (kBrickA * kBrickB) +
-                                (xa % kBrickA) * kBrickB;
-                for (int64_t xb = 0; xb < nb; ++xb) out[(xb / kBrickB) * (kBrickA * kBrickB) + xb % kBrickB] = in[xb];
-            }
+        for (int64_t mid = 0; mid < P1; ++mid)
+            for (int64_t xw = 0; xw < nw; ++xw)
+                for (int64_t xa = 0; xa < na; ++xa) {
+                    const uint32_t* in = row + ((mid * nw + xw) * na + xa) * nb;
+                    // brick (W, X, Z) of this row and the cell's place inside it
+                    const int64_t W = nd == 3 ? 0 : mid * NW + xw / bd.a0;
+                    const int64_t wofs = nd == 3 ? 0 : (xw % bd.a0) * half;
+                    uint32_t* out = buf.data() + ((W * NX + xa / bd.a) * NZ) * (pair_rows ? half : 32) + wofs +
+                                    (xa % bd.a) * bd.b;
+                    for (int64_t xb = 0; xb < nb; ++xb) out[(xb / bd.b) * (pair_rows ? half : 32) + xb % bd.b] = in[xb];
+                }
         const int64_t lr = shard_local_of(r, G, b);
-        OLAP_CUDA_TRY(cudaMemcpy(dst + lr * ic->row_cells * 4, buf.data(), ic->row_cells * 4, cudaMemcpyHostToDevice));
+        if (pair_rows)  // half-bricks: 64 B of every 128-B brick of inner row lr / 2
+            OLAP_CUDA_TRY(cudaMemcpy2D(dst + ((lr >> 1) * ic->row_cells + (lr & 1) * half) * 4, 128, buf.data(),
+                                       half * 4, half * 4, NX * NZ, cudaMemcpyHostToDevice));
+        else
+            OLAP_CUDA_TRY(cudaMemcpy(dst + lr * ic->row_cells * 4, buf.data(), ic->row_cells * 4, cudaMemcpyHostToDevice));
     }
     return OLAP_OK;
 }
@@ -2358,8 +2425,8 @@ int cube_geometry(const olap_cube* c, int* nd, int64_t* n, int* dtype, int64_t* 
     *nshards = c->sh.nshards;
     return OLAP_OK;
 }
-// OLAP_LAYOUT_ROWMAJOR or OLAP_LAYOUT_BRICK (roll-up reads raw cells and needs row-major)
-int cube_layout(const olap_cube* c) { return c->inner ? OLAP_LAYOUT_BRICK : OLAP_LAYOUT_ROWMAJOR; }
+// OLAP_LAYOUT_ROWMAJOR, _BRICK or _BRICK3 (roll-up reads raw cells and needs row-major)
+int cube_layout(const olap_cube* c) { return c->layout; }
 }  // namespace olap
 
 extern "C" {
@@ -2472,24 +2539,41 @@ int olap_cube_create_layout(int ndims, const int64_t* extents, int dtype, const 
                             int layout, olap_cube** out) {
     clear_error();
     if (layout == OLAP_LAYOUT_ROWMAJOR) return olap_cube_create(ndims, extents, dtype, shard, device, out);
-    if (layout != OLAP_LAYOUT_BRICK) return set_error(OLAP_E_INVALID, "unknown layout %d", layout);
+    if (layout != OLAP_LAYOUT_BRICK && layout != OLAP_LAYOUT_BRICK3)
+        return set_error(OLAP_E_INVALID, "unknown layout %d", layout);
     if (!out || !extents) return set_error(OLAP_E_INVALID, "olap_cube_create_layout: NULL argument");
     if (ndims < 3 || ndims > kMaxDims - 2)
         return set_error(OLAP_E_INVALID, "bricked layout needs ndims in [3,%d], got %d", kMaxDims - 2, ndims);
     for (int k = 0; k < ndims; ++k)
         if (extents[k] < 1) return set_error(OLAP_E_INVALID, "extent[%d] = %lld < 1", k, (long long)extents[k]);
+    olap_shard sh{1, 0, 1};
+    if (shard) sh = *shard;
+    if (sh.nshards < 1 || sh.shard < 0 || sh.shard >= sh.nshards || sh.block < 1)
+        return set_error(OLAP_E_INVALID, "bad shard {%lld,%lld,%lld}", (long long)sh.nshards, (long long)sh.shard,
+                         (long long)sh.block);
+    const BrickDims bd = brick_dims(layout);
+    // 2 x 4 x 4 bricks of a 3-D cube pair SHARD-LOCAL rows: the inner cube is this shard's own
+    // (unsharded, ceil(local rows / 2) inner rows); otherwise dim 0 stays unbricked and the inner
+    // cube is sharded like the logical one.
+    const bool pair_rows = ndims == 3 && bd.a0 == 2;
+    const int64_t lrows = shard_rows(extents[0], sh.nshards, sh.shard, sh.block);
     int64_t e[kMaxDims];
-    for (int k = 0; k < ndims - 2; ++k) e[k] = extents[k];
-    e[ndims - 2] = (extents[ndims - 2] + kBrickA - 1) / kBrickA;
-    e[ndims - 1] = (extents[ndims - 1] + kBrickB - 1) / kBrickB;
-    e[ndims] = kBrickA;
-    e[ndims + 1] = kBrickB;
+    for (int k = 0; k < ndims - 3; ++k) e[k] = extents[k];
+    e[ndims - 3] = pair_rows ? std::max<int64_t>(1, (lrows + 1) / 2) : (extents[ndims - 3] + bd.a0 - 1) / bd.a0;
+    e[ndims - 2] = (extents[ndims - 2] + bd.a - 1) / bd.a;
+    e[ndims - 1] = (extents[ndims - 1] + bd.b - 1) / bd.b;
+    e[ndims] = 32;
     olap_cube* ic = nullptr;
-    int rc = olap_cube_create(ndims + 2, e, dtype, shard, device, &ic);
+    int rc = olap_cube_create(ndims + 1, e, dtype, pair_rows ? nullptr : &sh, device, &ic);
     if (rc) return rc;
     if ((ic->local_cells >> 5) >= (1ll << 32)) {  // brick indices are 32-bit (2^32 bricks = 512 GiB per shard)
         olap_cube_destroy(ic);
         return set_error(OLAP_E_UNSUPPORTED, "a bricked shard must hold < 2^32 bricks");
+    }
+    // padding cells (ragged bricks, the unpaired last local row) read as 0 (they are always masked)
+    if (cudaMemset(ic->d_cells, 0, ic->local_cells * 4) != cudaSuccess) {
+        olap_cube_destroy(ic);
+        return set_error(OLAP_E_CUDA, "cudaMemset of the brick array failed");
     }
     DeviceGuard dg(device);
     olap_cube* c = new (std::nothrow) olap_cube();
@@ -2499,17 +2583,18 @@ int olap_cube_create_layout(int ndims, const int64_t* extents, int dtype, const 
     }
     ic->tiles_on = false;  // bricked queries run brick_reduce_kernel on the inner cube, never its tile path
     c->inner = ic;
+    c->layout = layout;
     c->nd = ndims;
     c->dtype = dtype;
     c->device = device;
-    c->sh = ic->sh;
+    c->sh = sh;
     for (int k = 0; k < ndims; ++k) c->n[k] = extents[k];
     c->pitch = c->n[ndims - 1];
     c->stride[ndims - 1] = 1;
     for (int k = ndims - 2; k >= 0; --k) c->stride[k] = c->stride[k + 1] * c->n[k + 1];
     c->lrow_cells = c->stride[0];
     c->row_cells = ic->row_cells;  // storage
-    c->local_rows = ic->local_rows;
+    c->local_rows = lrows;
     c->local_cells = ic->local_cells;
     c->d_cells = ic->d_cells;
     c->num_sms = ic->num_sms;
@@ -2626,13 +2711,19 @@ int olap_cube_fill(olap_cube* c, int generator, uint64_t seed, const double* par
     if (c->inner) {
         const olap_cube* ic = c->inner;
         OLAP_CUDA_TRY(cudaEventSynchronize(ic->ws_done));
-        const int64_t NX = ic->n[c->nd - 2], NZ = ic->n[c->nd - 1];
+        const int nd = c->nd;
+        const BrickDims bd = brick_dims(c->layout);
+        const int64_t NW = ic->n[nd - 3], NX = ic->n[nd - 2], NZ = ic->n[nd - 1];
+        int64_t P1 = 1;  // digits of dims 1..N-4 per dim-0 row
+        for (int k = 1; k <= nd - 4; ++k) P1 *= c->n[k];
         if (c->dtype == OLAP_INT32)
             fill_brick_kernel<int32_t><<<grid, 256, 0, c->stream>>>(static_cast<int32_t*>(c->d_cells), make_geo(c),
-                                                                    ic->row_cells, NX, NZ, generator, seed, fp);
+                                                                    ic->local_cells, NW, NX, NZ, bd.a0, bd.a, bd.b, P1,
+                                                                    generator, seed, fp);
         else
             fill_brick_kernel<float><<<grid, 256, 0, c->stream>>>(static_cast<float*>(c->d_cells), make_geo(c),
-                                                                  ic->row_cells, NX, NZ, generator, seed, fp);
+                                                                  ic->local_cells, NW, NX, NZ, bd.a0, bd.a, bd.b, P1,
+                                                                  generator, seed, fp);
         OLAP_CUDA_TRY(cudaGetLastError());
         OLAP_CUDA_TRY(cudaStreamSynchronize(c->stream));
         return OLAP_OK;

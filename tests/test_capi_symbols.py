@@ -59,7 +59,8 @@ def test_layout_arguments_validated_before_the_device():
     with OLAP_E_INVALID on any box (argument checks come before any CUDA call)."""
     import paper_conf_ipps_malikrse12_b200 as olap
     for ext, layout in (((4, 4, 4), 7), ((10, 20), olap.LAYOUT_BRICK), ((2,) * 7, olap.LAYOUT_BRICK),
-                        ((4, 0, 4), olap.LAYOUT_BRICK)):
+                        ((4, 0, 4), olap.LAYOUT_BRICK), ((10, 20), olap.LAYOUT_BRICK3),
+                        ((2,) * 7, olap.LAYOUT_BRICK3), ((0, 4, 4), olap.LAYOUT_BRICK3)):
         with pytest.raises(olap.OlapError) as ei:
             olap.Cube(ext, np.float32, layout=layout)
         assert ei.value.status == olap.E_INVALID, (ext, layout)
