@@ -9,8 +9,8 @@
 // query (Eq. 12: bytes = rows x C_QD x 4).  B200 design: a SHARED scan — one persistent
 // launch per batch streams every column once, tile by tile, into shared memory, and
 // every warp evaluates its share of the batch's queries on the staged tile (each
-// condition one unsigned range compare).  Per-(block, query) partials are folded in
-// fixed block order by a second kernel, so results are deterministic.
+// condition one unsigned range compare).  Per-(tile range, query) partials are folded in
+// fixed range order by a second kernel, so results are deterministic.
 #include <algorithm>
 #include <climits>
 #include <cstring>
@@ -47,7 +47,7 @@ struct TQuery {
     TCond c[kMaxConds];
 };
 
-struct TPartial {  // per (block, query)
+struct TPartial {  // per (tile range, query)
     long long sum;     // int64 wraparound sum or double bits
     int64_t count;     // matching rows
     int32_t code_max;  // order-preserving code of MAX (INT_MIN = none)
@@ -181,47 +181,71 @@ __global__ void table_prep_boxes_kernel(int64_t nq, int ncols, TableCols tc, Box
     note_columns(t, colmask);
 }
 
+// A query in the scan's shared-memory form (48 B, three broadcast LDS.128): the header, then its
+// first kInlineConds conditions (ascending span); further conditions are read from its TQuery.
+constexpr int kInlineConds = 4;
+struct SQ {
+    int32_t ncond;     // < 0: the query reads nothing (invalid or impossible)
+    int32_t q;         // query index (TQuery of conditions beyond kInlineConds; partial slot)
+    int32_t meta;      // data_col | fl << 8 (float data) | opk << 9 (0 SUM / AVG, 1 MIN, 2 MAX, 3 COUNT)
+    uint32_t colpack;  // column of inline condition k in bits 4k .. 4k+3
+    uint32_t lo[kInlineConds];
+    uint32_t span[kInlineConds];
+};
+static_assert(sizeof(SQ) == 48, "three 16-B words per query");
+
 // One query on one staged tile.  Lane l owns the row quads 4l..4l+3 + 128 i (i < 8): every
 // condition column is read with one LDS.128 per quad (lane-consecutive 16-B chunks, no bank
 // conflicts) and evaluated into a 32-bit pass mask (bit 4i + j = row 128 i + 4 l + j);
 // COUNT is a popcount, and only matching rows touch the data column, folding only the
-// accumulator the op needs (OPK: 0 SUM / AVG, 1 MIN, 2 MAX, 3 COUNT).
+// accumulator the op needs (OPK: 0 SUM / AVG, 1 MIN, 2 MAX, 3 COUNT).  Returns false when no
+// row of the tile matches (s, cnt, cmx, cmn untouched); else every lane holds the warp's totals.
 __device__ __forceinline__ uint32_t quad_pass(uint4 x, uint32_t lo, uint32_t span) {
     return (uint32_t)(x.x - lo <= span) | (uint32_t)(x.y - lo <= span) << 1 | (uint32_t)(x.z - lo <= span) << 2 |
            (uint32_t)(x.w - lo <= span) << 3;
 }
 template <bool FLOAT_DATA, int OPK>
-__device__ __forceinline__ void scan_query_tile(const uint32_t* __restrict__ smem, int rows, const TQuery& tq, int lane,
-                                                long long& s, int64_t& cnt, int32_t& cmx, int32_t& cmn) {
+__device__ __forceinline__ bool scan_query_tile(const uint32_t* __restrict__ smem, int rows, const SQ* sq,
+                                                const TQuery* __restrict__ qs, int lane, long long& s, int32_t& cnt,
+                                                int32_t& cmx, int32_t& cmn) {
     static_assert(kTileRows == 1024, "one 32-bit pass mask per lane");
     uint32_t pass = rows >= kTileRows ? 0xFFFFFFFFu : 0u;
     if (rows < kTileRows)
         for (int b = 0; b < 32; ++b)
             if (128 * (b >> 2) + 4 * lane + (b & 3) < rows) pass |= 1u << b;
-    const int nc = tq.ncond;
+    const int nc = sq->ncond;
     for (int k = 0; k < nc && pass; ++k) {
-        const TCond c = tq.c[k];
+        uint32_t col, lo, span;
+        if (k < kInlineConds) {  // shared memory (broadcast)
+            col = (sq->colpack >> (4 * k)) & 15u;
+            lo = sq->lo[k];
+            span = sq->span[k];
+        } else {
+            const TCond c = qs[sq->q].c[k];
+            col = (uint32_t)c.col;
+            lo = c.lo;
+            span = c.span;
+        }
         if (__popc(pass) <= kSparseRows) {  // few survivors: check them one by one
-            const uint32_t* col = smem + c.col * kTileRows + 4 * lane;
+            const uint32_t* cp = smem + col * kTileRows + 4 * lane;
             uint32_t left = pass;
             while (left) {
                 const int b = __ffs(left) - 1;
                 left &= left - 1;
-                if (col[128 * (b >> 2) + (b & 3)] - c.lo > c.span) pass &= ~(1u << b);
+                if (cp[128 * (b >> 2) + (b & 3)] - lo > span) pass &= ~(1u << b);
             }
             continue;
         }
-        const uint4* col = reinterpret_cast<const uint4*>(smem + c.col * kTileRows) + lane;
+        const uint4* cp = reinterpret_cast<const uint4*>(smem + col * kTileRows) + lane;
         uint32_t m = 0;
 #pragma unroll
-        for (int i = 0; i < 8; ++i) m |= quad_pass(col[32 * i], c.lo, c.span) << (4 * i);
+        for (int i = 0; i < 8; ++i) m |= quad_pass(cp[32 * i], lo, span) << (4 * i);
         pass &= m;
     }
-    // no row of the tile matches (most tiles of a query with equality predicates): the
-    // fold below would add +0 / INT_MIN codes, which leaves s, cnt, cmx, cmn bit-identical
-    if (!__any_sync(0xffffffffu, pass)) return;
+    // no row of the tile matches (most tiles of a query with equality predicates)
+    if (!__any_sync(0xffffffffu, pass)) return false;
     int32_t n = __popc(pass);
-    const uint32_t* data = smem + tq.data_col * kTileRows + 4 * lane;
+    const uint32_t* data = smem + (sq->meta & 0xff) * kTileRows + 4 * lane;
     unsigned long long si = 0ull;
     double sf = 0.0;
     float fmn = __int_as_float(0x7f800000), fmx = __int_as_float(0xff800000);
@@ -243,24 +267,21 @@ __device__ __forceinline__ void scan_query_tile(const uint32_t* __restrict__ sme
             if (OPK == 2) imx = max(imx, v);
         }
     }
-    // warp reduction in fixed order
-    long long sb = FLOAT_DATA ? __double_as_longlong(sf) : (long long)si;
-    int32_t mx = FLOAT_DATA ? tf32_code(fmx) : imx, mn = ~(FLOAT_DATA ? tf32_code(fmn) : imn);
-    if (n == 0) mx = mn = INT_MIN;
+    // warp reduction in fixed order (only the op's accumulator)
+    if (OPK == 0) {
+        long long sb = FLOAT_DATA ? __double_as_longlong(sf) : (long long)si;
 #pragma unroll
-    for (int o = 16; o; o >>= 1) {
-        const long long so = __shfl_xor_sync(0xffffffffu, sb, o);
-        sb = FLOAT_DATA ? __double_as_longlong(__longlong_as_double(sb) + __longlong_as_double(so))
-                        : (long long)((unsigned long long)sb + (unsigned long long)so);
-        n += __shfl_xor_sync(0xffffffffu, n, o);
+        for (int o = 16; o; o >>= 1) {
+            const long long so = __shfl_xor_sync(0xffffffffu, sb, o);
+            sb = FLOAT_DATA ? __double_as_longlong(__longlong_as_double(sb) + __longlong_as_double(so))
+                            : (long long)((unsigned long long)sb + (unsigned long long)so);
+        }
+        s = sb;
     }
-    mx = __reduce_max_sync(0xffffffffu, mx);
-    mn = __reduce_max_sync(0xffffffffu, mn);
-    s = FLOAT_DATA ? __double_as_longlong(__longlong_as_double(s) + __longlong_as_double(sb))
-                   : (long long)((unsigned long long)s + (unsigned long long)sb);
-    cnt += n;
-    cmx = max(cmx, mx);
-    cmn = max(cmn, mn);
+    cnt = __reduce_add_sync(0xffffffffu, (uint32_t)n);
+    if (OPK == 2) cmx = __reduce_max_sync(0xffffffffu, n ? (FLOAT_DATA ? tf32_code(fmx) : imx) : INT_MIN);
+    if (OPK == 1) cmn = __reduce_max_sync(0xffffffffu, n ? ~(FLOAT_DATA ? tf32_code(fmn) : imn) : INT_MIN);
+    return true;
 }
 
 // Scan instantiation of a query: (float data, op) -> 0..7; 8 = skipped (invalid / empty).
@@ -273,9 +294,9 @@ __device__ __forceinline__ int scan_class(const TableCols& tc, const TQuery& tq)
 // Batch order for the scan, grouped by scan_class: the warps of a block (and the blocks
 // of the grid) then run the same scan_query_tile instantiation at the same time instead of
 // cycling through eight code paths per tile (instruction-cache misses were the top stall,
-// "no_instruction", in profiles/ncu_table_scan_r01s4.txt).  The order inside a class is
+// "no_instruction", in profiles/r01/ncu_table_scan_r01s4.txt).  The order inside a class is
 // whatever the shared atomics give: each query's partials are still folded in tile and
-// block order, so results do not depend on it.
+// range order, so results do not depend on it.
 __global__ void __launch_bounds__(1024) table_order_kernel(TableCols tc, int64_t nq, const TQuery* __restrict__ qs,
                                                            int32_t* __restrict__ perm) {
     __shared__ unsigned long long cnt[9];
@@ -296,38 +317,76 @@ __global__ void __launch_bounds__(1024) table_order_kernel(TableCols tc, int64_t
         perm[atomicAdd(&cnt[scan_class(tc, qs[q])], 1ull)] = (int32_t)q;
 }
 
-// The shared scan.  Block b stages tiles b, b+G, ... (all columns) into shared memory;
-// warp w evaluates queries w, w+8, ... on every staged tile.
+// The shared scan, query-chunked.  The batch (in scan order) is cut into chunks of kChunkQ =
+// 256 queries and the table into `nranges` contiguous tile ranges; block (range, chunk) -- the
+// chunks of one range adjacent in blockIdx, so they run together and share each tile through
+// L2 -- keeps its chunk's queries (SQ) and their partials in shared memory, stages its tiles
+// one by one (every referenced column) and runs the chunk's queries on each, the warps claiming
+// them one by one.  No per-(query, tile) global traffic; one partial per (range, query) at the
+// end, folded in range order by table_final_kernel.
 // OLAP_SCAN_MINBLOCKS: tuning knob (resident blocks per SM the register budget must allow).
-// Not the default: an explicit minimum of 1 let ptxas take 96 registers (2 blocks/SM,
-// T 38.3k -> 25.2k q/s), while the bare bound gives 48 (5 blocks/SM).
+constexpr int kChunkQ = kScanWarps * 32;
 #ifdef OLAP_SCAN_MINBLOCKS
 #define OLAP_SCAN_BOUNDS __launch_bounds__(kScanThreads, OLAP_SCAN_MINBLOCKS)
 #else
 #define OLAP_SCAN_BOUNDS __launch_bounds__(kScanThreads)
 #endif
 __global__ void OLAP_SCAN_BOUNDS table_scan_kernel(TableCols tc, int ncols, int64_t nrows, int64_t nq,
-                                                                  const TQuery* __restrict__ qs,
-                                                                  TPartial* __restrict__ part,
-                                                                  const uint32_t* __restrict__ colmask,
-                                                                  const int32_t* __restrict__ perm) {
-    extern __shared__ uint32_t smem[];  // ncols x kTileRows (only the batch's columns are staged)
+                                                   const TQuery* __restrict__ qs, TPartial* __restrict__ part,
+                                                   const uint32_t* __restrict__ colmask,
+                                                   const int32_t* __restrict__ perm, int nchunks,
+                                                   int64_t tiles_per_range) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    SQ* sq = reinterpret_cast<SQ*>(smem_raw);                         // kChunkQ queries
+    TPartial* acc = reinterpret_cast<TPartial*>(sq + kChunkQ);        // their partials
+    int* ctr = reinterpret_cast<int*>(acc + kChunkQ);                 // per-tile claim counters (2)
+    uint32_t* smem = reinterpret_cast<uint32_t*>(ctr + 4);            // ncols x kTileRows (the batch's columns)
     const uint32_t used = *colmask;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int chunk = (int)(blockIdx.x % (unsigned)nchunks);
+    const int64_t range = blockIdx.x / (unsigned)nchunks;
     const int64_t ntiles = (nrows + kTileRows - 1) / kTileRows;
-    TPartial* mine = part + (int64_t)blockIdx.x * nq;
-    for (int64_t q = threadIdx.x; q < nq; q += kScanThreads) {
-        TPartial p;
-        p.sum = 0;
-        p.count = 0;
-        p.code_max = INT_MIN;
-        p.code_min = INT_MIN;
-        mine[q] = p;
+    const int64_t t0 = range * tiles_per_range, t1 = min(ntiles, t0 + tiles_per_range);
+    // the chunk's queries in scan form
+    for (int i = threadIdx.x; i < kChunkQ; i += kScanThreads) {
+        const int64_t idx = (int64_t)chunk * kChunkQ + i;
+        SQ d;
+        memset(&d, 0, sizeof(d));
+        d.ncond = -1;
+        d.q = -1;
+        if (idx < nq) {
+            const int32_t q = perm[idx];
+            const TQuery& t = qs[q];
+            d.q = q;
+            if (!t.flags && t.ncond >= 0) {
+                d.ncond = t.ncond;
+                const int opk = t.op == OLAP_MIN ? 1 : t.op == OLAP_MAX ? 2 : t.op == OLAP_COUNT ? 3 : 0;
+                d.meta = t.data_col | (tc.dtype[t.data_col] == OLAP_FLOAT32 ? 1 : 0) << 8 | opk << 9;
+                for (int k = 0; k < kInlineConds && k < t.ncond; ++k) {
+                    d.colpack |= (uint32_t)t.c[k].col << (4 * k);
+                    d.lo[k] = t.c[k].lo;
+                    d.span[k] = t.c[k].span;
+                }
+            }
+        }
+        sq[i] = d;
     }
-    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    // the chunk's partials live in shared memory; per tile, warps claim the chunk's queries one at
+    // a time from a shared counter (ping-pong per tile parity), so uneven query costs balance
+    // inside the tile and the barrier waits only for the last query
+    for (int i = threadIdx.x; i < kChunkQ; i += kScanThreads) {
+        acc[i].sum = 0;
+        acc[i].count = 0;
+        acc[i].code_max = INT_MIN;
+        acc[i].code_min = INT_MIN;
+    }
+    if (threadIdx.x == 0) ctr[0] = ctr[1] = 0;
+    const int nlive = (int)min((int64_t)kChunkQ, nq - (int64_t)chunk * kChunkQ);
+    for (int64_t t = t0; t < t1; ++t) {
         const int64_t r0 = t * kTileRows;
         const int rows = (int)min((int64_t)kTileRows, nrows - r0);
-        __syncthreads();  // previous tile fully consumed
+        const int par = (int)(t & 1);
+        __syncthreads();  // previous tile fully consumed (first pass: SQ, partials, counters written)
         for (int c = 0; c < ncols; ++c) {
             if (!((used >> c) & 1u)) continue;
             const uint32_t* src = tc.col[c] + r0;
@@ -339,39 +398,46 @@ __global__ void OLAP_SCAN_BOUNDS table_scan_kernel(TableCols tc, int ncols, int6
                 for (int r = threadIdx.x; r < rows; r += kScanThreads) dst[r] = __ldg(src + r);
             }
         }
+        if (threadIdx.x == 0) ctr[par ^ 1] = 0;  // the next tile's counter (nobody claims from it now)
         __syncthreads();
-        for (int64_t i = w; i < nq; i += kScanWarps) {
-            const int64_t q = perm[i];
-            const TQuery& tq = qs[q];
-            if (tq.flags || tq.ncond < 0) continue;
-            TPartial p = mine[q];  // warp w owns these partials: no race
-            long long s = p.sum;
-            int64_t cnt = p.count;
-            int32_t cmx = p.code_max, cmn = p.code_min;
-            const int opk = tq.op == OLAP_MIN ? 1 : tq.op == OLAP_MAX ? 2 : tq.op == OLAP_COUNT ? 3 : 0;
-            if (tc.dtype[tq.data_col] == OLAP_FLOAT32) {
-                if (opk == 0) scan_query_tile<true, 0>(smem, rows, tq, lane, s, cnt, cmx, cmn);
-                else if (opk == 1) scan_query_tile<true, 1>(smem, rows, tq, lane, s, cnt, cmx, cmn);
-                else if (opk == 2) scan_query_tile<true, 2>(smem, rows, tq, lane, s, cnt, cmx, cmn);
-                else scan_query_tile<true, 3>(smem, rows, tq, lane, s, cnt, cmx, cmn);
-            } else {
-                if (opk == 0) scan_query_tile<false, 0>(smem, rows, tq, lane, s, cnt, cmx, cmn);
-                else if (opk == 1) scan_query_tile<false, 1>(smem, rows, tq, lane, s, cnt, cmx, cmn);
-                else if (opk == 2) scan_query_tile<false, 2>(smem, rows, tq, lane, s, cnt, cmx, cmn);
-                else scan_query_tile<false, 3>(smem, rows, tq, lane, s, cnt, cmx, cmn);
+        for (;;) {
+            int i = 0;
+            if (lane == 0) i = atomicAdd(&ctr[par], 1);
+            i = __shfl_sync(0xffffffffu, i, 0);
+            if (i >= nlive) break;
+            const SQ* d = sq + i;
+            const int32_t meta = d->meta;  // broadcast
+            if (d->ncond < 0) continue;
+            long long ts = 0;
+            int32_t tn = 0, tmx = INT_MIN, tmn = INT_MIN;
+            const int cls = meta >> 8;  // fl | opk << 1
+            bool hit;
+            switch (cls) {
+                case 0: hit = scan_query_tile<false, 0>(smem, rows, d, qs, lane, ts, tn, tmx, tmn); break;
+                case 2: hit = scan_query_tile<false, 1>(smem, rows, d, qs, lane, ts, tn, tmx, tmn); break;
+                case 4: hit = scan_query_tile<false, 2>(smem, rows, d, qs, lane, ts, tn, tmx, tmn); break;
+                case 6: hit = scan_query_tile<false, 3>(smem, rows, d, qs, lane, ts, tn, tmx, tmn); break;
+                case 1: hit = scan_query_tile<true, 0>(smem, rows, d, qs, lane, ts, tn, tmx, tmn); break;
+                case 3: hit = scan_query_tile<true, 1>(smem, rows, d, qs, lane, ts, tn, tmx, tmn); break;
+                case 5: hit = scan_query_tile<true, 2>(smem, rows, d, qs, lane, ts, tn, tmx, tmn); break;
+                default: hit = scan_query_tile<true, 3>(smem, rows, d, qs, lane, ts, tn, tmx, tmn); break;
             }
-            if (lane == 0) {
-                p.sum = s;
-                p.count = cnt;
-                p.code_max = cmx;
-                p.code_min = cmn;
-                mine[q] = p;
+            if (hit && lane == 0) {  // one warp per (query, tile); tiles in order: deterministic
+                TPartial& p = acc[i];
+                p.sum = (cls & 1) ? __double_as_longlong(__longlong_as_double(p.sum) + __longlong_as_double(ts))
+                                  : (long long)((unsigned long long)p.sum + (unsigned long long)ts);
+                p.count += tn;
+                p.code_max = max(p.code_max, tmx);
+                p.code_min = max(p.code_min, tmn);
             }
         }
     }
+    __syncthreads();
+    for (int i = threadIdx.x; i < nlive; i += kScanThreads)
+        if (sq[i].q >= 0) part[range * nq + sq[i].q] = acc[i];
 }
 
-// fold per-block partials in block order -> results
+// fold per-range partials in range order -> results
 __global__ void table_final_kernel(TableCols tc, int64_t nq, int nblocks, const TQuery* __restrict__ qs,
                                    const TPartial* __restrict__ part, olap_result* __restrict__ out) {
     const int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
@@ -470,6 +536,10 @@ struct olap_table_part {
 };
 
 namespace {
+
+size_t scan_smem_bytes(int ncols) {
+    return (sizeof(SQ) + sizeof(TPartial)) * kChunkQ + 4 * sizeof(int) + sizeof(uint32_t) * kTileRows * ncols;
+}
 
 struct TDevGuard {
     int prev = -1;
@@ -576,8 +646,18 @@ int ensure_staging(olap_table* t, int64_t nq, int64_t nconds) {
 // scan + fold, after a prep kernel has written w.d_qs and w.d_colmask on `st`
 int launch_scan_fold(olap_table* t, TWork& w, int64_t nq, olap_result* d_res, cudaStream_t st) {
     const TableCols tc = cols_of(t);
-    const size_t smem = sizeof(uint32_t) * kTileRows * t->ncols;
+    const size_t smem = scan_smem_bytes(t->ncols);
     if (nq > INT32_MAX) return set_error(OLAP_E_INVALID, "table batch of %lld queries: at most 2^31-1", (long long)nq);
+    // (range, chunk) blocks: one resident wave when the batch has at most w.blocks chunks
+    const int64_t nchunks = (nq + kChunkQ - 1) / kChunkQ;
+    if (nchunks > INT32_MAX / 2) return set_error(OLAP_E_INVALID, "table batch too large");
+    const int64_t ntiles = (t->nrows + kTileRows - 1) / kTileRows;
+    int64_t nranges = std::max<int64_t>(1, w.blocks / nchunks);
+    nranges = std::min(nranges, ntiles);
+    const int64_t per = (ntiles + nranges - 1) / nranges;
+    nranges = (ntiles + per - 1) / per;
+    const int64_t grid = nranges * nchunks;
+    if (grid > INT32_MAX) return set_error(OLAP_E_INVALID, "table batch too large");
     table_order_kernel<<<1, 1024, 0, st>>>(tc, nq, w.d_qs, w.d_perm);
     const bool prof = t->prof && &w == &t->work && !stream_capturing(st);
     if (prof) {
@@ -588,13 +668,13 @@ int launch_scan_fold(olap_table* t, TWork& w, int64_t nq, olap_result* d_res, cu
         }
         OLAP_CUDA_TRY(cudaEventRecord(t->ev[t->ev_used], st));
     }
-    table_scan_kernel<<<w.blocks, kScanThreads, smem, st>>>(tc, t->ncols, t->nrows, nq, w.d_qs, w.d_part, w.d_colmask,
-                                                            w.d_perm);
+    table_scan_kernel<<<(unsigned)grid, kScanThreads, smem, st>>>(tc, t->ncols, t->nrows, nq, w.d_qs, w.d_part,
+                                                                   w.d_colmask, w.d_perm, (int)nchunks, per);
     if (prof) {
         OLAP_CUDA_TRY(cudaEventRecord(t->ev[t->ev_used + 1], st));
         t->ev_used += 2;
     }
-    table_final_kernel<<<(int)((nq + 255) / 256), 256, 0, st>>>(tc, nq, w.blocks, w.d_qs, w.d_part, d_res);
+    table_final_kernel<<<(int)((nq + 255) / 256), 256, 0, st>>>(tc, nq, (int)nranges, w.d_qs, w.d_part, d_res);
     OLAP_CUDA_TRY(cudaGetLastError());
     if (!stream_capturing(st)) OLAP_CUDA_TRY(cudaEventRecord(w.done, st));
     __atomic_fetch_add(&t->launches, 4, __ATOMIC_RELAXED);
@@ -652,7 +732,7 @@ int olap_table_create(int64_t nrows, int ncols, const int32_t* dtypes, int devic
     }
     cudaStreamCreateWithFlags(&t->stream, cudaStreamNonBlocking);
     cudaDeviceGetAttribute(&t->num_sms, cudaDevAttrMultiProcessorCount, device);
-    const size_t smem = sizeof(uint32_t) * kTileRows * ncols;
+    const size_t smem = scan_smem_bytes(ncols);
     if (smem > 48 * 1024)
         cudaFuncSetAttribute(table_scan_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     int bps = 0;

@@ -530,7 +530,7 @@ def test_c5_slice_full_size_sampled():
 
 def test_c5_slice_bricked_full_size_sampled():
     """C5 as bench.py runs it: the 128 GiB slice in the bricked layout (R26)."""
-    _sampled_full_size("C5", 50, 400, 2_000_000, np.array([2, 1, 1, 1], float), layout=olap.LAYOUT_BRICK)
+    _sampled_full_size("C5", 50, 400, 2_000_000, np.array([2, 1, 1, 1], float), layout=olap.LAYOUT_BRICK3)
 
 
 # ------------------------------------------------------------------ fact tables (NEXT #1)
@@ -578,6 +578,38 @@ def test_table_scan_parity(nrows):
     assert (np.abs(got["d"] - ref["d"]) <= tol).all()
     with pytest.raises(olap.OlapError):
         t.query([([(5, 0, 1)], 4, olap.SUM)])             # condition on a float column
+
+
+def test_table_scan_chunks_and_long_conditions():
+    """The scan keeps 256-query chunks in shared memory with their first 4 conditions inline:
+    batches of 1 .. 1,300 queries (ragged last chunk) and queries with 5-9 conditions (the rest
+    read from the query descriptor) against oracle.tablescan."""
+    nrows = 70_001
+    rng = np.random.default_rng(77)
+    cols = _table_cols(nrows, rng)
+    t = olap.Table(nrows, [c.dtype for c in cols])
+    for i, c in enumerate(cols):
+        t.load_column(i, c)
+    qs = _table_queries(rng, 1300)
+    for k in range(0, 1300, 7):  # every 7th query: 5-9 conditions, repeated columns narrowing the range
+        conds = []
+        for j in range(5 + k % 5):
+            c = j % 4
+            n = (40, 7, 13, 5)[c]
+            conds.append((c, int(rng.integers(-1, 2 + j % 3)), int(n - rng.integers(0, 2 + j % 3))))
+        qs[k] = (conds, int(rng.integers(4, 6)), int(rng.integers(0, 5)))
+    for nq in (1, 255, 256, 257, 1300):
+        sub = qs[:nq]
+        got = t.query(sub)
+        ref = oracle.tablescan(cols, sub, nthreads=oracle.max_threads())
+        ops = np.array([q[2] for q in sub], np.int32)
+        isf = np.array([cols[q[1]].dtype == np.float32 for q in sub])
+        assert np.array_equal(got["flags"], ref["flags"]) and np.array_equal(got["i"], ref["i"]), nq
+        ex = ~isf | (ops == olap.MIN) | (ops == olap.MAX) | (ops == olap.COUNT)
+        assert np.array_equal(got["d"][ex], ref["d"][ex]), nq
+        assert (np.abs(got["d"] - ref["d"]) <= 1e-6 * np.abs(ref["d"]) + 1e-300).all(), nq
+    # deterministic: the same batch twice gives bit-identical results
+    assert np.array_equal(t.query(qs).view(np.uint8), t.query(qs).view(np.uint8))
 
 
 # ------------------------------------------------------------------ multi-resolution cube set (NEXT #3)
