@@ -661,12 +661,18 @@ def run_resolution(args, rank, world):
     for k in range(warm):
         cs.query(*batches_[k])
     torch.cuda.synchronize()
+    k0 = sum(c.stats()[0] for c in cubes.values())
+    clocks = Clocks(0)
+    clocks.mark(True)
     t0 = time.perf_counter()
     used_hist = np.zeros(3, np.int64)
     for k in range(warm, warm + steps):
         _, used = cs.query(*batches_[k])
         used_hist += np.bincount(used[used >= 0], minlength=3)
     routed_s = time.perf_counter() - t0
+    clocks.mark(False)
+    clk = clocks.stop()
+    launches = sum(c.stats()[0] for c in cubes.values()) - k0
     # the same queries answered on the day cube only (conditions converted to days)
     conv = [(h.convert(b[0], b[1], 2), b[2]) for b in batches_]
     for k in range(warm):
@@ -685,7 +691,10 @@ def run_resolution(args, rank, world):
                    "rollup_s": rollup_s, "queries_per_level_used": used_hist.tolist()},
         "day_cube_only": {"value": nq * steps / day_s, "unit": "queries/s"},
         "e2e": {"value": nq * steps / routed_s, "unit": "queries/s", "api": "olap_cubeset_query (host buffers)"},
-        "cpu_baseline": None, "roofline": None, "gpu_launches": None,
+        "cpu_baseline": None, "roofline": None, "gpu_launches": int(launches), "clocks": clk,
+        "note": "NEXT #3 (cube set + Eq. 2 routing): host-timed through the public API (routing is host logic, "
+                "every routed sub-batch an olap_query_batch); no roofline (the per-cube kernels are the C1/C2 "
+                "paths) and no CPU baseline for this secondary line",
     }
     print(json.dumps(line), flush=True)
     return 0

@@ -80,6 +80,7 @@ struct SDesc {
 };
 static_assert(sizeof(SDesc) == 128, "one line per query");
 
+
 // ------------------------------------------------------------------ mbarrier / bulk copy (PTX)
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -450,30 +451,37 @@ __device__ __forceinline__ void build_pair_desc(const TGeo& tg, const TDesc& d, 
 // level j holds one entry per aligned block of 2^j slots, combined from level j-1 (float SUM: the fp32
 // tree continues, so a level-5 entry is an fp32 tree of 256 cells, depth 8, reading R8').  Any slot
 // range [a, b) is the union of at most two entries per level (plus whole level-kTreeTop entries):
-// a run's interior costs O(log) lookups instead of one per slot.  Entries live at padded indices
-// (sw(i) = i + i / 32: one spare entry per 32) so that lanes walking runs one 32-slot row apart hit
-// different banks at every level.  Written by the producer warp once per tile.
+// a run's interior costs O(log) lookups instead of one per slot.  Each level is stored TRANSPOSED
+// over 256-cell rows: node n of level j (row n >> (5 - j), column n mod 2^(5-j)) sits at column x
+// kTreeRows + row.  The same node of runs one or more rows apart is then consecutive entries (no
+// bank conflicts across lanes walking such runs, and a run-to-run step is a constant address
+// increment); kTreeRows is odd so that the columns of one row spread over the banks too.  Written
+// by the producer warp once per tile.
 constexpr int kTileSlots = (int)((kTileCellsMax + 7) / 8);
 #ifndef OLAP_COL_SLOTS
 #define OLAP_COL_SLOTS 4
 #endif
 constexpr uint32_t kColSlots = OLAP_COL_SLOTS;  // runs of at most this many slots: column mode on raw cells
 #ifndef OLAP_PAT_MAX_RUNS
-#define OLAP_PAT_MAX_RUNS 16
+#define OLAP_PAT_MAX_RUNS (1u << 30)
 #endif
-// pairs of at most this many runs take the per-query pattern (long runs, few of them: C3); more
-// runs are walked through the trees one run per lane (C2a measured equal either way)
+// pairs of at most this many runs take the per-query pattern (every row-aligned pair by default;
+// before the transposed trees, pairs of > 16 runs were walked one run per lane at equal speed)
 constexpr uint32_t kPatMaxRuns = OLAP_PAT_MAX_RUNS;
-constexpr int lvl_size(int j) { return (((kTileSlots + (1 << j) - 1) >> j) + 1 + 31) & ~31; }
+constexpr int kTreeRows = (kTileSlots + 31) / 32 + ((((kTileSlots + 31) / 32) & 1) ? 0 : 1);  // odd
+constexpr int lvl_size(int j) { return (32 >> j) * kTreeRows; }
 constexpr int lvl_off(int j) { return j == 0 ? 0 : lvl_off(j - 1) + lvl_size(j - 1); }
-constexpr int kTreeEntries = lvl_off(kTreeTop + 1) + lvl_off(kTreeTop + 1) / 32 + 1;  // padded
-__device__ __forceinline__ uint32_t sw(uint32_t i) { return i + (i >> 5); }
+constexpr int kTreeEntries = lvl_off(kTreeTop + 1);
 __device__ __forceinline__ uint32_t lvl_off_dev(int j) {
     // lvl_off(j) for j in [0, kTreeTop] (constexpr table folded by the compiler)
     constexpr uint32_t o[kTreeTop + 1] = {lvl_off(0), lvl_off(1), lvl_off(2), lvl_off(3), lvl_off(4), lvl_off(5)};
     return o[j];
 }
 __constant__ uint32_t kLvlOff[kTreeTop + 1] = {lvl_off(0), lvl_off(1), lvl_off(2), lvl_off(3), lvl_off(4), lvl_off(5)};
+// entry index of node n at level j
+__device__ __forceinline__ uint32_t tidx(int j, uint32_t n) {
+    return lvl_off_dev(j) + (n & ((32u >> j) - 1u)) * (uint32_t)kTreeRows + (n >> (5 - j));
+}
 template <class Acc> struct SumEntry;
 template <> struct SumEntry<AccF> { using T = float; };
 template <> struct SumEntry<AccI> { using T = long long; };
@@ -506,11 +514,11 @@ __device__ __forceinline__ void summarize_tile(const uint32_t* __restrict__ sb, 
                                                int lane) {
     TreeView<Acc> tv(base);
     uint32_t n = (ncell + 7) >> 3;
-    for (uint32_t s = lane; s < n; s += 32) {
+    // level 0: slot s = lane + 32 it is column lane of row it
+    for (uint32_t s = lane, i = lane * (uint32_t)kTreeRows; s < n; s += 32, ++i) {
         const uint4 a = *reinterpret_cast<const uint4*>(sb + 8 * s);
         const uint4 b = *reinterpret_cast<const uint4*>(sb + 8 * s + 4);
         const uint32_t v[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
-        const uint32_t i = sw(s);
         if constexpr (std::is_same<Acc, AccF>::value) {
             tv.sum[i] = slot_tree<8>(v);
             float mn = __uint_as_float(v[0]), mx = mn;
@@ -540,10 +548,12 @@ __device__ __forceinline__ void summarize_tile(const uint32_t* __restrict__ sb, 
 #pragma unroll 1
     for (int j = 1; j <= kTreeTop; ++j) {
         __syncwarp();
-        const uint32_t o0 = lvl_off_dev(j - 1), o1 = lvl_off_dev(j);
         n = (n + 1) >> 1;
         for (uint32_t k = lane; k < n; k += 32) {
-            const uint32_t c0 = sw(o0 + 2 * k), c1 = sw(o0 + 2 * k + 1), d = sw(o1 + k);
+            // node k = (column c, row r) of level j; its children are columns 2c, 2c + 1 of row r
+            const uint32_t c = k & ((32u >> j) - 1u), r = k >> (5 - j);
+            const uint32_t d = lvl_off_dev(j) + c * (uint32_t)kTreeRows + r;
+            const uint32_t c0 = lvl_off_dev(j - 1) + 2 * c * (uint32_t)kTreeRows + r, c1 = c0 + (uint32_t)kTreeRows;
             if constexpr (std::is_same<Acc, AccF>::value) {
                 tv.sum[d] = tv.sum[c0] + tv.sum[c1];
                 tv.mn[d] = __float_as_int(fminf(__int_as_float(tv.mn[c0]), __int_as_float(tv.mn[c1])));
@@ -614,14 +624,13 @@ __device__ __forceinline__ void fold_range(const TreeView<Acc>& tv, uint32_t a, 
 #pragma unroll
     for (int j = 0; j < kTreeTop; ++j) {
         if (a >= b) return;
-        const uint32_t o = lvl_off_dev(j);
-        if (a & 1u) fold_entry<Acc, OPC>(tv, sw(o + a++), acc);
-        if (b & 1u) fold_entry<Acc, OPC>(tv, sw(o + --b), acc);
+        if (a & 1u) fold_entry<Acc, OPC>(tv, tidx(j, a++), acc);
+        if (b & 1u) fold_entry<Acc, OPC>(tv, tidx(j, --b), acc);
         a >>= 1;
         b >>= 1;
     }
-    const uint32_t o = lvl_off_dev(kTreeTop);
-    for (; a < b; ++a) fold_entry<Acc, OPC>(tv, sw(o + a), acc);
+    const uint32_t o = lvl_off_dev(kTreeTop);  // one node per row: column 0
+    for (; a < b; ++a) fold_entry<Acc, OPC>(tv, o + a, acc);
 }
 
 template <typename T, class Acc, int OPC>
@@ -683,12 +692,14 @@ __device__ __forceinline__ void pair_summary(const uint32_t* __restrict__ sb, un
     }
 }
 
-// A pair whose runs all start at the same slot of a 32-slot row (SDesc.npat >= 0): the interior
-// of every run is the same K tree entries (level j, node (rb >> j) + off, rb = the run's row start
-// slot) and the same E edge cells.  One unit = one tree entry or one edge cell of one run; lanes =
-// (run group, unit) with U = K + E <= 32 units per run and 32 / U runs per step, every lane keeping
-// one unit for the whole pair: a step is one load and one fold per lane, no decomposition, no
-// divisions, addresses advanced by fixed increments (kt rows outside, the inner digit inside).
+// A pair whose runs all start at the same slot of a 32-slot (256-cell) row (SDesc.npat >= 0): the
+// interior of every run is the same K tree entries (level j, node (rb >> j) + off, rb = the run's
+// row start slot) and the same E edge cells.  One unit = one tree entry or one edge cell of one run;
+// lanes = (run group, unit) with U = K + E <= 32 units per run and 32 / U runs per step, every lane
+// keeping one unit for the whole pair.  Runs start whole rows apart and the trees are stored
+// transposed over rows, so a lane's address advances by a fixed byte step per run (inner digit) and
+// per kt row: a step is one load, one fold and one add per lane -- no decomposition, no division,
+// no per-load index arithmetic.
 template <typename T, class Acc, int OPC>
 __device__ __forceinline__ void pair_pattern(const uint32_t* __restrict__ sb, unsigned char* __restrict__ tree,
                                              uint32_t al, uint32_t h0, uint32_t L, uint32_t rad, uint32_t na,
@@ -702,44 +713,46 @@ __device__ __forceinline__ void pair_pattern(const uint32_t* __restrict__ sb, un
     const uint32_t ulane = (uint32_t)lane;
     const uint32_t g = small_div(32u, U), grp = small_div(ulane, U), u = ulane - grp * U;
     const uint32_t pw = __shfl_sync(0xffffffffu, patw, (int)(u >> 1) & 7);
+    if (na > rad) {  // runs are (kt row, inner digit) pairs either way: split the longer side among the groups
+        const uint32_t t = na;
+        na = rad;
+        rad = t;
+        const uint32_t ts = rs;
+        rs = skt;
+        skt = ts;
+    }
     if (grp >= g) return;
     const bool is_tree = u < K;
     constexpr bool wide_sum = std::is_same<Acc, AccI>::value && OPC == OPC_SUM;  // int64 tree entries
-    const uint32_t rs8 = rs >> 3, skt8 = skt >> 3;  // row-aligned: multiples of 32 slots
-    uint32_t pos, dinner, dkt, base, sh;
+    uint32_t addr, step_in, step_kt;  // shared-memory byte address of run (grp, kt row 0) and its steps
     if (is_tree) {
         const uint32_t pt = (u & 1u) ? pw >> 16 : pw & 0xffffu;
         const uint32_t j = pt >> 13, off = pt & 0x1fffu;
-        const uint32_t rb0 = (al >> 3) & ~31u;
-        pos = kLvlOff[j] + (rb0 >> j) + off + ((grp * rs8) >> j);
-        dinner = (g * rs8) >> j;
-        dkt = skt8 >> j;
+        const uint32_t row0 = al >> 8, rsr = rs >> 8, sktr = skt >> 8;  // rows of 256 cells
+        const uint32_t idx = kLvlOff[j] + (off & ((32u >> j) - 1u)) * (uint32_t)kTreeRows + (off >> (5 - j)) +
+                             row0 + grp * rsr;
         const TreeView<Acc> tv(tree);
-        base = smem_addr_u32(OPC == OPC_SUM ? (const void*)tv.sum : (OPC == OPC_MIN ? (const void*)tv.mn
-                                                                                     : (const void*)tv.mx));
-        sh = wide_sum ? 3u : 2u;
+        const uint32_t esz = wide_sum ? 8u : 4u;
+        addr = smem_addr_u32(OPC == OPC_SUM ? (const void*)tv.sum
+                                            : (OPC == OPC_MIN ? (const void*)tv.mn : (const void*)tv.mx)) + idx * esz;
+        step_in = g * rsr * esz;
+        step_kt = sktr * esz;
     } else {
         const uint32_t e = u - K;
-        pos = al + (e < E1 ? h0 + e : 8 * (nslot - 1) + (e - E1)) + grp * rs;
-        dinner = g * rs;
-        dkt = skt;
-        base = smem_addr_u32(sb);
-        sh = 2u;
+        addr = smem_addr_u32(sb) + 4u * (al + (e < E1 ? h0 + e : 8 * (nslot - 1) + (e - E1)) + grp * rs);
+        step_in = 4u * g * rs;
+        step_kt = 4u * skt;
     }
-    auto fold_one = [&](uint32_t p) {
-        const uint32_t addr = base + ((is_tree ? sw(p) : p) << sh);
-        if constexpr (wide_sum) {
-            long long x;
-            if (is_tree) asm volatile("ld.shared.s64 %0, [%1];" : "=l"(x) : "r"(addr));
-            else {
-                int32_t y;
-                asm volatile("ld.shared.s32 %0, [%1];" : "=r"(y) : "r"(addr));
-                x = y;
-            }
+    auto fold_one = [&](uint32_t a) {
+        if constexpr (wide_sum) {  // tree lanes: 64-bit entry (two 32-bit halves); edge lanes: one cell
+            uint32_t lo, hi = 0;
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(lo) : "r"(a));
+            if (is_tree) asm volatile("ld.shared.u32 %0, [%1];" : "=r"(hi) : "r"(a + 4u));
+            const long long x = is_tree ? (long long)(((unsigned long long)hi << 32) | lo) : (long long)(int32_t)lo;
             acc.s += (unsigned long long)x;
         } else {
             uint32_t v;
-            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
             if constexpr (OPC == OPC_SUM) acc.s += (double)__uint_as_float(v);
             else if constexpr (OPC == OPC_MIN) {
                 if constexpr (std::is_same<Acc, AccF>::value) acc.mn = fminf(acc.mn, __uint_as_float(v));
@@ -751,13 +764,28 @@ __device__ __forceinline__ void pair_pattern(const uint32_t* __restrict__ sb, un
         }
     };
     (void)sizeof(ST);
-    for (uint32_t kr = 0; kr < na; ++kr, pos += dkt) {
-        uint32_t p = pos, ri = grp;
-        for (; ri + g < rad; ri += 2 * g, p += 2 * dinner) {  // two runs per lane in flight
-            fold_one(p);
-            fold_one(p + dinner);
+    constexpr bool fsum = std::is_same<Acc, AccF>::value && OPC == OPC_SUM;
+    for (uint32_t kr = 0; kr < na; ++kr, addr += step_kt) {
+        uint32_t a = addr, ri = grp;
+        for (; ri + 3 * g < rad; ri += 4 * g, a += 4 * step_in) {  // four runs per lane in flight
+            if constexpr (fsum) {
+                // float SUM: the four values (tree entries of depth <= 8, or cells) as one fp32 tree of
+                // depth 2, then one conversion and one fp64 add (reading R8': fp32 depth <= 10)
+                uint32_t v0, v1, v2, v3;
+                asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v0) : "r"(a));
+                asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v1) : "r"(a + step_in));
+                asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v2) : "r"(a + 2 * step_in));
+                asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v3) : "r"(a + 3 * step_in));
+                acc.s += (double)((__uint_as_float(v0) + __uint_as_float(v1)) +
+                                  (__uint_as_float(v2) + __uint_as_float(v3)));
+            } else {
+                fold_one(a);
+                fold_one(a + step_in);
+                fold_one(a + 2 * step_in);
+                fold_one(a + 3 * step_in);
+            }
         }
-        if (ri < rad) fold_one(p);
+        for (; ri < rad; ri += g, a += step_in) fold_one(a);
     }
 }
 
