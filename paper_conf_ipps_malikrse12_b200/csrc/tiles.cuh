@@ -95,7 +95,7 @@ __device__ __forceinline__ void mbar_arrive_tx(uint64_t* b, uint32_t bytes) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
 }
 // A wait that never completes is a bug (a phase nobody will reach); rather than hang the GPU, a
-// waiter that has spun for ~8 s traps the kernel (cudaErrorLaunchFailure: an error, not a hang).
+// waiter that has waited ~8 s traps the kernel (cudaErrorLaunchFailure: an error, not a hang).
 constexpr long long kWaitTrapCycles = 16ll * 1000 * 1000 * 1000;
 __device__ __forceinline__ bool mbar_try(uint64_t* b, uint32_t parity) {
     uint32_t ok = 0;
@@ -110,30 +110,35 @@ __device__ __forceinline__ bool mbar_try(uint64_t* b, uint32_t parity) {
         : "memory");
     return ok != 0;
 }
-// producer side: back off between probes (keeps the spin off the issue slots)
-__device__ __forceinline__ void mbar_wait_sleep(uint64_t* b, uint32_t parity) {
-    if (mbar_try(b, parity)) return;
-    const long long t0 = clock64();
-    for (;;) {
-        if (mbar_try(b, parity)) return;
-        __nanosleep(256);
-        if (clock64() - t0 > kWaitTrapCycles) __trap();
-    }
+// try_wait with a suspend-time hint: the warp is suspended in hardware until the phase completes
+// (or the hint expires) instead of spinning on the issue slots the reducing warps need (a spin
+// loop with __nanosleep took 13% of the kernel's instructions once the consumers got faster)
+__device__ __forceinline__ bool mbar_try_suspend(uint64_t* b, uint32_t parity, uint32_t hint_ns) {
+    uint32_t ok = 0;
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n"
+        "selp.u32 %0, 1, 0, p;\n"
+        "}\n"
+        : "=r"(ok)
+        : "r"(smem_u32(b)), "r"(parity), "r"(hint_ns)
+        : "memory");
+    return ok != 0;
 }
-#ifndef OLAP_WAIT_NS
-#define OLAP_WAIT_NS 128
+#ifndef OLAP_WAIT_HINT_NS
+#define OLAP_WAIT_HINT_NS 1000000u
 #endif
 __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
     if (mbar_try(b, parity)) return;  // the common case: one probe
-    // a consumer waiting for the next stage sleeps between probes: a spinning warp would take
-    // issue slots from the warps still reducing (ncu: 7% of the kernel's instructions)
     const long long t0 = clock64();
     for (;;) {
-        if (OLAP_WAIT_NS) __nanosleep(OLAP_WAIT_NS);
-        if (mbar_try(b, parity)) return;
+        if (mbar_try_suspend(b, parity, OLAP_WAIT_HINT_NS)) return;
         if (clock64() - t0 > kWaitTrapCycles) __trap();
     }
 }
+// producer side: the same wait
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* b, uint32_t parity) { mbar_wait(b, parity); }
 // global -> shared bulk copy completing on mbarrier b (bytes: multiple of 16, both ends 16-B aligned)
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* b) {
     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
