@@ -662,17 +662,26 @@ def run_resolution(args, rank, world):
         cs.query(*batches_[k])
     torch.cuda.synchronize()
     k0 = sum(c.stats()[0] for c in cubes.values())
-    clocks = Clocks(0)
-    clocks.mark(True)
     t0 = time.perf_counter()
     used_hist = np.zeros(3, np.int64)
     for k in range(warm, warm + steps):
         _, used = cs.query(*batches_[k])
         used_hist += np.bincount(used[used >= 0], minlength=3)
     routed_s = time.perf_counter() - t0
+    launches = sum(c.stats()[0] for c in cubes.values()) - k0
+    # this line is host-bound (routing, many small synchronous batches) and a running nvidia-smi
+    # sampler slows such a loop ~2.6x (driver contention, measured): the clocks come from a second,
+    # identical pass over the same batches with the sampler on
+    clocks = Clocks(0)
+    clocks.mark(True)
+    t0 = time.perf_counter()
+    for k in range(warm, warm + steps):
+        cs.query(*batches_[k])
+    sampled_s = time.perf_counter() - t0
     clocks.mark(False)
     clk = clocks.stop()
-    launches = sum(c.stats()[0] for c in cubes.values()) - k0
+    if clk is not None:
+        clk["pass"] = f"repeat of the timed loop with the sampler running ({nq * steps / sampled_s:.0f} q/s there)"
     # the same queries answered on the day cube only (conditions converted to days)
     conv = [(h.convert(b[0], b[1], 2), b[2]) for b in batches_]
     for k in range(warm):

@@ -80,6 +80,32 @@ struct SDesc {
 };
 static_assert(sizeof(SDesc) == 128, "one line per query");
 
+// A run of L cells starting at cell h0 of its first 8-cell slot covers nslot slots.  Its tree
+// interior is slots [i0, i1) -- every FULL slot, the first and last included when they are
+// whole -- and its edge cells are E1 cells of a partial first slot (h0 ..) and E2 of a partial
+// last slot (0 .. E2-1).
+struct RunSplit {
+    uint32_t nslot, i0, i1, E1, E2;
+};
+__host__ __device__ __forceinline__ RunSplit run_split(uint32_t h0, uint32_t L) {
+    RunSplit r;
+    r.nslot = (h0 + L + 7) >> 3;
+    if (r.nslot == 1) {
+        const bool full = L == 8;  // h0 = 0
+        r.i0 = full ? 0u : 1u;
+        r.i1 = full ? 1u : 0u;
+        r.E1 = full ? 0u : L;
+        r.E2 = 0;
+    } else {
+        const uint32_t tail = h0 + L - 8 * (r.nslot - 1);
+        r.i0 = h0 ? 1u : 0u;
+        r.i1 = r.nslot - (tail < 8 ? 1u : 0u);
+        r.E1 = h0 ? 8 - h0 : 0u;
+        r.E2 = tail < 8 ? tail : 0u;
+    }
+    return r;
+}
+
 
 // ------------------------------------------------------------------ mbarrier / bulk copy (PTX)
 
@@ -265,11 +291,11 @@ __global__ void __launch_bounds__(kDescThreads) tile_desc_kernel(Geo geo, TGeo t
             if (sd.mode && !d.span && (d.nrd == 0 || (d.rs[0] & 255) == 0) && (tg.stride[kt] & 255) == 0) {
                 const uint32_t h0 = (uint32_t)(d.base_in & 7);
                 const uint32_t c0 = (uint32_t)(((d.base_in - h0) >> 3) & 31);
-                const uint32_t nslot = (uint32_t)((h0 + d.L + 7) >> 3);
+                const RunSplit rsp = run_split(h0, (uint32_t)d.L);
                 int np2 = 0;
                 bool ok = true;
-                if (nslot > 2) {
-                    uint32_t a = c0 + 1, b = c0 + nslot - 1;
+                if (rsp.i0 < rsp.i1) {
+                    uint32_t a = c0 + rsp.i0, b = c0 + rsp.i1;
                     auto emit = [&](uint32_t j, uint32_t n) {
                         if (np2 >= 16 || n >= 8192u) ok = false;
                         else sd.pat[np2++] = (uint16_t)(j << 13 | n);
@@ -587,6 +613,7 @@ __constant__ uint32_t kSmallInv[33] = {0,    65536, 32768, 21846, 16384, 13108, 
                                         2979, 2850,  2731,  2622,  2521,  2428,  2341,  2260, 2185, 2115, 2048};
 __device__ __forceinline__ uint32_t small_div(uint32_t n, uint32_t d) { return (n * kSmallInv[d]) >> 16; }
 
+
 struct RunWalk {  // lane's run cursor: off(r) for r = my, my + g, my + 2g, ...
     uint32_t off, x0, rad, dstep, s0, dcarry;
     __device__ __forceinline__ void init(uint32_t my, uint32_t g, uint32_t rad_, FastDiv fr, uint32_t rs,
@@ -643,12 +670,12 @@ __device__ __forceinline__ void pair_summary(const uint32_t* __restrict__ sb, un
                                              uint32_t al, uint32_t h0, uint32_t L, uint32_t R, uint32_t rad,
                                              uint32_t na, FastDiv fr, uint32_t rs, uint32_t skt, Acc& acc, int lane) {
     const TreeView<Acc> tv(tree);
-    const uint32_t nslot = (h0 + L + 7) >> 3;
-    const uint32_t tail = h0 + L - 8 * (nslot - 1);
+    const RunSplit rsp = run_split(h0, L);
+    const uint32_t nslot = rsp.nslot;
     const uint32_t ulane = (uint32_t)lane;
     // ---- interior slots through the trees: lane = (run, chunk)
-    if (nslot > 2) {
-        const uint32_t ni = nslot - 2;
+    if (rsp.i0 < rsp.i1) {
+        const uint32_t ni = rsp.i1 - rsp.i0;
         // C = 2^lgc chunks per run: the largest power of two with C * min(R, 32) <= 32
         const uint32_t lgc = R >= 32 ? 0u : 31u - __clz(small_div(32u, R));
         const uint32_t C = 1u << lgc;
@@ -659,7 +686,7 @@ __device__ __forceinline__ void pair_summary(const uint32_t* __restrict__ sb, un
         w.init(my, g, rad, fr, rs, skt);
         for (uint32_t r0 = 0; r0 < R; r0 += g) {
             if (r0 + my < R) {
-                const uint32_t s1 = ((al + w.off) >> 3) + 1u;
+                const uint32_t s1 = ((al + w.off) >> 3) + rsp.i0;
                 fold_range<Acc, OPC>(tv, s1 + ca, s1 + cb, acc);
             }
             w.step();
@@ -667,7 +694,8 @@ __device__ __forceinline__ void pair_summary(const uint32_t* __restrict__ sb, un
     }
     // ---- edge cells: E1 of the first slot (h0 ..), E2 of the last (0 .. tail-1); lanes = (run, cell),
     // g = 32 / E runs per step; kt rows outside, the inner digit inside (offsets advance by g * rs)
-    const uint32_t E1 = nslot == 1 ? L : 8 - h0, E2 = nslot >= 2 ? tail : 0u, E = E1 + E2;
+    const uint32_t E1 = rsp.E1, E2 = rsp.E2, E = E1 + E2;
+    if (E == 0) return;
     const uint32_t g = small_div(32u, E), grp = small_div(ulane, E), e = ulane - grp * E;
     if (grp >= g) return;
     const uint32_t cofs = e < E1 ? h0 + e : 8 * (nslot - 1) + (e - E1);
@@ -711,9 +739,8 @@ __device__ __forceinline__ void pair_pattern(const uint32_t* __restrict__ sb, un
                                              uint32_t rs, uint32_t skt, uint32_t K, uint32_t patw, Acc& acc,
                                              int lane) {
     using ST = typename SumEntry<Acc>::T;
-    const uint32_t nslot = (h0 + L + 7) >> 3;
-    const uint32_t tail = h0 + L - 8 * (nslot - 1);
-    const uint32_t E1 = nslot == 1 ? L : 8 - h0, E2 = nslot >= 2 ? tail : 0u;
+    const RunSplit rsp = run_split(h0, L);
+    const uint32_t nslot = rsp.nslot, E1 = rsp.E1, E2 = rsp.E2;
     const uint32_t U = K + E1 + E2;
     const uint32_t ulane = (uint32_t)lane;
     const uint32_t g = small_div(32u, U), grp = small_div(ulane, U), u = ulane - grp * U;
@@ -958,9 +985,8 @@ __global__ void __launch_bounds__(kTileThreads, 1)
                     if (opc == OPC_SUM) stream_cols<Acc, OPC_SUM, 8, 2>(sb, qd, acc, lane);
                     else if (opc == OPC_MIN) stream_cols<Acc, OPC_MIN, 8, 2>(sb, qd, acc, lane);
                     else stream_cols<Acc, OPC_MAX, 8, 2>(sb, qd, acc, lane);
-                } else if (w3.z >= 0 && !span && R <= kPatMaxRuns && (uint32_t)w3.z + ((h0 + L + 7) >> 3 == 1 ? L : 8 - h0) +
-                                                        (((h0 + L + 7) >> 3) >= 2 ? h0 + L - 8 * (((h0 + L + 7) >> 3) - 1)
-                                                                                  : 0u) <= 32u) {
+                } else if (w3.z >= 0 && !span && R <= kPatMaxRuns &&
+                           (uint32_t)w3.z + run_split(h0, L).E1 + run_split(h0, L).E2 <= 32u) {
                     // row-aligned runs: the precomputed per-query pattern, one unit per lane
                     const uint32_t K = (uint32_t)w3.z;
                     if (opc == OPC_SUM) pair_pattern<T, Acc, OPC_SUM>(sb, sm, al, h0, L, rad, na, rs, skt, K, patw, acc, lane);

@@ -44,6 +44,8 @@ def main():
     data = json.load(open(tp)) if os.path.exists(tp) else {}
     for p in sorted(glob.glob(os.path.join(ROOT, "gpurun_out", "traffic_*.csv"))):
         w = os.path.basename(p)[len("traffic_"):-4]
+        if w not in ("C1", "C2a", "C2b", "C3", "C4", "C5", "T", "R"):  # experiment captures are not bench workloads
+            continue
         try:
             data[w] = parse(p)
         except StopIteration:
