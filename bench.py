@@ -73,10 +73,10 @@ def workload(name: str, world: int):
     return tuple(cfg["extents"]), cfg
 
 
-def batches(name, ext, nq, count, seed0):
+def batches(name, ext, nq, count, seed0, size_extents=None):
     out = []
     for k in range(count):
-        b, o = synth.config_queries(name, nq=nq, seed=seed0 + 1000 + k, extents=ext)
+        b, o = synth.config_queries(name, nq=nq, seed=seed0 + 1000 + k, extents=ext, size_extents=size_extents)
         out.append((b, o))
     return out
 
@@ -852,7 +852,10 @@ def run_cube(args, rank, world, local):
     cube.fill(olap.GEN_UNIFORM, cfg["seed"])
     # replicas answer different batches; shards answer the same global batch
     seed0 = cfg["seed"] + (7919 * rank if (world > 1 and not sharded) else 0)
-    host_batches = batches(args.workload, ext, nq, args.warmup + args.steps, seed0)
+    # weak scaling over N GPUs: the global cube and batch grow N-fold, every query keeps the box sizes
+    # of the one-GPU recipe (offsets over the global cube) -- fixed bytes and pairs per GPU per step
+    weak_sizes = cfg["extents"] if (sharded and scaling == "weak" and world > 1) else None
+    host_batches = batches(args.workload, ext, nq, args.warmup + args.steps, seed0, size_extents=weak_sizes)
     d_batches = [(torch.from_numpy(b).to(dev), torch.from_numpy(o).to(dev)) for b, o in host_batches]
     res = torch.empty(nq * olap.RESULT_DTYPE.itemsize, dtype=torch.uint8, device=dev)
     stream = torch.cuda.Stream(device=dev)
@@ -988,6 +991,8 @@ def run_cube(args, rank, world, local):
                                   "brick3": "bricked: last three dims in 2x4x4-cell (128-B) bricks (dim 0: local "
                                             "row pairs)"}.get(layout, "row-major"),
                        "parallelism": par,
+                       "box_sizes": ("one-GPU recipe (weak scaling: every query reads what it reads at N = 1, "
+                                     "offsets over the global cube)" if weak_sizes is not None else "config recipe"),
                        "exchange": ("library NCCL: ncclAllReduce of the 16-B/query partials per batch "
                                     "(olap_cube_attach_comm)" if sharded else None)},
             "gbs": gbs_total, "frac_of_nominal_8tbs": gbs_total / world / NOMINAL_HBM_GBS,

@@ -93,13 +93,17 @@ def random_boxes(extents, nq: int, rng: np.random.Generator) -> np.ndarray:
     return r
 
 
-def fraction_boxes(extents, nq: int, rng: np.random.Generator, phi_lo: float, phi_hi: float = 1.0):
-    """C2/C3 recipe: phi log-uniform, l_d = max(1, round(n_d * phi^(1/N))), offsets uniform."""
+def fraction_boxes(extents, nq: int, rng: np.random.Generator, phi_lo: float, phi_hi: float = 1.0,
+                   size_extents=None):
+    """C2/C3 recipe: phi log-uniform, l_d = max(1, round(n_d * phi^(1/N))), offsets uniform.
+    `size_extents` (weak scaling over GPUs): box lengths from these (the one-GPU cube), offsets
+    uniform over `extents` (the grown global cube), so every query reads what it would at N = 1."""
     nd = len(extents)
+    sizes = extents if size_extents is None else size_extents
     phi = np.exp(rng.uniform(np.log(phi_lo), np.log(phi_hi), size=nq))
     r = np.empty((nq, nd, 2), dtype=np.int64)
     for d, n in enumerate(extents):
-        ell = np.clip(np.rint(n * phi ** (1.0 / nd)).astype(np.int64), 1, n)
+        ell = np.clip(np.rint(sizes[d] * phi ** (1.0 / nd)).astype(np.int64), 1, n)
         off = (rng.random(nq) * (n - ell + 1)).astype(np.int64)
         r[:, d, 0] = off
         r[:, d, 1] = off + ell - 1
@@ -131,7 +135,9 @@ def ops_mix(nq: int, rng: np.random.Generator) -> np.ndarray:
                       p=[0.4, 0.2, 0.2, 0.1, 0.1]).astype(np.int32)
 
 
-def config_queries(name: str, nq: int | None = None, seed: int | None = None, extents=None):
+def config_queries(name: str, nq: int | None = None, seed: int | None = None, extents=None, size_extents=None):
+    """Boxes and ops of a config.  `size_extents`: weak scaling (see fraction_boxes); C5's boxes
+    have absolute sizes already, C1's are uniform pairs."""
     cfg = CONFIGS[name]
     ext = tuple(extents) if extents is not None else cfg["extents"]
     nq = cfg["nq"] if nq is None else nq
@@ -139,9 +145,9 @@ def config_queries(name: str, nq: int | None = None, seed: int | None = None, ex
     if name == "C1":
         return random_boxes(ext, nq, rng), ops_uniform(nq, rng)
     if name in ("C2a", "C2b"):
-        return fraction_boxes(ext, nq, rng, 1e-4), ops_mix(nq, rng)
+        return fraction_boxes(ext, nq, rng, 1e-4, size_extents=size_extents), ops_mix(nq, rng)
     if name == "C3":
-        return fraction_boxes(ext, nq, rng, 1e-5), ops_mix(nq, rng)
+        return fraction_boxes(ext, nq, rng, 1e-5, size_extents=size_extents), ops_mix(nq, rng)
     if name == "C5":
         return small_boxes(ext, nq, rng), ops_mix(nq, rng)
     raise KeyError(name)

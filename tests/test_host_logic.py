@@ -148,6 +148,25 @@ def test_bench_scaling_modes():
     assert bench.default_scaling("C3") == "strong" and bench.default_scaling("C2a") == "weak"
 
 
+def test_bench_weak_scaling_keeps_per_query_work():
+    """Weak scaling over N GPUs: the batch of N x 4,096 queries on the N-fold cube keeps the box
+    sizes of the one-GPU recipe (the same phi draws give the same lengths), offsets span the global
+    cube, so the bytes per GPU per step stay those of N = 1 and queries/s can grow N-fold."""
+    import bench
+    import synth
+    base = synth.CONFIGS["C2a"]["extents"]
+    ext, nq = bench.scaled_workload("C2a", 4, "weak")
+    one = synth.config_queries("C2a", nq=nq, seed=99, extents=base)[0]
+    weak = bench.batches("C2a", ext, nq, 1, 99 - 1000, size_extents=base)[0][0]
+    assert np.array_equal(weak[:, :, 1] - weak[:, :, 0], one[:, :, 1] - one[:, :, 0])
+    assert (weak[:, :, 0] >= 0).all() and (weak[:, :, 1] < np.array(ext)).all()
+    assert weak[:, 0, 1].max() >= base[0]  # offsets reach beyond the one-GPU rows
+    # block-cyclic shards (b = 1) own rows r = g mod N: each GPU's owned rows sum to ~1/N of them
+    owned = [sum(len(range(lo + ((g - lo) % 4), hi + 1, 4)) for lo, hi in weak[:, 0]) for g in range(4)]
+    total = int((weak[:, 0, 1] - weak[:, 0, 0] + 1).sum())
+    assert sum(owned) == total and max(owned) <= 1.05 * total / 4
+
+
 def test_bench_refuses_mismatched_world():
     """--gpus N under a launcher that started a different number of ranks is an error, never a
     silent 1-GPU run (VERDICT r1 weak #6)."""
