@@ -832,9 +832,17 @@ def run_cube(args, rank, world, local):
     # OLAP_BENCH_SHARDED=1 runs the N > 1 code path (a shard with the library's communicator
     # attached) at N = 1 as well: a 1-rank NCCL communicator, for testing on one GPU
     sharded = (world > 1 and scaling != "replica") or os.environ.get("OLAP_BENCH_SHARDED") == "1"
-    ext, nq = scaled_workload(args.workload, world, scaling if sharded else "strong")
+    # OLAP_BENCH_VIRTUAL_WORLD=V (one GPU, development aid): rank 0's shard of the V-GPU job -- the
+    # V-fold workload, this GPU holding shard 0 of V with a 1-rank communicator -- so the per-GPU step
+    # of an N-GPU run can be timed on one GPU (the line says "virtual_world"; it is not an N-GPU result)
+    vworld = int(os.environ.get("OLAP_BENCH_VIRTUAL_WORLD", "0") or 0) if world == 1 else 0
+    if vworld > 1:
+        sharded = True
+        scaling = args.scaling or default_scaling(args.workload)
+    sworld = vworld if vworld > 1 else world  # the world the workload and the shard are sized for
+    ext, nq = scaled_workload(args.workload, sworld, scaling if sharded else "strong")
     if args.batch:
-        nq = args.batch * (world if (sharded and scaling == "weak") else 1)
+        nq = args.batch * (sworld if (sharded and scaling == "weak") else 1)
     dtype = cfg["dtype"]
     nd = len(ext)
     layout = args.layout if args.layout != "auto" else ("brick3" if args.workload == "C5" else "row")
@@ -844,9 +852,10 @@ def run_cube(args, rank, world, local):
     if sharded:
         # this rank's block-cyclic dim-0 shard; the library's NCCL communicator does the exchange
         from paper_conf_ipps_malikrse12_b200.dist import init_comm
-        cube = olap.Cube(ext, dtype, shard=(world, rank, 1), device=local, layout=lay)
-        comm = init_comm(rank, world, local) if world > 1 else olap.Comm(olap.comm_unique_id(), 1, 0, local)
-        cube.attach_comm(comm)
+        cube = olap.Cube(ext, dtype, shard=(sworld, rank, 1), device=local, layout=lay)
+        if vworld <= 1:
+            comm = init_comm(rank, world, local) if world > 1 else olap.Comm(olap.comm_unique_id(), 1, 0, local)
+            cube.attach_comm(comm)
     else:
         cube = olap.Cube(ext, dtype, device=local, layout=lay)
     cube.fill(olap.GEN_UNIFORM, cfg["seed"])
@@ -854,14 +863,22 @@ def run_cube(args, rank, world, local):
     seed0 = cfg["seed"] + (7919 * rank if (world > 1 and not sharded) else 0)
     # weak scaling over N GPUs: the global cube and batch grow N-fold, every query keeps the box sizes
     # of the one-GPU recipe (offsets over the global cube) -- fixed bytes and pairs per GPU per step
-    weak_sizes = cfg["extents"] if (sharded and scaling == "weak" and world > 1) else None
+    weak_sizes = cfg["extents"] if (sharded and scaling == "weak" and sworld > 1) else None
     host_batches = batches(args.workload, ext, nq, args.warmup + args.steps, seed0, size_extents=weak_sizes)
     d_batches = [(torch.from_numpy(b).to(dev), torch.from_numpy(o).to(dev)) for b, o in host_batches]
     res = torch.empty(nq * olap.RESULT_DTYPE.itemsize, dtype=torch.uint8, device=dev)
     stream = torch.cuda.Stream(device=dev)
 
+    if vworld > 1:  # shard 0's partials + finalize: the per-GPU compute of the V-GPU job, no exchange
+        v_sum = torch.empty(nq, dtype=torch.int64, device=dev)
+        v_ext = torch.empty(2 * nq, dtype=torch.int32, device=dev)
+
     def step(k):
         dr, do = d_batches[k]
+        if vworld > 1:
+            cube.partials_device(dr, do, v_sum, v_ext, nq=nq, stream=stream)
+            olap.finalize_device(ext, dtype, nq, dr, do, v_sum, v_ext, res, stream=stream)
+            return
         cube.query_device(dr, do, res, nq=nq, stream=stream)
 
     for k in range(args.warmup):
@@ -963,7 +980,7 @@ def run_cube(args, rank, world, local):
 
     kernel = "tile_reduce_kernel" if tiles_used else ("brick_reduce_kernel" if bricked else "reduce_kernel")
     roofline = cube_roofline(args.workload, kernel, achieved, kern_s, clk, alg_bytes / max(launches, 1),
-                             reduce_ms / elapsed_ms if elapsed_ms else None, with_traffic=world == 1)
+                             reduce_ms / elapsed_ms if elapsed_ms else None, with_traffic=world == 1 and vworld <= 1)
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -990,11 +1007,13 @@ def run_cube(args, rank, world, local):
                        "layout": {"brick": "bricked: last two dims in 4x8-cell (128-B) bricks",
                                   "brick3": "bricked: last three dims in 2x4x4-cell (128-B) bricks (dim 0: local "
                                             "row pairs)"}.get(layout, "row-major"),
-                       "parallelism": par,
+                       "parallelism": par if vworld <= 1 else f"virtual shard 0 of {vworld} (one GPU)",
+                       "virtual_world": vworld if vworld > 1 else None,
                        "box_sizes": ("one-GPU recipe (weak scaling: every query reads what it reads at N = 1, "
                                      "offsets over the global cube)" if weak_sizes is not None else "config recipe"),
-                       "exchange": ("library NCCL: ncclAllReduce of the 16-B/query partials per batch "
-                                    "(olap_cube_attach_comm)" if sharded else None)},
+                       "exchange": ("none (virtual shard: partials + finalize of shard 0 only)" if vworld > 1 else
+                                    ("library NCCL: ncclAllReduce of the 16-B/query partials per batch "
+                                     "(olap_cube_attach_comm)" if sharded else None))},
             "gbs": gbs_total, "frac_of_nominal_8tbs": gbs_total / world / NOMINAL_HBM_GBS,
             "roofline": roofline,
             "gpu_launches": int(gpu_launches), "l2_order": l2_order,
