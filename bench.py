@@ -852,7 +852,8 @@ def run_cube(args, rank, world, local):
     if sharded:
         # this rank's block-cyclic dim-0 shard; the library's NCCL communicator does the exchange
         from paper_conf_ipps_malikrse12_b200.dist import init_comm
-        cube = olap.Cube(ext, dtype, shard=(sworld, rank, 1), device=local, layout=lay)
+        vshard = int(os.environ.get("OLAP_BENCH_VIRTUAL_SHARD", "0") or 0) if vworld > 1 else rank
+        cube = olap.Cube(ext, dtype, shard=(sworld, vshard, args.shard_block), device=local, layout=lay)
         if vworld <= 1:
             comm = init_comm(rank, world, local) if world > 1 else olap.Comm(olap.comm_unique_id(), 1, 0, local)
             cube.attach_comm(comm)
@@ -1007,7 +1008,8 @@ def run_cube(args, rank, world, local):
                        "layout": {"brick": "bricked: last two dims in 4x8-cell (128-B) bricks",
                                   "brick3": "bricked: last three dims in 2x4x4-cell (128-B) bricks (dim 0: local "
                                             "row pairs)"}.get(layout, "row-major"),
-                       "parallelism": par if vworld <= 1 else f"virtual shard 0 of {vworld} (one GPU)",
+                       "parallelism": par if vworld <= 1 else f"virtual shard {vshard} of {vworld} (one GPU)",
+                       "shard_block": args.shard_block if sharded else None,
                        "virtual_world": vworld if vworld > 1 else None,
                        "box_sizes": ("one-GPU recipe (weak scaling: every query reads what it reads at N = 1, "
                                      "offsets over the global cube)" if weak_sizes is not None else "config recipe"),
@@ -1048,6 +1050,9 @@ def main():
                     help="also time the e2e queries as one olap_query_stream in batches of this size")
     ap.add_argument("--graph", action="store_true", help="replay each step as a captured CUDA graph (N=1)")
     ap.add_argument("--batch", type=int, default=0, help="queries per batch per GPU (default: the config's)")
+    ap.add_argument("--shard-block", type=int, default=None,
+                    help="block-cyclic dim-0 shard block b (rows; DESIGN.md §5, §8): row r lives on GPU (r / b) mod N; "
+                         "default 4 for C5 (small boxes: fewer (query, GPU) splits), else 1")
     ap.add_argument("--layout", default="auto", choices=["auto", "row", "brick", "brick3"],
                     help="cube layout in HBM (auto: 2x4x4 bricks for C5's small boxes, row-major otherwise; "
                          "DESIGN.md §5)")
@@ -1057,6 +1062,8 @@ def main():
     launched = "WORLD_SIZE" in os.environ
     if args.gpus is None:
         args.gpus = world
+    if args.shard_block is None:
+        args.shard_block = 4 if args.workload == "C5" else 1
     if not launched and args.gpus > 1:
         return launch_ranks(args.gpus)
     if world != args.gpus:
