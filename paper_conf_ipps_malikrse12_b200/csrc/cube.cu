@@ -1852,6 +1852,7 @@ struct olap_cube {
     unsigned int* d_tcount = nullptr;  // ntiles + 1
     unsigned int* d_tstart = nullptr;  // ntiles + 1
     uint32_t* d_nonempty = nullptr;    // ntiles
+    QDesc* d_tpds = nullptr;           // num_sms x kTileConsumers fallback descriptors of tile_reduce_kernel
     uint32_t* d_list = nullptr;        // pairs_cap
     long long* d_partial = nullptr;    // pairs_cap
     void* d_cubtmp = nullptr;
@@ -1965,6 +1966,8 @@ void free_ws(olap_cube* c) {
     cudaFree(c->d_tcount);
     cudaFree(c->d_tstart);
     cudaFree(c->d_nonempty);
+    cudaFree(c->d_tpds);
+    c->d_tpds = nullptr;
     cudaFree(c->d_list);
     cudaFree(c->d_partial);
     cudaFree(c->d_cubtmp);
@@ -1992,6 +1995,7 @@ void ensure_tile_ws(olap_cube* c, int64_t cap) {
         ok = cudaMalloc(&c->d_tcount, sizeof(unsigned int) * (3 * nt + 1)) == cudaSuccess &&
              cudaMalloc(&c->d_tstart, sizeof(unsigned int) * (3 * nt + 1)) == cudaSuccess &&
              cudaMalloc(&c->d_nonempty, sizeof(uint32_t) * nt) == cudaSuccess &&
+             cudaMalloc(&c->d_tpds, sizeof(QDesc) * (size_t)c->num_sms * kTileConsumers) == cudaSuccess &&
              cudaMalloc(&c->d_list, sizeof(uint32_t) * c->pairs_cap) == cudaSuccess &&
              cudaMalloc(&c->d_partial, sizeof(long long) * c->pairs_cap) == cudaSuccess;
         if (ok) {
@@ -2143,11 +2147,11 @@ int run_partials(olap_cube* c, int64_t nq, const olap_range* d_ranges, const int
         if (c->dtype == OLAP_INT32)
             tile_reduce_kernel<int32_t, AccI><<<c->num_sms, kTileThreads, tile_smem_bytes<AccI>(), st>>>(
                 static_cast<const int32_t*>(c->d_cells), tg, c->d_tdesc, c->d_sdesc, c->d_pstart, c->d_tstart,
-                c->d_nonempty, c->d_list, c->d_ctl, c->d_partial);
+                c->d_nonempty, c->d_list, c->d_ctl, c->d_partial, c->d_tpds);
         else
             tile_reduce_kernel<float, AccF><<<c->num_sms, kTileThreads, tile_smem_bytes<AccF>(), st>>>(
                 static_cast<const float*>(c->d_cells), tg, c->d_tdesc, c->d_sdesc, c->d_pstart, c->d_tstart,
-                c->d_nonempty, c->d_list, c->d_ctl, c->d_partial);
+                c->d_nonempty, c->d_list, c->d_ctl, c->d_partial, c->d_tpds);
         OLAP_CUDA_TRY(cudaGetLastError());
         if (prof) OLAP_CUDA_TRY(cudaEventRecord(t1, st));
         const int fg = (int)std::min<int64_t>(nq, (int64_t)c->num_sms * 8);
@@ -2378,9 +2382,10 @@ void make_tiles(olap_cube* c) {
         t.stride[k] = nd == 1 ? 1 : c->stride[k];
     }
     int kt = 0;
-    while (t.stride[kt] > kTileCellsMax) ++kt;
+    const int64_t tcap = tile_cells_max(c->dtype == OLAP_FLOAT32);
+    while (t.stride[kt] > tcap) ++kt;
     t.kt = kt;
-    int64_t ctmax = std::max<int64_t>(1, kTileCellsMax / t.stride[kt]);
+    int64_t ctmax = std::max<int64_t>(1, tcap / t.stride[kt]);
     const int64_t ekt = std::max<int64_t>(t.ext[kt], 1);
     const int64_t nch = (ekt + ctmax - 1) / ctmax;
     int64_t ct = (ekt + nch - 1) / nch;

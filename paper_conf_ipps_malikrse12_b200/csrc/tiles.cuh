@@ -24,8 +24,11 @@
 // -> tile_reduce_kernel -> pair_fold_kernel.  Every kernel of the path not chosen exits
 // at once.
 
-#ifndef OLAP_TILE_CELLS
-#define OLAP_TILE_CELLS 12288
+#ifndef OLAP_TILE_CELLS_F
+#define OLAP_TILE_CELLS_F 16384
+#endif
+#ifndef OLAP_TILE_CELLS_I
+#define OLAP_TILE_CELLS_I 12288
 #endif
 #ifndef OLAP_TILE_NO_SUMMARY
 #define OLAP_TILE_NO_SUMMARY 0  // 1: every pair through the item-path streamers (A/B of the summary path)
@@ -33,7 +36,11 @@
 #ifndef OLAP_TILE_STAGES
 #define OLAP_TILE_STAGES 2
 #endif
-constexpr int64_t kTileCellsMax = OLAP_TILE_CELLS;  // 48 KiB of 4-byte cells per tile (2 stages + slot trees)
+// Cells per tile: 64 KiB for float32 cubes, 48 KiB for int32 (whose SUM trees hold int64 entries):
+// two stages of cells + slot trees fill the 227 KiB of shared memory.  Fewer, bigger tiles mean fewer
+// (query, tile) pairs, and the per-pair set-up is a large part of the work (32-KiB tiles: C2a -22%).
+constexpr int64_t kTileCellsF = OLAP_TILE_CELLS_F, kTileCellsI = OLAP_TILE_CELLS_I;
+__host__ __device__ constexpr int64_t tile_cells_max(bool is_float) { return is_float ? kTileCellsF : kTileCellsI; }
 constexpr int kTileStages = OLAP_TILE_STAGES;
 #ifndef OLAP_TILE_WARPS
 #define OLAP_TILE_WARPS 32
@@ -488,7 +495,7 @@ __device__ __forceinline__ void build_pair_desc(const TGeo& tg, const TDesc& d, 
 // bank conflicts across lanes walking such runs, and a run-to-run step is a constant address
 // increment); kTreeRows is odd so that the columns of one row spread over the banks too.  Written
 // by the producer warp once per tile.
-constexpr int kTileSlots = (int)((kTileCellsMax + 7) / 8);
+template <class Acc> struct TreeGeo;  // slot-tree geometry of the tile size of Acc's dtype (below)
 #ifndef OLAP_COL_SLOTS
 #define OLAP_COL_SLOTS 4
 #endif
@@ -499,32 +506,31 @@ constexpr uint32_t kColSlots = OLAP_COL_SLOTS;  // runs of at most this many slo
 // pairs of at most this many runs take the per-query pattern (every row-aligned pair by default;
 // before the transposed trees, pairs of > 16 runs were walked one run per lane at equal speed)
 constexpr uint32_t kPatMaxRuns = OLAP_PAT_MAX_RUNS;
-constexpr int kTreeRows = (kTileSlots + 31) / 32 + ((((kTileSlots + 31) / 32) & 1) ? 0 : 1);  // odd
-constexpr int lvl_size(int j) { return (32 >> j) * kTreeRows; }
-constexpr int lvl_off(int j) { return j == 0 ? 0 : lvl_off(j - 1) + lvl_size(j - 1); }
-constexpr int kTreeEntries = lvl_off(kTreeTop + 1);
-__device__ __forceinline__ uint32_t lvl_off_dev(int j) {
-    // lvl_off(j) for j in [0, kTreeTop] (constexpr table folded by the compiler)
-    constexpr uint32_t o[kTreeTop + 1] = {lvl_off(0), lvl_off(1), lvl_off(2), lvl_off(3), lvl_off(4), lvl_off(5)};
-    return o[j];
-}
-__constant__ uint32_t kLvlOff[kTreeTop + 1] = {lvl_off(0), lvl_off(1), lvl_off(2), lvl_off(3), lvl_off(4), lvl_off(5)};
-// entry index of node n at level j
-__device__ __forceinline__ uint32_t tidx(int j, uint32_t n) {
-    return lvl_off_dev(j) + (n & ((32u >> j) - 1u)) * (uint32_t)kTreeRows + (n >> (5 - j));
-}
+template <class Acc>
+struct TreeGeo {
+    static constexpr int slots = (int)((tile_cells_max(std::is_same<Acc, AccF>::value) + 7) / 8);
+    static constexpr int rows = (slots + 31) / 32 + ((((slots + 31) / 32) & 1) ? 0 : 1);  // odd
+    static constexpr int entries = 63 * rows;  // levels 0..5: (32 + 16 + .. + 1) columns of `rows` entries
+    // first entry of level j: rows x (32 + 16 + .. + (32 >> (j - 1))) = rows x (64 - (64 >> j))
+    __host__ __device__ static constexpr uint32_t lvl_off(int j) { return (uint32_t)rows * (64u - (64u >> j)); }
+    // entry index of node n at level j
+    __device__ static __forceinline__ uint32_t tidx(int j, uint32_t n) {
+        return lvl_off(j) + (n & ((32u >> j) - 1u)) * (uint32_t)rows + (n >> (5 - j));
+    }
+};
 template <class Acc> struct SumEntry;
 template <> struct SumEntry<AccF> { using T = float; };
 template <> struct SumEntry<AccI> { using T = long long; };
 template <class Acc>
 constexpr size_t tile_sum_bytes() {  // one stage: sum, min, max trees
-    return ((size_t)kTreeEntries * sizeof(typename SumEntry<Acc>::T) + 2 * (size_t)kTreeEntries * 4 + 127) &
+    return ((size_t)TreeGeo<Acc>::entries * sizeof(typename SumEntry<Acc>::T) + 2 * (size_t)TreeGeo<Acc>::entries * 4 + 127) &
            ~size_t(127);
 }
 template <class Acc>
 constexpr size_t tile_smem_bytes() {
-    return (size_t)kTileStages * (kTileCellsMax + kTileSlack) * 4 + kTileStages * tile_sum_bytes<Acc>() +
-           kTileStages * sizeof(TileMeta) + 3 * kTileStages * sizeof(uint64_t) + kTileConsumers * sizeof(QDesc) + 256;
+    return (size_t)kTileStages * (tile_cells_max(std::is_same<Acc, AccF>::value) + kTileSlack) * 4 +
+           kTileStages * tile_sum_bytes<Acc>() +
+           kTileStages * sizeof(TileMeta) + 3 * kTileStages * sizeof(uint64_t) + 256;
 }
 
 template <class Acc>
@@ -535,8 +541,8 @@ struct TreeView {
     int32_t* mx;
     __device__ __forceinline__ explicit TreeView(unsigned char* base)
         : sum(reinterpret_cast<ST*>(base)),
-          mn(reinterpret_cast<int32_t*>(base + (size_t)kTreeEntries * sizeof(ST))),
-          mx(mn + kTreeEntries) {}
+          mn(reinterpret_cast<int32_t*>(base + (size_t)TreeGeo<Acc>::entries * sizeof(ST))),
+          mx(mn + TreeGeo<Acc>::entries) {}
 };
 
 // producer warp: the slot trees of the tile staged in `sb` (cells [0, ncell))
@@ -546,7 +552,8 @@ __device__ __forceinline__ void summarize_tile(const uint32_t* __restrict__ sb, 
     TreeView<Acc> tv(base);
     uint32_t n = (ncell + 7) >> 3;
     // level 0: slot s = lane + 32 it is column lane of row it
-    for (uint32_t s = lane, i = lane * (uint32_t)kTreeRows; s < n; s += 32, ++i) {
+    using TG = TreeGeo<Acc>;
+    for (uint32_t s = lane, i = lane * (uint32_t)TG::rows; s < n; s += 32, ++i) {
         const uint4 a = *reinterpret_cast<const uint4*>(sb + 8 * s);
         const uint4 b = *reinterpret_cast<const uint4*>(sb + 8 * s + 4);
         const uint32_t v[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
@@ -583,8 +590,8 @@ __device__ __forceinline__ void summarize_tile(const uint32_t* __restrict__ sb, 
         for (uint32_t k = lane; k < n; k += 32) {
             // node k = (column c, row r) of level j; its children are columns 2c, 2c + 1 of row r
             const uint32_t c = k & ((32u >> j) - 1u), r = k >> (5 - j);
-            const uint32_t d = lvl_off_dev(j) + c * (uint32_t)kTreeRows + r;
-            const uint32_t c0 = lvl_off_dev(j - 1) + 2 * c * (uint32_t)kTreeRows + r, c1 = c0 + (uint32_t)kTreeRows;
+            const uint32_t d = TG::lvl_off(j) + c * (uint32_t)TG::rows + r;
+            const uint32_t c0 = TG::lvl_off(j - 1) + 2 * c * (uint32_t)TG::rows + r, c1 = c0 + (uint32_t)TG::rows;
             if constexpr (std::is_same<Acc, AccF>::value) {
                 tv.sum[d] = tv.sum[c0] + tv.sum[c1];
                 tv.mn[d] = __float_as_int(fminf(__int_as_float(tv.mn[c0]), __int_as_float(tv.mn[c1])));
@@ -656,12 +663,12 @@ __device__ __forceinline__ void fold_range(const TreeView<Acc>& tv, uint32_t a, 
 #pragma unroll
     for (int j = 0; j < kTreeTop; ++j) {
         if (a >= b) return;
-        if (a & 1u) fold_entry<Acc, OPC>(tv, tidx(j, a++), acc);
-        if (b & 1u) fold_entry<Acc, OPC>(tv, tidx(j, --b), acc);
+        if (a & 1u) fold_entry<Acc, OPC>(tv, TreeGeo<Acc>::tidx(j, a++), acc);
+        if (b & 1u) fold_entry<Acc, OPC>(tv, TreeGeo<Acc>::tidx(j, --b), acc);
         a >>= 1;
         b >>= 1;
     }
-    const uint32_t o = lvl_off_dev(kTreeTop);  // one node per row: column 0
+    const uint32_t o = TreeGeo<Acc>::lvl_off(kTreeTop);  // one node per row: column 0
     for (; a < b; ++a) fold_entry<Acc, OPC>(tv, o + a, acc);
 }
 
@@ -761,7 +768,8 @@ __device__ __forceinline__ void pair_pattern(const uint32_t* __restrict__ sb, un
         const uint32_t pt = (u & 1u) ? pw >> 16 : pw & 0xffffu;
         const uint32_t j = pt >> 13, off = pt & 0x1fffu;
         const uint32_t row0 = al >> 8, rsr = rs >> 8, sktr = skt >> 8;  // rows of 256 cells
-        const uint32_t idx = kLvlOff[j] + (off & ((32u >> j) - 1u)) * (uint32_t)kTreeRows + (off >> (5 - j)) +
+        const uint32_t idx = TreeGeo<Acc>::lvl_off((int)j) + (off & ((32u >> j) - 1u)) * (uint32_t)TreeGeo<Acc>::rows +
+                             (off >> (5 - j)) +
                              row0 + grp * rsr;
         const TreeView<Acc> tv(tree);
         const uint32_t esz = wide_sum ? 8u : 4u;
@@ -838,17 +846,21 @@ __global__ void __launch_bounds__(kTileThreads, 1)
     tile_reduce_kernel(const T* __restrict__ cube, TGeo tg, const TDesc* __restrict__ tdesc,
                        const SDesc* __restrict__ sdesc, const int64_t* __restrict__ pair_start,
                        const unsigned int* __restrict__ tile_start, const uint32_t* __restrict__ nonempty,
-                       const uint32_t* __restrict__ list, int32_t* ctl, long long* __restrict__ partial) {
+                       const uint32_t* __restrict__ list, int32_t* ctl, long long* __restrict__ partial,
+                       QDesc* __restrict__ pds_g) {
     if (!*(volatile int32_t*)ctl) return;
     extern __shared__ __align__(128) unsigned char smem[];
-    constexpr size_t kBufBytes = (size_t)(kTileCellsMax + kTileSlack) * 4;
-    uint32_t* buf = reinterpret_cast<uint32_t*>(smem);  // kTileStages x (kTileCellsMax + kTileSlack) cells
+    constexpr int64_t kCells = tile_cells_max(std::is_same<Acc, AccF>::value);
+    constexpr size_t kBufBytes = (size_t)(kCells + kTileSlack) * 4;
+    uint32_t* buf = reinterpret_cast<uint32_t*>(smem);  // kTileStages x (kCells + kTileSlack) cells
     unsigned char* sums = smem + kTileStages * kBufBytes;  // kTileStages x tile_sum_bytes
     TileMeta* meta = reinterpret_cast<TileMeta*>(sums + kTileStages * tile_sum_bytes<Acc>());
     uint64_t* full = reinterpret_cast<uint64_t*>(meta + kTileStages);
     uint64_t* empty = full + kTileStages;
     uint64_t* ready = empty + kTileStages;
-    QDesc* pds = reinterpret_cast<QDesc*>(ready + kTileStages);
+    // the general-geometry fallback's per-warp descriptors live in global memory (L1-resident):
+    // shared memory holds two 64-KiB float stages with their trees and nothing else fits
+    QDesc* pds = pds_g + (size_t)blockIdx.x * kTileConsumers;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     if (threadIdx.x == 0) {
         for (int s = 0; s < kTileStages; ++s) {
@@ -859,7 +871,7 @@ __global__ void __launch_bounds__(kTileThreads, 1)
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
-    const int64_t bufcells = kTileCellsMax + kTileSlack;
+    const int64_t bufcells = kCells + kTileSlack;
     if (w == 0) {
         // producer warp: pop a non-empty tile, stage it with bulk copies (lane 0), wait for it to
         // land, write its slot summaries (all lanes), then release it to the consumers (ready)
