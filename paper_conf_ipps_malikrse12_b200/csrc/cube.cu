@@ -583,12 +583,25 @@ __device__ __forceinline__ void lds_slot(uint32_t pa, uint32_t pb, uint32_t (&v)
 
 // NRD = digits of a run's start (0: one run; 1: r * rs0; 2: (r mod rad0) * rs0 + (r div rad0) * rs1).
 // The lane's run advances by g per step; its offset is updated incrementally (one carry test).
+// n / d for d in [1, 32] and n < 2^27 by one 64-bit multiply-high: q = (n * ceil(2^32 / d)) >> 32
+// (exact: the excess n * (ceil(2^32/d) - 2^32/d) / 2^32 < 2^-5 <= 1/d); a runtime 32-bit division
+// is ~20 instructions, and column mode needed three per pair
+__constant__ unsigned long long kInv32[33] = {
+    0ull,          4294967296ull, 2147483648ull, 1431655766ull, 1073741824ull, 858993460ull, 715827883ull,
+    613566757ull,  536870912ull,  477218589ull,  429496730ull,  390451573ull,  357913942ull, 330382100ull,
+    306783379ull,  286331154ull,  268435456ull,  252645136ull,  238609295ull,  226050911ull, 214748365ull,
+    204522253ull,  195225787ull,  186737709ull,  178956971ull,  171798692ull,  165191050ull, 159072863ull,
+    153391690ull,  148102321ull,  143165577ull,  138547333ull,  134217728ull};
+__device__ __forceinline__ uint32_t div_le32(uint32_t n, uint32_t d) {
+    return (uint32_t)(((unsigned long long)n * kInv32[d]) >> 32);
+}
+
 template <class Acc, int OPC, int V, int NRD>
 __device__ __forceinline__ void stream_cols(const uint32_t* __restrict__ sb, const QDesc& d, Acc& acc, int lane) {
     static_assert(V == 4 || V == 8, "column mode reads 16-B slots");
     const uint32_t nslot = (uint32_t)d.nslot;
-    const uint32_t g = 32u / nslot;
-    const uint32_t grp = (uint32_t)lane / nslot;
+    const uint32_t g = div_le32(32u, nslot);  // nslot <= 32 in column mode
+    const uint32_t grp = div_le32((uint32_t)lane, nslot);
     const uint32_t R = (uint32_t)d.R;
     const bool act = grp < g && grp < R;
     // idle lanes read the last active lane's slot (same address or the other half of it), so in a
@@ -637,7 +650,7 @@ __device__ __forceinline__ void stream_cols(const uint32_t* __restrict__ sb, con
             }
         }
     };
-    const uint32_t full = (R / g) * g;  // steps in which every group has a run
+    const uint32_t full = div_le32(R, g) * g;  // steps in which every group has a run (R < 2^27: one tile / item)
     uint32_t r0 = 0;
     for (; r0 + 2 * g <= full; r0 += 2 * g) {
         uint32_t v0[V], v1[V];
