@@ -1000,7 +1000,7 @@ def run_cube(args, rank, world, local):
                        "l2": ("no flush: C1's 4 MiB cube is L2-resident by design (flagged)" if args.workload == "C1"
                               else "no flush: cube > L2 (126 MB) and every step reads >> L2"),
                        "accumulation": ("int32 cells, int64 SUM" if dtype == np.int32 else
-                                        ("f32 cells, SUM in fp32 trees of <= 16 cells then f64 (reading R8')"
+                                        ("f32 cells, SUM in fp32 trees (slot trees of up to 256 cells, quads of them; depth <= 10) then f64 (reading R8')"
                                          if tiles_used else
                                          ("f32 cells, SUM in fp32 trees of 8 cells of a brick then f64"
                                           if bricked else "f32 cells, f64 SUM"))),
