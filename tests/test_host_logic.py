@@ -176,3 +176,17 @@ def test_bench_refuses_mismatched_world():
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "1"],
                        capture_output=True, text=True, env=env, timeout=120)
     assert r.returncode != 0 and "WORLD_SIZE=1" in (r.stderr + r.stdout)
+
+
+def test_column_mode_reciprocal_table():
+    """cube.cu's kInv32 (column mode's division-free n / d, d <= 32) holds ceil(2^32 / d), and the
+    multiply-high quotient is exact for every n < 2^27 it is used on (brute force at the edges)."""
+    import os
+    import re
+    src = open(os.path.join(ROOT, "paper_conf_ipps_malikrse12_b200", "csrc", "cube.cu")).read()
+    body = re.search(r"kInv32\[33\] = \{([^}]*)\}", src).group(1)
+    tab = [int(x.strip().rstrip("ul")) for x in body.replace("\n", " ").split(",") if x.strip()]
+    assert tab == [0] + [-(-(1 << 32) // d) for d in range(1, 33)]
+    for d in range(1, 33):
+        for n in list(range(0, 4096)) + [(1 << 27) - k for k in range(1, 4096)]:
+            assert (n * tab[d]) >> 32 == n // d
