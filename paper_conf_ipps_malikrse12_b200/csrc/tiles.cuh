@@ -497,7 +497,7 @@ __device__ __forceinline__ void build_pair_desc(const TGeo& tg, const TDesc& d, 
 // by the producer warp once per tile.
 template <class Acc> struct TreeGeo;  // slot-tree geometry of the tile size of Acc's dtype (below)
 #ifndef OLAP_COL_SLOTS
-#define OLAP_COL_SLOTS 4
+#define OLAP_COL_SLOTS 6
 #endif
 constexpr uint32_t kColSlots = OLAP_COL_SLOTS;  // runs of at most this many slots: column mode on raw cells
 #ifndef OLAP_PAT_MAX_RUNS
@@ -984,7 +984,7 @@ __global__ void __launch_bounds__(kTileThreads, 1)
                 Acc acc;
                 acc.init();
                 if (((h0 + L + 7) >> 3) <= kColSlots) {
-                    // short runs (<= 4 slots): column mode over the raw cells, 8+ runs per step
+                    // short runs (<= kColSlots = 6 slots): column mode over the raw cells, 5+ runs per step
                     QDesc qd;
                     qd.nslot = (h0 + L + 7) >> 3;
                     qd.R = R;
